@@ -1,0 +1,343 @@
+#!/usr/bin/env python
+"""Benchmark: indexing throughput of the B200 indexer on BASELINE.json configs[1]
+(ClueWeb09-shaped synthetic, 1 GiB of raw text per GPU).
+
+One step = one pass of the whole hot path over one batch: index_reset + index_add_stream (1 GiB,
+device-resident) + index_finalize (the final inverted file on the device).  Timed with CUDA events
+on the stream the library launches on, after W warm-up steps, bracketed by barrier + synchronize,
+max over ranks.  Inputs (1 GiB) are larger than L2 (126 MB), so no L2 flush is needed.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config 2]
+
+N > 1 (torchrun): every rank indexes its own 1 GiB document shard (chunk index = rank) into a
+local dictionary; scaling is weak.  ``--impl reference`` times the CPU oracle (the reference arm of
+this tier) on a bounded document prefix of the same workload, on rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import gen  # noqa: E402
+
+METRIC = "indexing throughput, MB/s of raw text (1 MB = 10^6 B)"
+WORKLOAD = {2: "clueweb09-shaped synthetic, 1 GiB per GPU (BASELINE configs[1])"}
+HBM_FALLBACK_GBS = 6650.0
+
+# Algorithmic bytes per launch of each timed kernel, given the chunk's
+# T (text bytes), N (kept tokens), P (postings).
+KERNEL_BYTES = {
+    "tokenize_count": lambda T, N, P: T,                  # read the text once
+    "tokenize_emit": lambda T, N, P: T + 8 * N,           # read text, write (slot u32, doc u32) per token
+    "slot_to_tid": lambda T, N, P: 8 * N,                 # read + write u32 per token
+    "map_rank": lambda T, N, P: 8 * N,                    # read + write u32 per token
+    "sort_hist": lambda T, N, P: 4 * N,                   # read u32 keys
+    "sort_scatter": lambda T, N, P: 16 * N,               # read + write (u32 key, u32 doc) per token
+    "rle_emit": lambda T, N, P: 8 * N + 8 * P,            # read (key, doc), write (docid, tf)
+}
+
+
+def measured_peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy bandwidth)"
+    except Exception:
+        return HBM_FALLBACK_GBS, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "50"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 8:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                smax.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[4:8]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def corpus(cfg_id: int, chunk: int, chunk_bytes: int | None = None):
+    cfg = gen.CONFIGS[cfg_id]
+    if chunk_bytes is not None:
+        cfg = cfg.scaled(chunk_bytes=chunk_bytes)
+    return gen.generate(cfg, chunk=chunk)
+
+
+def oracle_rate(text, doc_off, target_s: float = 8.0):
+    """Time the CPU oracle (single thread, as it stands) on a bounded document prefix."""
+    import oracle
+
+    def run(nbytes):
+        nd = int(np.searchsorted(doc_off, nbytes, side="right")) - 1
+        nd = max(1, min(nd, len(doc_off) - 1))
+        t0 = time.perf_counter()
+        o = oracle.Oracle()
+        o.add(text[: int(doc_off[nd])], doc_off[: nd + 1])
+        o.serialize()
+        dt = time.perf_counter() - t0
+        return int(doc_off[nd]), nd, dt
+
+    b, nd, dt = run(2 << 20)
+    want = int(min(len(text), max(b, b / max(dt, 1e-6) * target_s)))
+    b, nd, dt = run(want)
+    return {"value": b / dt / 1e6, "unit": "MB/s", "cores": 1, "kind": "oracle",
+            "sample": f"first {nd} documents ({b} bytes) of the same corpus, oracle_add + serialize, 1 thread, "
+                      f"{dt:.1f} s"}
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    import oracle
+
+    sample_bytes = 4 << 20
+    text, doc_off = corpus(args.config, 0, chunk_bytes=sample_bytes)
+    nd = len(doc_off) - 1
+
+    def step():
+        o = oracle.Oracle()
+        o.add(text, doc_off)
+        o.serialize()
+        o.close()
+
+    for _ in range(args.warmup):
+        step()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        step()
+    dt = (time.perf_counter() - t0) / args.steps
+    val = len(text) / dt / 1e6
+    line = {
+        "impl": "reference", "metric": METRIC, "value": val, "unit": "MB/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": WORKLOAD.get(args.config, str(args.config)),
+                   "sample": f"{nd} documents, {len(text)} bytes (document prefix of the same generator stream)"},
+        "cpu_baseline": {"value": val, "unit": "MB/s", "cores": 1, "kind": "oracle",
+                         "sample": f"first {nd} documents ({len(text)} B) per step, std::map oracle, 1 thread"},
+        "e2e": {"value": val, "unit": "MB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", type=int, default=2)
+    ap.add_argument("--chunk-bytes", type=int, default=None, help="override bytes per GPU (debug)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    args = ap.parse_args()
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_weij11_b200 as wj
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    text, doc_off = corpus(args.config, rank, args.chunk_bytes)
+    T = len(text)
+    text_h = torch.from_numpy(text).pin_memory()
+    off_h = torch.from_numpy(doc_off.astype(np.int64)).pin_memory()
+    text_d = text_h.cuda()
+    off_d = off_h.cuda()
+    torch.cuda.synchronize()
+
+    ix = wj.Index(device=local, profile=True)
+
+    def step(t, o):
+        ix.reset()
+        ix.add_stream(t, o)
+        ix.finalize()
+
+    for _ in range(args.warmup):
+        step(text_d, off_d)
+    torch.cuda.synchronize()
+    s0 = ix.stats()
+    N, P, V = s0["n_tokens"], s0["n_postings"], s0["n_terms"]
+
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.15)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(args.steps):
+        step(text_d, off_d)
+    e1.record()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    ms = e0.elapsed_time(e1) / args.steps
+    s1 = ix.stats()
+    if world > 1:
+        t = torch.tensor([ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+
+    total_bytes = T * world
+    value = total_bytes / (ms / 1e3) / 1e6
+    launches = (s1["kernel_launches"] - s0["kernel_launches"]) / args.steps
+
+    # roofline of the dominant timed kernel (CUDA events around each launch, same stream)
+    peak, peak_src = measured_peak()
+    kms = {k: s1["kernel_ms"][k] - s0["kernel_ms"][k] for k in wj.KERNELS}
+    kcnt = {k: s1["kernel_count"][k] - s0["kernel_count"][k] for k in wj.KERNELS}
+    dom = max((k for k in KERNEL_BYTES if kcnt.get(k)), key=lambda k: kms[k])
+    per_launch_ms = kms[dom] / kcnt[dom]
+    launches_per_step = kcnt[dom] / args.steps
+    bytes_per_launch = KERNEL_BYTES[dom](T, N, P) if dom not in ("sort_hist", "sort_scatter") else KERNEL_BYTES[dom](T, N, P)
+    achieved = bytes_per_launch / (per_launch_ms / 1e3) / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get(dom)
+        except Exception:
+            traffic = None
+    # whole-step compulsory bytes: T + 8P + sum(len + 28) over terms
+    b_min = T + 8 * P + s1["n_term_bytes"] + 28 * V
+    step_gbs = b_min * world / (ms / 1e3) / 1e9
+
+    phases = {k: (s1["phase_ms"][k] - s0["phase_ms"][k]) / args.steps for k in wj.PHASES}
+    kernels = {k: {"ms_per_step": kms[k] / args.steps, "launches_per_step": kcnt[k] / args.steps} for k in wj.KERNELS}
+
+    # e2e through the public API with host buffers: H2D of the chunk inside, D2H of the whole index
+    e2e = None
+    if args.e2e_steps > 0:
+        ix.reset()
+        ix.add_stream(text_h, off_h)
+        ix.finalize()
+        out_bytes = ix.serialized_size()
+        out_h = torch.empty(out_bytes, dtype=torch.uint8, pin_memory=True)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        f0 = torch.cuda.Event(enable_timing=True)
+        f1 = torch.cuda.Event(enable_timing=True)
+        f0.record()
+        for _ in range(args.e2e_steps):
+            ix.reset()
+            ix.add_stream(text_h, off_h)
+            ix.finalize()
+            ix.serialize_into(out_h.data_ptr(), out_bytes)
+        f1.record()
+        torch.cuda.synchronize()
+        ems = f0.elapsed_time(f1) / args.e2e_steps
+        if world > 1:
+            t = torch.tensor([ems], device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ems = float(t.item())
+        e2e = {"value": total_bytes / (ems / 1e3) / 1e6, "unit": "MB/s", "ms_per_step": ems,
+               "h2d_bytes_per_step": T + 8 * len(doc_off), "d2h_bytes_per_step": out_bytes,
+               "what": "index_add_stream(pinned host text + doc_off) + index_finalize + index_serialize to pinned host"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = oracle_rate(text, doc_off)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "MB/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic (gen/wjgen.cpp seeded generator)",
+            "config": {"workload": WORKLOAD.get(args.config, str(args.config)), "bytes_per_gpu": T,
+                       "docs_per_gpu": len(doc_off) - 1, "tokens_per_gpu": N, "terms_per_gpu": V,
+                       "postings_per_gpu": P, "l2": "no flush: 1 GiB input per step > 126 MB L2",
+                       "parallelism": "single GPU" if world == 1 else f"{world} document shards, local dictionaries"},
+            "mib_per_s": total_bytes / (ms / 1e3) / 2**20,
+            "tokens_per_s": N * world / (ms / 1e3),
+            "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                         "algorithmic_bytes_per_launch": bytes_per_launch, "ms_per_launch": per_launch_ms,
+                         "launches_per_step": launches_per_step},
+            "roofline_step": {"bytes_min": b_min, "achieved": step_gbs, "peak": peak * world, "unit": "GB/s",
+                              "frac": step_gbs / (peak * world),
+                              "def": "B_min = T + 8P + sum(len+28) over terms (SURVEY 8(d)) / step time"},
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": int(round(launches * args.steps)),
+            "gpu_launches_per_step": launches,
+            "clocks": clk,
+            "phases_ms_per_step": phases,
+            "kernels": kernels,
+            "paper_context": "262.76 MB/s end-to-end on ClueWeb09 (2x X5560 + 2x C1060, Table VI); not this workload",
+        }
+        print(json.dumps(line), flush=True)
+    ix.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,1002 @@
+// Engine + C ABI (include/wjindex.h): owns device state, orders the kernels of one chunk and of
+// finalize on the context stream, and turns CUDA errors into wj_status codes.
+#include <algorithm>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/wjindex.h"
+#include "common.cuh"
+#include "dict.cuh"
+#include "postings.cuh"
+#include "radix.cuh"
+#include "scan.cuh"
+#include "tokenize.cuh"
+
+using namespace wj;
+
+namespace {
+
+struct StatusError {
+  int code;
+  std::string msg;
+};
+
+struct DevBuf {
+  void* p = nullptr;
+  size_t cap = 0;  // bytes
+};
+
+struct PhaseRec {
+  int phase;
+  cudaEvent_t a, b;
+  uint64_t launches;
+};
+struct KernelRec {
+  int k;
+  cudaEvent_t a, b;
+};
+
+template <typename T>
+__global__ void k_fill(T* p, uint64_t n, T v) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) p[i] = v;
+}
+
+__global__ void k_update_counts(uint32_t* coll_n, const uint32_t* nlo, const uint32_t* nhi) {
+  const uint32_t b = blockIdx.x * blockDim.x + threadIdx.x;
+  if (b < kCollections) coll_n[b] += nhi[b] - nlo[b];
+}
+
+// doc_off validation: doc_off[0]==0, non-decreasing, doc_off[n]==n_bytes
+__global__ void k_check_docoff(const uint64_t* d, uint64_t n_docs, uint64_t n_bytes, uint32_t* bad) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i > n_docs) return;
+  bool ok = true;
+  if (i == 0) ok = d[0] == 0;
+  else ok = d[i - 1] <= d[i];
+  if (i == n_docs) ok = ok && d[i] == n_bytes;
+  if (!ok) atomicExch(bad, 1u);
+}
+
+struct NonZero64 {
+  const uint64_t* t;
+  __device__ __forceinline__ uint32_t operator()(uint64_t i) const { return t[i] != 0 ? 1u : 0u; }
+};
+struct IsMiss {
+  const uint32_t* t;
+  __device__ __forceinline__ uint32_t operator()(uint64_t i) const { return t[i] == kMiss ? 1u : 0u; }
+};
+struct ArenaSize {
+  const uint32_t* sorted_u;
+  const uint32_t* u_len;
+  const uint32_t* u_bucket;
+  __device__ __forceinline__ uint32_t operator()(uint64_t k) const {
+    const uint32_t u = sorted_u[k];
+    return 1u + u_len[u] - bucket_plen(u_bucket[u]);
+  }
+};
+
+inline unsigned grid_for(uint64_t n, unsigned block) { return (unsigned)((n + block - 1) / block); }
+
+}  // namespace
+
+struct wj_index {
+  int device = 0;
+  int rank = 0, world = 1;
+  cudaStream_t st = nullptr;
+  bool own_stream = false;
+  uint32_t flags = 0;
+  std::string err;
+  bool finalized = false;
+  bool broken = false;
+
+  // counters
+  uint64_t n_docs = 0, n_tokens = 0, n_dropped = 0, n_chunks = 0, launches = 0, syncs = 0;
+  uint64_t unique_last = 0, new_last = 0, n_nodes = 0, height_max = 0;
+  uint32_t V = 0;
+  uint64_t arena_used = 0;
+  uint64_t table_est = 0;
+  uint64_t P = 0, TB = 0;
+
+  // persistent dictionary
+  DevBuf nodes, coll_root, coll_n, coll_base, coll_base2, e_tid, e_bkt, e_tid2, e_bkt2, arena, t_arena, t_cache,
+      t_bucket;
+  // device scalars: [0] tokens, [1] dropped, [2] U, [3] Nnew, [4] arena total, [5] overflow|bad,
+  // [6] tid counter (u32 view), [7] level count, [8] P, [9] TB, [10] bad doc_off
+  DevBuf scal;
+  uint64_t* h_scal = nullptr;  // pinned
+  // token stream (termID, docID) of all chunks
+  DevBuf g_tid, g_doc;
+  // chunk scratch
+  DevBuf text_stage, doc_stage, seg_cnt, table, uid, u_ref, u_len, u_bucket, u_cache, u_key, u_tid, u_rank, midx, nk_key,
+      nk_val, nk_key2, nk_val2, aoff, ns_tid, ns_bucket, ns_rank, nlo, nhi, nbase, lvA[4], lvB[4], child_off, root_idx,
+      scan_scr, hist, hist_scan, dbg_start, dbg_len, dbg_off, dbg_out, dbg_slot, dbg_doc, lexg, qbuf, qres;
+  // finalize
+  DevBuf rank_of, term_at, sk1, sv1, pidx, out_doc, out_tf, post_off, df, cf, term_off, term_bytes;
+  uint32_t* f_key = nullptr;   // sorted keys (term ranks)
+  uint32_t* f_doc = nullptr;   // sorted docIDs
+  // profiling
+  std::vector<PhaseRec> recs;
+  std::vector<cudaEvent_t> ev_pool;
+  size_t ev_used = 0;
+  int cur_phase = -1;
+  uint64_t phase_launch0 = 0;
+  double phase_ms[WJ_PHASE_COUNT] = {0};
+  uint64_t phase_launches[WJ_PHASE_COUNT] = {0};
+  std::vector<KernelRec> krecs;
+  double kernel_ms[WJ_KERNEL_COUNT] = {0};
+  uint64_t kernel_count[WJ_KERNEL_COUNT] = {0};
+  size_t device_bytes = 0;
+
+  // ---------------------------------------------------------------- memory
+  void* grow(DevBuf& b, size_t bytes, bool keep = false, size_t keep_bytes = 0) {
+    if (bytes <= b.cap && b.p) return b.p;
+    size_t nc = std::max(bytes, b.cap + b.cap / 2);
+    nc = (nc + 255) & ~(size_t)255;
+    void* np = nullptr;
+    cudaError_t e = cudaMalloc(&np, nc);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      throw StatusError{WJ_ERR_OOM, "cudaMalloc(" + std::to_string(nc) + ") failed: " + cudaGetErrorString(e)};
+    }
+    if (keep && b.p && keep_bytes) WJ_CUDA_CHECK(cudaMemcpyAsync(np, b.p, keep_bytes, cudaMemcpyDeviceToDevice, st));
+    if (b.p) {
+      WJ_CUDA_CHECK(cudaStreamSynchronize(st));
+      WJ_CUDA_CHECK(cudaFree(b.p));
+      device_bytes -= b.cap;
+    }
+    b.p = np;
+    b.cap = nc;
+    device_bytes += nc;
+    return np;
+  }
+  template <typename T>
+  T* buf(DevBuf& b, uint64_t n) { return (T*)grow(b, std::max<uint64_t>(n, 1) * sizeof(T)); }
+  template <typename T>
+  T* buf_keep(DevBuf& b, uint64_t n, uint64_t used) {
+    return (T*)grow(b, std::max<uint64_t>(n, 1) * sizeof(T), true, used * sizeof(T));
+  }
+  void free_all() {
+    DevBuf* all[] = {&nodes, &coll_root, &coll_n, &coll_base, &coll_base2, &e_tid, &e_bkt, &e_tid2, &e_bkt2, &arena,
+                     &t_arena, &t_cache, &t_bucket, &scal, &g_tid, &g_doc, &text_stage, &doc_stage, &seg_cnt, &table,
+                     &uid, &u_ref, &u_len, &u_bucket, &u_cache, &u_key, &u_tid, &u_rank, &midx, &nk_key, &nk_val,
+                     &nk_key2, &nk_val2, &aoff, &ns_tid, &ns_bucket, &ns_rank, &nlo, &nhi, &nbase, &child_off,
+                     &root_idx, &scan_scr, &hist, &hist_scan, &dbg_start, &dbg_len, &dbg_off, &dbg_out, &dbg_slot,
+                     &dbg_doc, &lexg, &qbuf, &qres, &rank_of, &term_at, &sk1, &sv1, &pidx, &out_doc, &out_tf,
+                     &post_off, &df, &cf, &term_off, &term_bytes};
+    for (DevBuf* b : all) {
+      if (b->p) cudaFree(b->p);
+      b->p = nullptr;
+      b->cap = 0;
+    }
+    for (int i = 0; i < 4; ++i) {
+      if (lvA[i].p) cudaFree(lvA[i].p);
+      if (lvB[i].p) cudaFree(lvB[i].p);
+      lvA[i] = DevBuf{};
+      lvB[i] = DevBuf{};
+    }
+  }
+
+  void* scan_scratch(uint64_t n, size_t elem) {
+    const uint64_t tiles = (n + kScanTile - 1) / kScanTile;
+    return grow(scan_scr, (size_t)(tiles + 2) * elem * 2 + 1024);
+  }
+
+  // ---------------------------------------------------------------- launch bookkeeping
+  void launched(int n = 1) {
+    launches += n;
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) throw CudaError(e, "kernel launch", __FILE__, __LINE__);
+  }
+  void sync() {
+    WJ_CUDA_CHECK(cudaStreamSynchronize(st));
+    ++syncs;
+  }
+  cudaEvent_t ev() {
+    if (ev_used == ev_pool.size()) {
+      cudaEvent_t e;
+      WJ_CUDA_CHECK(cudaEventCreate(&e));
+      ev_pool.push_back(e);
+    }
+    return ev_pool[ev_used++];
+  }
+  void phase(int p) {
+    if (!(flags & WJ_FLAG_PROFILE)) { cur_phase = p; return; }
+    if (cur_phase >= 0) {
+      PhaseRec& r = recs.back();
+      WJ_CUDA_CHECK(cudaEventRecord(r.b, st));
+      r.launches = launches - phase_launch0;
+    }
+    cur_phase = p;
+    if (p >= 0) {
+      PhaseRec r{p, ev(), ev(), 0};
+      WJ_CUDA_CHECK(cudaEventRecord(r.a, st));
+      recs.push_back(r);
+      phase_launch0 = launches;
+    }
+  }
+  // times one launch (or a few) of kernel k with CUDA events when profiling
+  template <class F>
+  void ktime(int k, F&& launch) {
+    if (!(flags & WJ_FLAG_PROFILE)) { launch(); return; }
+    KernelRec r{k, ev(), ev()};
+    WJ_CUDA_CHECK(cudaEventRecord(r.a, st));
+    launch();
+    WJ_CUDA_CHECK(cudaEventRecord(r.b, st));
+    krecs.push_back(r);
+  }
+  void collect_phases() {
+    if (recs.empty() && krecs.empty()) return;
+    if (cur_phase >= 0) phase(-1);
+    sync();
+    for (auto& r : recs) {
+      float ms = 0;
+      WJ_CUDA_CHECK(cudaEventElapsedTime(&ms, r.a, r.b));
+      phase_ms[r.phase] += ms;
+      phase_launches[r.phase] += r.launches;
+    }
+    for (auto& r : krecs) {
+      float ms = 0;
+      WJ_CUDA_CHECK(cudaEventElapsedTime(&ms, r.a, r.b));
+      kernel_ms[r.k] += ms;
+      kernel_count[r.k] += 1;
+    }
+    recs.clear();
+    krecs.clear();
+    ev_used = 0;
+  }
+  uint64_t* dscal() { return (uint64_t*)scal.p; }
+  void readback(int first, int count) {
+    WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + first, dscal() + first, count * sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+    sync();
+  }
+
+  template <typename T, typename F>
+  void scan(F in, uint64_t n, T* out, T* d_total) {
+    void* s = scan_scratch(n, sizeof(T));
+    launched(0);
+    launches += exclusive_scan<T, F>(in, n, out, d_total, s, st);
+    launched(0);
+  }
+
+  // ---------------------------------------------------------------- init / reset
+  void reset_state() {
+    collect_phases();
+    n_docs = n_tokens = n_dropped = n_chunks = 0;
+    unique_last = new_last = n_nodes = height_max = 0;
+    V = 0;
+    arena_used = 0;
+    P = TB = 0;
+    finalized = false;
+    f_key = f_doc = nullptr;
+    cur_phase = -1;
+    uint32_t* cn = buf<uint32_t>(coll_n, kCollections + 1);
+    uint32_t* cb = buf<uint32_t>(coll_base, kCollections + 1);
+    uint32_t* cr = buf<uint32_t>(coll_root, kCollections + 1);
+    WJ_CUDA_CHECK(cudaMemsetAsync(cn, 0, (kCollections + 1) * 4, st));
+    WJ_CUDA_CHECK(cudaMemsetAsync(cb, 0, (kCollections + 1) * 4, st));
+    WJ_CUDA_CHECK(cudaMemsetAsync(cr, 0xFF, (kCollections + 1) * 4, st));
+    buf<uint64_t>(scal, 16);
+    WJ_CUDA_CHECK(cudaMemsetAsync(scal.p, 0, 16 * 8, st));
+    sync();
+  }
+
+  // ---------------------------------------------------------------- chunk staging
+  static bool is_device_ptr(const void* p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+      cudaGetLastError();
+      return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+  }
+
+  void stage(const void* bytes, uint64_t n_bytes, const uint64_t* doc_off, uint64_t nd, const uint8_t** text_d,
+             const uint64_t** off_d) {
+    const bool dev_text = n_bytes == 0 || is_device_ptr(bytes);
+    const bool dev_off = is_device_ptr(doc_off);
+    if (!dev_off) {
+      // host doc_off: validate here (cheap) before copying
+      if (doc_off[0] != 0 || doc_off[nd] != n_bytes) throw StatusError{WJ_ERR_INVALID_ARG, "doc_off[0] must be 0 and doc_off[n_docs] == n_bytes"};
+      for (uint64_t i = 0; i < nd; ++i)
+        if (doc_off[i] > doc_off[i + 1]) throw StatusError{WJ_ERR_INVALID_ARG, "doc_off must be non-decreasing"};
+    }
+    const bool any_host = !dev_text || !dev_off;
+    if (any_host) phase(WJ_PHASE_H2D);
+    if (dev_text && ((uintptr_t)bytes & 15) == 0) {
+      *text_d = (const uint8_t*)bytes;
+    } else {
+      uint8_t* t = buf<uint8_t>(text_stage, n_bytes + 16);
+      if (n_bytes) WJ_CUDA_CHECK(cudaMemcpyAsync(t, bytes, n_bytes, dev_text ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, st));
+      *text_d = t;
+    }
+    if (dev_off) {
+      *off_d = doc_off;
+    } else {
+      uint64_t* o = buf<uint64_t>(doc_stage, nd + 1);
+      WJ_CUDA_CHECK(cudaMemcpyAsync(o, doc_off, (nd + 1) * 8, cudaMemcpyHostToDevice, st));
+      *off_d = o;
+    }
+    uint32_t* bad = (uint32_t*)(dscal() + 10);
+    WJ_CUDA_CHECK(cudaMemsetAsync(bad, 0, 8, st));
+    if (dev_off) {
+      k_check_docoff<<<grid_for(nd + 1, 256), 256, 0, st>>>(*off_d, nd, n_bytes, bad);
+      launched();
+    }
+  }
+
+  // K1 count + scan; returns kept tokens of the chunk (host sync)
+  uint64_t count_tokens(const ChunkView& cv, uint64_t n_segs) {
+    uint32_t* cnt = buf<uint32_t>(seg_cnt, n_segs + 1);
+    const uint64_t warps = (n_segs + kSegsPerWarp - 1) / kSegsPerWarp;
+    const unsigned grid = (unsigned)((warps + kTokWarps - 1) / kTokWarps);
+    WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 1, 0, 8, st));
+    ktime(WJ_KERNEL_TOKENIZE_COUNT, [&] {
+      k_tokenize<false><<<grid, kTokThreads, 0, st>>>(cv, n_segs, cnt, nullptr, EmitOut{}, (unsigned long long*)(dscal() + 1));
+      launched();
+    });
+    scan<uint32_t>(ArrayIn<uint32_t>{cnt}, n_segs, cnt, (uint32_t*)(dscal() + 0));
+    // dscal[0] low 32 bits = tokens; clear the high half first is unnecessary: read as u32
+    readback(0, 2);
+    readback(10, 1);
+    if ((uint32_t)h_scal[10]) throw StatusError{WJ_ERR_INVALID_ARG, "doc_off must start at 0, be non-decreasing and end at n_bytes"};
+    return (uint32_t)h_scal[0];
+  }
+
+  void emit_tokens(const ChunkView& cv, uint64_t n_segs, uint32_t* slot_out, uint32_t* doc_out, uint32_t doc_base,
+                   uint64_t C, uint32_t* dstart, uint32_t* dlen) {
+    uint64_t* tab = buf<uint64_t>(table, C);
+    WJ_CUDA_CHECK(cudaMemsetAsync(tab, 0, C * 8, st));
+    WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 5, 0, 8, st));
+    EmitOut eo;
+    eo.table = tab;
+    eo.mask = (uint32_t)(C - 1);
+    eo.doc_base = doc_base;
+    eo.slot = slot_out;
+    eo.doc = doc_out;
+    eo.dbg_start = dstart;
+    eo.dbg_len = dlen;
+    eo.overflow = (uint32_t*)(dscal() + 5);
+    const uint64_t warps = (n_segs + kSegsPerWarp - 1) / kSegsPerWarp;
+    const unsigned grid = (unsigned)((warps + kTokWarps - 1) / kTokWarps);
+    ktime(WJ_KERNEL_TOKENIZE_EMIT, [&] {
+      k_tokenize<true><<<grid, kTokThreads, 0, st>>>(cv, n_segs, nullptr, (const uint32_t*)seg_cnt.p, eo, nullptr);
+      launched();
+    });
+  }
+
+  static uint64_t pow2_at_least(uint64_t x) {
+    uint64_t c = 1;
+    while (c < x) c <<= 1;
+    return c;
+  }
+
+  // ---------------------------------------------------------------- one chunk
+  void add_chunk(const void* bytes, uint64_t n_bytes, const uint64_t* doc_off_in, uint64_t nd) {
+    if (n_docs + nd > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 documents"};
+    const uint8_t* text = nullptr;
+    const uint64_t* off = nullptr;
+    stage(bytes, n_bytes, doc_off_in, nd, &text, &off);
+    const uint32_t doc_base = (uint32_t)n_docs;
+    ++n_chunks;
+    if (nd == 0 || n_bytes == 0) {
+      n_docs += nd;
+      phase(-1);
+      return;
+    }
+    ChunkView cv{text, n_bytes, off, nd};
+    const uint64_t n_segs = (n_bytes + kSegBytes - 1) / kSegBytes;
+
+    phase(WJ_PHASE_TOKENIZE);
+    const uint64_t Nc = count_tokens(cv, n_segs);
+    n_dropped += h_scal[1];
+    if (n_tokens + Nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 tokens in one index"};
+    uint32_t* gt = buf_keep<uint32_t>(g_tid, n_tokens + Nc, n_tokens);
+    uint32_t* gd = buf_keep<uint32_t>(g_doc, n_tokens + Nc, n_tokens);
+    if (Nc == 0) {
+      n_docs += nd;
+      phase(-1);
+      return;
+    }
+    uint64_t est = std::max<uint64_t>({table_est, Nc / 24, 4096});
+    est = std::min<uint64_t>(est, Nc + 16);
+    uint64_t C = pow2_at_least(2 * est);
+    uint32_t* slot_uid = nullptr;
+    uint64_t U = 0;
+    for (;;) {
+      emit_tokens(cv, n_segs, gt + n_tokens, gd + n_tokens, doc_base, C, nullptr, nullptr);
+      phase(WJ_PHASE_UNIQUE);
+      slot_uid = buf<uint32_t>(uid, C);
+      scan<uint32_t>(NonZero64{(const uint64_t*)table.p}, C, slot_uid, (uint32_t*)(dscal() + 2));
+      WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 2) + 1, 0, 4, st));
+      readback(2, 4);
+      U = (uint32_t)h_scal[2];
+      if (((uint32_t)h_scal[5]) == 0) break;
+      C *= 2;  // probe sequence overflow: retry with a larger table
+      phase(WJ_PHASE_TOKENIZE);
+    }
+    unique_last = U;
+    table_est = (U * 5) / 4;
+
+    // unique terms: first occurrence, Table I bucket, stripped-suffix cache, sort key
+    uint32_t* ur = buf<uint32_t>(u_ref, U);
+    uint32_t* ul = buf<uint32_t>(u_len, U);
+    uint32_t* ub = buf<uint32_t>(u_bucket, U);
+    uint32_t* uc = buf<uint32_t>(u_cache, U);
+    uint64_t* uk = buf<uint64_t>(u_key, U);
+    uint32_t* ut = buf<uint32_t>(u_tid, U);
+    uint32_t* urk = buf<uint32_t>(u_rank, U);
+    k_unique_gather<<<grid_for(C, 256), 256, 0, st>>>((const uint64_t*)table.p, (uint32_t)C, slot_uid, text, ur, ul, ub,
+                                                      uc, uk);
+    launched();
+
+    // K3 probe
+    phase(WJ_PHASE_PROBE);
+    DictView dv{(const Node*)nodes.p, (const uint32_t*)coll_root.p, (const uint32_t*)coll_n.p, (const uint8_t*)arena.p};
+    if (V > 0) {
+      UniqueView uv{text, ur, ul, ub, uc};
+      const unsigned blocks = (unsigned)std::min<uint64_t>((U + 7) / 8, 148ull * 64);
+      ktime(WJ_KERNEL_PROBE, [&] {
+        k_probe<<<blocks, 256, 0, st>>>(dv, uv, (uint32_t)U, ut, urk);
+        launched();
+      });
+    } else {
+      k_fill<uint32_t><<<grid_for(U, 256), 256, 0, st>>>(ut, U, kMiss);
+      k_fill<uint32_t><<<grid_for(U, 256), 256, 0, st>>>(urk, U, 0u);
+      launched(2);
+    }
+
+    // K4 insert
+    phase(WJ_PHASE_INSERT);
+    uint32_t* mi = buf<uint32_t>(midx, U);
+    scan<uint32_t>(IsMiss{ut}, U, mi, (uint32_t*)(dscal() + 3));
+    WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 3) + 1, 0, 4, st));
+    readback(3, 1);
+    const uint64_t Nn = (uint32_t)h_scal[3];
+    new_last = Nn;
+    if (Nn > 0) {
+      if ((uint64_t)V + Nn > 0xFFFFFFFEull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-2 terms"};
+      insert_new(text, U, Nn);
+      phase(WJ_PHASE_REBUILD);
+      rebuild();
+    }
+
+    // termIDs into the stream (the postings input)
+    phase(WJ_PHASE_STREAM);
+    ktime(WJ_KERNEL_SLOT_TO_TID, [&] {
+      k_slot_to_tid<<<grid_for(Nc, 256), 256, 0, st>>>(gt + n_tokens, Nc, slot_uid, ut);
+      launched();
+    });
+    n_tokens += Nc;
+    n_docs += nd;
+    phase(-1);
+  }
+
+  void insert_new(const uint8_t* text, uint64_t U, uint64_t Nn) {
+    uint64_t* kk = buf<uint64_t>(nk_key, Nn);
+    uint32_t* kv = buf<uint32_t>(nk_val, Nn);
+    uint64_t* kk2 = buf<uint64_t>(nk_key2, Nn);
+    uint32_t* kv2 = buf<uint32_t>(nk_val2, Nn);
+    k_miss_compact<<<grid_for(U, 256), 256, 0, st>>>((const uint32_t*)u_tid.p, (const uint32_t*)midx.p,
+                                                     (const uint64_t*)u_key.p, (uint32_t)U, kk, kv);
+    launched();
+    // sort new terms by (collection, suffix): 8-bit LSD over the 63-bit key, then tie runs
+    const size_t hb = radix_hist_bytes(Nn);
+    uint32_t* h1 = (uint32_t*)grow(hist, hb);
+    uint32_t* h2 = (uint32_t*)grow(hist_scan, hb);
+    void* ss = scan_scratch((uint64_t)radix_plan(Nn).ctas * kRsBins, 4);
+    const bool in2 = sort_pairs<uint64_t>(kk, kv, kk2, kv2, Nn, 0, 64, h1, h2, ss, false);
+    uint64_t* sk = in2 ? kk2 : kk;
+    uint32_t* sv = in2 ? kv2 : kv;
+    k_tie_fix<<<grid_for(Nn, 256), 256, 0, st>>>(sk, sv, (uint32_t)Nn, text, (const uint32_t*)u_ref.p,
+                                                 (const uint32_t*)u_len.p);
+    launched();
+    // arena offsets
+    uint32_t* ao = buf<uint32_t>(aoff, Nn);
+    scan<uint32_t>(ArenaSize{sv, (const uint32_t*)u_len.p, (const uint32_t*)u_bucket.p}, Nn, ao,
+                   (uint32_t*)(dscal() + 4));
+    WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 4) + 1, 0, 4, st));
+    readback(4, 1);
+    const uint64_t A = (uint32_t)h_scal[4];
+    if (arena_used + A >= 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "string arena exceeds 4 GiB"};
+    uint8_t* ar = buf_keep<uint8_t>(arena, arena_used + A, arena_used);
+    const uint64_t Vn = (uint64_t)V + Nn;
+    uint32_t* ta = buf_keep<uint32_t>(t_arena, Vn, V);
+    uint32_t* tc = buf_keep<uint32_t>(t_cache, Vn, V);
+    uint32_t* tb = buf_keep<uint32_t>(t_bucket, Vn, V);
+    uint32_t* nt = buf<uint32_t>(ns_tid, Nn);
+    uint32_t* nb = buf<uint32_t>(ns_bucket, Nn);
+    uint32_t* nr = buf<uint32_t>(ns_rank, Nn);
+    uint32_t* counter = (uint32_t*)(dscal() + 6);
+    k_fill<uint32_t><<<1, 1, 0, st>>>(counter, 1, V);
+    launched();
+    k_new_terms<<<grid_for(Nn, 256), 256, 0, st>>>(sv, (uint32_t)Nn, ao, arena_used, text, (const uint32_t*)u_ref.p,
+                                                   (const uint32_t*)u_len.p, (const uint32_t*)u_bucket.p,
+                                                   (const uint32_t*)u_cache.p, (const uint32_t*)u_rank.p,
+                                                   (uint32_t*)u_tid.p, counter, ar, ta, tc, tb, nt, nb, nr);
+    launched();
+    arena_used += A;
+    // merge into the sorted key order E of every collection
+    uint32_t* lo = buf<uint32_t>(nlo, kCollections + 1);
+    uint32_t* hi = buf<uint32_t>(nhi, kCollections + 1);
+    WJ_CUDA_CHECK(cudaMemsetAsync(lo, 0, (kCollections + 1) * 4, st));
+    WJ_CUDA_CHECK(cudaMemsetAsync(hi, 0, (kCollections + 1) * 4, st));
+    k_new_ranges<<<grid_for(Nn, 256), 256, 0, st>>>(nb, (uint32_t)Nn, lo, hi);
+    launched();
+    uint32_t* cb2 = buf<uint32_t>(coll_base2, kCollections + 1);
+    scan<uint32_t>(NewCount{(const uint32_t*)coll_n.p, lo, hi}, kCollections, cb2, cb2 + kCollections);
+    uint32_t* et2 = buf<uint32_t>(e_tid2, Vn);
+    uint32_t* eb2 = buf<uint32_t>(e_bkt2, Vn);
+    k_place_new<<<grid_for(Nn, 256), 256, 0, st>>>(nt, nb, nr, (uint32_t)Nn, lo, cb2, et2, eb2);
+    launched();
+    if (V > 0) {
+      k_place_old<<<grid_for(V, 256), 256, 0, st>>>((const uint32_t*)e_tid.p, (const uint32_t*)e_bkt.p, V,
+                                                    (const uint32_t*)coll_base.p, nr, lo, hi, cb2, et2, eb2);
+      launched();
+    }
+    k_update_counts<<<grid_for(kCollections, 256), 256, 0, st>>>((uint32_t*)coll_n.p, lo, hi);
+    launched();
+    std::swap(e_tid, e_tid2);
+    std::swap(e_bkt, e_bkt2);
+    std::swap(coll_base, coll_base2);
+    V = (uint32_t)Vn;
+  }
+
+  void rebuild() {
+    // level 0: one root per non-empty collection
+    uint32_t* ri = buf<uint32_t>(root_idx, kCollections + 1);
+    scan<uint32_t>(NonEmpty{(const uint32_t*)coll_n.p}, kCollections, ri, (uint32_t*)(dscal() + 7));
+    WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 7) + 1, 0, 4, st));
+    readback(7, 1);
+    uint64_t L = (uint32_t)h_scal[7];
+    // worst case nodes: every non-root node holds >= 15 keys
+    const uint64_t max_nodes = (uint64_t)V / 15 + L + 16;
+    Node* nd = (Node*)grow(nodes, max_nodes * sizeof(Node));
+    DevBuf* cur = lvA;
+    DevBuf* nxt = lvB;
+    auto level = [&](DevBuf* lv, uint64_t n) {
+      return Level{buf<uint32_t>(lv[0], n), buf<uint32_t>(lv[1], n), buf<uint32_t>(lv[2], n), buf<uint32_t>(lv[3], n)};
+    };
+    Level lc = level(cur, L);
+    k_roots<<<grid_for(kCollections, 256), 256, 0, st>>>((const uint32_t*)coll_n.p, ri, (uint32_t*)coll_root.p, lc);
+    launched();
+    uint64_t base = 0;
+    uint32_t depth = 0;
+    while (L > 0) {
+      ++depth;
+      uint32_t* co = buf<uint32_t>(child_off, L + 1);
+      scan<uint32_t>(ChildCount{lc.m, lc.h}, L, co, (uint32_t*)(dscal() + 7));
+      WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 7) + 1, 0, 4, st));
+      readback(7, 1);
+      const uint64_t Ln = (uint32_t)h_scal[7];
+      if (base + L + Ln > max_nodes) throw StatusError{WJ_ERR_CAPACITY, "B-tree node pool overflow (internal)"};
+      Level ln = level(nxt, Ln);
+      lc = level(cur, L);  // (re)fetch pointers: level() may not reallocate cur, but keep it explicit
+      const unsigned blocks = (unsigned)std::min<uint64_t>((L + 7) / 8, 148ull * 64);
+      k_build_level<<<blocks, 256, 0, st>>>(lc, (uint32_t)L, (uint32_t)base, co, (uint32_t)(base + L), ln,
+                                            (const uint32_t*)e_tid.p, (const uint32_t*)coll_base.p,
+                                            (const uint32_t*)t_arena.p, (const uint32_t*)t_cache.p, nd);
+      launched();
+      base += L;
+      L = Ln;
+      std::swap(cur, nxt);
+      lc = ln;
+    }
+    n_nodes = base;
+    height_max = depth;
+  }
+
+  // stable LSD radix sort driver (radix.cuh kernels); timed = token-stream sort
+  template <typename K>
+  bool sort_pairs(K* k0, uint32_t* v0, K* k1, uint32_t* v1, uint64_t n, int begin_bit, int end_bit, uint32_t* h1,
+                  uint32_t* h2, void* ss, bool timed) {
+    if (n <= 1 || end_bit <= begin_bit) return false;
+    const RadixPlan p = radix_plan(n);
+    bool in1 = false;
+    for (int shift = begin_bit; shift < end_bit; shift += 8) {
+      K* ki = in1 ? k1 : k0;
+      uint32_t* vi = in1 ? v1 : v0;
+      K* ko = in1 ? k0 : k1;
+      uint32_t* vo = in1 ? v0 : v1;
+      auto hist_launch = [&] {
+        k_radix_hist<K><<<p.ctas, kRsThreads, 0, st>>>(ki, n, p.per, shift, h1);
+        launched();
+      };
+      if (timed) ktime(WJ_KERNEL_SORT_HIST, hist_launch); else hist_launch();
+      launches += exclusive_scan<uint32_t>(ArrayIn<uint32_t>{h1}, (uint64_t)kRsBins * p.ctas, h2, (uint32_t*)nullptr, ss, st);
+      launched(0);
+      auto scatter_launch = [&] {
+        k_radix_scatter<K><<<p.ctas, kRsThreads, 0, st>>>(ki, vi, ko, vo, n, p.per, shift, h2);
+        launched();
+      };
+      if (timed) ktime(WJ_KERNEL_SORT_SCATTER, scatter_launch); else scatter_launch();
+      in1 = !in1;
+    }
+    return in1;
+  }
+
+  // ---------------------------------------------------------------- finalize
+  void finalize() {
+    const uint64_t N = n_tokens;
+    uint32_t* ro = buf<uint32_t>(rank_of, V);
+    uint32_t* ta = buf<uint32_t>(term_at, V);
+    if (V > 0) {
+      phase(WJ_PHASE_LEXRANK);
+      LexGroups* g = (LexGroups*)grow(lexg, sizeof(LexGroups));
+      k_lex_groups<<<1, 32, 0, st>>>((const uint32_t*)e_tid.p, (const uint32_t*)coll_base.p,
+                                     (const uint32_t*)coll_n.p, (const uint32_t*)t_cache.p, g);
+      launched();
+      k_lexrank<<<grid_for(V, 256), 256, 0, st>>>((const uint32_t*)e_tid.p, (const uint32_t*)e_bkt.p, V,
+                                                  (const uint32_t*)coll_base.p, (const uint32_t*)coll_n.p, g,
+                                                  (const uint8_t*)arena.p, (const uint32_t*)t_arena.p,
+                                                  (const uint32_t*)t_bucket.p, (const uint32_t*)t_cache.p, ro, ta);
+      launched();
+    }
+    uint64_t* po = buf<uint64_t>(post_off, (uint64_t)V + 1);
+    uint32_t* dfp = buf<uint32_t>(df, V);
+    uint64_t* cfp = buf<uint64_t>(cf, V);
+    P = 0;
+    if (N > 0) {
+      phase(WJ_PHASE_SORT);
+      uint32_t* kt = (uint32_t*)g_tid.p;
+      uint32_t* dt = (uint32_t*)g_doc.p;
+      ktime(WJ_KERNEL_MAP_RANK, [&] {
+        k_map_rank<<<grid_for(N, 256), 256, 0, st>>>(kt, N, ro);
+        launched();
+      });
+      uint32_t* k1 = buf<uint32_t>(sk1, N);
+      uint32_t* v1 = buf<uint32_t>(sv1, N);
+      int bits = 0;
+      while (bits < 32 && ((uint64_t)1 << bits) < V) ++bits;
+      const size_t hb = radix_hist_bytes(N);
+      uint32_t* h1 = (uint32_t*)grow(hist, hb);
+      uint32_t* h2 = (uint32_t*)grow(hist_scan, hb);
+      void* ss = scan_scratch((uint64_t)radix_plan(N).ctas * kRsBins, 4);
+      const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, N, 0, bits, h1, h2, ss, true);
+      f_key = in1 ? k1 : kt;
+      f_doc = in1 ? v1 : dt;
+      uint32_t* spare_k = in1 ? kt : k1;  // free N-sized buffers for pstart / tstart
+      uint32_t* spare_v = in1 ? dt : v1;
+
+      phase(WJ_PHASE_POSTINGS);
+      uint32_t* pi = buf<uint32_t>(pidx, N);
+      scan<uint32_t>(NewPosting{f_key, f_doc}, N, pi, (uint32_t*)(dscal() + 8));
+      WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 8) + 1, 0, 4, st));
+      readback(8, 1);
+      P = (uint32_t)h_scal[8];
+      uint32_t* od = buf<uint32_t>(out_doc, P);
+      uint32_t* of = buf<uint32_t>(out_tf, P);
+      ktime(WJ_KERNEL_RLE_EMIT, [&] {
+        k_rle_emit<<<grid_for(N, 256), 256, 0, st>>>(f_key, f_doc, N, pi, od, spare_k, po, spare_v);
+        launched();
+      });
+      k_rle_tf<<<grid_for(P, 256), 256, 0, st>>>(spare_k, P, N, of);
+      launched();
+      k_df_cf<<<grid_for((uint64_t)V + 1, 256), 256, 0, st>>>(po, spare_v, V, P, N, dfp, cfp);
+      launched();
+    } else {
+      WJ_CUDA_CHECK(cudaMemsetAsync(po, 0, 8, st));
+    }
+    phase(WJ_PHASE_DICT);
+    uint64_t* to = buf<uint64_t>(term_off, (uint64_t)V + 1);
+    TB = 0;
+    if (V > 0) {
+      scan<uint64_t>(TermFullLen{ta, (const uint32_t*)t_bucket.p, (const uint32_t*)t_arena.p, (const uint8_t*)arena.p},
+                     V, to, to + V);
+      WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 9, to + V, 8, cudaMemcpyDeviceToHost, st));
+      sync();
+      TB = h_scal[9];
+      uint8_t* tbp = buf<uint8_t>(term_bytes, TB);
+      k_term_bytes<<<grid_for(V, 256), 256, 0, st>>>(ta, V, (const uint32_t*)t_bucket.p, (const uint32_t*)t_arena.p,
+                                                     (const uint8_t*)arena.p, to, tbp);
+      launched();
+    } else {
+      WJ_CUDA_CHECK(cudaMemsetAsync(to, 0, 8, st));
+    }
+    phase(-1);
+    sync();
+    finalized = true;
+  }
+
+  // ---------------------------------------------------------------- serialize
+  uint64_t serialized_size() const {
+    auto pad8 = [](uint64_t x) { return (x + 7) & ~7ull; };
+    return 64 + 8 * ((uint64_t)V + 1) + pad8(TB) + pad8(4ull * V) + 8ull * V + 8 * ((uint64_t)V + 1) + pad8(4 * P) +
+           pad8(4 * P);
+  }
+  void serialize(uint8_t* out) {
+    auto pad8 = [](uint64_t x) { return (x + 7) & ~7ull; };
+    uint64_t hdr[8];
+    memcpy(hdr, "WJINV001", 8);
+    hdr[1] = n_docs; hdr[2] = n_tokens; hdr[3] = n_dropped; hdr[4] = V; hdr[5] = P; hdr[6] = TB; hdr[7] = 0;
+    memcpy(out, hdr, 64);
+    uint64_t p = 64;
+    auto d2h = [&](const void* src, uint64_t bytes, uint64_t padded) {
+      if (bytes) WJ_CUDA_CHECK(cudaMemcpyAsync(out + p, src, bytes, cudaMemcpyDeviceToHost, st));
+      if (padded > bytes) memset(out + p + bytes, 0, padded - bytes);
+      p += padded;
+    };
+    d2h(term_off.p, 8 * ((uint64_t)V + 1), 8 * ((uint64_t)V + 1));
+    d2h(term_bytes.p, TB, pad8(TB));
+    d2h(df.p, 4ull * V, pad8(4ull * V));
+    d2h(cf.p, 8ull * V, 8ull * V);
+    d2h(post_off.p, 8 * ((uint64_t)V + 1), 8 * ((uint64_t)V + 1));
+    d2h(out_doc.p, 4 * P, pad8(4 * P));
+    d2h(out_tf.p, 4 * P, pad8(4 * P));
+    sync();
+  }
+};
+
+// ====================================================================== C ABI
+namespace {
+
+template <class F>
+int guarded(wj_index* ix, F&& f) {
+  try {
+    if (ix->broken) {
+      ix->err = "context unusable after an earlier CUDA error";
+      return WJ_ERR_CUDA;
+    }
+    WJ_CUDA_CHECK(cudaSetDevice(ix->device));
+    return f();
+  } catch (const StatusError& e) {
+    ix->err = e.msg;
+    return e.code;
+  } catch (const CudaError& e) {
+    ix->err = std::string("CUDA error ") + cudaGetErrorString(e.err) + " at " + e.file + ":" + std::to_string(e.line) +
+              " (" + e.expr + ")";
+    if (e.err == cudaErrorMemoryAllocation) return WJ_ERR_OOM;
+    ix->broken = true;
+    return WJ_ERR_CUDA;
+  } catch (const std::bad_alloc&) {
+    ix->err = "host allocation failed";
+    return WJ_ERR_OOM;
+  }
+}
+
+thread_local std::string g_init_err;
+
+}  // namespace
+
+extern "C" {
+
+int index_init(wj_index** out, const wj_config* cfg) {
+  if (!out || !cfg) return WJ_ERR_INVALID_ARG;
+  *out = nullptr;
+  if (cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~WJ_FLAG_PROFILE) || cfg->reserved) {
+    g_init_err = "invalid config";
+    return WJ_ERR_INVALID_ARG;
+  }
+  if (cfg->world > 1) {
+    g_init_err = "world > 1 is not supported by this build";
+    return WJ_ERR_INVALID_ARG;
+  }
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    g_init_err = "no CUDA device";
+    return WJ_ERR_CUDA;
+  }
+  if (cfg->device < 0 || cfg->device >= ndev) {
+    g_init_err = "bad device ordinal";
+    return WJ_ERR_INVALID_ARG;
+  }
+  wj_index* ix = new (std::nothrow) wj_index();
+  if (!ix) return WJ_ERR_OOM;
+  ix->device = cfg->device;
+  ix->rank = cfg->rank;
+  ix->world = cfg->world;
+  ix->flags = cfg->flags;
+  int rc = guarded(ix, [&]() {
+    if (cfg->stream) {
+      ix->st = (cudaStream_t)cfg->stream;
+    } else {
+      WJ_CUDA_CHECK(cudaStreamCreateWithFlags(&ix->st, cudaStreamNonBlocking));
+      ix->own_stream = true;
+    }
+    WJ_CUDA_CHECK(cudaHostAlloc(&ix->h_scal, 16 * sizeof(uint64_t), cudaHostAllocDefault));
+    ix->reset_state();
+    return WJ_OK;
+  });
+  if (rc != WJ_OK) {
+    g_init_err = ix->err;
+    index_destroy(ix);
+    return rc;
+  }
+  *out = ix;
+  return WJ_OK;
+}
+
+int index_add_stream(wj_index* ix, const void* bytes, uint64_t n_bytes, const uint64_t* doc_off, uint64_t n_docs) {
+  if (!ix) return WJ_ERR_INVALID_ARG;
+  return guarded(ix, [&]() {
+    if (ix->finalized) throw StatusError{WJ_ERR_STATE, "index_add_stream after index_finalize"};
+    if (!doc_off || (n_bytes && !bytes)) throw StatusError{WJ_ERR_INVALID_ARG, "NULL bytes or doc_off"};
+    if (n_bytes >= 0xFFFFFFFFull) throw StatusError{WJ_ERR_INVALID_ARG, "n_bytes must be < 2^32 per call"};
+    if (n_docs == 0 && n_bytes != 0) throw StatusError{WJ_ERR_INVALID_ARG, "n_bytes > 0 with no documents"};
+    ix->add_chunk(bytes, n_bytes, doc_off, n_docs);
+    return WJ_OK;
+  });
+}
+
+int index_finalize(wj_index* ix) {
+  if (!ix) return WJ_ERR_INVALID_ARG;
+  return guarded(ix, [&]() {
+    if (ix->finalized) throw StatusError{WJ_ERR_STATE, "index_finalize called twice"};
+    ix->finalize();
+    return WJ_OK;
+  });
+}
+
+int index_read_postings(wj_index* ix, const uint8_t* term, uint32_t len, uint32_t* docids, uint32_t* tfs, uint64_t cap,
+                        uint64_t* n_out) {
+  if (!ix || !n_out || (!term && len)) return WJ_ERR_INVALID_ARG;
+  return guarded(ix, [&]() {
+    if (!ix->finalized) throw StatusError{WJ_ERR_STATE, "index_read_postings before index_finalize"};
+    *n_out = 0;
+    if (len == 0 || len > kMaxTermLen || ix->V == 0) return (int)WJ_NOT_FOUND;
+    for (uint32_t i = 0; i < len; ++i) {  // only token bytes can be terms (reading S1)
+      const uint8_t c = term[i];
+      const bool tok = (c >= '0' && c <= '9') || (c >= 'A' && c <= 'Z') || (c >= 'a' && c <= 'z') || c >= 0x80;
+      if (!tok) return (int)WJ_NOT_FOUND;
+    }
+    uint8_t* q = (uint8_t*)ix->grow(ix->qbuf, 512);
+    QueryResult* r = (QueryResult*)ix->grow(ix->qres, sizeof(QueryResult));
+    WJ_CUDA_CHECK(cudaMemcpyAsync(q, term, len, cudaMemcpyHostToDevice, ix->st));
+    DictView dv{(const Node*)ix->nodes.p, (const uint32_t*)ix->coll_root.p, (const uint32_t*)ix->coll_n.p,
+                (const uint8_t*)ix->arena.p};
+    k_query<<<1, 32, 0, ix->st>>>(dv, q, len, (const uint32_t*)ix->rank_of.p, (const uint64_t*)ix->post_off.p, r);
+    ix->launched();
+    QueryResult h;
+    WJ_CUDA_CHECK(cudaMemcpyAsync(&h, r, sizeof(h), cudaMemcpyDeviceToHost, ix->st));
+    ix->sync();
+    if (h.tid == kMiss) return (int)WJ_NOT_FOUND;
+    const uint64_t df = h.hi - h.lo;
+    *n_out = df;
+    if (cap < df) return (int)WJ_ERR_BUFFER_TOO_SMALL;
+    if (df && (!docids || !tfs)) throw StatusError{WJ_ERR_INVALID_ARG, "NULL output arrays"};
+    if (df) {
+      WJ_CUDA_CHECK(cudaMemcpyAsync(docids, (const uint32_t*)ix->out_doc.p + h.lo, df * 4, cudaMemcpyDeviceToHost, ix->st));
+      WJ_CUDA_CHECK(cudaMemcpyAsync(tfs, (const uint32_t*)ix->out_tf.p + h.lo, df * 4, cudaMemcpyDeviceToHost, ix->st));
+      ix->sync();
+    }
+    return (int)WJ_OK;
+  });
+}
+
+int index_serialize(wj_index* ix, uint8_t* buf, uint64_t cap, uint64_t* n_out) {
+  if (!ix || !n_out) return WJ_ERR_INVALID_ARG;
+  return guarded(ix, [&]() {
+    if (!ix->finalized) throw StatusError{WJ_ERR_STATE, "index_serialize before index_finalize"};
+    const uint64_t n = ix->serialized_size();
+    *n_out = n;
+    if (!buf) return (int)WJ_OK;
+    if (cap < n) return (int)WJ_ERR_BUFFER_TOO_SMALL;
+    ix->serialize(buf);
+    return (int)WJ_OK;
+  });
+}
+
+int index_stats(wj_index* ix, wj_stats* out) {
+  if (!ix || !out) return WJ_ERR_INVALID_ARG;
+  return guarded(ix, [&]() {
+    ix->collect_phases();
+    ix->sync();
+    memset(out, 0, sizeof(*out));
+    out->n_docs = ix->n_docs;
+    out->n_tokens = ix->n_tokens;
+    out->n_dropped = ix->n_dropped;
+    out->n_terms = ix->V;
+    out->n_postings = ix->P;
+    out->n_term_bytes = ix->TB;
+    out->n_chunks = ix->n_chunks;
+    out->kernel_launches = ix->launches;
+    out->host_syncs = ix->syncs;
+    out->unique_terms_last = ix->unique_last;
+    out->new_terms_last = ix->new_last;
+    out->btree_nodes = ix->n_nodes;
+    out->btree_height_max = ix->height_max;
+    out->exchange_bytes = 0;
+    out->device_bytes = ix->device_bytes;
+    for (int i = 0; i < WJ_PHASE_COUNT; ++i) {
+      out->phase_ms[i] = ix->phase_ms[i];
+      out->phase_launches[i] = ix->phase_launches[i];
+    }
+    for (int i = 0; i < WJ_KERNEL_COUNT; ++i) {
+      out->kernel_ms[i] = ix->kernel_ms[i];
+      out->kernel_count[i] = ix->kernel_count[i];
+    }
+    return (int)WJ_OK;
+  });
+}
+
+int index_reset(wj_index* ix) {
+  if (!ix) return WJ_ERR_INVALID_ARG;
+  return guarded(ix, [&]() {
+    ix->reset_state();
+    return (int)WJ_OK;
+  });
+}
+
+int index_debug_tokens(wj_index* ix, const void* bytes, uint64_t n_bytes, const uint64_t* doc_off, uint64_t n_docs,
+                       uint32_t doc_base, uint8_t* out, uint64_t cap, uint64_t* n_out) {
+  if (!ix || !n_out || !doc_off) return WJ_ERR_INVALID_ARG;
+  return guarded(ix, [&]() {
+    if (n_bytes >= 0xFFFFFFFFull) throw StatusError{WJ_ERR_INVALID_ARG, "n_bytes must be < 2^32"};
+    *n_out = 0;
+    if (n_docs == 0 || n_bytes == 0) return (int)WJ_OK;
+    const uint8_t* text = nullptr;
+    const uint64_t* off = nullptr;
+    ix->stage(bytes, n_bytes, doc_off, n_docs, &text, &off);
+    ChunkView cv{text, n_bytes, off, n_docs};
+    const uint64_t n_segs = (n_bytes + kSegBytes - 1) / kSegBytes;
+    const uint64_t Nc = ix->count_tokens(cv, n_segs);
+    if (Nc == 0) return (int)WJ_OK;
+    uint32_t* sl = ix->buf<uint32_t>(ix->dbg_slot, Nc);
+    uint32_t* dd = ix->buf<uint32_t>(ix->dbg_doc, Nc);
+    uint32_t* ds = ix->buf<uint32_t>(ix->dbg_start, Nc);
+    uint32_t* dl = ix->buf<uint32_t>(ix->dbg_len, Nc);
+    uint64_t C = wj_index::pow2_at_least(2 * Nc + 16);
+    ix->emit_tokens(cv, n_segs, sl, dd, doc_base, C, ds, dl);
+    uint64_t* doff = ix->buf<uint64_t>(ix->dbg_off, Nc + 1);
+    ix->scan<uint64_t>(DumpSize{dl}, Nc, doff, doff + Nc);
+    WJ_CUDA_CHECK(cudaMemcpyAsync(ix->h_scal + 9, doff + Nc, 8, cudaMemcpyDeviceToHost, ix->st));
+    ix->sync();
+    const uint64_t total = ix->h_scal[9];
+    *n_out = total;
+    if (!out) return (int)WJ_OK;
+    if (cap < total) return (int)WJ_ERR_BUFFER_TOO_SMALL;
+    uint8_t* dbo = ix->buf<uint8_t>(ix->dbg_out, total);
+    k_dump_tokens<<<grid_for(Nc, 256), 256, 0, ix->st>>>(text, ds, dl, dd, Nc, doff, dbo);
+    ix->launched();
+    WJ_CUDA_CHECK(cudaMemcpyAsync(out, dbo, total, cudaMemcpyDeviceToHost, ix->st));
+    ix->sync();
+    return (int)WJ_OK;
+  });
+}
+
+int index_debug_btree(wj_index* ix, void* nodes, uint64_t node_cap, uint64_t* n_nodes, uint32_t* collections,
+                      uint8_t* arena, uint64_t arena_cap, uint64_t* arena_bytes) {
+  if (!ix || !n_nodes || !arena_bytes) return WJ_ERR_INVALID_ARG;
+  return guarded(ix, [&]() {
+    ix->sync();
+    *n_nodes = ix->n_nodes;
+    *arena_bytes = ix->arena_used;
+    if (nodes) {
+      if (node_cap < ix->n_nodes) return (int)WJ_ERR_BUFFER_TOO_SMALL;
+      if (ix->n_nodes) WJ_CUDA_CHECK(cudaMemcpy(nodes, ix->nodes.p, ix->n_nodes * sizeof(Node), cudaMemcpyDeviceToHost));
+    }
+    if (collections) {
+      std::vector<uint32_t> r(kCollections), n(kCollections);
+      WJ_CUDA_CHECK(cudaMemcpy(r.data(), ix->coll_root.p, kCollections * 4, cudaMemcpyDeviceToHost));
+      WJ_CUDA_CHECK(cudaMemcpy(n.data(), ix->coll_n.p, kCollections * 4, cudaMemcpyDeviceToHost));
+      for (uint32_t b = 0; b < kCollections; ++b) {
+        collections[3 * b] = r[b];
+        collections[3 * b + 1] = n[b];
+        collections[3 * b + 2] = height_of(n[b]);
+      }
+    }
+    if (arena) {
+      if (arena_cap < ix->arena_used) return (int)WJ_ERR_BUFFER_TOO_SMALL;
+      if (ix->arena_used) WJ_CUDA_CHECK(cudaMemcpy(arena, ix->arena.p, ix->arena_used, cudaMemcpyDeviceToHost));
+    }
+    return (int)WJ_OK;
+  });
+}
+
+const char* index_last_error(const wj_index* ix) { return ix ? ix->err.c_str() : g_init_err.c_str(); }
+
+void index_destroy(wj_index* ix) {
+  if (!ix) return;
+  cudaSetDevice(ix->device);
+  if (ix->st) cudaStreamSynchronize(ix->st);
+  ix->free_all();
+  for (auto e : ix->ev_pool) cudaEventDestroy(e);
+  if (ix->h_scal) cudaFreeHost(ix->h_scal);
+  if (ix->own_stream && ix->st) cudaStreamDestroy(ix->st);
+  delete ix;
+}
+
+}  // extern "C"
