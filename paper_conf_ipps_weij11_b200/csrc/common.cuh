@@ -30,6 +30,12 @@ struct alignas(128) Node {
 static_assert(sizeof(Node) == 512, "Table II: a B-tree node is 512 bytes");
 static_assert(4 + 31 * 4 + 4 + 31 * 4 + 32 * 4 + 31 * 4 + 4 == 512, "Table II field sizes");
 
+// Chunk-local term table slot (K1 emit): 16 bytes, claimed once by CAS on meta.
+struct __align__(16) Slot {
+  unsigned long long meta;  // bits 0-31 first-occurrence offset, 32-39 length, 40-63 hash tag; 0 = empty
+  unsigned long long pfx;   // first 8 folded bytes (little-endian, zero padded); 0 until published
+};
+
 __host__ __device__ inline uint32_t ceil_div32(uint64_t a, uint32_t b) { return (uint32_t)((a + b - 1) / b); }
 
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }

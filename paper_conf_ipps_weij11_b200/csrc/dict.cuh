@@ -191,12 +191,12 @@ __global__ void k_probe(DictView dv, UniqueView uv, uint32_t U, uint32_t* tid_ou
 }
 
 // unique gather: occupied slot i -> unique index uid[i]; term info from the first occurrence
-__global__ void k_unique_gather(const uint64_t* table, uint32_t C, const uint32_t* uid, const uint8_t* text,
+__global__ void k_unique_gather(const Slot* table, uint32_t C, const uint32_t* uid, const uint8_t* text,
                                 uint32_t* u_ref, uint32_t* u_len, uint32_t* u_bucket, uint32_t* u_cache,
                                 uint64_t* u_key) {
   const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= C) return;
-  const uint64_t e = table[i];
+  const uint64_t e = table[i].meta;
   if (e == 0) return;
   const uint32_t u = uid[i];
   const uint32_t ref = (uint32_t)e, len = (uint32_t)(e >> 32) & 0xFFu;

@@ -60,9 +60,9 @@ __global__ void k_check_docoff(const uint64_t* d, uint64_t n_docs, uint64_t n_by
   if (!ok) atomicExch(bad, 1u);
 }
 
-struct NonZero64 {
-  const uint64_t* t;
-  __device__ __forceinline__ uint32_t operator()(uint64_t i) const { return t[i] != 0 ? 1u : 0u; }
+struct NonZeroSlot {
+  const Slot* t;
+  __device__ __forceinline__ uint32_t operator()(uint64_t i) const { return t[i].meta != 0 ? 1u : 0u; }
 };
 struct IsMiss {
   const uint32_t* t;
@@ -112,7 +112,7 @@ struct wj_index {
   // chunk scratch
   DevBuf text_stage, doc_stage, seg_cnt, table, uid, u_ref, u_len, u_bucket, u_cache, u_key, u_tid, u_rank, midx, nk_key,
       nk_val, nk_key2, nk_val2, aoff, ns_tid, ns_bucket, ns_rank, nlo, nhi, nbase, lvA[4], lvB[4], child_off, root_idx,
-      scan_scr, hist, hist_scan, dbg_start, dbg_len, dbg_off, dbg_out, dbg_slot, dbg_doc, lexg, qbuf, qres;
+      scan_scr, hist, hist_scan, os_hist, os_look, os_ctr, kstart, dbg_start, dbg_len, dbg_off, dbg_out, dbg_slot, dbg_doc, lexg, qbuf, qres;
   // finalize
   DevBuf rank_of, term_at, sk1, sv1, pidx, out_doc, out_tf, post_off, df, cf, term_off, term_bytes;
   uint32_t* f_key = nullptr;   // sorted keys (term ranks)
@@ -163,7 +163,7 @@ struct wj_index {
                      &t_arena, &t_cache, &t_bucket, &scal, &g_tid, &g_doc, &text_stage, &doc_stage, &seg_cnt, &table,
                      &uid, &u_ref, &u_len, &u_bucket, &u_cache, &u_key, &u_tid, &u_rank, &midx, &nk_key, &nk_val,
                      &nk_key2, &nk_val2, &aoff, &ns_tid, &ns_bucket, &ns_rank, &nlo, &nhi, &nbase, &child_off,
-                     &root_idx, &scan_scr, &hist, &hist_scan, &dbg_start, &dbg_len, &dbg_off, &dbg_out, &dbg_slot,
+                     &root_idx, &scan_scr, &hist, &hist_scan, &os_hist, &os_look, &os_ctr, &kstart, &dbg_start, &dbg_len, &dbg_off, &dbg_out, &dbg_slot,
                      &dbg_doc, &lexg, &qbuf, &qres, &rank_of, &term_at, &sk1, &sv1, &pidx, &out_doc, &out_tf,
                      &post_off, &df, &cf, &term_off, &term_bytes};
     for (DevBuf* b : all) {
@@ -329,16 +329,18 @@ struct wj_index {
 
   // K1 count + scan; returns kept tokens of the chunk (host sync)
   uint64_t count_tokens(const ChunkView& cv, uint64_t n_segs) {
-    uint32_t* cnt = buf<uint32_t>(seg_cnt, n_segs + 1);
-    const uint64_t warps = (n_segs + kSegsPerWarp - 1) / kSegsPerWarp;
-    const unsigned grid = (unsigned)((warps + kTokWarps - 1) / kTokWarps);
+    const uint64_t ranges = (n_segs + kSegsPerWarp - 1) / kSegsPerWarp;
+    const unsigned grid = (unsigned)((ranges + kTokWarps - 1) / kTokWarps);
+    uint32_t* cnt = buf<uint32_t>(seg_cnt, ranges + 1);
+    uint64_t* ks = buf<uint64_t>(kstart, ranges);
+    k_warp_kstart<<<grid_for(ranges, 256), 256, 0, st>>>(cv, ranges, ks);
+    launched();
     WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 1, 0, 8, st));
     ktime(WJ_KERNEL_TOKENIZE_COUNT, [&] {
-      k_tokenize<false><<<grid, kTokThreads, 0, st>>>(cv, n_segs, cnt, nullptr, EmitOut{}, (unsigned long long*)(dscal() + 1));
+      k_tok_count<<<grid, kTokThreads, 0, st>>>(cv, n_segs, ks, cnt, (unsigned long long*)(dscal() + 1));
       launched();
     });
-    scan<uint32_t>(ArrayIn<uint32_t>{cnt}, n_segs, cnt, (uint32_t*)(dscal() + 0));
-    // dscal[0] low 32 bits = tokens; clear the high half first is unnecessary: read as u32
+    scan<uint32_t>(ArrayIn<uint32_t>{cnt}, ranges, cnt, (uint32_t*)(dscal() + 0));
     readback(0, 2);
     readback(10, 1);
     if ((uint32_t)h_scal[10]) throw StatusError{WJ_ERR_INVALID_ARG, "doc_off must start at 0, be non-decreasing and end at n_bytes"};
@@ -347,8 +349,8 @@ struct wj_index {
 
   void emit_tokens(const ChunkView& cv, uint64_t n_segs, uint32_t* slot_out, uint32_t* doc_out, uint32_t doc_base,
                    uint64_t C, uint32_t* dstart, uint32_t* dlen) {
-    uint64_t* tab = buf<uint64_t>(table, C);
-    WJ_CUDA_CHECK(cudaMemsetAsync(tab, 0, C * 8, st));
+    Slot* tab = buf<Slot>(table, C);
+    WJ_CUDA_CHECK(cudaMemsetAsync(tab, 0, C * sizeof(Slot), st));
     WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 5, 0, 8, st));
     EmitOut eo;
     eo.table = tab;
@@ -359,10 +361,10 @@ struct wj_index {
     eo.dbg_start = dstart;
     eo.dbg_len = dlen;
     eo.overflow = (uint32_t*)(dscal() + 5);
-    const uint64_t warps = (n_segs + kSegsPerWarp - 1) / kSegsPerWarp;
-    const unsigned grid = (unsigned)((warps + kTokWarps - 1) / kTokWarps);
+    const uint64_t ranges = (n_segs + kSegsPerWarp - 1) / kSegsPerWarp;
+    const unsigned grid = (unsigned)((ranges + kTokWarps - 1) / kTokWarps);
     ktime(WJ_KERNEL_TOKENIZE_EMIT, [&] {
-      k_tokenize<true><<<grid, kTokThreads, 0, st>>>(cv, n_segs, nullptr, (const uint32_t*)seg_cnt.p, eo, nullptr);
+      k_tok_emit<<<grid, kTokThreads, 0, st>>>(cv, n_segs, (const uint64_t*)kstart.p, (const uint32_t*)seg_cnt.p, eo);
       launched();
     });
   }
@@ -400,16 +402,18 @@ struct wj_index {
       phase(-1);
       return;
     }
-    uint64_t est = std::max<uint64_t>({table_est, Nc / 24, 4096});
+    // capacity ~1.5-3x the expected unique terms (U/N ~ 1/30 on Zipf text; the next chunk uses
+    // the last U); a probe-sequence overflow retries with a doubled table
+    uint64_t est = std::max<uint64_t>({table_est, Nc / 32, 4096});
     est = std::min<uint64_t>(est, Nc + 16);
-    uint64_t C = pow2_at_least(2 * est);
+    uint64_t C = pow2_at_least(est + est / 2);
     uint32_t* slot_uid = nullptr;
     uint64_t U = 0;
     for (;;) {
       emit_tokens(cv, n_segs, gt + n_tokens, gd + n_tokens, doc_base, C, nullptr, nullptr);
       phase(WJ_PHASE_UNIQUE);
       slot_uid = buf<uint32_t>(uid, C);
-      scan<uint32_t>(NonZero64{(const uint64_t*)table.p}, C, slot_uid, (uint32_t*)(dscal() + 2));
+      scan<uint32_t>(NonZeroSlot{(const Slot*)table.p}, C, slot_uid, (uint32_t*)(dscal() + 2));
       WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 2) + 1, 0, 4, st));
       readback(2, 4);
       U = (uint32_t)h_scal[2];
@@ -428,7 +432,7 @@ struct wj_index {
     uint64_t* uk = buf<uint64_t>(u_key, U);
     uint32_t* ut = buf<uint32_t>(u_tid, U);
     uint32_t* urk = buf<uint32_t>(u_rank, U);
-    k_unique_gather<<<grid_for(C, 256), 256, 0, st>>>((const uint64_t*)table.p, (uint32_t)C, slot_uid, text, ur, ul, ub,
+    k_unique_gather<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, (uint32_t)C, slot_uid, text, ur, ul, ub,
                                                       uc, uk);
     launched();
 
@@ -483,11 +487,7 @@ struct wj_index {
                                                      (const uint64_t*)u_key.p, (uint32_t)U, kk, kv);
     launched();
     // sort new terms by (collection, suffix): 8-bit LSD over the 63-bit key, then tie runs
-    const size_t hb = radix_hist_bytes(Nn);
-    uint32_t* h1 = (uint32_t*)grow(hist, hb);
-    uint32_t* h2 = (uint32_t*)grow(hist_scan, hb);
-    void* ss = scan_scratch((uint64_t)radix_plan(Nn).ctas * kRsBins, 4);
-    const bool in2 = sort_pairs<uint64_t>(kk, kv, kk2, kv2, Nn, 0, 64, h1, h2, ss, false);
+    const bool in2 = sort_pairs<uint64_t>(kk, kv, kk2, kv2, Nn, 0, 63, nullptr, false);
     uint64_t* sk = in2 ? kk2 : kk;
     uint32_t* sv = in2 ? kv2 : kv;
     k_tie_fix<<<grid_for(Nn, 256), 256, 0, st>>>(sk, sv, (uint32_t)Nn, text, (const uint32_t*)u_ref.p,
@@ -588,30 +588,41 @@ struct wj_index {
     height_max = depth;
   }
 
-  // stable LSD radix sort driver (radix.cuh kernels); timed = token-stream sort
+  // stable LSD radix sort driver: onesweep (radix.cuh).  rank_of != nullptr maps keys first.
   template <typename K>
-  bool sort_pairs(K* k0, uint32_t* v0, K* k1, uint32_t* v1, uint64_t n, int begin_bit, int end_bit, uint32_t* h1,
-                  uint32_t* h2, void* ss, bool timed) {
-    if (n <= 1 || end_bit <= begin_bit) return false;
-    const RadixPlan p = radix_plan(n);
+  bool sort_pairs(K* k0, uint32_t* v0, K* k1, uint32_t* v1, uint64_t n, int begin_bit, int end_bit,
+                  const uint32_t* rank_of, bool timed) {
+    if (n == 0) return false;
+    const int passes = end_bit > begin_bit ? (end_bit - begin_bit + 7) / 8 : 0;
+    if (n == 1 && !rank_of) return false;
+    uint32_t* gh = buf<uint32_t>(os_hist, (uint64_t)std::max(passes, 1) * 256);
+    WJ_CUDA_CHECK(cudaMemsetAsync(gh, 0, (size_t)std::max(passes, 1) * 256 * 4, st));
+    const unsigned hb = (unsigned)std::min<uint64_t>((n + 255) / 256, 148ull * 8);
+    auto hist_launch = [&] {
+      k_os_hist<K><<<hb, 256, 0, st>>>(k0, n, begin_bit, passes, rank_of, gh);
+      launched();
+    };
+    if (timed) ktime(WJ_KERNEL_SORT_HIST, hist_launch); else hist_launch();
+    if (passes == 0 || n == 1) return false;
+    k_os_hist_scan<<<passes, 256, 0, st>>>(gh);
+    launched();
+    const uint64_t tiles = (n + kOsTile - 1) / kOsTile;
+    uint64_t* lk = buf<uint64_t>(os_look, (uint64_t)passes * tiles * 256);
+    uint32_t* ctr = buf<uint32_t>(os_ctr, passes);
+    WJ_CUDA_CHECK(cudaMemsetAsync(lk, 0, (size_t)passes * tiles * 256 * 8, st));
+    WJ_CUDA_CHECK(cudaMemsetAsync(ctr, 0, (size_t)passes * 4, st));
     bool in1 = false;
-    for (int shift = begin_bit; shift < end_bit; shift += 8) {
+    for (int p = 0; p < passes; ++p) {
       K* ki = in1 ? k1 : k0;
       uint32_t* vi = in1 ? v1 : v0;
       K* ko = in1 ? k0 : k1;
       uint32_t* vo = in1 ? v0 : v1;
-      auto hist_launch = [&] {
-        k_radix_hist<K><<<p.ctas, kRsThreads, 0, st>>>(ki, n, p.per, shift, h1);
+      auto pass_launch = [&] {
+        k_os_pass<K><<<(unsigned)tiles, kOsThreads, os_smem_bytes<K>(), st>>>(
+            ki, vi, ko, vo, n, begin_bit + 8 * p, gh + 256 * p, lk + (uint64_t)p * tiles * 256, ctr + p);
         launched();
       };
-      if (timed) ktime(WJ_KERNEL_SORT_HIST, hist_launch); else hist_launch();
-      launches += exclusive_scan<uint32_t>(ArrayIn<uint32_t>{h1}, (uint64_t)kRsBins * p.ctas, h2, (uint32_t*)nullptr, ss, st);
-      launched(0);
-      auto scatter_launch = [&] {
-        k_radix_scatter<K><<<p.ctas, kRsThreads, 0, st>>>(ki, vi, ko, vo, n, p.per, shift, h2);
-        launched();
-      };
-      if (timed) ktime(WJ_KERNEL_SORT_SCATTER, scatter_launch); else scatter_launch();
+      if (timed) ktime(WJ_KERNEL_SORT_SCATTER, pass_launch); else pass_launch();
       in1 = !in1;
     }
     return in1;
@@ -642,19 +653,12 @@ struct wj_index {
       phase(WJ_PHASE_SORT);
       uint32_t* kt = (uint32_t*)g_tid.p;
       uint32_t* dt = (uint32_t*)g_doc.p;
-      ktime(WJ_KERNEL_MAP_RANK, [&] {
-        k_map_rank<<<grid_for(N, 256), 256, 0, st>>>(kt, N, ro);
-        launched();
-      });
       uint32_t* k1 = buf<uint32_t>(sk1, N);
       uint32_t* v1 = buf<uint32_t>(sv1, N);
       int bits = 0;
       while (bits < 32 && ((uint64_t)1 << bits) < V) ++bits;
-      const size_t hb = radix_hist_bytes(N);
-      uint32_t* h1 = (uint32_t*)grow(hist, hb);
-      uint32_t* h2 = (uint32_t*)grow(hist_scan, hb);
-      void* ss = scan_scratch((uint64_t)radix_plan(N).ctas * kRsBins, 4);
-      const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, N, 0, bits, h1, h2, ss, true);
+      // termID -> rank is fused into the histogram pass; stable sort by rank keeps docIDs ascending
+      const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, N, 0, bits, ro, true);
       f_key = in1 ? k1 : kt;
       f_doc = in1 ? v1 : dt;
       uint32_t* spare_k = in1 ? kt : k1;  // free N-sized buffers for pstart / tstart
@@ -797,6 +801,10 @@ int index_init(wj_index** out, const wj_config* cfg) {
       ix->own_stream = true;
     }
     WJ_CUDA_CHECK(cudaHostAlloc(&ix->h_scal, 16 * sizeof(uint64_t), cudaHostAllocDefault));
+    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_os_pass<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)os_smem_bytes<uint64_t>()));
+    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_os_pass<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)os_smem_bytes<uint32_t>()));
     ix->reset_state();
     return WJ_OK;
   });

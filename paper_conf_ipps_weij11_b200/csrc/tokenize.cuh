@@ -5,13 +5,20 @@
 // character and hence a trie index can be calculated as a byproduct".  Readings S1 (token
 // bytes), S2 (ASCII folding), S4 (drop > 255 bytes), S16 (empty documents).
 //
-// B200 design: a warp owns a 512-byte segment (16 B per lane, one coalesced 128-bit load per lane),
-// classifies bytes with SWAR, finds token starts/ends with funnel shifts and shuffles, and walks
-// the document boundaries (doc_off) with a per-warp cursor.  Pass 1 counts kept tokens per
-// segment; a scan gives output offsets; pass 2 re-tokenises and, per token, hashes the folded
-// bytes into a chunk-local open-addressing table (one 64-bit CAS claims a slot; equal strings are
-// confirmed against the first occurrence in the immutable text), so the dictionary (K3/K4) sees
-// each distinct term of the chunk once instead of once per token.
+// B200 design.  A warp owns a range of 4 x 512-byte segments.  Per segment every lane classifies
+// its 16 bytes with SWAR (one 128-bit load per lane), document starts come from doc_off through a
+// per-warp cursor (fast path: no boundary in the segment), token starts are `tok & ~prev_tok |
+// doc_start`, ends are the next terminator found in-lane, in a later lane (ballot + one shuffle) or
+// past the segment (one lane scans forward).
+//   * k_tok_count: kept tokens per warp range (a fast path avoids per-token work unless a run of
+//     16 token bytes could hide a > 255-byte token).
+//   * k_tok_emit: stages the range (+1 segment) in shared memory, queues (start, len) of kept tokens
+//     in text order, then processes them one token per lane (full SIMT width): fold, hash, find/claim
+//     the term's slot in a chunk-local open-addressing table of 16-byte slots {first-occurrence
+//     offset | len | 24-bit tag, first 8 folded bytes}.  A token of <= 8 bytes is resolved from the
+//     slot alone; longer ones compare the remaining bytes with the first occurrence in the
+//     (immutable) text.  Writes (slot, docID) at the token's scanned position (coalesced).
+// The dictionary (K3/K4) then sees each distinct term of the chunk once instead of once per token.
 #pragma once
 #include "common.cuh"
 
@@ -20,7 +27,9 @@ namespace wj {
 constexpr int kSegBytes = 512;
 constexpr int kTokThreads = 256;
 constexpr int kTokWarps = kTokThreads / 32;
-constexpr int kSegsPerWarp = 8;
+constexpr int kSegsPerWarp = 4;
+constexpr int kWinBytes = (kSegsPerWarp + 1) * kSegBytes + 16;  // staged range + 1 segment + pad
+constexpr int kQueueCap = kSegBytes;                            // >= tokens of one segment
 
 struct ChunkView {
   const uint8_t* text;     // 16-byte aligned device pointer
@@ -30,7 +39,7 @@ struct ChunkView {
 };
 
 struct EmitOut {
-  uint64_t* table;         // chunk hash table (u64 slots, 0 = empty)
+  Slot* table;             // chunk hash table
   uint32_t mask;           // capacity - 1 (power of two)
   uint32_t doc_base;       // global DocID of local document 0
   uint32_t* slot;          // per kept token: table slot
@@ -48,225 +57,331 @@ __device__ __forceinline__ uint64_t lower_bound_u64(const uint64_t* a, uint64_t 
   return lo;
 }
 
-__device__ __forceinline__ uint64_t term_hash(const TermWords& tw, uint32_t len) {
-  uint64_t h = 0x9E3779B97F4A7C15ull ^ ((uint64_t)len * 0xA0761D6478BD642Full);
-  const uint32_t nw = (len + 3) >> 2;
-  for (uint32_t k = 0; k < nw; ++k) {
-    h = (h ^ tw.word(k)) * 0xff51afd7ed558ccdull;
-    h ^= h >> 29;
-  }
-  return fmix64(h);
-}
-
-__device__ __forceinline__ bool term_equal(const uint8_t* text, uint32_t a, uint32_t b, uint32_t len) {
-  if (a == b) return true;
-  TermWords A(text, a, len), B(text, b, len);
-  const uint32_t nw = (len + 3) >> 2;
-  for (uint32_t k = 0; k < nw; ++k)
-    if (A.word(k) != B.word(k)) return false;
-  return true;
-}
-
-// Slot word: bits 0-31 start offset of the first occurrence, 32-39 length, 40-63 hash tag.
-__device__ __forceinline__ uint32_t table_insert(const uint8_t* text, uint64_t* table, uint32_t mask, uint64_t h,
-                                                 uint32_t s, uint32_t len, uint32_t* overflow) {
-  const uint64_t mine = (uint64_t)s | ((uint64_t)len << 32) | (h & 0xFFFFFF0000000000ull);
-  uint32_t i = (uint32_t)h & mask;
-  for (int probe = 0; probe < 8192; ++probe) {
-    uint64_t cur = *(volatile uint64_t*)(table + i);
-    if (cur == 0) {
-      const unsigned long long prev = atomicCAS((unsigned long long*)(table + i), 0ull, (unsigned long long)mine);
-      if (prev == 0) return i;
-      cur = prev;
+// The lane's 16 bytes of segment `seg` (zero past the end of the chunk).
+__device__ __forceinline__ uint4 load_lane16(const ChunkView& cv, uint64_t seg) {
+  const uint64_t p0 = seg * kSegBytes + 16 * lane_id();
+  if (p0 + 16 <= cv.n_bytes) return __ldg((const uint4*)(cv.text + p0));
+  uint32_t wv[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    uint32_t x = 0;
+#pragma unroll
+    for (int b = 0; b < 4; ++b) {
+      const uint64_t p = p0 + 4 * q + b;
+      if (p < cv.n_bytes) x |= (uint32_t)cv.text[p] << (8 * b);
     }
-    if ((cur >> 32) == (mine >> 32) && term_equal(text, (uint32_t)cur, s, len)) return i;
+    wv[q] = x;
+  }
+  return make_uint4(wv[0], wv[1], wv[2], wv[3]);
+}
+
+// Per-lane view of one segment.
+struct SegBits {
+  uint32_t tm;      // 16-bit token-byte mask
+  uint32_t startm;  // token starts
+  uint32_t termm;   // terminators: non-token byte or document start
+  uint64_t k_lo, k_hi;  // doc_off indices of the boundaries inside the segment: [k_lo, k_hi)
+};
+
+// Classifies one segment; kcur = first boundary index (k >= 1) with doc_off[k] >= segment start;
+// prev = token bit of the byte before the segment (lane 0's left neighbour).
+__device__ __forceinline__ SegBits seg_bits(const ChunkView& cv, uint64_t seg, uint4 v, uint32_t prev,
+                                            uint64_t& kcur, uint32_t* bnd_smem) {
+  const uint32_t lane = lane_id();
+  const uint64_t s0 = seg * kSegBytes;
+  const uint64_t p0 = s0 + 16 * lane;
+  uint32_t tm = tokmask4(v.x) | (tokmask4(v.y) << 4) | (tokmask4(v.z) << 8) | (tokmask4(v.w) << 12);
+  if (p0 >= cv.n_bytes) tm = 0;
+  else if (p0 + 16 > cv.n_bytes) tm &= (1u << (uint32_t)(cv.n_bytes - p0)) - 1u;
+  SegBits sb;
+  sb.k_lo = kcur;
+  const uint64_t s1 = s0 + kSegBytes;
+  uint32_t bm = 0;
+  const uint64_t nb = (kcur < cv.n_docs) ? cv.doc_off[kcur] : ~0ull;  // warp-uniform
+  if (nb < s1) {
+    bnd_smem[lane] = 0;
+    __syncwarp();
+    for (;;) {
+      const uint64_t k = kcur + lane;
+      const uint64_t x = (k < cv.n_docs) ? cv.doc_off[k] : ~0ull;
+      const bool in = x < s1;
+      if (in) atomicOr(&bnd_smem[(uint32_t)(x - s0) >> 4], 1u << ((uint32_t)(x - s0) & 15u));
+      const uint32_t b = __ballot_sync(0xffffffffu, in);
+      kcur += __popc(b);
+      if (b != 0xffffffffu) break;
+    }
+    __syncwarp();
+    bm = bnd_smem[lane];
+    __syncwarp();
+  }
+  sb.k_hi = kcur;
+  uint32_t pv = __shfl_up_sync(0xffffffffu, tm >> 15, 1) & 1u;
+  if (lane == 0) pv = prev;
+  sb.tm = tm;
+  sb.startm = tm & (~((tm << 1) | pv) | bm) & 0xFFFFu;
+  sb.termm = (~tm | bm) & 0xFFFFu;
+  return sb;
+}
+
+// segment-relative position of the first terminator in a later lane, or 0xFFFF
+__device__ __forceinline__ uint32_t next_term_later(uint32_t termm) {
+  const uint32_t lane = lane_id();
+  const uint32_t ft = termm ? 16 * lane + __ffs(termm) - 1 : 0xFFFFu;
+  const uint32_t later = __ballot_sync(0xffffffffu, termm != 0) & ~((2u << lane) - 1u);
+  const uint32_t v = __shfl_sync(0xffffffffu, ft, later ? __ffs(later) - 1 : lane);
+  return later ? v : 0xFFFFu;
+}
+
+// End of the token starting at absolute position sabs whose run reaches the end of its segment
+// (s1): the first non-token byte or document start at or after s1, capped at sabs + 256.
+__device__ __forceinline__ uint64_t far_end(const ChunkView& cv, uint64_t sabs, uint64_t s1, uint64_t k_hi) {
+  uint64_t limit = (k_hi < cv.n_docs) ? cv.doc_off[k_hi] : cv.n_bytes;
+  if (limit > cv.n_bytes) limit = cv.n_bytes;
+  if (limit > sabs + kMaxTermLen + 1) limit = sabs + kMaxTermLen + 1;
+  uint64_t p = s1;
+  while (p < limit) {
+    uint32_t word = 0;
+    if (p + 4 <= cv.n_bytes) word = __ldg((const uint32_t*)(cv.text + p));
+    else for (int b = 0; b < 4; ++b) if (p + b < cv.n_bytes) word |= (uint32_t)cv.text[p + b] << (8 * b);
+    const uint32_t t4 = tokmask4(word);
+    if (t4 != 0xFu) { p += __ffs(~t4) - 1; break; }
+    p += 4;
+  }
+  return p > limit ? limit : p;
+}
+
+// The far end of the segment's last token, computed by the lane holding it (0 elsewhere / if none).
+__device__ __forceinline__ uint64_t seg_far_end(const ChunkView& cv, const SegBits& sb, uint64_t seg, uint32_t nt) {
+  const uint32_t lane = lane_id();
+  const uint32_t has = __ballot_sync(0xffffffffu, sb.startm != 0);
+  uint64_t fe = 0;
+  if (has && (int)lane == 31 - __clz(has)) {
+    const int j = 31 - __clz(sb.startm);
+    if ((sb.termm & ~((2u << j) - 1u)) == 0 && nt == 0xFFFFu)
+      fe = far_end(cv, seg * kSegBytes + 16 * lane + j, (seg + 1) * kSegBytes, sb.k_hi);
+  }
+  return fe;
+}
+
+__device__ __forceinline__ uint64_t token_end(const SegBits& sb, uint32_t nt, uint64_t fe, uint64_t s0, uint64_t p0,
+                                              int j) {
+  const uint32_t above = sb.termm & ~((2u << j) - 1u);
+  if (above) return p0 + (__ffs(above) - 1);
+  if (nt != 0xFFFFu) return s0 + nt;
+  return fe;
+}
+
+// first boundary index k >= 1 with doc_off[k] >= start of each warp's segment range
+__global__ void k_warp_kstart(ChunkView cv, uint64_t warps, uint64_t* kstart) {
+  const uint64_t gw = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (gw >= warps) return;
+  kstart[gw] = lower_bound_u64(cv.doc_off, 1, cv.n_docs > 0 ? cv.n_docs : 1, gw * kSegsPerWarp * kSegBytes);
+}
+
+__device__ __forceinline__ uint32_t prev_token_bit(const ChunkView& cv, uint64_t s0) {
+  return (s0 > 0 && s0 - 1 < cv.n_bytes) ? (tokmask4(cv.text[s0 - 1]) & 1u) : 0u;
+}
+
+// ------------------------------------------------------------------ pass 1: count
+__global__ void __launch_bounds__(kTokThreads) k_tok_count(ChunkView cv, uint64_t n_segs, const uint64_t* kstart,
+                                                           uint32_t* range_count, unsigned long long* dropped) {
+  __shared__ uint32_t bnd[kTokWarps][32];
+  const uint32_t lane = lane_id();
+  const int w = threadIdx.x >> 5;
+  const uint64_t gw = (uint64_t)blockIdx.x * kTokWarps + w;
+  const uint64_t sb0 = gw * kSegsPerWarp;
+  if (sb0 >= n_segs) return;
+  const uint64_t se = min(sb0 + kSegsPerWarp, n_segs);
+  uint64_t kcur = kstart[gw];
+  uint32_t prev = prev_token_bit(cv, sb0 * kSegBytes);
+  uint32_t cnt = 0, drop = 0;
+  uint4 vnext = load_lane16(cv, sb0);
+  for (uint64_t seg = sb0; seg < se; ++seg) {
+    const uint4 v = vnext;
+    if (seg + 1 < se) vnext = load_lane16(cv, seg + 1);
+    const SegBits sb = seg_bits(cv, seg, v, prev, kcur, bnd[w]);
+    prev = __shfl_sync(0xffffffffu, sb.tm, 31) >> 15;
+    const uint32_t nt = next_term_later(sb.termm);
+    const uint64_t fe = seg_far_end(cv, sb, seg, nt);
+    const uint64_t s0 = seg * kSegBytes, p0 = s0 + 16 * lane;
+    const bool maybe_long = __ballot_sync(0xffffffffu, sb.tm == 0xFFFFu) != 0;
+    if (!maybe_long) {
+      // only a token running past the segment can exceed 255 bytes
+      uint32_t c = __popc(sb.startm);
+      if (fe && fe - (p0 + 31 - __clz(sb.startm)) > kMaxTermLen) { --c; ++drop; }
+      cnt += c;
+    } else {
+      uint32_t sm = sb.startm;
+      while (sm) {
+        const int j = __ffs(sm) - 1;
+        sm &= sm - 1;
+        if (token_end(sb, nt, fe, s0, p0, j) - (p0 + j) <= kMaxTermLen) ++cnt; else ++drop;
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
+    drop += __shfl_xor_sync(0xffffffffu, drop, o);
+  }
+  if (lane == 0) {
+    range_count[gw] = cnt;
+    if (drop) atomicAdd(dropped, (unsigned long long)drop);
+  }
+}
+
+// ------------------------------------------------------------------ pass 2: emit
+// k-th little-endian word of the folded term starting at window byte s (len bytes), zero padded
+__device__ __forceinline__ uint32_t win_word(const uint32_t* win32, uint32_t s, uint32_t len, uint32_t k) {
+  const uint32_t a = (s >> 2) + k, sh = (s & 3) * 8;
+  uint32_t w = __funnelshift_r(win32[a], win32[a + 1], sh);
+  const uint32_t rem = len - 4 * k;
+  if (rem < 4) w &= (1u << (rem * 8)) - 1u;
+  return lower4(w);
+}
+
+__device__ __forceinline__ uint64_t mix_hash(uint64_t h, uint64_t x) {
+  h = (h ^ x) * 0xff51afd7ed558ccdull;
+  return h ^ (h >> 29);
+}
+
+__device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* table, uint32_t mask, uint64_t h,
+                                                 uint32_t s_abs, uint32_t len, uint64_t mypfx,
+                                                 const uint32_t* win32, uint32_t s_win, uint32_t* overflow) {
+  const uint64_t mine = (uint64_t)s_abs | ((uint64_t)len << 32) | (h & 0xFFFFFF0000000000ull);
+  uint32_t i = (uint32_t)h & mask;
+  for (int probe = 0; probe < 4096; ++probe) {
+    // Slots are claimed once (CAS on meta) and their pfx published once, so a cached read can
+    // only be stale-empty: the CAS or the volatile re-read below resolves it.
+    const ulonglong2 e = *(const ulonglong2*)(table + i);
+    uint64_t meta = e.x, pfx = e.y;
+    if (meta == 0) {
+      const unsigned long long prev = atomicCAS(&table[i].meta, 0ull, (unsigned long long)mine);
+      if (prev == 0) {
+        *(volatile unsigned long long*)&table[i].pfx = mypfx;
+        return i;
+      }
+      meta = prev;
+      pfx = 0;
+    }
+    if ((meta >> 32) == (mine >> 32)) {
+      while (pfx == 0) pfx = *(volatile unsigned long long*)&table[i].pfx;
+      if (pfx == mypfx) {
+        if (len <= 8) return i;
+        const TermWords other(text, (uint32_t)meta, len);
+        bool eq = true;
+        for (uint32_t k = 2; k * 4 < len; ++k)
+          if (other.word(k) != win_word(win32, s_win, len, k)) { eq = false; break; }
+        if (eq) return i;
+      }
+    }
     i = (i + 1) & mask;
   }
   atomicExch(overflow, 1u);
   return kMiss;
 }
 
-// Per-warp view of one segment after classification.
-struct SegState {
-  uint32_t startm;   // lane-local 16-bit mask of token starts
-  uint32_t termm;    // lane-local 16-bit mask of terminators (non-token byte or doc start)
-  uint32_t next_t;   // segment-relative position of the first terminator in a later lane (or 0xFFFF)
-  uint32_t far_end;  // absolute end of the token running past the segment (valid in the last-start lane)
-  uint64_t k_lo, k_hi;  // doc_off boundary index range for this segment
-};
-
-// Classifies segment `seg` for the calling warp; kcur = first doc boundary index >= segment start.
-__device__ __forceinline__ SegState classify_segment(const ChunkView& cv, uint64_t seg, uint64_t& kcur,
-                                                     uint32_t* bnd_smem /* 32 words, this warp */) {
-  const uint32_t lane = lane_id();
-  const uint64_t s0 = seg * kSegBytes;
-  const uint64_t p0 = s0 + 16 * lane;
-  uint32_t wv[4];
-  if (p0 + 16 <= cv.n_bytes) {
-    const uint4 v = __ldg((const uint4*)(cv.text + p0));
-    wv[0] = v.x; wv[1] = v.y; wv[2] = v.z; wv[3] = v.w;
-  } else {
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      uint32_t x = 0;
-#pragma unroll
-      for (int b = 0; b < 4; ++b) {
-        const uint64_t p = p0 + 4 * q + b;
-        if (p < cv.n_bytes) x |= (uint32_t)cv.text[p] << (8 * b);
-      }
-      wv[q] = x;
-    }
-  }
-  uint32_t tm = tokmask4(wv[0]) | (tokmask4(wv[1]) << 4) | (tokmask4(wv[2]) << 8) | (tokmask4(wv[3]) << 12);
-  if (p0 >= cv.n_bytes) tm = 0;
-  else if (p0 + 16 > cv.n_bytes) tm &= (1u << (uint32_t)(cv.n_bytes - p0)) - 1u;
-
-  // document boundaries (doc_off[k], 1 <= k < n_docs) inside [s0, s0+512)
-  bnd_smem[lane] = 0;
-  __syncwarp();
-  const uint64_t s1 = s0 + kSegBytes;
-  SegState st;
-  st.k_lo = kcur;
-  for (;;) {
-    const uint64_t k = kcur + lane;
-    const uint64_t x = (k < cv.n_docs) ? cv.doc_off[k] : ~0ull;
-    const bool in = x < s1;
-    if (in) atomicOr(&bnd_smem[(uint32_t)(x - s0) >> 4], 1u << ((uint32_t)(x - s0) & 15u));
-    const uint32_t b = __ballot_sync(0xffffffffu, in);
-    kcur += __popc(b);
-    if (b != 0xffffffffu) break;
-  }
-  st.k_hi = kcur;
-  __syncwarp();
-  const uint32_t bm = bnd_smem[lane];
-
-  // previous byte's token bit (for lane 0: last byte of the previous segment)
-  uint32_t prev = __shfl_up_sync(0xffffffffu, tm >> 15, 1) & 1u;
-  if (lane == 0) prev = (s0 > 0 && s0 - 1 < cv.n_bytes) ? ((tokmask4(cv.text[s0 - 1]) & 1u)) : 0u;
-  st.startm = tm & ((~((tm << 1) | prev)) | bm) & 0xFFFFu;
-  st.termm = (~tm | bm) & 0xFFFFu;
-
-  // first terminator in any later lane
-  uint32_t f = st.termm ? (16 * lane + __ffs(st.termm) - 1) : 0xFFFFu;
-  // suffix-min over lanes > lane
-  uint32_t m = f;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    uint32_t u = __shfl_down_sync(0xffffffffu, m, o);
-    if (lane + o < 32) m = min(m, u);
-  }
-  uint32_t nt = __shfl_down_sync(0xffffffffu, m, 1);
-  if (lane == 31) nt = 0xFFFFu;
-  st.next_t = nt;
-
-  // the last start of the segment may run past it: find its end in global memory
-  st.far_end = 0;
-  const uint32_t has = __ballot_sync(0xffffffffu, st.startm != 0);
-  if (has) {
-    const int last_lane = 31 - __clz(has);
-    if ((int)lane == last_lane) {
-      const int j = 31 - __clz(st.startm);
-      const uint32_t above = st.termm & ~((2u << j) - 1u);
-      if (above == 0 && nt == 0xFFFFu) {
-        const uint64_t sabs = p0 + j;
-        uint64_t limit = (st.k_hi < cv.n_docs) ? cv.doc_off[st.k_hi] : cv.n_bytes;
-        if (limit > cv.n_bytes) limit = cv.n_bytes;
-        if (limit > sabs + kMaxTermLen + 1) limit = sabs + kMaxTermLen + 1;
-        uint64_t p = s1;
-        while (p < limit) {
-          uint32_t word = 0;
-          if (p + 4 <= cv.n_bytes) word = __ldg((const uint32_t*)(cv.text + p));
-          else for (int b = 0; b < 4; ++b) if (p + b < cv.n_bytes) word |= (uint32_t)cv.text[p + b] << (8 * b);
-          const uint32_t t4 = tokmask4(word);
-          if (t4 != 0xFu) { p += __ffs(~t4) - 1; break; }
-          p += 4;
-        }
-        if (p > limit) p = limit;
-        st.far_end = (uint32_t)p;
-      }
-    }
-  }
-  return st;
-}
-
-// End (absolute) of the token starting at lane-local bit j.
-__device__ __forceinline__ uint64_t token_end(const SegState& st, uint64_t p0, uint64_t s0, int j) {
-  const uint32_t above = st.termm & ~((2u << j) - 1u);
-  if (above) return p0 + (__ffs(above) - 1);
-  if (st.next_t != 0xFFFFu) return s0 + st.next_t;
-  return st.far_end;
-}
-
-template <bool EMIT>
-__global__ void __launch_bounds__(kTokThreads) k_tokenize(ChunkView cv, uint64_t n_segs, uint32_t* seg_count,
-                                                          const uint32_t* seg_off, EmitOut eo,
-                                                          unsigned long long* dropped) {
+__global__ void __launch_bounds__(kTokThreads) k_tok_emit(ChunkView cv, uint64_t n_segs, const uint64_t* kstart,
+                                                          const uint32_t* range_off, EmitOut eo) {
+  __shared__ __align__(16) uint32_t win[kTokWarps][kWinBytes / 4];
+  __shared__ uint32_t queue[kTokWarps][kQueueCap];
   __shared__ uint32_t bnd[kTokWarps][32];
   const uint32_t lane = lane_id();
   const int w = threadIdx.x >> 5;
   const uint64_t gw = (uint64_t)blockIdx.x * kTokWarps + w;
-  const uint64_t seg_begin = gw * kSegsPerWarp;
-  if (seg_begin >= n_segs) return;
-  const uint64_t seg_end = min(seg_begin + kSegsPerWarp, n_segs);
-  // first boundary index k >= 1 with doc_off[k] >= segment start
-  uint64_t kcur = 0;
-  if (lane == 0) kcur = lower_bound_u64(cv.doc_off, 1, cv.n_docs > 0 ? cv.n_docs : 1, seg_begin * kSegBytes);
-  kcur = __shfl_sync(0xffffffffu, kcur, 0);
-  uint32_t drop_acc = 0;
-  for (uint64_t seg = seg_begin; seg < seg_end; ++seg) {
-    const SegState st = classify_segment(cv, seg, kcur, bnd[w]);
-    const uint64_t s0 = seg * kSegBytes;
-    const uint64_t p0 = s0 + 16 * lane;
-    uint32_t nvalid = 0, ndrop = 0;
-    uint32_t sm = st.startm;
-    while (sm) {
-      const int j = __ffs(sm) - 1;
-      sm &= sm - 1;
-      const uint64_t e = token_end(st, p0, s0, j);
-      if (e - (p0 + j) <= kMaxTermLen) ++nvalid; else ++ndrop;
-    }
-    drop_acc += ndrop;
-    if (!EMIT) {
-      uint32_t tot = nvalid;
+  const uint64_t sb0 = gw * kSegsPerWarp;
+  if (sb0 >= n_segs) return;
+  const uint64_t se = min(sb0 + kSegsPerWarp, n_segs);
+  const uint64_t B0 = sb0 * kSegBytes;
+  uint32_t* w32 = win[w];
+  uint32_t* q = queue[w];
+  // stage the range and one more segment (tokens may run past the range)
+  uint4 v[kSegsPerWarp + 1];
 #pragma unroll
-      for (int o = 16; o > 0; o >>= 1) tot += __shfl_xor_sync(0xffffffffu, tot, o);
-      if (lane == 0) seg_count[seg] = tot;
-    } else {
-      // exclusive prefix of nvalid over lanes
-      uint32_t inc = nvalid;
+  for (int j = 0; j <= kSegsPerWarp; ++j) v[j] = load_lane16(cv, sb0 + j);
 #pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
-        if ((int)lane >= o) inc += u;
-      }
-      uint64_t out = (uint64_t)seg_off[seg] + (inc - nvalid);
-      sm = st.startm;
-      while (sm) {
-        const int j = __ffs(sm) - 1;
-        sm &= sm - 1;
-        const uint64_t s = p0 + j;
-        const uint64_t e = token_end(st, p0, s0, j);
-        const uint32_t len = (uint32_t)(e - s);
-        if (len > kMaxTermLen) continue;
-        // DocID: number of doc_off[k] <= s, k < n_docs, minus one (reading S9/S16)
-        uint64_t k = st.k_lo;
-        while (k < st.k_hi && cv.doc_off[k] <= s) ++k;
-        const uint32_t doc = eo.doc_base + (uint32_t)(k - 1);
-        const TermWords tw(cv.text, s, len);
-        const uint64_t h = term_hash(tw, len);
-        const uint32_t slot = table_insert(cv.text, eo.table, eo.mask, h, (uint32_t)s, len, eo.overflow);
+  for (int j = 0; j <= kSegsPerWarp; ++j) *(uint4*)&w32[(j * kSegBytes + 16 * lane) / 4] = v[j];
+  if (lane < 4) w32[(kWinBytes - 16) / 4 + lane] = 0;
+  __syncwarp();
+
+  const uint64_t k_range_lo = kstart[gw];
+  uint64_t kcur = k_range_lo;
+  uint32_t prev = prev_token_bit(cv, B0);
+  uint32_t qn = 0;
+  uint64_t obase = range_off[gw];
+  uint64_t k_range_hi = k_range_lo;
+
+  auto flush = [&]() {
+    for (uint32_t r = 0; r < qn; r += 32) {
+      const uint32_t idx = r + lane;
+      if (idx < qn) {
+        const uint32_t e = q[idx];
+        const uint32_t s_win = e >> 8, len = e & 255u;
+        const uint32_t s_abs = (uint32_t)(B0 + s_win);
+        uint32_t wd[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) wd[k] = (4u * k < len) ? win_word(w32, s_win, len, k) : 0u;
+        uint64_t h = 0x9E3779B97F4A7C15ull ^ ((uint64_t)len * 0xA0761D6478BD642Full);
+        h = mix_hash(h, (uint64_t)wd[0] | ((uint64_t)wd[1] << 32));
+        h = mix_hash(h, (uint64_t)wd[2] | ((uint64_t)wd[3] << 32));
+        for (uint32_t k = 4; k * 4 < len; k += 2) {
+          const uint32_t a = win_word(w32, s_win, len, k);
+          const uint32_t b = ((k + 1) * 4 < len) ? win_word(w32, s_win, len, k + 1) : 0u;
+          h = mix_hash(h, (uint64_t)a | ((uint64_t)b << 32));
+        }
+        h = fmix64(h);
+        // DocID = (number of doc_off[k] <= s, k < n_docs) - 1 (readings S9, S16)
+        uint64_t lo = k_range_lo, hi = k_range_hi;
+        while (lo < hi) {
+          const uint64_t mid = (lo + hi) >> 1;
+          if (cv.doc_off[mid] <= s_abs) lo = mid + 1; else hi = mid;
+        }
+        const uint32_t doc = eo.doc_base + (uint32_t)(lo - 1);
+        const uint64_t pfx = (uint64_t)wd[0] | ((uint64_t)wd[1] << 32);
+        const uint32_t slot = table_insert(cv.text, eo.table, eo.mask, h, s_abs, len, pfx, w32, s_win, eo.overflow);
+        const uint64_t out = obase + idx;
         eo.slot[out] = slot;
         eo.doc[out] = doc;
-        if (eo.dbg_start) { eo.dbg_start[out] = (uint32_t)s; eo.dbg_len[out] = len; }
-        ++out;
+        if (eo.dbg_start) { eo.dbg_start[out] = s_abs; eo.dbg_len[out] = len; }
       }
     }
-  }
-  if (!EMIT) {
+    obase += qn;
+    qn = 0;
+    __syncwarp();
+  };
+
+  for (uint64_t seg = sb0; seg < se; ++seg) {
+    const int j = (int)(seg - sb0);
+    const uint4 vv = *(const uint4*)&w32[(j * kSegBytes + 16 * lane) / 4];
+    const SegBits sb = seg_bits(cv, seg, vv, prev, kcur, bnd[w]);
+    prev = __shfl_sync(0xffffffffu, sb.tm, 31) >> 15;
+    k_range_hi = kcur;
+    const uint32_t nt = next_term_later(sb.termm);
+    const uint64_t fe = seg_far_end(cv, sb, seg, nt);
+    const uint64_t s0 = seg * kSegBytes, p0 = s0 + 16 * lane;
+    uint32_t c = 0;
+    for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
+      const int jb = __ffs(sm) - 1;
+      c += (token_end(sb, nt, fe, s0, p0, jb) - (p0 + jb) <= kMaxTermLen) ? 1u : 0u;
+    }
+    uint32_t inc = c;
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) drop_acc += __shfl_xor_sync(0xffffffffu, drop_acc, o);
-    if (lane == 0 && drop_acc) atomicAdd(dropped, (unsigned long long)drop_acc);
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
+      if ((int)lane >= o) inc += u;
+    }
+    const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
+    if (qn + tot > (uint32_t)kQueueCap) flush();
+    uint32_t pos = qn + inc - c;
+    for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
+      const int jb = __ffs(sm) - 1;
+      const uint64_t len = token_end(sb, nt, fe, s0, p0, jb) - (p0 + jb);
+      if (len <= kMaxTermLen) q[pos++] = ((uint32_t)(p0 + jb - B0) << 8) | (uint32_t)len;
+    }
+    qn += tot;
+    __syncwarp();
   }
+  flush();
 }
 
 }  // namespace wj
