@@ -30,11 +30,16 @@ struct alignas(128) Node {
 static_assert(sizeof(Node) == 512, "Table II: a B-tree node is 512 bytes");
 static_assert(4 + 31 * 4 + 4 + 31 * 4 + 32 * 4 + 31 * 4 + 4 == 512, "Table II field sizes");
 
-// Chunk-local term table slot (K1 emit): 16 bytes, claimed once by CAS on meta.
+// Chunk-local term table slot (K1 emit): 16 bytes, claimed once by CAS on k0, k1 published after.
+//   k0 = len (8 bits) | hash tag (24 bits) << 8 | folded bytes 0-3 << 32      (0 = empty)
+//   k1 = folded bytes 4-10 (56 bits) | 1 << 56                                   (0 = unpublished)
+// Terms of <= 11 bytes are identified by (k0, k1) alone; longer ones also compare bytes 8.. with
+// their first occurrence (offset in a side array written by the inserter before publishing k1).
 struct __align__(16) Slot {
-  unsigned long long meta;  // bits 0-31 first-occurrence offset, 32-39 length, 40-63 hash tag; 0 = empty
-  unsigned long long pfx;   // first 8 folded bytes (little-endian, zero padded); 0 until published
+  unsigned long long k0;
+  unsigned long long k1;
 };
+constexpr uint32_t kSlotBytes = 11;
 
 __host__ __device__ inline uint32_t ceil_div32(uint64_t a, uint32_t b) { return (uint32_t)((a + b - 1) / b); }
 

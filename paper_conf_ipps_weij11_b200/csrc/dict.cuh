@@ -191,15 +191,16 @@ __global__ void k_probe(DictView dv, UniqueView uv, uint32_t U, uint32_t* tid_ou
 }
 
 // unique gather: occupied slot i -> unique index uid[i]; term info from the first occurrence
-__global__ void k_unique_gather(const Slot* table, uint32_t C, const uint32_t* uid, const uint8_t* text,
+__global__ void k_unique_gather(const Slot* table, const uint32_t* slot_ref, uint32_t C, const uint32_t* uid,
+                                const uint8_t* text,
                                 uint32_t* u_ref, uint32_t* u_len, uint32_t* u_bucket, uint32_t* u_cache,
                                 uint64_t* u_key) {
   const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= C) return;
-  const uint64_t e = table[i].meta;
+  const uint64_t e = table[i].k0;
   if (e == 0) return;
   const uint32_t u = uid[i];
-  const uint32_t ref = (uint32_t)e, len = (uint32_t)(e >> 32) & 0xFFu;
+  const uint32_t ref = slot_ref[i], len = (uint32_t)e & 0xFFu;
   const TermInfo ti = term_info(text, ref, len);
   u_ref[u] = ref; u_len[u] = len; u_bucket[u] = ti.bucket; u_cache[u] = ti.cache; u_key[u] = ti.key;
 }

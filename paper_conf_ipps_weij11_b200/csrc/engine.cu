@@ -62,7 +62,7 @@ __global__ void k_check_docoff(const uint64_t* d, uint64_t n_docs, uint64_t n_by
 
 struct NonZeroSlot {
   const Slot* t;
-  __device__ __forceinline__ uint32_t operator()(uint64_t i) const { return t[i].meta != 0 ? 1u : 0u; }
+  __device__ __forceinline__ uint32_t operator()(uint64_t i) const { return t[i].k0 != 0 ? 1u : 0u; }
 };
 struct IsMiss {
   const uint32_t* t;
@@ -112,9 +112,13 @@ struct wj_index {
   // chunk scratch
   DevBuf text_stage, doc_stage, seg_cnt, table, uid, u_ref, u_len, u_bucket, u_cache, u_key, u_tid, u_rank, midx, nk_key,
       nk_val, nk_key2, nk_val2, aoff, ns_tid, ns_bucket, ns_rank, nlo, nhi, nbase, lvA[4], lvB[4], child_off, root_idx,
-      scan_scr, hist, hist_scan, os_hist, os_look, os_ctr, kstart, dbg_start, dbg_len, dbg_off, dbg_out, dbg_slot, dbg_doc, lexg, qbuf, qres;
+      scan_scr, hist, hist_scan, os_hist, os_look, os_ctr, kstart, slotref, dbg_start, dbg_len, dbg_off, dbg_out, dbg_slot, dbg_doc, lexg, qbuf, qres;
   // finalize
   DevBuf rank_of, term_at, sk1, sv1, pidx, out_doc, out_tf, post_off, df, cf, term_off, term_bytes;
+  std::vector<DevBuf> chunk_map;        // per chunk: slot -> termID (-> rank at finalize)
+  std::vector<uint64_t> chunk_tok;      // per chunk: first token index in the stream
+  std::vector<uint32_t> chunk_C;        // per chunk: table capacity
+  DevBuf rle_look, rle_p0, rle_lead;
   uint32_t* f_key = nullptr;   // sorted keys (term ranks)
   uint32_t* f_doc = nullptr;   // sorted docIDs
   // profiling
@@ -163,7 +167,7 @@ struct wj_index {
                      &t_arena, &t_cache, &t_bucket, &scal, &g_tid, &g_doc, &text_stage, &doc_stage, &seg_cnt, &table,
                      &uid, &u_ref, &u_len, &u_bucket, &u_cache, &u_key, &u_tid, &u_rank, &midx, &nk_key, &nk_val,
                      &nk_key2, &nk_val2, &aoff, &ns_tid, &ns_bucket, &ns_rank, &nlo, &nhi, &nbase, &child_off,
-                     &root_idx, &scan_scr, &hist, &hist_scan, &os_hist, &os_look, &os_ctr, &kstart, &dbg_start, &dbg_len, &dbg_off, &dbg_out, &dbg_slot,
+                     &root_idx, &scan_scr, &hist, &hist_scan, &os_hist, &os_look, &os_ctr, &kstart, &slotref, &dbg_start, &dbg_len, &dbg_off, &dbg_out, &dbg_slot,
                      &dbg_doc, &lexg, &qbuf, &qres, &rank_of, &term_at, &sk1, &sv1, &pidx, &out_doc, &out_tf,
                      &post_off, &df, &cf, &term_off, &term_bytes};
     for (DevBuf* b : all) {
@@ -171,6 +175,9 @@ struct wj_index {
       b->p = nullptr;
       b->cap = 0;
     }
+    for (auto& b : chunk_map) if (b.p) cudaFree(b.p);
+    chunk_map.clear();
+    for (DevBuf* b : {&rle_look, &rle_p0, &rle_lead}) { if (b->p) cudaFree(b->p); *b = DevBuf{}; }
     for (int i = 0; i < 4; ++i) {
       if (lvA[i].p) cudaFree(lvA[i].p);
       if (lvB[i].p) cudaFree(lvB[i].p);
@@ -264,6 +271,8 @@ struct wj_index {
   // ---------------------------------------------------------------- init / reset
   void reset_state() {
     collect_phases();
+    chunk_tok.clear();
+    chunk_C.clear();
     n_docs = n_tokens = n_dropped = n_chunks = 0;
     unique_last = new_last = n_nodes = height_max = 0;
     V = 0;
@@ -337,7 +346,7 @@ struct wj_index {
     launched();
     WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 1, 0, 8, st));
     ktime(WJ_KERNEL_TOKENIZE_COUNT, [&] {
-      k_tok_count<<<grid, kTokThreads, 0, st>>>(cv, n_segs, ks, cnt, (unsigned long long*)(dscal() + 1));
+      k_tok_count<<<grid, kTokThreads, 0, st>>>(cv, (uint32_t)n_segs, ks, cnt, (unsigned long long*)(dscal() + 1));
       launched();
     });
     scan<uint32_t>(ArrayIn<uint32_t>{cnt}, ranges, cnt, (uint32_t*)(dscal() + 0));
@@ -354,6 +363,7 @@ struct wj_index {
     WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 5, 0, 8, st));
     EmitOut eo;
     eo.table = tab;
+    eo.slot_ref = buf<uint32_t>(slotref, C);
     eo.mask = (uint32_t)(C - 1);
     eo.doc_base = doc_base;
     eo.slot = slot_out;
@@ -364,7 +374,7 @@ struct wj_index {
     const uint64_t ranges = (n_segs + kSegsPerWarp - 1) / kSegsPerWarp;
     const unsigned grid = (unsigned)((ranges + kTokWarps - 1) / kTokWarps);
     ktime(WJ_KERNEL_TOKENIZE_EMIT, [&] {
-      k_tok_emit<<<grid, kTokThreads, 0, st>>>(cv, n_segs, (const uint64_t*)kstart.p, (const uint32_t*)seg_cnt.p, eo);
+      k_tok_emit<<<grid, kTokThreads, 0, st>>>(cv, (uint32_t)n_segs, (const uint64_t*)kstart.p, (const uint32_t*)seg_cnt.p, eo);
       launched();
     });
   }
@@ -432,7 +442,7 @@ struct wj_index {
     uint64_t* uk = buf<uint64_t>(u_key, U);
     uint32_t* ut = buf<uint32_t>(u_tid, U);
     uint32_t* urk = buf<uint32_t>(u_rank, U);
-    k_unique_gather<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, (uint32_t)C, slot_uid, text, ur, ul, ub,
+    k_unique_gather<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, (const uint32_t*)slotref.p, (uint32_t)C, slot_uid, text, ur, ul, ub,
                                                       uc, uk);
     launched();
 
@@ -467,12 +477,17 @@ struct wj_index {
       rebuild();
     }
 
-    // termIDs into the stream (the postings input)
+    // the chunk's (slot, docID) stream is the postings input; keep its slot -> termID map
     phase(WJ_PHASE_STREAM);
+    const size_t ci = chunk_tok.size();
+    if (chunk_map.size() <= ci) chunk_map.emplace_back();
+    uint32_t* cmap = buf<uint32_t>(chunk_map[ci], C);
     ktime(WJ_KERNEL_SLOT_TO_TID, [&] {
-      k_slot_to_tid<<<grid_for(Nc, 256), 256, 0, st>>>(gt + n_tokens, Nc, slot_uid, ut);
+      k_slot_map<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, slot_uid, ut, (uint32_t)C, cmap);
       launched();
     });
+    chunk_tok.push_back(n_tokens);
+    chunk_C.push_back((uint32_t)C);
     n_tokens += Nc;
     n_docs += nd;
     phase(-1);
@@ -591,18 +606,27 @@ struct wj_index {
   // stable LSD radix sort driver: onesweep (radix.cuh).  rank_of != nullptr maps keys first.
   template <typename K>
   bool sort_pairs(K* k0, uint32_t* v0, K* k1, uint32_t* v1, uint64_t n, int begin_bit, int end_bit,
-                  const uint32_t* rank_of, bool timed) {
+                  const uint32_t* rank_of, bool timed,
+                  const std::vector<std::pair<uint64_t, const uint32_t*>>* segs = nullptr) {
     if (n == 0) return false;
     const int passes = end_bit > begin_bit ? (end_bit - begin_bit + 7) / 8 : 0;
-    if (n == 1 && !rank_of) return false;
+    if (n == 1 && !rank_of && !segs) return false;
     uint32_t* gh = buf<uint32_t>(os_hist, (uint64_t)std::max(passes, 1) * 256);
     WJ_CUDA_CHECK(cudaMemsetAsync(gh, 0, (size_t)std::max(passes, 1) * 256 * 4, st));
-    const unsigned hb = (unsigned)std::min<uint64_t>((n + 255) / 256, 148ull * 8);
-    auto hist_launch = [&] {
-      k_os_hist<K><<<hb, 256, 0, st>>>(k0, n, begin_bit, passes, rank_of, gh);
-      launched();
-    };
-    if (timed) ktime(WJ_KERNEL_SORT_HIST, hist_launch); else hist_launch();
+    // histogram of every digit; segs (optional): per stream segment a key map (slot -> rank)
+    const size_t nseg = segs ? segs->size() : 1;
+    for (size_t sgi = 0; sgi < nseg; ++sgi) {
+      const uint64_t off = segs ? (*segs)[sgi].first : 0;
+      const uint64_t end = segs ? (sgi + 1 < nseg ? (*segs)[sgi + 1].first : n) : n;
+      const uint32_t* map = segs ? (*segs)[sgi].second : rank_of;
+      if (end <= off) continue;
+      const unsigned hb = (unsigned)std::min<uint64_t>((end - off + 255) / 256, 148ull * 8);
+      auto hist_launch = [&] {
+        k_os_hist<K><<<hb, 256, 0, st>>>(k0 + off, end - off, begin_bit, passes, map, gh);
+        launched();
+      };
+      if (timed) ktime(WJ_KERNEL_SORT_HIST, hist_launch); else hist_launch();
+    }
     if (passes == 0 || n == 1) return false;
     k_os_hist_scan<<<passes, 256, 0, st>>>(gh);
     launched();
@@ -657,28 +681,45 @@ struct wj_index {
       uint32_t* v1 = buf<uint32_t>(sv1, N);
       int bits = 0;
       while (bits < 32 && ((uint64_t)1 << bits) < V) ++bits;
-      // termID -> rank is fused into the histogram pass; stable sort by rank keeps docIDs ascending
-      const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, N, 0, bits, ro, true);
+      // per chunk: slot -> termID -> rank map; applied in the histogram pass; the stable sort by
+      // rank keeps docIDs ascending within every term
+      std::vector<std::pair<uint64_t, const uint32_t*>> segs;
+      for (size_t c = 0; c < chunk_tok.size(); ++c) {
+        uint32_t* m = (uint32_t*)chunk_map[c].p;
+        k_map_compose<<<grid_for(chunk_C[c], 256), 256, 0, st>>>(m, chunk_C[c], ro);
+        launched();
+        segs.emplace_back(chunk_tok[c], m);
+      }
+      const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, N, 0, bits, nullptr, true, &segs);
       f_key = in1 ? k1 : kt;
       f_doc = in1 ? v1 : dt;
       uint32_t* spare_k = in1 ? kt : k1;  // free N-sized buffers for pstart / tstart
       uint32_t* spare_v = in1 ? dt : v1;
 
       phase(WJ_PHASE_POSTINGS);
-      uint32_t* pi = buf<uint32_t>(pidx, N);
-      scan<uint32_t>(NewPosting{f_key, f_doc}, N, pi, (uint32_t*)(dscal() + 8));
+      const uint64_t tiles = (N + kRleTile - 1) / kRleTile;
+      uint64_t* lk = buf<uint64_t>(rle_look, tiles);
+      uint32_t* tp0 = buf<uint32_t>(rle_p0, tiles);
+      uint32_t* tld = buf<uint32_t>(rle_lead, tiles);
+      uint32_t* ctr = buf<uint32_t>(os_ctr, 4);
+      WJ_CUDA_CHECK(cudaMemsetAsync(lk, 0, tiles * 8, st));
+      WJ_CUDA_CHECK(cudaMemsetAsync(ctr, 0, 4, st));
+      // P <= N: size the outputs by N, no host round trip before the pass
+      uint32_t* od = buf<uint32_t>(out_doc, N);
+      uint32_t* of = buf<uint32_t>(out_tf, N);
+      uint32_t* tstart_p = spare_v;  // N >= V entries
+      (void)spare_k;
+      ktime(WJ_KERNEL_RLE_EMIT, [&] {
+        k_rle_fused<<<(unsigned)tiles, kRleThreads, 0, st>>>(f_key, f_doc, N, od, of, po, tstart_p, lk, ctr, tp0, tld,
+                                                            (uint32_t*)(dscal() + 8));
+        launched();
+      });
+      k_rle_fixup<<<grid_for(tiles, 256), 256, 0, st>>>(tp0, tld, (uint32_t)tiles, of);
+      launched();
       WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 8) + 1, 0, 4, st));
       readback(8, 1);
       P = (uint32_t)h_scal[8];
-      uint32_t* od = buf<uint32_t>(out_doc, P);
-      uint32_t* of = buf<uint32_t>(out_tf, P);
-      ktime(WJ_KERNEL_RLE_EMIT, [&] {
-        k_rle_emit<<<grid_for(N, 256), 256, 0, st>>>(f_key, f_doc, N, pi, od, spare_k, po, spare_v);
-        launched();
-      });
-      k_rle_tf<<<grid_for(P, 256), 256, 0, st>>>(spare_k, P, N, of);
-      launched();
-      k_df_cf<<<grid_for((uint64_t)V + 1, 256), 256, 0, st>>>(po, spare_v, V, P, N, dfp, cfp);
+      k_df_cf<<<grid_for((uint64_t)V + 1, 256), 256, 0, st>>>(po, tstart_p, V, P, N, dfp, cfp);
       launched();
     } else {
       WJ_CUDA_CHECK(cudaMemsetAsync(po, 0, 8, st));

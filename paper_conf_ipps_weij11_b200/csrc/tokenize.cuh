@@ -40,6 +40,7 @@ struct ChunkView {
 
 struct EmitOut {
   Slot* table;             // chunk hash table
+  uint32_t* slot_ref;      // per slot: first-occurrence offset (written by the inserter)
   uint32_t mask;           // capacity - 1 (power of two)
   uint32_t doc_base;       // global DocID of local document 0
   uint32_t* slot;          // per kept token: table slot
@@ -57,10 +58,11 @@ __device__ __forceinline__ uint64_t lower_bound_u64(const uint64_t* a, uint64_t 
   return lo;
 }
 
-// The lane's 16 bytes of segment `seg` (zero past the end of the chunk).
-__device__ __forceinline__ uint4 load_lane16(const ChunkView& cv, uint64_t seg) {
-  const uint64_t p0 = seg * kSegBytes + 16 * lane_id();
-  if (p0 + 16 <= cv.n_bytes) return __ldg((const uint4*)(cv.text + p0));
+// The lane's 16 bytes of segment `seg` (zero past the end of the chunk).  Streaming loads
+// (evict-first): the text is read once per pass and must not push the term table out of L2.
+__device__ __forceinline__ uint4 load_lane16(const ChunkView& cv, uint32_t seg) {
+  const uint64_t p0 = (uint64_t)seg * kSegBytes + 16 * lane_id();
+  if (p0 + 16 <= cv.n_bytes) return __ldcs((const uint4*)(cv.text + p0));
   uint32_t wv[4];
 #pragma unroll
   for (int q = 0; q < 4; ++q) {
@@ -75,27 +77,24 @@ __device__ __forceinline__ uint4 load_lane16(const ChunkView& cv, uint64_t seg) 
   return make_uint4(wv[0], wv[1], wv[2], wv[3]);
 }
 
+constexpr uint32_t kNone = 0xFFFFu;
+
 // Per-lane view of one segment.
 struct SegBits {
   uint32_t tm;      // 16-bit token-byte mask
   uint32_t startm;  // token starts
   uint32_t termm;   // terminators: non-token byte or document start
-  uint64_t k_lo, k_hi;  // doc_off indices of the boundaries inside the segment: [k_lo, k_hi)
 };
 
-// Classifies one segment; kcur = first boundary index (k >= 1) with doc_off[k] >= segment start;
-// prev = token bit of the byte before the segment (lane 0's left neighbour).
-__device__ __forceinline__ SegBits seg_bits(const ChunkView& cv, uint64_t seg, uint4 v, uint32_t prev,
+// Classifies one segment; kcur = first boundary index (k >= 1) with doc_off[k] >= segment start
+// (advanced past the segment); prev = token bit of the byte before the segment.
+__device__ __forceinline__ SegBits seg_bits(const ChunkView& cv, uint32_t s0, uint4 v, uint32_t prev,
                                             uint64_t& kcur, uint32_t* bnd_smem) {
   const uint32_t lane = lane_id();
-  const uint64_t s0 = seg * kSegBytes;
-  const uint64_t p0 = s0 + 16 * lane;
+  const uint64_t p0 = (uint64_t)s0 + 16 * lane;
   uint32_t tm = tokmask4(v.x) | (tokmask4(v.y) << 4) | (tokmask4(v.z) << 8) | (tokmask4(v.w) << 12);
-  if (p0 >= cv.n_bytes) tm = 0;
-  else if (p0 + 16 > cv.n_bytes) tm &= (1u << (uint32_t)(cv.n_bytes - p0)) - 1u;
-  SegBits sb;
-  sb.k_lo = kcur;
-  const uint64_t s1 = s0 + kSegBytes;
+  if (p0 + 16 > cv.n_bytes) tm = p0 >= cv.n_bytes ? 0u : tm & ((1u << (uint32_t)(cv.n_bytes - p0)) - 1u);
+  const uint64_t s1 = (uint64_t)s0 + kSegBytes;
   uint32_t bm = 0;
   const uint64_t nb = (kcur < cv.n_docs) ? cv.doc_off[kcur] : ~0ull;  // warp-uniform
   if (nb < s1) {
@@ -114,61 +113,58 @@ __device__ __forceinline__ SegBits seg_bits(const ChunkView& cv, uint64_t seg, u
     bm = bnd_smem[lane];
     __syncwarp();
   }
-  sb.k_hi = kcur;
   uint32_t pv = __shfl_up_sync(0xffffffffu, tm >> 15, 1) & 1u;
   if (lane == 0) pv = prev;
+  SegBits sb;
   sb.tm = tm;
   sb.startm = tm & (~((tm << 1) | pv) | bm) & 0xFFFFu;
   sb.termm = (~tm | bm) & 0xFFFFu;
   return sb;
 }
 
-// segment-relative position of the first terminator in a later lane, or 0xFFFF
-__device__ __forceinline__ uint32_t next_term_later(uint32_t termm) {
+// Token structure of a segment that needs cross-lane information.
+struct SegTok {
+  uint32_t anyterm;    // ballot of lanes holding a terminator
+  uint32_t nt;         // per lane: first terminator in a later lane (segment-relative) or kNone
+  int open_lane;       // lane of the segment's last start if its token runs past the segment, else -1
+  uint32_t open_pos;   // its segment-relative position
+};
+
+__device__ __forceinline__ SegTok seg_tok(const SegBits& sb) {
   const uint32_t lane = lane_id();
-  const uint32_t ft = termm ? 16 * lane + __ffs(termm) - 1 : 0xFFFFu;
-  const uint32_t later = __ballot_sync(0xffffffffu, termm != 0) & ~((2u << lane) - 1u);
+  SegTok t;
+  t.anyterm = __ballot_sync(0xffffffffu, sb.termm != 0);
+  const uint32_t ft = sb.termm ? 16 * lane + __ffs(sb.termm) - 1 : kNone;
+  const uint32_t later = t.anyterm & ~((2u << lane) - 1u);
   const uint32_t v = __shfl_sync(0xffffffffu, ft, later ? __ffs(later) - 1 : lane);
-  return later ? v : 0xFFFFu;
-}
-
-// End of the token starting at absolute position sabs whose run reaches the end of its segment
-// (s1): the first non-token byte or document start at or after s1, capped at sabs + 256.
-__device__ __forceinline__ uint64_t far_end(const ChunkView& cv, uint64_t sabs, uint64_t s1, uint64_t k_hi) {
-  uint64_t limit = (k_hi < cv.n_docs) ? cv.doc_off[k_hi] : cv.n_bytes;
-  if (limit > cv.n_bytes) limit = cv.n_bytes;
-  if (limit > sabs + kMaxTermLen + 1) limit = sabs + kMaxTermLen + 1;
-  uint64_t p = s1;
-  while (p < limit) {
-    uint32_t word = 0;
-    if (p + 4 <= cv.n_bytes) word = __ldg((const uint32_t*)(cv.text + p));
-    else for (int b = 0; b < 4; ++b) if (p + b < cv.n_bytes) word |= (uint32_t)cv.text[p + b] << (8 * b);
-    const uint32_t t4 = tokmask4(word);
-    if (t4 != 0xFu) { p += __ffs(~t4) - 1; break; }
-    p += 4;
+  t.nt = later ? v : kNone;
+  t.open_lane = -1;
+  t.open_pos = 0;
+  const uint32_t hasS = __ballot_sync(0xffffffffu, sb.startm != 0);
+  if (hasS) {
+    const int H = 31 - __clz(hasS);
+    const int j = 31 - __clz(sb.startm | 1u);
+    const bool op = ((int)lane == H) && (sb.termm & ~((2u << j) - 1u)) == 0 && t.nt == kNone;
+    if (__ballot_sync(0xffffffffu, op)) {
+      t.open_lane = H;
+      t.open_pos = 16 * H + __shfl_sync(0xffffffffu, (uint32_t)j, H);
+    }
   }
-  return p > limit ? limit : p;
+  return t;
 }
 
-// The far end of the segment's last token, computed by the lane holding it (0 elsewhere / if none).
-__device__ __forceinline__ uint64_t seg_far_end(const ChunkView& cv, const SegBits& sb, uint64_t seg, uint32_t nt) {
+// segment-relative first terminator of the segment (warp-uniform), kNone if none
+__device__ __forceinline__ uint32_t first_term(const SegBits& sb, const SegTok& t) {
   const uint32_t lane = lane_id();
-  const uint32_t has = __ballot_sync(0xffffffffu, sb.startm != 0);
-  uint64_t fe = 0;
-  if (has && (int)lane == 31 - __clz(has)) {
-    const int j = 31 - __clz(sb.startm);
-    if ((sb.termm & ~((2u << j) - 1u)) == 0 && nt == 0xFFFFu)
-      fe = far_end(cv, seg * kSegBytes + 16 * lane + j, (seg + 1) * kSegBytes, sb.k_hi);
-  }
-  return fe;
+  const uint32_t ft = sb.termm ? 16 * lane + __ffs(sb.termm) - 1 : kNone;
+  const uint32_t v = __shfl_sync(0xffffffffu, ft, t.anyterm ? __ffs(t.anyterm) - 1 : 0);
+  return t.anyterm ? v : kNone;
 }
 
-__device__ __forceinline__ uint64_t token_end(const SegBits& sb, uint32_t nt, uint64_t fe, uint64_t s0, uint64_t p0,
-                                              int j) {
+// segment-relative end of the (non-open) token starting at lane bit j
+__device__ __forceinline__ uint32_t tok_end_rel(const SegBits& sb, const SegTok& t, int j) {
   const uint32_t above = sb.termm & ~((2u << j) - 1u);
-  if (above) return p0 + (__ffs(above) - 1);
-  if (nt != 0xFFFFu) return s0 + nt;
-  return fe;
+  return above ? 16 * lane_id() + __ffs(above) - 1 : t.nt;
 }
 
 // first boundary index k >= 1 with doc_off[k] >= start of each warp's segment range
@@ -183,41 +179,59 @@ __device__ __forceinline__ uint32_t prev_token_bit(const ChunkView& cv, uint64_t
 }
 
 // ------------------------------------------------------------------ pass 1: count
-__global__ void __launch_bounds__(kTokThreads) k_tok_count(ChunkView cv, uint64_t n_segs, const uint64_t* kstart,
+// A token that runs past the end of its segment ("open") is resolved by the first terminator of
+// the next segment (the warp reads one look-ahead segment past its range), so no lane ever scans
+// forward; only a run of 16 token bytes in a lane can hide a > 255-byte token inside a segment.
+__global__ void __launch_bounds__(kTokThreads) k_tok_count(ChunkView cv, uint32_t n_segs, const uint64_t* kstart,
                                                            uint32_t* range_count, unsigned long long* dropped) {
   __shared__ uint32_t bnd[kTokWarps][32];
   const uint32_t lane = lane_id();
   const int w = threadIdx.x >> 5;
-  const uint64_t gw = (uint64_t)blockIdx.x * kTokWarps + w;
-  const uint64_t sb0 = gw * kSegsPerWarp;
+  const uint32_t gw = blockIdx.x * kTokWarps + w;
+  const uint32_t sb0 = gw * kSegsPerWarp;
   if (sb0 >= n_segs) return;
-  const uint64_t se = min(sb0 + kSegsPerWarp, n_segs);
+  const uint32_t se = min(sb0 + kSegsPerWarp, n_segs);
+  const uint32_t last = se < n_segs ? se : se - 1;  // includes the look-ahead segment
   uint64_t kcur = kstart[gw];
-  uint32_t prev = prev_token_bit(cv, sb0 * kSegBytes);
+  uint32_t prev = prev_token_bit(cv, (uint64_t)sb0 * kSegBytes);
   uint32_t cnt = 0, drop = 0;
-  uint4 vnext = load_lane16(cv, sb0);
-  for (uint64_t seg = sb0; seg < se; ++seg) {
-    const uint4 v = vnext;
-    if (seg + 1 < se) vnext = load_lane16(cv, seg + 1);
-    const SegBits sb = seg_bits(cv, seg, v, prev, kcur, bnd[w]);
+  bool open = false;
+  uint32_t open_start = 0;
+  uint4 vr[kSegsPerWarp + 1];
+#pragma unroll
+  for (int j = 0; j <= kSegsPerWarp; ++j) vr[j] = (sb0 + j <= last) ? load_lane16(cv, sb0 + j) : make_uint4(0, 0, 0, 0);
+#pragma unroll
+  for (int jj = 0; jj <= kSegsPerWarp; ++jj) {
+    const uint32_t seg = sb0 + jj;
+    if (seg > last) break;
+    const uint4 v = vr[jj];
+    const uint32_t s0 = seg * kSegBytes;
+    const SegBits sb = seg_bits(cv, s0, v, prev, kcur, bnd[w]);
     prev = __shfl_sync(0xffffffffu, sb.tm, 31) >> 15;
-    const uint32_t nt = next_term_later(sb.termm);
-    const uint64_t fe = seg_far_end(cv, sb, seg, nt);
-    const uint64_t s0 = seg * kSegBytes, p0 = s0 + 16 * lane;
-    const bool maybe_long = __ballot_sync(0xffffffffu, sb.tm == 0xFFFFu) != 0;
-    if (!maybe_long) {
-      // only a token running past the segment can exceed 255 bytes
-      uint32_t c = __popc(sb.startm);
-      if (fe && fe - (p0 + 31 - __clz(sb.startm)) > kMaxTermLen) { --c; ++drop; }
-      cnt += c;
-    } else {
-      uint32_t sm = sb.startm;
-      while (sm) {
+    const SegTok tk = seg_tok(sb);
+    if (open) {
+      const uint32_t ft = first_term(sb, tk);
+      if (lane == 0) {
+        if (ft != kNone && s0 + ft - open_start <= kMaxTermLen) ++cnt; else ++drop;
+      }
+      open = false;
+    }
+    if (seg == se) break;  // look-ahead segment: resolution only
+    uint32_t c = __popc(sb.startm);
+    if ((int)lane == tk.open_lane) --c;
+    if (tk.open_lane >= 0) { open = true; open_start = s0 + tk.open_pos; }
+    if (__ballot_sync(0xffffffffu, sb.tm == 0xFFFFu)) {
+      for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
         const int j = __ffs(sm) - 1;
-        sm &= sm - 1;
-        if (token_end(sb, nt, fe, s0, p0, j) - (p0 + j) <= kMaxTermLen) ++cnt; else ++drop;
+        const uint32_t pos = 16 * lane + j;
+        if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
+        if (tok_end_rel(sb, tk, j) - pos > kMaxTermLen) { --c; ++drop; }
       }
     }
+    cnt += c;
+  }
+  if (open && lane == 0) {  // chunk end
+    if (cv.n_bytes - open_start <= kMaxTermLen) ++cnt; else ++drop;
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {
@@ -245,30 +259,31 @@ __device__ __forceinline__ uint64_t mix_hash(uint64_t h, uint64_t x) {
   return h ^ (h >> 29);
 }
 
-__device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* table, uint32_t mask, uint64_t h,
-                                                 uint32_t s_abs, uint32_t len, uint64_t mypfx,
+__device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* table, uint32_t* slot_ref, uint32_t mask,
+                                                 uint64_t h, uint64_t k0, uint64_t k1, uint32_t s_abs, uint32_t len,
                                                  const uint32_t* win32, uint32_t s_win, uint32_t* overflow) {
-  const uint64_t mine = (uint64_t)s_abs | ((uint64_t)len << 32) | (h & 0xFFFFFF0000000000ull);
   uint32_t i = (uint32_t)h & mask;
   for (int probe = 0; probe < 4096; ++probe) {
-    // Slots are claimed once (CAS on meta) and their pfx published once, so a cached read can
-    // only be stale-empty: the CAS or the volatile re-read below resolves it.
-    const ulonglong2 e = *(const ulonglong2*)(table + i);
-    uint64_t meta = e.x, pfx = e.y;
-    if (meta == 0) {
-      const unsigned long long prev = atomicCAS(&table[i].meta, 0ull, (unsigned long long)mine);
+    // Slots are claimed once (CAS on k0) and published once (k1), so a cached read can only be
+    // stale-empty: the CAS or the volatile re-read below resolves it.
+    ulonglong2 e = *(const ulonglong2*)(table + i);
+    if (e.x == 0) {
+      const unsigned long long prev = atomicCAS(&table[i].k0, 0ull, (unsigned long long)k0);
       if (prev == 0) {
-        *(volatile unsigned long long*)&table[i].pfx = mypfx;
+        slot_ref[i] = s_abs;
+        if (len > kSlotBytes) __threadfence();  // only > 11-byte terms are compared via slot_ref
+        *(volatile unsigned long long*)&table[i].k1 = k1;
         return i;
       }
-      meta = prev;
-      pfx = 0;
+      e.x = prev;
+      e.y = 0;
     }
-    if ((meta >> 32) == (mine >> 32)) {
-      while (pfx == 0) pfx = *(volatile unsigned long long*)&table[i].pfx;
-      if (pfx == mypfx) {
-        if (len <= 8) return i;
-        const TermWords other(text, (uint32_t)meta, len);
+    if (e.x == k0) {
+      while (e.y == 0) e.y = *(volatile unsigned long long*)&table[i].k1;
+      if (e.y == k1) {
+        if (len <= kSlotBytes) return i;
+        const uint32_t r = *(volatile uint32_t*)&slot_ref[i];
+        const TermWords other(text, r, len);
         bool eq = true;
         for (uint32_t k = 2; k * 4 < len; ++k)
           if (other.word(k) != win_word(win32, s_win, len, k)) { eq = false; break; }
@@ -281,21 +296,22 @@ __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* tabl
   return kMiss;
 }
 
-__global__ void __launch_bounds__(kTokThreads) k_tok_emit(ChunkView cv, uint64_t n_segs, const uint64_t* kstart,
+__global__ void __launch_bounds__(kTokThreads) k_tok_emit(ChunkView cv, uint32_t n_segs, const uint64_t* kstart,
                                                           const uint32_t* range_off, EmitOut eo) {
   __shared__ __align__(16) uint32_t win[kTokWarps][kWinBytes / 4];
-  __shared__ uint32_t queue[kTokWarps][kQueueCap];
+  __shared__ uint32_t queue[kTokWarps][kQueueCap + 1];
   __shared__ uint32_t bnd[kTokWarps][32];
   const uint32_t lane = lane_id();
   const int w = threadIdx.x >> 5;
-  const uint64_t gw = (uint64_t)blockIdx.x * kTokWarps + w;
-  const uint64_t sb0 = gw * kSegsPerWarp;
+  const uint32_t gw = blockIdx.x * kTokWarps + w;
+  const uint32_t sb0 = gw * kSegsPerWarp;
   if (sb0 >= n_segs) return;
-  const uint64_t se = min(sb0 + kSegsPerWarp, n_segs);
-  const uint64_t B0 = sb0 * kSegBytes;
+  const uint32_t se = min(sb0 + kSegsPerWarp, n_segs);
+  const uint32_t last = se < n_segs ? se : se - 1;
+  const uint32_t B0 = sb0 * kSegBytes;
   uint32_t* w32 = win[w];
   uint32_t* q = queue[w];
-  // stage the range and one more segment (tokens may run past the range)
+  // stage the range and the look-ahead segment (tokens may run past the range)
   uint4 v[kSegsPerWarp + 1];
 #pragma unroll
   for (int j = 0; j <= kSegsPerWarp; ++j) v[j] = load_lane16(cv, sb0 + j);
@@ -310,6 +326,8 @@ __global__ void __launch_bounds__(kTokThreads) k_tok_emit(ChunkView cv, uint64_t
   uint32_t qn = 0;
   uint64_t obase = range_off[gw];
   uint64_t k_range_hi = k_range_lo;
+  bool open = false;
+  uint32_t open_start = 0;
 
   auto flush = [&]() {
     for (uint32_t r = 0; r < qn; r += 32) {
@@ -317,7 +335,7 @@ __global__ void __launch_bounds__(kTokThreads) k_tok_emit(ChunkView cv, uint64_t
       if (idx < qn) {
         const uint32_t e = q[idx];
         const uint32_t s_win = e >> 8, len = e & 255u;
-        const uint32_t s_abs = (uint32_t)(B0 + s_win);
+        const uint32_t s_abs = B0 + s_win;
         uint32_t wd[4];
 #pragma unroll
         for (int k = 0; k < 4; ++k) wd[k] = (4u * k < len) ? win_word(w32, s_win, len, k) : 0u;
@@ -337,11 +355,13 @@ __global__ void __launch_bounds__(kTokThreads) k_tok_emit(ChunkView cv, uint64_t
           if (cv.doc_off[mid] <= s_abs) lo = mid + 1; else hi = mid;
         }
         const uint32_t doc = eo.doc_base + (uint32_t)(lo - 1);
-        const uint64_t pfx = (uint64_t)wd[0] | ((uint64_t)wd[1] << 32);
-        const uint32_t slot = table_insert(cv.text, eo.table, eo.mask, h, s_abs, len, pfx, w32, s_win, eo.overflow);
+        const uint64_t k0 = (uint64_t)len | (((h >> 40) & 0xFFFFFFull) << 8) | ((uint64_t)wd[0] << 32);
+        const uint64_t k1 = (uint64_t)wd[1] | ((uint64_t)(wd[2] & 0xFFFFFFu) << 32) | (1ull << 56);
+        const uint32_t slot =
+            table_insert(cv.text, eo.table, eo.slot_ref, eo.mask, h, k0, k1, s_abs, len, w32, s_win, eo.overflow);
         const uint64_t out = obase + idx;
-        eo.slot[out] = slot;
-        eo.doc[out] = doc;
+        __stcs(eo.slot + out, slot);
+        __stcs(eo.doc + out, doc);
         if (eo.dbg_start) { eo.dbg_start[out] = s_abs; eo.dbg_len[out] = len; }
       }
     }
@@ -350,19 +370,31 @@ __global__ void __launch_bounds__(kTokThreads) k_tok_emit(ChunkView cv, uint64_t
     __syncwarp();
   };
 
-  for (uint64_t seg = sb0; seg < se; ++seg) {
-    const int j = (int)(seg - sb0);
+  for (uint32_t seg = sb0; seg <= last; ++seg) {
+    const uint32_t j = seg - sb0;
+    const uint32_t s0 = seg * kSegBytes;
     const uint4 vv = *(const uint4*)&w32[(j * kSegBytes + 16 * lane) / 4];
-    const SegBits sb = seg_bits(cv, seg, vv, prev, kcur, bnd[w]);
+    const SegBits sb = seg_bits(cv, s0, vv, prev, kcur, bnd[w]);
     prev = __shfl_sync(0xffffffffu, sb.tm, 31) >> 15;
+    const SegTok tk = seg_tok(sb);
+    if (open) {  // the previous segment's last token ends in this one
+      const uint32_t ft = first_term(sb, tk);
+      if (ft != kNone && s0 + ft - open_start <= kMaxTermLen) {
+        if (qn + 1 > (uint32_t)kQueueCap) flush();
+        if (lane == 0) q[qn] = ((open_start - B0) << 8) | (s0 + ft - open_start);
+        ++qn;
+        __syncwarp();
+      }
+      open = false;
+    }
+    if (seg == se) break;
     k_range_hi = kcur;
-    const uint32_t nt = next_term_later(sb.termm);
-    const uint64_t fe = seg_far_end(cv, sb, seg, nt);
-    const uint64_t s0 = seg * kSegBytes, p0 = s0 + 16 * lane;
     uint32_t c = 0;
     for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
       const int jb = __ffs(sm) - 1;
-      c += (token_end(sb, nt, fe, s0, p0, jb) - (p0 + jb) <= kMaxTermLen) ? 1u : 0u;
+      const uint32_t pos = 16 * lane + jb;
+      if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
+      c += (tok_end_rel(sb, tk, jb) - pos <= kMaxTermLen) ? 1u : 0u;
     }
     uint32_t inc = c;
 #pragma unroll
@@ -372,14 +404,26 @@ __global__ void __launch_bounds__(kTokThreads) k_tok_emit(ChunkView cv, uint64_t
     }
     const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
     if (qn + tot > (uint32_t)kQueueCap) flush();
-    uint32_t pos = qn + inc - c;
+    uint32_t pos_q = qn + inc - c;
     for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
       const int jb = __ffs(sm) - 1;
-      const uint64_t len = token_end(sb, nt, fe, s0, p0, jb) - (p0 + jb);
-      if (len <= kMaxTermLen) q[pos++] = ((uint32_t)(p0 + jb - B0) << 8) | (uint32_t)len;
+      const uint32_t pos = 16 * lane + jb;
+      if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
+      const uint32_t len = tok_end_rel(sb, tk, jb) - pos;
+      if (len <= kMaxTermLen) q[pos_q++] = ((s0 + pos - B0) << 8) | len;
     }
     qn += tot;
+    if (tk.open_lane >= 0) { open = true; open_start = s0 + tk.open_pos; }
     __syncwarp();
+  }
+  k_range_hi = kcur;
+  if (open) {  // chunk end
+    if (cv.n_bytes - open_start <= kMaxTermLen) {
+      if (qn + 1 > (uint32_t)kQueueCap) flush();
+      if (lane == 0) q[qn] = ((open_start - B0) << 8) | (uint32_t)(cv.n_bytes - open_start);
+      ++qn;
+      __syncwarp();
+    }
   }
   flush();
 }
