@@ -70,6 +70,50 @@ __device__ __forceinline__ TermInfo term_info(const uint8_t* text, uint64_t ref,
 
 __host__ __device__ __forceinline__ uint32_t bucket_plen(uint32_t b) { return b == 0 ? 0u : (b <= 36 ? 1u : 3u); }
 
+// Folded byte i of a chunk unique term: the first 16 bytes are held in w (built from its table slot),
+// longer terms read the rest from their first occurrence in the chunk text.
+__device__ __forceinline__ uint32_t ubyte(const uint4& w, const uint8_t* text, uint32_t ref, uint32_t i) {
+  if (i < 16) {
+    const uint32_t x = i < 8 ? (i < 4 ? w.x : w.y) : (i < 12 ? w.z : w.w);
+    return (x >> (8 * (i & 3))) & 0xFFu;
+  }
+  const uint32_t c = text[ref + i];
+  return (c - 'A' < 26u) ? c + 32 : c;
+}
+
+// Table I index etc. of a unique term given its first 16 folded bytes (w) and length.
+__device__ __forceinline__ TermInfo term_info_w(const uint4& w, const uint8_t* text, uint32_t ref, uint32_t len) {
+  bool digits = true;
+  const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+  for (uint32_t k = 0; k < 4; ++k) {
+    if (4 * k >= len) break;
+    const uint32_t rem = len - 4 * k;
+    const uint32_t valid = rem >= 4 ? 0x80808080u : (0x80808080u & ((1u << (8 * rem)) - 1u));
+    if ((digit4(ws[k]) & valid) != valid) digits = false;
+  }
+  for (uint32_t i = 16; i < len && digits; ++i) digits = ubyte(w, text, ref, i) - '0' < 10u;
+  const uint32_t b0 = ws[0] & 0xFFu, b1 = (ws[0] >> 8) & 0xFFu, b2 = (ws[0] >> 16) & 0xFFu;
+  TermInfo ti;
+  if (digits) { ti.bucket = 1 + (b0 - '0'); ti.plen = 1; }
+  else if (is_letter(b0)) {
+    if (len > 3 && is_letter(b1) && is_letter(b2)) { ti.bucket = 37 + 676 * (b0 - 'a') + 26 * (b1 - 'a') + (b2 - 'a'); ti.plen = 3; }
+    else { ti.bucket = 11 + (b0 - 'a'); ti.plen = 1; }
+  } else { ti.bucket = 0; ti.plen = 0; }
+  ti.slen = len - ti.plen;
+  uint32_t c = 0;
+  uint64_t k6 = 0;
+#pragma unroll
+  for (uint32_t i = 0; i < 6; ++i) {
+    const uint32_t b = (ti.plen + i < len) ? ubyte(w, text, ref, ti.plen + i) : 0u;
+    if (i < 4) c |= b << (24 - 8 * i);
+    k6 |= (uint64_t)b << (40 - 8 * i);
+  }
+  ti.cache = c;
+  ti.key = ((uint64_t)ti.bucket << 48) | k6;
+  return ti;
+}
+
 __host__ __device__ __forceinline__ uint32_t prefix_byte(uint32_t b, uint32_t i) {
   if (b <= 10) return '0' + (b - 1);
   if (b <= 36) return 'a' + (b - 11);
@@ -83,24 +127,24 @@ __device__ __forceinline__ uint32_t text_sfx_byte(const uint8_t* text, uint64_t 
   return (c - 'A' < 26u) ? c + 32 : c;
 }
 
-// sign(chunk term suffix - arena term), given that the first 4 suffix bytes are equal.
-__device__ __forceinline__ int cmp_sfx_arena(const uint8_t* text, uint64_t ref, uint32_t plen, uint32_t slen,
-                                             const uint8_t* arena, uint32_t aoff) {
+// sign(unique term suffix - arena term), given that the first 4 suffix bytes are equal.
+__device__ __forceinline__ int cmp_sfx_arena(const uint4& w, const uint8_t* text, uint32_t ref, uint32_t plen,
+                                             uint32_t slen, const uint8_t* arena, uint32_t aoff) {
   const uint32_t alen = arena[aoff];
   const uint32_t m = slen < alen ? slen : alen;
   for (uint32_t i = 4; i < m; ++i) {
-    const uint32_t x = text_sfx_byte(text, ref, plen, i), y = arena[aoff + 1 + i];
+    const uint32_t x = ubyte(w, text, ref, plen + i), y = arena[aoff + 1 + i];
     if (x != y) return x < y ? -1 : 1;
   }
   return slen == alen ? 0 : (slen < alen ? -1 : 1);
 }
 
-// sign(chunk term a - chunk term b) on suffixes, starting at byte `from`.
-__device__ __forceinline__ int cmp_sfx_sfx(const uint8_t* text, uint64_t ra, uint32_t la, uint64_t rb, uint32_t lb,
-                                           uint32_t plen, uint32_t from) {
+// sign(unique a - unique b) on suffixes (same prefix length), starting at suffix byte `from`.
+__device__ __forceinline__ int cmp_sfx_sfx(const uint4& wa, uint32_t ra, uint32_t la, const uint4& wb, uint32_t rb,
+                                           uint32_t lb, const uint8_t* text, uint32_t plen, uint32_t from) {
   const uint32_t m = la < lb ? la : lb;
   for (uint32_t i = from; i < m; ++i) {
-    const uint32_t x = text_sfx_byte(text, ra, plen, i), y = text_sfx_byte(text, rb, plen, i);
+    const uint32_t x = ubyte(wa, text, ra, plen + i), y = ubyte(wb, text, rb, plen + i);
     if (x != y) return x < y ? -1 : 1;
   }
   return la == lb ? 0 : (la < lb ? -1 : 1);
@@ -142,6 +186,7 @@ struct DictView {
 
 struct UniqueView {
   const uint8_t* text;
+  const uint4* w;
   const uint32_t* ref;
   const uint32_t* len;
   const uint32_t* bucket;
@@ -149,8 +194,8 @@ struct UniqueView {
 };
 
 // Warp-cooperative descent for one key.  Returns termID (tid) or kMiss with *ins_rank set.
-__device__ __forceinline__ uint32_t probe_key(const DictView& dv, const uint8_t* text, uint64_t ref, uint32_t len,
-                                              uint32_t bucket, uint32_t cache, uint32_t* ins_rank) {
+__device__ __forceinline__ uint32_t probe_key(const DictView& dv, const uint4& w, const uint8_t* text, uint32_t ref,
+                                              uint32_t len, uint32_t bucket, uint32_t cache, uint32_t* ins_rank) {
   const uint32_t lane = lane_id();
   const uint32_t n = dv.coll_n[bucket];
   if (n == 0) { *ins_rank = 0; return kMiss; }
@@ -164,7 +209,7 @@ __device__ __forceinline__ uint32_t probe_key(const DictView& dv, const uint8_t*
     int cmp = 0;
     if (valid) {
       if (cache != wv) cmp = cache < wv ? -1 : 1;
-      else if (slen >= 4) cmp = cmp_sfx_arena(text, ref, plen, slen, dv.arena, __ldg(&nd->str[lane - 1]));
+      else if (slen >= 4) cmp = cmp_sfx_arena(w, text, ref, plen, slen, dv.arena, __ldg(&nd->str[lane - 1]));
     }
     const uint32_t eq = __ballot_sync(0xffffffffu, valid && cmp == 0);
     if (eq) {
@@ -185,24 +230,32 @@ __global__ void k_probe(DictView dv, UniqueView uv, uint32_t U, uint32_t* tid_ou
   const uint32_t warps = gridDim.x * (blockDim.x >> 5);
   for (uint32_t u = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); u < U; u += warps) {
     uint32_t r = 0;
-    const uint32_t t = probe_key(dv, uv.text, uv.ref[u], uv.len[u], uv.bucket[u], uv.cache[u], &r);
+    const uint32_t t = probe_key(dv, uv.w[u], uv.text, uv.ref[u], uv.len[u], uv.bucket[u], uv.cache[u], &r);
     if (lane_id() == 0) { tid_out[u] = t; rank_out[u] = r; }
   }
 }
 
-// unique gather: occupied slot i -> unique index uid[i]; term info from the first occurrence
+// unique gather (slot order, sequential): occupied slot i -> unique index uid[i]; the term's first
+// 11 folded bytes come from the slot itself, longer terms read their first occurrence
 __global__ void k_unique_gather(const Slot* table, const uint32_t* slot_ref, uint32_t C, const uint32_t* uid,
-                                const uint8_t* text,
-                                uint32_t* u_ref, uint32_t* u_len, uint32_t* u_bucket, uint32_t* u_cache,
-                                uint64_t* u_key) {
+                                const uint8_t* text, uint4* u_w, uint32_t* u_ref, uint32_t* u_len, uint32_t* u_bucket,
+                                uint32_t* u_cache, uint64_t* u_key) {
   const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= C) return;
-  const uint64_t e = table[i].k0;
-  if (e == 0) return;
+  const ulonglong2 e = *(const ulonglong2*)(table + i);
+  if (e.x == 0) return;
   const uint32_t u = uid[i];
-  const uint32_t ref = slot_ref[i], len = (uint32_t)e & 0xFFu;
-  const TermInfo ti = term_info(text, ref, len);
-  u_ref[u] = ref; u_len[u] = len; u_bucket[u] = ti.bucket; u_cache[u] = ti.cache; u_key[u] = ti.key;
+  const uint32_t len = (uint32_t)e.x & 0xFFu;
+  const uint32_t ref = slot_ref[i];
+  uint4 w;
+  if (len <= kSlotBytes) {
+    w = make_uint4((uint32_t)(e.x >> 32), (uint32_t)e.y, (uint32_t)(e.y >> 32) & 0xFFFFFFu, 0u);
+  } else {
+    const TermWords tw(text, ref, len);
+    w = make_uint4(tw.word(0), tw.word(1), tw.word(2), tw.word(3));
+  }
+  const TermInfo ti = term_info_w(w, text, ref, len);
+  u_w[u] = w; u_ref[u] = ref; u_len[u] = len; u_bucket[u] = ti.bucket; u_cache[u] = ti.cache; u_key[u] = ti.key;
 }
 
 // compact the misses: nk_key/nk_val in unique order (radix-sorted next)
@@ -217,8 +270,8 @@ __global__ void k_miss_compact(const uint32_t* u_tid, const uint32_t* midx, cons
 
 // Runs of equal (bucket, 6-byte) keys are ordered by the rest of the suffix (insertion sort by the
 // run's first thread; runs are rare and short: two new terms sharing bucket + 6 suffix bytes).
-__global__ void k_tie_fix(const uint64_t* key, uint32_t* val, uint32_t N, const uint8_t* text, const uint32_t* u_ref,
-                          const uint32_t* u_len) {
+__global__ void k_tie_fix(const uint64_t* key, uint32_t* val, uint32_t N, const uint8_t* text, const uint4* u_w,
+                          const uint32_t* u_ref, const uint32_t* u_len) {
   const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= N) return;
   if (i > 0 && key[i - 1] == key[i]) return;
@@ -228,11 +281,12 @@ __global__ void k_tie_fix(const uint64_t* key, uint32_t* val, uint32_t N, const 
   const uint32_t plen = bucket_plen((uint32_t)(key[i] >> 48));
   for (uint32_t a = i + 1; a < e; ++a) {
     const uint32_t x = val[a];
+    const uint4 wx = u_w[x];
     const uint32_t rx = u_ref[x], lx = u_len[x] - plen;
     uint32_t b = a;
     while (b > i) {
       const uint32_t y = val[b - 1];
-      if (cmp_sfx_sfx(text, u_ref[y], u_len[y] - plen, rx, lx, plen, 6) <= 0) break;
+      if (cmp_sfx_sfx(u_w[y], u_ref[y], u_len[y] - plen, wx, rx, lx, text, plen, 6) <= 0) break;
       val[b] = y;
       --b;
     }
@@ -243,7 +297,7 @@ __global__ void k_tie_fix(const uint64_t* key, uint32_t* val, uint32_t N, const 
 // New terms in sorted order: termIDs by warp-aggregated atomics (the paper's GPU indexer assigns
 // postings pointers as it inserts), arena append <len><suffix> (Fig. 6), per-term columns.
 __global__ void k_new_terms(const uint32_t* sorted_u, uint32_t N, const uint32_t* aoff, uint64_t arena_base,
-                            const uint8_t* text, const uint32_t* u_ref, const uint32_t* u_len,
+                            const uint8_t* text, const uint4* u_w, const uint32_t* u_ref, const uint32_t* u_len,
                             const uint32_t* u_bucket, const uint32_t* u_cache, const uint32_t* u_rank,
                             uint32_t* u_tid, uint32_t* tid_counter, uint8_t* arena, uint32_t* t_arena,
                             uint32_t* t_cache, uint32_t* t_bucket, uint32_t* ns_tid, uint32_t* ns_bucket,
@@ -261,7 +315,8 @@ __global__ void k_new_terms(const uint32_t* sorted_u, uint32_t N, const uint32_t
   const uint32_t b = u_bucket[u], plen = bucket_plen(b), ref = u_ref[u], slen = u_len[u] - plen;
   const uint64_t off = arena_base + aoff[k];
   arena[off] = (uint8_t)slen;
-  for (uint32_t i = 0; i < slen; ++i) arena[off + 1 + i] = (uint8_t)text_sfx_byte(text, ref, plen, i);
+  const uint4 w = u_w[u];
+  for (uint32_t i = 0; i < slen; ++i) arena[off + 1 + i] = (uint8_t)ubyte(w, text, ref, plen + i);
   t_arena[tid] = (uint32_t)off;
   t_cache[tid] = u_cache[u];
   t_bucket[tid] = b;

@@ -110,7 +110,7 @@ struct wj_index {
   // token stream (termID, docID) of all chunks
   DevBuf g_tid, g_doc;
   // chunk scratch
-  DevBuf text_stage, doc_stage, seg_cnt, table, uid, u_ref, u_len, u_bucket, u_cache, u_key, u_tid, u_rank, midx, nk_key,
+  DevBuf text_stage, doc_stage, seg_cnt, table, uid, u_w, u_ref, u_len, u_bucket, u_cache, u_key, u_tid, u_rank, midx, nk_key,
       nk_val, nk_key2, nk_val2, aoff, ns_tid, ns_bucket, ns_rank, nlo, nhi, nbase, lvA[4], lvB[4], child_off, root_idx,
       scan_scr, hist, hist_scan, os_hist, os_look, os_ctr, kstart, slotref, dbg_start, dbg_len, dbg_off, dbg_out, dbg_slot, dbg_doc, lexg, qbuf, qres;
   // finalize
@@ -165,7 +165,7 @@ struct wj_index {
   void free_all() {
     DevBuf* all[] = {&nodes, &coll_root, &coll_n, &coll_base, &coll_base2, &e_tid, &e_bkt, &e_tid2, &e_bkt2, &arena,
                      &t_arena, &t_cache, &t_bucket, &scal, &g_tid, &g_doc, &text_stage, &doc_stage, &seg_cnt, &table,
-                     &uid, &u_ref, &u_len, &u_bucket, &u_cache, &u_key, &u_tid, &u_rank, &midx, &nk_key, &nk_val,
+                     &uid, &u_w, &u_ref, &u_len, &u_bucket, &u_cache, &u_key, &u_tid, &u_rank, &midx, &nk_key, &nk_val,
                      &nk_key2, &nk_val2, &aoff, &ns_tid, &ns_bucket, &ns_rank, &nlo, &nhi, &nbase, &child_off,
                      &root_idx, &scan_scr, &hist, &hist_scan, &os_hist, &os_look, &os_ctr, &kstart, &slotref, &dbg_start, &dbg_len, &dbg_off, &dbg_out, &dbg_slot,
                      &dbg_doc, &lexg, &qbuf, &qres, &rank_of, &term_at, &sk1, &sv1, &pidx, &out_doc, &out_tf,
@@ -379,6 +379,32 @@ struct wj_index {
     });
   }
 
+  // L2 persisting access-policy window on the context stream (best effort; cleared with bytes == 0)
+  size_t l2_persist_max = 0;
+  void set_l2_window(void* p, size_t bytes) {
+    if (l2_persist_max == 0) {
+      int v = 0;
+      cudaDeviceGetAttribute(&v, cudaDevAttrMaxPersistingL2CacheSize, device);
+      l2_persist_max = v > 0 ? (size_t)v : 1;
+      if (v > 0 && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)v) != cudaSuccess) cudaGetLastError();
+    }
+    if (l2_persist_max <= 1) return;
+    cudaStreamAttrValue a;
+    memset(&a, 0, sizeof(a));
+    if (bytes) {
+      int maxw = 0;
+      cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, device);
+      const size_t win = std::min(bytes, (size_t)maxw);
+      a.accessPolicyWindow.base_ptr = p;
+      a.accessPolicyWindow.num_bytes = win;
+      a.accessPolicyWindow.hitRatio = (float)std::min(1.0, (double)l2_persist_max / (double)win);
+      a.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+      a.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    }
+    if (cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &a) != cudaSuccess) cudaGetLastError();
+    if (!bytes && cudaCtxResetPersistingL2Cache() != cudaSuccess) cudaGetLastError();
+  }
+
   static uint64_t pow2_at_least(uint64_t x) {
     uint64_t c = 1;
     while (c < x) c <<= 1;
@@ -405,8 +431,8 @@ struct wj_index {
     const uint64_t Nc = count_tokens(cv, n_segs);
     n_dropped += h_scal[1];
     if (n_tokens + Nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 tokens in one index"};
-    uint32_t* gt = buf_keep<uint32_t>(g_tid, n_tokens + Nc, n_tokens);
-    uint32_t* gd = buf_keep<uint32_t>(g_doc, n_tokens + Nc, n_tokens);
+    uint32_t* gt = buf_keep<uint32_t>(g_tid, n_tokens + Nc + 16, n_tokens);  // +16: TMA round-up reads
+    uint32_t* gd = buf_keep<uint32_t>(g_doc, n_tokens + Nc + 16, n_tokens);
     if (Nc == 0) {
       n_docs += nd;
       phase(-1);
@@ -435,6 +461,7 @@ struct wj_index {
     table_est = (U * 5) / 4;
 
     // unique terms: first occurrence, Table I bucket, stripped-suffix cache, sort key
+    uint4* uw = buf<uint4>(u_w, U);
     uint32_t* ur = buf<uint32_t>(u_ref, U);
     uint32_t* ul = buf<uint32_t>(u_len, U);
     uint32_t* ub = buf<uint32_t>(u_bucket, U);
@@ -442,7 +469,7 @@ struct wj_index {
     uint64_t* uk = buf<uint64_t>(u_key, U);
     uint32_t* ut = buf<uint32_t>(u_tid, U);
     uint32_t* urk = buf<uint32_t>(u_rank, U);
-    k_unique_gather<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, (const uint32_t*)slotref.p, (uint32_t)C, slot_uid, text, ur, ul, ub,
+    k_unique_gather<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, (const uint32_t*)slotref.p, (uint32_t)C, slot_uid, text, uw, ur, ul, ub,
                                                       uc, uk);
     launched();
 
@@ -450,7 +477,7 @@ struct wj_index {
     phase(WJ_PHASE_PROBE);
     DictView dv{(const Node*)nodes.p, (const uint32_t*)coll_root.p, (const uint32_t*)coll_n.p, (const uint8_t*)arena.p};
     if (V > 0) {
-      UniqueView uv{text, ur, ul, ub, uc};
+      UniqueView uv{text, uw, ur, ul, ub, uc};
       const unsigned blocks = (unsigned)std::min<uint64_t>((U + 7) / 8, 148ull * 64);
       ktime(WJ_KERNEL_PROBE, [&] {
         k_probe<<<blocks, 256, 0, st>>>(dv, uv, (uint32_t)U, ut, urk);
@@ -494,10 +521,10 @@ struct wj_index {
   }
 
   void insert_new(const uint8_t* text, uint64_t U, uint64_t Nn) {
-    uint64_t* kk = buf<uint64_t>(nk_key, Nn);
-    uint32_t* kv = buf<uint32_t>(nk_val, Nn);
-    uint64_t* kk2 = buf<uint64_t>(nk_key2, Nn);
-    uint32_t* kv2 = buf<uint32_t>(nk_val2, Nn);
+    uint64_t* kk = buf<uint64_t>(nk_key, Nn + 16);
+    uint32_t* kv = buf<uint32_t>(nk_val, Nn + 16);
+    uint64_t* kk2 = buf<uint64_t>(nk_key2, Nn + 16);
+    uint32_t* kv2 = buf<uint32_t>(nk_val2, Nn + 16);
     k_miss_compact<<<grid_for(U, 256), 256, 0, st>>>((const uint32_t*)u_tid.p, (const uint32_t*)midx.p,
                                                      (const uint64_t*)u_key.p, (uint32_t)U, kk, kv);
     launched();
@@ -505,7 +532,7 @@ struct wj_index {
     const bool in2 = sort_pairs<uint64_t>(kk, kv, kk2, kv2, Nn, 0, 63, nullptr, false);
     uint64_t* sk = in2 ? kk2 : kk;
     uint32_t* sv = in2 ? kv2 : kv;
-    k_tie_fix<<<grid_for(Nn, 256), 256, 0, st>>>(sk, sv, (uint32_t)Nn, text, (const uint32_t*)u_ref.p,
+    k_tie_fix<<<grid_for(Nn, 256), 256, 0, st>>>(sk, sv, (uint32_t)Nn, text, (const uint4*)u_w.p, (const uint32_t*)u_ref.p,
                                                  (const uint32_t*)u_len.p);
     launched();
     // arena offsets
@@ -527,7 +554,8 @@ struct wj_index {
     uint32_t* counter = (uint32_t*)(dscal() + 6);
     k_fill<uint32_t><<<1, 1, 0, st>>>(counter, 1, V);
     launched();
-    k_new_terms<<<grid_for(Nn, 256), 256, 0, st>>>(sv, (uint32_t)Nn, ao, arena_used, text, (const uint32_t*)u_ref.p,
+    k_new_terms<<<grid_for(Nn, 256), 256, 0, st>>>(sv, (uint32_t)Nn, ao, arena_used, text, (const uint4*)u_w.p,
+                                                   (const uint32_t*)u_ref.p,
                                                    (const uint32_t*)u_len.p, (const uint32_t*)u_bucket.p,
                                                    (const uint32_t*)u_cache.p, (const uint32_t*)u_rank.p,
                                                    (uint32_t*)u_tid.p, counter, ar, ta, tc, tb, nt, nb, nr);
@@ -603,50 +631,56 @@ struct wj_index {
     height_max = depth;
   }
 
-  // stable LSD radix sort driver: onesweep (radix.cuh).  rank_of != nullptr maps keys first.
+  // stable LSD radix sort driver (radix.cuh: per pass k_rs_up + scan + k_rs_down).  segs (optional):
+  // per stream segment a key map applied in place by the first upsweep (slot -> rank).
   template <typename K>
   bool sort_pairs(K* k0, uint32_t* v0, K* k1, uint32_t* v1, uint64_t n, int begin_bit, int end_bit,
                   const uint32_t* rank_of, bool timed,
                   const std::vector<std::pair<uint64_t, const uint32_t*>>* segs = nullptr) {
     if (n == 0) return false;
     const int passes = end_bit > begin_bit ? (end_bit - begin_bit + 7) / 8 : 0;
-    if (n == 1 && !rank_of && !segs) return false;
-    uint32_t* gh = buf<uint32_t>(os_hist, (uint64_t)std::max(passes, 1) * 256);
-    WJ_CUDA_CHECK(cudaMemsetAsync(gh, 0, (size_t)std::max(passes, 1) * 256 * 4, st));
-    // histogram of every digit; segs (optional): per stream segment a key map (slot -> rank)
-    const size_t nseg = segs ? segs->size() : 1;
-    for (size_t sgi = 0; sgi < nseg; ++sgi) {
-      const uint64_t off = segs ? (*segs)[sgi].first : 0;
-      const uint64_t end = segs ? (sgi + 1 < nseg ? (*segs)[sgi + 1].first : n) : n;
-      const uint32_t* map = segs ? (*segs)[sgi].second : rank_of;
-      if (end <= off) continue;
-      const unsigned hb = (unsigned)std::min<uint64_t>((end - off + 255) / 256, 148ull * 8);
-      auto hist_launch = [&] {
-        k_os_hist<K><<<hb, 256, 0, st>>>(k0 + off, end - off, begin_bit, passes, map, gh);
-        launched();
-      };
-      if (timed) ktime(WJ_KERNEL_SORT_HIST, hist_launch); else hist_launch();
+    // apply key maps (when there is nothing to sort the map is still applied)
+    auto map_only = [&](uint64_t off, uint64_t cnt, const uint32_t* map) {
+      k_map_rank<<<grid_for(cnt, 256), 256, 0, st>>>((uint32_t*)(k0 + off), cnt, map);
+      launched();
+    };
+    const bool multi_map = segs && segs->size() > 1;
+    if (segs && (passes == 0 || n == 1 || multi_map)) {
+      for (size_t i = 0; i < segs->size(); ++i) {
+        const uint64_t off = (*segs)[i].first;
+        const uint64_t end = i + 1 < segs->size() ? (*segs)[i + 1].first : n;
+        if (end > off) {
+          if (timed) ktime(WJ_KERNEL_SORT_HIST, [&] { map_only(off, end - off, (*segs)[i].second); });
+          else map_only(off, end - off, (*segs)[i].second);
+        }
+      }
     }
     if (passes == 0 || n == 1) return false;
-    k_os_hist_scan<<<passes, 256, 0, st>>>(gh);
-    launched();
-    const uint64_t tiles = (n + kOsTile - 1) / kOsTile;
-    uint64_t* lk = buf<uint64_t>(os_look, (uint64_t)passes * tiles * 256);
-    uint32_t* ctr = buf<uint32_t>(os_ctr, passes);
-    WJ_CUDA_CHECK(cudaMemsetAsync(lk, 0, (size_t)passes * tiles * 256 * 8, st));
-    WJ_CUDA_CHECK(cudaMemsetAsync(ctr, 0, (size_t)passes * 4, st));
+    const uint32_t* first_map = (segs && !multi_map) ? (*segs)[0].second : rank_of;
+    uint64_t per = (n + kRsCtas - 1) / kRsCtas;
+    per = (per + kOsTile - 1) / kOsTile * kOsTile;
+    const uint32_t G = (uint32_t)((n + per - 1) / per);
+    uint32_t* h1 = buf<uint32_t>(hist, (uint64_t)256 * G);
+    uint32_t* h2 = buf<uint32_t>(hist_scan, (uint64_t)256 * G);
     bool in1 = false;
     for (int p = 0; p < passes; ++p) {
       K* ki = in1 ? k1 : k0;
       uint32_t* vi = in1 ? v1 : v0;
       K* ko = in1 ? k0 : k1;
       uint32_t* vo = in1 ? v0 : v1;
-      auto pass_launch = [&] {
-        k_os_pass<K><<<(unsigned)tiles, kOsThreads, os_smem_bytes<K>(), st>>>(
-            ki, vi, ko, vo, n, begin_bit + 8 * p, gh + 256 * p, lk + (uint64_t)p * tiles * 256, ctr + p);
+      const int shift = begin_bit + 8 * p;
+      const uint32_t* mp = p == 0 ? first_map : nullptr;
+      auto up = [&] {
+        k_rs_up<K><<<G, 256, 0, st>>>(ki, n, per, shift, mp, h1);
         launched();
       };
-      if (timed) ktime(WJ_KERNEL_SORT_SCATTER, pass_launch); else pass_launch();
+      if (timed) ktime(WJ_KERNEL_SORT_HIST, up); else up();
+      scan<uint32_t>(ArrayIn<uint32_t>{h1}, (uint64_t)256 * G, h2, (uint32_t*)nullptr);
+      auto down = [&] {
+        k_rs_down2<K><<<G, kDsThreads, ds_smem_bytes<K>(), st>>>(ki, vi, ko, vo, n, per, shift, h2);
+        launched();
+      };
+      if (timed) ktime(WJ_KERNEL_SORT_SCATTER, down); else down();
       in1 = !in1;
     }
     return in1;
@@ -677,8 +711,8 @@ struct wj_index {
       phase(WJ_PHASE_SORT);
       uint32_t* kt = (uint32_t*)g_tid.p;
       uint32_t* dt = (uint32_t*)g_doc.p;
-      uint32_t* k1 = buf<uint32_t>(sk1, N);
-      uint32_t* v1 = buf<uint32_t>(sv1, N);
+      uint32_t* k1 = buf<uint32_t>(sk1, N + 16);
+      uint32_t* v1 = buf<uint32_t>(sv1, N + 16);
       int bits = 0;
       while (bits < 32 && ((uint64_t)1 << bits) < V) ++bits;
       // per chunk: slot -> termID -> rank map; applied in the histogram pass; the stable sort by
@@ -697,24 +731,24 @@ struct wj_index {
       uint32_t* spare_v = in1 ? dt : v1;
 
       phase(WJ_PHASE_POSTINGS);
-      const uint64_t tiles = (N + kRleTile - 1) / kRleTile;
-      uint64_t* lk = buf<uint64_t>(rle_look, tiles);
-      uint32_t* tp0 = buf<uint32_t>(rle_p0, tiles);
-      uint32_t* tld = buf<uint32_t>(rle_lead, tiles);
-      uint32_t* ctr = buf<uint32_t>(os_ctr, 4);
-      WJ_CUDA_CHECK(cudaMemsetAsync(lk, 0, tiles * 8, st));
-      WJ_CUDA_CHECK(cudaMemsetAsync(ctr, 0, 4, st));
+      uint64_t per = (N + 148 * 2 - 1) / (148 * 2);
+      per = (per + kRleTile - 1) / kRleTile * kRleTile;
+      const uint32_t G = (uint32_t)((N + per - 1) / per);
+      uint32_t* rc = buf<uint32_t>(rle_p0, (uint64_t)G + 1);
+      uint32_t* rl = buf<uint32_t>(rle_lead, (uint64_t)G + 1);
       // P <= N: size the outputs by N, no host round trip before the pass
       uint32_t* od = buf<uint32_t>(out_doc, N);
       uint32_t* of = buf<uint32_t>(out_tf, N);
       uint32_t* tstart_p = spare_v;  // N >= V entries
       (void)spare_k;
       ktime(WJ_KERNEL_RLE_EMIT, [&] {
-        k_rle_fused<<<(unsigned)tiles, kRleThreads, 0, st>>>(f_key, f_doc, N, od, of, po, tstart_p, lk, ctr, tp0, tld,
-                                                            (uint32_t*)(dscal() + 8));
+        k_rle_count<<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc);
+        launched();
+        scan<uint32_t>(ArrayIn<uint32_t>{rc}, G, rc, (uint32_t*)(dscal() + 8));
+        k_rle_write_tma<<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, od, of, po, tstart_p, rl);
         launched();
       });
-      k_rle_fixup<<<grid_for(tiles, 256), 256, 0, st>>>(tp0, tld, (uint32_t)tiles, of);
+      k_rle_fixup<<<grid_for(G, 256), 256, 0, st>>>(rc, rl, G, of);
       launched();
       WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 8) + 1, 0, 4, st));
       readback(8, 1);
@@ -846,6 +880,20 @@ int index_init(wj_index** out, const wj_config* cfg) {
                                        (int)os_smem_bytes<uint64_t>()));
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_os_pass<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)os_smem_bytes<uint32_t>()));
+    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_os_pass_tma<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)os_tma_smem_bytes<uint64_t>()));
+    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_os_pass_tma<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)os_tma_smem_bytes<uint32_t>()));
+    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rs_down<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)os_tma_smem_bytes<uint64_t>()));
+    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rs_down<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)os_tma_smem_bytes<uint32_t>()));
+    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rs_down2<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)ds_smem_bytes<uint64_t>()));
+    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rs_down2<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)ds_smem_bytes<uint32_t>()));
+    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rle_write_tma, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)rle_smem_bytes()));
     ix->reset_state();
     return WJ_OK;
   });

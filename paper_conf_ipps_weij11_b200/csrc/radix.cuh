@@ -2,8 +2,10 @@
 // Stability (equal keys keep input order) is what turns the docID-ordered token stream into
 // docID-sorted postings: within one term, tokens stay in submission order.
 #pragma once
+#include <type_traits>
 #include "common.cuh"
 #include "scan.cuh"
+#include "tma.cuh"
 
 namespace wj {
 
@@ -155,8 +157,21 @@ __global__ void __launch_bounds__(256) k_os_hist_scan(uint32_t* ghist) {
   h[threadIdx.x] = ex;
 }
 
+// Lanes holding the same 8-bit digit (a warp-wide multi-split with 8 ballots: cheaper than
+// MATCH.ANY on sm_100a); `valid` lanes only.
+__device__ __forceinline__ uint32_t digit_peers(uint32_t d, bool valid) {
+  uint32_t peers = __ballot_sync(0xffffffffu, valid);
+#pragma unroll
+  for (int b = 0; b < 8; ++b) {
+    const bool bit = (d >> b) & 1u;
+    const uint32_t m = __ballot_sync(0xffffffffu, bit);
+    peers &= bit ? m : ~m;
+  }
+  return peers;
+}
+
 template <typename K>
-__global__ void __launch_bounds__(kOsThreads, 3) k_os_pass(const K* __restrict__ kin, const uint32_t* __restrict__ vin,
+__global__ void __launch_bounds__(kOsThreads, 4) k_os_pass(const K* __restrict__ kin, const uint32_t* __restrict__ vin,
                                                         K* __restrict__ kout, uint32_t* __restrict__ vout, uint64_t n,
                                                         int shift, const uint32_t* __restrict__ gofs,
                                                         uint64_t* look, uint32_t* tile_ctr) {
@@ -186,9 +201,9 @@ __global__ void __launch_bounds__(kOsThreads, 3) k_os_pass(const K* __restrict__
   for (int k = 0; k < kOsItems; ++k) {
     const uint64_t i = base + (uint64_t)w * (32 * kOsItems) + k * 32 + lane;
     const bool valid = i < n;
-    const uint32_t d = valid ? (uint32_t)((key[k] >> shift) & 255u) : 256u;
-    const uint32_t peers = __match_any_sync(0xffffffffu, d);
-    const int leader = __ffs(peers) - 1;
+    const uint32_t d = (uint32_t)((key[k] >> shift) & 255u);
+    const uint32_t peers = digit_peers(d, valid);
+    const int leader = valid ? __ffs(peers) - 1 : (int)lane;
     uint32_t old = 0;
     if (valid && (int)lane == leader) {
       old = wcnt[w][d];
@@ -246,6 +261,458 @@ __global__ void __launch_bounds__(kOsThreads, 3) k_os_pass(const K* __restrict__
     const uint32_t pos = dig_glob[(uint32_t)((kk >> shift) & 255u)] + j;
     kout[pos] = kk;
     vout[pos] = sv[j];
+  }
+}
+
+// Persistent onesweep pass with TMA: each CTA claims tiles in order (atomic counter), prefetches the
+// next tile's keys and values into the other half of a 2-stage shared-memory ring with one
+// cp.async.bulk each (completion on an mbarrier), ranks the current tile from shared memory,
+// publishes / looks back, stages the tile in digit order in the same buffer and writes it out.
+template <typename K>
+inline size_t os_tma_smem_bytes() { return 2 * (size_t)kOsTile * (sizeof(K) + sizeof(uint32_t)); }
+
+template <typename K>
+__global__ void __launch_bounds__(kOsThreads, 2) k_os_pass_tma(const K* __restrict__ kin, const uint32_t* __restrict__ vin,
+                                                            K* __restrict__ kout, uint32_t* __restrict__ vout, uint64_t n,
+                                                            int shift, const uint32_t* __restrict__ gofs, uint64_t* look,
+                                                            uint32_t* tile_ctr, uint32_t ntiles) {
+  extern __shared__ __align__(128) unsigned char os_smem[];
+  __shared__ __align__(8) uint64_t bar[2];
+  __shared__ uint32_t wcnt[kOsWarps][256];
+  __shared__ uint32_t dig_off[256];
+  __shared__ uint32_t dig_glob[256];
+  __shared__ uint32_t s_tile[2];
+  const size_t stage_bytes = (size_t)kOsTile * (sizeof(K) + sizeof(uint32_t));
+  auto skey = [&](int s) { return (K*)(os_smem + s * stage_bytes); };
+  auto sval = [&](int s) { return (uint32_t*)(os_smem + s * stage_bytes + (size_t)kOsTile * sizeof(K)); };
+  const uint32_t lane = lane_id();
+  const int w = threadIdx.x >> 5;
+  const uint32_t lt = (1u << lane) - 1u;
+
+  auto issue = [&](int s, uint32_t tile) {  // thread 0
+    const uint64_t base = (uint64_t)tile * kOsTile;
+    const uint32_t cnt = (uint32_t)((n - base) < (uint64_t)kOsTile ? (n - base) : (uint64_t)kOsTile);
+    const uint32_t bk = (uint32_t)((cnt * sizeof(K) + 15) & ~(size_t)15);
+    const uint32_t bv = (cnt * 4 + 15) & ~15u;
+    fence_proxy_async_smem();
+    mbar_arrive_expect_tx(&bar[s], bk + bv);
+    tma_load_1d(skey(s), kin + base, bk, &bar[s]);
+    tma_load_1d(sval(s), vin + base, bv, &bar[s]);
+  };
+
+  if (threadIdx.x == 0) {
+    mbar_init(&bar[0], 1);
+    mbar_init(&bar[1], 1);
+    fence_mbar_init();
+  }
+  for (int x = 0; x < kOsWarps; ++x) wcnt[x][threadIdx.x] = 0;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const uint32_t t = atomicAdd(tile_ctr, 1u);
+    s_tile[0] = t;
+    if (t < ntiles) issue(0, t);
+  }
+  __syncthreads();
+  uint32_t parity = 0u;  // bit s: phase of stage s
+  int s = 0;
+  for (;;) {
+    const uint32_t tile = s_tile[s];
+    if (tile >= ntiles) break;
+    if (threadIdx.x == 0) {  // prefetch the next tile into the other stage
+      const uint32_t t2 = atomicAdd(tile_ctr, 1u);
+      s_tile[s ^ 1] = t2;
+      if (t2 < ntiles) issue(s ^ 1, t2);
+    }
+    mbar_wait(&bar[s], (parity >> s) & 1u);
+    parity ^= 1u << s;
+    const uint64_t base = (uint64_t)tile * kOsTile;
+    const K* sk = skey(s);
+    uint32_t* sv = sval(s);
+    K key[kOsItems];
+    uint32_t val[kOsItems], rank[kOsItems];
+#pragma unroll
+    for (int k = 0; k < kOsItems; ++k) {
+      const uint32_t li = w * (32 * kOsItems) + k * 32 + lane;
+      key[k] = sk[li];
+      val[k] = sv[li];
+    }
+#pragma unroll
+    for (int k = 0; k < kOsItems; ++k) {
+      const uint64_t i = base + (uint64_t)w * (32 * kOsItems) + k * 32 + lane;
+      const bool valid = i < n;
+      const uint32_t d = (uint32_t)((key[k] >> shift) & 255u);
+      const uint32_t peers = digit_peers(d, valid);
+      const int leader = valid ? __ffs(peers) - 1 : (int)lane;
+      uint32_t old = 0;
+      if (valid && (int)lane == leader) {
+        old = wcnt[w][d];
+        wcnt[w][d] = old + __popc(peers);
+      }
+      old = __shfl_sync(0xffffffffu, old, leader);
+      rank[k] = old + __popc(peers & lt);
+      __syncwarp();
+    }
+    __syncthreads();
+    const uint32_t d = threadIdx.x;
+    uint32_t cnt = 0;
+#pragma unroll
+    for (int x = 0; x < kOsWarps; ++x) {
+      const uint32_t t = wcnt[x][d];
+      wcnt[x][d] = cnt;
+      cnt += t;
+    }
+    volatile uint64_t* lk = (volatile uint64_t*)look;
+    if (tile == 0) lk[d] = kLbPre | cnt;
+    else lk[(uint64_t)tile * 256 + d] = kLbAgg | cnt;
+    uint32_t tot;
+    const uint32_t toff = block_exclusive_sum<uint32_t>(cnt, tot);
+    dig_off[d] = toff;
+    uint64_t prefix = 0;
+    if (tile > 0) {
+      int64_t t = (int64_t)tile - 1;
+      for (;;) {
+        const uint64_t v = lk[(uint64_t)t * 256 + d];
+        if ((v & (kLbAgg | kLbPre)) == 0) continue;
+        prefix += v & kLbVal;
+        if (v & kLbPre) break;
+        --t;
+      }
+      lk[(uint64_t)tile * 256 + d] = kLbPre | (prefix + cnt);
+    }
+    dig_glob[d] = gofs[d] + (uint32_t)prefix - toff;
+    __syncthreads();
+    // stage in digit order (same buffer: every thread already holds its keys and values)
+    K* sko = (K*)sk;
+#pragma unroll
+    for (int k = 0; k < kOsItems; ++k) {
+      const uint64_t i = base + (uint64_t)w * (32 * kOsItems) + k * 32 + lane;
+      if (i < n) {
+        const uint32_t dk = (uint32_t)((key[k] >> shift) & 255u);
+        const uint32_t p = dig_off[dk] + wcnt[w][dk] + rank[k];
+        sko[p] = key[k];
+        sv[p] = val[k];
+      }
+    }
+    __syncthreads();
+    const uint32_t tn = (uint32_t)((n - base) < (uint64_t)kOsTile ? (n - base) : (uint64_t)kOsTile);
+    for (uint32_t j = threadIdx.x; j < tn; j += kOsThreads) {
+      const K kk = sko[j];
+      const uint32_t pos = dig_glob[(uint32_t)((kk >> shift) & 255u)] + j;
+      kout[pos] = kk;
+      vout[pos] = sv[j];
+    }
+#pragma unroll
+    for (int x = 0; x < kOsWarps; ++x) wcnt[x][threadIdx.x] = 0;
+    __syncthreads();
+    s ^= 1;
+  }
+}
+
+// ------------------------------------------------------------------ reduce-then-scan, TMA ring
+// Pass = upsweep (per-CTA-range digit histogram) + scan of the 256 x G counts (digit-major) +
+// downsweep: CTA c walks its contiguous range tile by tile with exact running digit offsets (no
+// look-back), the next tile's keys/values streaming into the other half of a 2-stage smem ring by
+// cp.async.bulk while the current tile is ranked, staged in digit order and written out.
+constexpr int kRsCtas = 148 * 2;
+
+template <typename K>
+__global__ void __launch_bounds__(256) k_rs_up(K* keys, uint64_t n, uint64_t per, int shift,
+                                               const uint32_t* __restrict__ map, uint32_t* hist) {
+  __shared__ uint32_t h[kOsWarps][256];
+  const int w = threadIdx.x >> 5;
+  for (int x = 0; x < kOsWarps; ++x) h[x][threadIdx.x] = 0;
+  __syncthreads();
+  const uint64_t lo = (uint64_t)blockIdx.x * per;  // multiple of the tile size: 16-byte aligned
+  const uint64_t hi = lo + per < n ? lo + per : n;
+  constexpr int V = 16 / sizeof(K);  // keys per 16-byte vector
+  const uint64_t nvec = (hi - lo) / V;
+  typedef typename std::conditional<sizeof(K) == 4, uint4, ulonglong2>::type Vec;
+  Vec* vp = (Vec*)(keys + lo);
+  constexpr int U = 4;  // vectors in flight per thread
+  uint64_t v0 = threadIdx.x;
+  for (; v0 + (U - 1) * 256 < nvec; v0 += U * 256) {
+    Vec x[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) x[u] = vp[v0 + u * 256];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      K* kk = (K*)&x[u];
+#pragma unroll
+      for (int j = 0; j < V; ++j) {
+        if (map) kk[j] = (K)__ldg(&map[(uint32_t)kk[j]]);
+        atomicAdd(&h[w][(uint32_t)(kk[j] >> shift) & 255u], 1u);
+      }
+      if (map) vp[v0 + u * 256] = x[u];
+    }
+  }
+  for (uint64_t v = v0; v < nvec; v += 256) {
+    Vec x = vp[v];
+    K* kk = (K*)&x;
+#pragma unroll
+    for (int j = 0; j < V; ++j) {
+      if (map) kk[j] = (K)__ldg(&map[(uint32_t)kk[j]]);
+      atomicAdd(&h[w][(uint32_t)(kk[j] >> shift) & 255u], 1u);
+    }
+    if (map) vp[v] = x;
+  }
+  for (uint64_t i = lo + nvec * V + threadIdx.x; i < hi; i += 256) {
+    K k = keys[i];
+    if (map) {
+      k = (K)__ldg(&map[(uint32_t)k]);
+      keys[i] = k;
+    }
+    atomicAdd(&h[w][(uint32_t)(k >> shift) & 255u], 1u);
+  }
+  __syncthreads();
+  uint32_t t = 0;
+#pragma unroll
+  for (int x = 0; x < kOsWarps; ++x) t += h[x][threadIdx.x];
+  hist[(uint64_t)threadIdx.x * gridDim.x + blockIdx.x] = t;
+}
+
+template <typename K>
+__global__ void __launch_bounds__(kOsThreads, 2) k_rs_down(const K* __restrict__ kin, const uint32_t* __restrict__ vin,
+                                                        K* __restrict__ kout, uint32_t* __restrict__ vout, uint64_t n,
+                                                        uint64_t per, int shift, const uint32_t* __restrict__ offs) {
+  extern __shared__ __align__(128) unsigned char os_smem[];
+  __shared__ __align__(8) uint64_t bar[2];
+  __shared__ uint32_t wcnt[kOsWarps][256];
+  __shared__ uint32_t dig_off[256];
+  __shared__ uint32_t dig_glob[256];
+  __shared__ uint32_t run_base[256];
+  const size_t stage_bytes = (size_t)kOsTile * (sizeof(K) + sizeof(uint32_t));
+  auto skey = [&](int s) { return (K*)(os_smem + s * stage_bytes); };
+  auto sval = [&](int s) { return (uint32_t*)(os_smem + s * stage_bytes + (size_t)kOsTile * sizeof(K)); };
+  const uint32_t lane = lane_id();
+  const int w = threadIdx.x >> 5;
+  const uint32_t lt = (1u << lane) - 1u;
+  const uint64_t lo = (uint64_t)blockIdx.x * per;
+  const uint64_t hi = lo + per < n ? lo + per : n;
+  if (lo >= hi) return;
+
+  auto issue = [&](int s, uint64_t base) {  // thread 0
+    const uint32_t cnt = (uint32_t)((hi - base) < (uint64_t)kOsTile ? (hi - base) : (uint64_t)kOsTile);
+    const uint32_t bk = (uint32_t)((cnt * sizeof(K) + 15) & ~(size_t)15);
+    const uint32_t bv = (cnt * 4 + 15) & ~15u;
+    fence_proxy_async_smem();
+    mbar_arrive_expect_tx(&bar[s], bk + bv);
+    tma_load_1d(skey(s), kin + base, bk, &bar[s]);
+    tma_load_1d(sval(s), vin + base, bv, &bar[s]);
+  };
+
+  if (threadIdx.x == 0) {
+    mbar_init(&bar[0], 1);
+    mbar_init(&bar[1], 1);
+    fence_mbar_init();
+  }
+  for (int x = 0; x < kOsWarps; ++x) wcnt[x][threadIdx.x] = 0;
+  run_base[threadIdx.x] = offs[(uint64_t)threadIdx.x * gridDim.x + blockIdx.x];
+  __syncthreads();
+  if (threadIdx.x == 0) issue(0, lo);
+  uint32_t parity = 0u;
+  int s = 0;
+  for (uint64_t base = lo; base < hi; base += kOsTile) {
+    if (threadIdx.x == 0 && base + kOsTile < hi) issue(s ^ 1, base + kOsTile);
+    mbar_wait(&bar[s], (parity >> s) & 1u);
+    parity ^= 1u << s;
+    const uint32_t tn = (uint32_t)((hi - base) < (uint64_t)kOsTile ? (hi - base) : (uint64_t)kOsTile);
+    K* sk = skey(s);
+    uint32_t* sv = sval(s);
+    K key[kOsItems];
+    uint32_t val[kOsItems], rank[kOsItems];
+#pragma unroll
+    for (int k = 0; k < kOsItems; ++k) {
+      const uint32_t li = w * (32 * kOsItems) + k * 32 + lane;
+      key[k] = sk[li];
+      val[k] = sv[li];
+    }
+    // peer masks by 8-ballot multisplit (no MATCH.ANY), then the per-warp running counters
+#pragma unroll
+    for (int k = 0; k < kOsItems; ++k) {
+      const uint32_t li = w * (32 * kOsItems) + k * 32 + lane;
+      rank[k] = digit_peers((uint32_t)((key[k] >> shift) & 255u), li < tn);
+    }
+#pragma unroll
+    for (int k = 0; k < kOsItems; ++k) {
+      const uint32_t li = w * (32 * kOsItems) + k * 32 + lane;
+      const bool valid = li < tn;
+      const uint32_t d = (uint32_t)((key[k] >> shift) & 255u);
+      const uint32_t peers = rank[k];
+      const int leader = valid ? __ffs(peers) - 1 : (int)lane;
+      uint32_t old = 0;
+      if (valid && (int)lane == leader) {
+        old = wcnt[w][d];
+        wcnt[w][d] = old + __popc(peers);
+      }
+      old = __shfl_sync(0xffffffffu, old, leader);
+      rank[k] = old + __popc(peers & lt);
+      __syncwarp();
+    }
+    __syncthreads();
+    const uint32_t d = threadIdx.x;
+    uint32_t cnt = 0;
+#pragma unroll
+    for (int x = 0; x < kOsWarps; ++x) {
+      const uint32_t t = wcnt[x][d];
+      wcnt[x][d] = cnt;
+      cnt += t;
+    }
+    uint32_t tot;
+    const uint32_t toff = block_exclusive_sum<uint32_t>(cnt, tot);
+    dig_off[d] = toff;
+    const uint32_t rb = run_base[d];
+    dig_glob[d] = rb - toff;
+    run_base[d] = rb + cnt;
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < kOsItems; ++k) {
+      const uint32_t li = w * (32 * kOsItems) + k * 32 + lane;
+      if (li < tn) {
+        const uint32_t dk = (uint32_t)((key[k] >> shift) & 255u);
+        const uint32_t p = dig_off[dk] + wcnt[w][dk] + rank[k];
+        sk[p] = key[k];
+        sv[p] = val[k];
+      }
+    }
+    __syncthreads();
+    for (uint32_t j = threadIdx.x; j < tn; j += kOsThreads) {
+      const K kk = sk[j];
+      const uint32_t pos = dig_glob[(uint32_t)((kk >> shift) & 255u)] + j;
+      kout[pos] = kk;
+      vout[pos] = sv[j];
+    }
+#pragma unroll
+    for (int x = 0; x < kOsWarps; ++x) wcnt[x][threadIdx.x] = 0;
+    __syncthreads();
+    s ^= 1;
+  }
+}
+
+// Downsweep v2: 512 threads x 8 items (tile 4096); the tile is never copied inside shared memory:
+// ranks produce an inverse permutation (u16) and the write-out gathers keys/values from the TMA
+// stage through it, so keys/values need no registers across barriers (occupancy: 32 warps/SM).
+constexpr int kDsThreads = 512;
+constexpr int kDsWarps = kDsThreads / 32;
+constexpr int kDsItems = 8;
+static_assert(kDsThreads * kDsItems == kOsTile, "tile");
+
+template <typename K>
+inline size_t ds_smem_bytes() { return 2 * (size_t)kOsTile * (sizeof(K) + sizeof(uint32_t)) + kOsTile * 2; }
+
+template <typename K>
+__global__ void __launch_bounds__(kDsThreads, 2) k_rs_down2(const K* __restrict__ kin, const uint32_t* __restrict__ vin,
+                                                         K* __restrict__ kout, uint32_t* __restrict__ vout, uint64_t n,
+                                                         uint64_t per, int shift, const uint32_t* __restrict__ offs) {
+  extern __shared__ __align__(128) unsigned char os_smem[];
+  __shared__ __align__(8) uint64_t bar[2];
+  __shared__ uint32_t wcnt[kDsWarps][256];
+  __shared__ uint32_t dig_off[256];
+  __shared__ uint32_t dig_glob[256];
+  __shared__ uint32_t run_base[256];
+  __shared__ uint32_t wtot[8];
+  const size_t stage_bytes = (size_t)kOsTile * (sizeof(K) + sizeof(uint32_t));
+  auto skey = [&](int s) { return (K*)(os_smem + s * stage_bytes); };
+  auto sval = [&](int s) { return (uint32_t*)(os_smem + s * stage_bytes + (size_t)kOsTile * sizeof(K)); };
+  uint16_t* inv = (uint16_t*)(os_smem + 2 * stage_bytes);
+  const uint32_t lane = lane_id();
+  const int w = threadIdx.x >> 5;
+  const uint32_t lt = (1u << lane) - 1u;
+  const uint64_t lo = (uint64_t)blockIdx.x * per;
+  const uint64_t hi = lo + per < n ? lo + per : n;
+  if (lo >= hi) return;
+
+  auto issue = [&](int s, uint64_t base) {  // thread 0
+    const uint32_t cnt = (uint32_t)((hi - base) < (uint64_t)kOsTile ? (hi - base) : (uint64_t)kOsTile);
+    const uint32_t bk = (uint32_t)((cnt * sizeof(K) + 15) & ~(size_t)15);
+    const uint32_t bv = (cnt * 4 + 15) & ~15u;
+    fence_proxy_async_smem();
+    mbar_arrive_expect_tx(&bar[s], bk + bv);
+    tma_load_1d(skey(s), kin + base, bk, &bar[s]);
+    tma_load_1d(sval(s), vin + base, bv, &bar[s]);
+  };
+
+  if (threadIdx.x == 0) {
+    mbar_init(&bar[0], 1);
+    mbar_init(&bar[1], 1);
+    fence_mbar_init();
+  }
+  for (int i = threadIdx.x; i < kDsWarps * 256; i += kDsThreads) (&wcnt[0][0])[i] = 0;
+  if (threadIdx.x < 256) run_base[threadIdx.x] = offs[(uint64_t)threadIdx.x * gridDim.x + blockIdx.x];
+  __syncthreads();
+  if (threadIdx.x == 0) issue(0, lo);
+  uint32_t parity = 0u;
+  int s = 0;
+  for (uint64_t base = lo; base < hi; base += kOsTile) {
+    if (threadIdx.x == 0 && base + kOsTile < hi) issue(s ^ 1, base + kOsTile);
+    mbar_wait(&bar[s], (parity >> s) & 1u);
+    parity ^= 1u << s;
+    const uint32_t tn = (uint32_t)((hi - base) < (uint64_t)kOsTile ? (hi - base) : (uint64_t)kOsTile);
+    const K* sk = skey(s);
+    const uint32_t* sv = sval(s);
+    uint32_t dg[kDsItems], rank[kDsItems];
+#pragma unroll
+    for (int k = 0; k < kDsItems; ++k) {
+      const uint32_t li = w * (32 * kDsItems) + k * 32 + lane;
+      dg[k] = (uint32_t)((sk[li] >> shift) & 255u);
+      rank[k] = digit_peers(dg[k], li < tn);
+    }
+#pragma unroll
+    for (int k = 0; k < kDsItems; ++k) {
+      const uint32_t li = w * (32 * kDsItems) + k * 32 + lane;
+      const bool valid = li < tn;
+      const uint32_t peers = rank[k];
+      const int leader = valid ? __ffs(peers) - 1 : (int)lane;
+      uint32_t old = 0;
+      if (valid && (int)lane == leader) {
+        old = wcnt[w][dg[k]];
+        wcnt[w][dg[k]] = old + __popc(peers);
+      }
+      old = __shfl_sync(0xffffffffu, old, leader);
+      rank[k] = old + __popc(peers & lt);
+      __syncwarp();
+    }
+    __syncthreads();
+    // per digit (threads 0..255): offsets across warps, tile count, tile-exclusive digit offset
+    uint32_t cnt = 0, inc = 0;
+    if (threadIdx.x < 256) {
+      const uint32_t d = threadIdx.x;
+#pragma unroll
+      for (int x = 0; x < kDsWarps; ++x) {
+        const uint32_t t = wcnt[x][d];
+        wcnt[x][d] = cnt;
+        cnt += t;
+      }
+      inc = warp_inclusive_sum<uint32_t>(cnt);
+      if (lane == 31) wtot[w] = inc;
+    }
+    __syncthreads();
+    if (threadIdx.x < 256) {
+      const uint32_t d = threadIdx.x;
+      uint32_t wp = 0;
+      for (int x = 0; x < w; ++x) wp += wtot[x];
+      const uint32_t toff = wp + inc - cnt;
+      dig_off[d] = toff;
+      const uint32_t rb = run_base[d];
+      dig_glob[d] = rb - toff;
+      run_base[d] = rb + cnt;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < kDsItems; ++k) {
+      const uint32_t li = w * (32 * kDsItems) + k * 32 + lane;
+      if (li < tn) inv[dig_off[dg[k]] + wcnt[w][dg[k]] + rank[k]] = (uint16_t)li;
+    }
+    __syncthreads();
+    for (uint32_t j = threadIdx.x; j < tn; j += kDsThreads) {
+      const uint32_t li = inv[j];
+      const K kk = sk[li];
+      const uint32_t pos = dig_glob[(uint32_t)((kk >> shift) & 255u)] + j;
+      kout[pos] = kk;
+      vout[pos] = sv[li];
+    }
+    for (int i = threadIdx.x; i < kDsWarps * 256; i += kDsThreads) (&wcnt[0][0])[i] = 0;
+    __syncthreads();
+    s ^= 1;
   }
 }
 

@@ -251,7 +251,7 @@ __device__ __forceinline__ uint32_t win_word(const uint32_t* win32, uint32_t s, 
   uint32_t w = __funnelshift_r(win32[a], win32[a + 1], sh);
   const uint32_t rem = len - 4 * k;
   if (rem < 4) w &= (1u << (rem * 8)) - 1u;
-  return lower4(w);
+  return w;  // the window is staged already folded (reading S2)
 }
 
 __device__ __forceinline__ uint64_t mix_hash(uint64_t h, uint64_t x) {
@@ -316,7 +316,9 @@ __global__ void __launch_bounds__(kTokThreads) k_tok_emit(ChunkView cv, uint32_t
 #pragma unroll
   for (int j = 0; j <= kSegsPerWarp; ++j) v[j] = load_lane16(cv, sb0 + j);
 #pragma unroll
-  for (int j = 0; j <= kSegsPerWarp; ++j) *(uint4*)&w32[(j * kSegBytes + 16 * lane) / 4] = v[j];
+  for (int j = 0; j <= kSegsPerWarp; ++j)  // fold A-Z once here (classification is case-blind)
+    *(uint4*)&w32[(j * kSegBytes + 16 * lane) / 4] =
+        make_uint4(lower4(v[j].x), lower4(v[j].y), lower4(v[j].z), lower4(v[j].w));
   if (lane < 4) w32[(kWinBytes - 16) / 4 + lane] = 0;
   __syncwarp();
 
