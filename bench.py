@@ -9,8 +9,10 @@ max over ranks.  Inputs (1 GiB) are larger than L2 (126 MB), so no L2 flush is n
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config 2]
 
-N > 1 (torchrun): every rank indexes its own 1 GiB document shard (chunk index = rank) into a
-local dictionary; scaling is weak.  ``--impl reference`` times the CPU oracle (the reference arm of
+N > 1 (torchrun): every rank submits its own 1 GiB document range (chunk index = rank; rank order =
+DocID order) and the library routes each term to the rank owning its trie collection (b mod N,
+PAPER.md P:210) with an NCCL all-to-all-v over NVLink; each rank builds its exclusive dictionary
+slice.  Per-GPU work is fixed as N grows: scaling is weak.  ``--impl reference`` times the CPU oracle (the reference arm of
 this tier) on a bounded document prefix of the same workload, on rank 0 only.
 """
 from __future__ import annotations
@@ -209,7 +211,12 @@ def main():
     off_d = off_h.cuda()
     torch.cuda.synchronize()
 
-    ix = wj.Index(device=local, profile=True)
+    if world > 1:
+        nid = [wj.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(nid, src=0)
+        ix = wj.Index(device=local, profile=True, rank=rank, world=world, nccl_id=nid[0])
+    else:
+        ix = wj.Index(device=local, profile=True)
 
     def step(t, o):
         ix.reset()
@@ -314,7 +321,9 @@ def main():
             "config": {"workload": WORKLOAD.get(args.config, str(args.config)), "bytes_per_gpu": T,
                        "docs_per_gpu": len(doc_off) - 1, "tokens_per_gpu": N, "terms_per_gpu": V,
                        "postings_per_gpu": P, "l2": "no flush: 1 GiB input per step > 126 MB L2",
-                       "parallelism": "single GPU" if world == 1 else f"{world} document shards, local dictionaries"},
+                       "parallelism": "single GPU" if world == 1 else
+                       f"{world} ranks: document ranges, trie collections b mod {world}, NCCL all-to-all-v"},
+            "exchange_bytes_per_step": (s1["exchange_bytes"]),
             "mib_per_s": total_bytes / (ms / 1e3) / 2**20,
             "tokens_per_s": N * world / (ms / 1e3),
             "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",

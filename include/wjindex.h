@@ -48,6 +48,8 @@ typedef enum {
 
 /* config.flags */
 #define WJ_FLAG_PROFILE 0x1u   /* record CUDA events per phase (index_stats.phase_ms)               */
+#define WJ_FLAG_LOOPBACK 0x2u  /* world > 1 inside one process: nccl_unique_id is a hub from        */
+                               /* index_loopback_create; one host thread per rank context (tests)   */
 
 typedef struct wj_index wj_index; /* opaque; all index state is owned by the library */
 
@@ -168,6 +170,26 @@ int index_debug_tokens(wj_index* ix, const void* bytes, uint64_t n_bytes, const 
 int index_debug_btree(wj_index* ix, void* nodes, uint64_t node_cap, uint64_t* n_nodes,
                       uint32_t* collections, uint8_t* arena, uint64_t arena_cap,
                       uint64_t* arena_bytes);
+
+/* Multi-GPU.  Rank r owns the trie collections b with b mod world == r
+ * and builds that exclusive dictionary slice; every index_add_stream call is collective and
+ * moves, per owner, the chunk's unique terms and (term, docID) token records with one all-to-all-v
+ * (NCCL over NVLink, or the loopback hub).  index_serialize returns the rank's slice (its terms;
+ * n_docs global, other header counts local); index_merge_serialized merges the slices of all ranks
+ * into the canonical global file (host, untimed).  index_read_postings answers owned terms only. */
+
+/* Writes a fresh 128-byte ncclUniqueId (rank 0 calls it and broadcasts the bytes).  WJ_ERR_NCCL if
+ * libnccl.so.2 cannot be loaded (override the path with the WJ_NCCL_LIB environment variable). */
+int index_nccl_unique_id(void* out128);
+
+/* In-process transport for world ranks driven by world host threads on one device (tests). */
+int index_loopback_create(int32_t world, void** hub);
+void index_loopback_destroy(void* hub);
+
+/* Merges k serialized slices (host memory) into the global serialized index; two-call sizing like
+ * index_serialize.  WJ_ERR_INVALID_ARG if a slice does not parse or n_docs differ. */
+int index_merge_serialized(int32_t k, const uint8_t* const* slices, const uint64_t* sizes, uint8_t* out, uint64_t cap,
+                           uint64_t* n_out);
 
 const char* index_last_error(const wj_index* ix);
 void index_destroy(wj_index* ix);

@@ -28,8 +28,10 @@ KERNELS = ["tokenize_count", "tokenize_emit", "probe", "slot_to_tid", "map_rank"
 N_COLLECTIONS = 17613
 
 EXPORTS = ["index_init", "index_add_stream", "index_finalize", "index_read_postings", "index_serialize",
-           "index_stats", "index_reset", "index_debug_tokens", "index_debug_btree", "index_last_error",
+           "index_stats", "index_reset", "index_debug_tokens", "index_debug_btree", "index_nccl_unique_id",
+           "index_loopback_create", "index_loopback_destroy", "index_merge_serialized", "index_last_error",
            "index_destroy"]
+WJ_FLAG_LOOPBACK = 2
 
 
 class WJError(RuntimeError):
@@ -81,10 +83,16 @@ def load_library():
         lib.index_last_error.argtypes = [vp]
         lib.index_last_error.restype = ctypes.c_char_p
         lib.index_destroy.argtypes = [vp]
+        lib.index_nccl_unique_id.argtypes = [vp]
+        lib.index_loopback_create.argtypes = [ctypes.c_int32, ctypes.POINTER(vp)]
+        lib.index_loopback_destroy.argtypes = [vp]
+        lib.index_merge_serialized.argtypes = [ctypes.c_int32, ctypes.POINTER(ctypes.c_void_p), ctypes.POINTER(ctypes.c_uint64),
+                                               vp, u64, P64]
         for f in EXPORTS:
-            if f not in ("index_last_error", "index_destroy"):
+            if f not in ("index_last_error", "index_destroy", "index_loopback_destroy"):
                 getattr(lib, f).restype = i32
         lib.index_destroy.restype = None
+        lib.index_loopback_destroy.restype = None
         _lib = lib
     return _lib
 
@@ -116,11 +124,20 @@ def _current_stream(device):
 class Index:
     """One indexing context on one GPU (index_init .. index_destroy)."""
 
-    def __init__(self, device: int = 0, stream=None, profile: bool = False, rank: int = 0, world: int = 1):
+    def __init__(self, device: int = 0, stream=None, profile: bool = False, rank: int = 0, world: int = 1,
+                 nccl_id: bytes | None = None, hub: "LoopbackHub | None" = None, own_stream: bool = False):
+        """world > 1: pass nccl_id (128 bytes from nccl_unique_id(), broadcast by the caller) or a
+        LoopbackHub shared by `world` contexts of this process (one host thread each)."""
         self._lib = load_library()
-        cfg = Config(device=device, rank=rank, world=world, nccl_unique_id=None,
-                     stream=stream if stream is not None else _current_stream(device),
-                     max_chunk_bytes=0, flags=WJ_FLAG_PROFILE if profile else 0, reserved=0)
+        flags = (WJ_FLAG_PROFILE if profile else 0) | (WJ_FLAG_LOOPBACK if hub is not None else 0)
+        self._nid = ctypes.create_string_buffer(bytes(nccl_id), 128) if nccl_id is not None else None
+        uid = hub._h if hub is not None else (ctypes.cast(self._nid, ctypes.c_void_p) if self._nid is not None else None)
+        if own_stream:
+            strm = ctypes.c_void_p(0)
+        else:
+            strm = stream if stream is not None else _current_stream(device)
+        cfg = Config(device=device, rank=rank, world=world, nccl_unique_id=uid, stream=strm,
+                     max_chunk_bytes=0, flags=flags, reserved=0)
         h = ctypes.c_void_p()
         rc = self._lib.index_init(ctypes.byref(h), ctypes.byref(cfg))
         if rc != WJ_OK:
@@ -232,6 +249,59 @@ class Index:
         self._check(self._lib.index_debug_btree(self._h, nodes.ctypes.data, nn.value, ctypes.byref(nn),
                                                 coll.ctypes.data, arena.ctypes.data, na.value, ctypes.byref(na)))
         return nodes, coll, arena[: na.value]
+
+
+class LoopbackHub:
+    """In-process exchange for `world` rank contexts driven by `world` host threads (one GPU)."""
+
+    def __init__(self, world: int):
+        self._lib = load_library()
+        h = ctypes.c_void_p()
+        rc = self._lib.index_loopback_create(world, ctypes.byref(h))
+        if rc != WJ_OK:
+            raise WJError(rc, "index_loopback_create")
+        self._h = h
+        self.world = world
+
+    def close(self):
+        if getattr(self, "_h", None):
+            self._lib.index_loopback_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        self.close()
+
+
+def nccl_unique_id() -> bytes:
+    lib = load_library()
+    buf = ctypes.create_string_buffer(128)
+    rc = lib.index_nccl_unique_id(buf)
+    if rc != WJ_OK:
+        raise WJError(rc, lib.index_last_error(None).decode())
+    return buf.raw
+
+
+def merge_serialized(slices) -> bytes:
+    """Merge the per-rank serialized slices into the global canonical inverted file (host)."""
+    lib = load_library()
+    k = len(slices)
+    arrs = [np.frombuffer(bytes(x), dtype=np.uint8) for x in slices]
+    ptrs = (ctypes.c_void_p * k)(*[a.ctypes.data for a in arrs])
+    sizes = (ctypes.c_uint64 * k)(*[a.size for a in arrs])
+    n = ctypes.c_uint64()
+    rc = lib.index_merge_serialized(k, ptrs, sizes, None, 0, ctypes.byref(n))
+    if rc != WJ_OK:
+        raise WJError(rc, lib.index_last_error(None).decode())
+    out = np.empty(n.value, dtype=np.uint8)
+    rc = lib.index_merge_serialized(k, ptrs, sizes, out.ctypes.data, n.value, ctypes.byref(n))
+    if rc != WJ_OK:
+        raise WJError(rc, lib.index_last_error(None).decode())
+    return out.tobytes()
+
+
+def owner_of(collection: int, world: int) -> int:
+    """Rank owning a trie collection: index i goes to GPU i mod N_2."""
+    return collection % world
 
 
 def build_index(text, doc_off, device: int = 0, chunks=None) -> bytes:

@@ -11,8 +11,20 @@ NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", 
               "-Xcompiler", "-fPIC", "-shared", "-Xptxas", "-v"]
 
 
+def nccl_include():
+    """nccl.h of the NCCL that torch ships (types only: libnccl is dlopen-ed at run time)."""
+    try:
+        import nvidia.nccl
+        base = os.path.dirname(nvidia.nccl.__file__) if nvidia.nccl.__file__ else list(nvidia.nccl.__path__)[0]
+    except Exception:
+        import site
+        base = os.path.join(site.getsitepackages()[0], "nvidia", "nccl")
+    return os.path.join(base, "include")
+
+
 def sources():
     return sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cuh"))
+                  + glob.glob(os.path.join(CSRC, "*.h"))
                   + glob.glob(os.path.join(INCLUDE, "*.h")))
 
 
@@ -21,7 +33,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and os.path.exists(LIB) and os.path.getmtime(LIB) >= newest:
         return LIB
     nvcc = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-    cmd = [nvcc, *NVCC_FLAGS, "-o", LIB, os.path.join(CSRC, "engine.cu")]
+    cmd = [nvcc, *NVCC_FLAGS, "-I", nccl_include(), "-o", LIB, os.path.join(CSRC, "engine.cu"), "-ldl"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError("nvcc failed:\n" + r.stderr[-8000:])

@@ -1,0 +1,88 @@
+// Multi-GPU pack / unpack kernels.
+//
+// Ownership: trie collection b belongs to rank b mod K — the paper's static split of collections
+// over GPUs, "assigning the trie collection TC_i with index i to the GPU whose index is given by
+// i mod N_2".  Each rank owns an exclusive slice of the dictionary.
+//
+// Per chunk, rank r has tokenised its own document range into a chunk table (unique terms) and a
+// (slot, docID) stream.  For every owner o it sends
+//   * the folded bytes of the unique terms it saw whose collection o owns, each followed by ' '
+//     (so the owner can run the received bytes through the same tokenizer/dedup kernels), and
+//   * one record (xid, docID) per token of those terms, in stream (= docID) order, xid = the
+//     term's index in the list sent to o.
+// The owner appends the records in source-rank order, so postings stay docID-sorted.
+#pragma once
+#include "common.cuh"
+#include "dict.cuh"
+
+namespace wj {
+
+__global__ void k_owner(const uint32_t* u_bucket, uint32_t U, uint32_t K, uint32_t* owner, uint32_t* iota,
+                        uint32_t* owner_cnt) {
+  const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
+  if (u >= U) return;
+  const uint32_t o = u_bucket[u] % K;
+  owner[u] = o;
+  iota[u] = u;
+  atomicAdd(&owner_cnt[o], 1u);
+}
+
+// xid = index of the unique term in the list sent to its owner (terms sorted stably by owner)
+__global__ void k_xid(const uint32_t* sorted_u, uint32_t U, const uint32_t* u_owner, const uint64_t* t_off,
+                      uint32_t* xid) {
+  const uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= U) return;
+  const uint32_t u = sorted_u[j];
+  xid[u] = j - (uint32_t)t_off[u_owner[u]];
+}
+
+struct PackTermSize {
+  const uint32_t* sorted_u;
+  const uint32_t* u_len;
+  __device__ __forceinline__ uint64_t operator()(uint64_t j) const { return (uint64_t)u_len[sorted_u[j]] + 1; }
+};
+
+__global__ void k_pack_terms(const uint32_t* sorted_u, uint32_t U, const uint64_t* boff, const uint4* u_w,
+                             const uint8_t* text, const uint32_t* u_ref, const uint32_t* u_len, uint8_t* out) {
+  const uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= U) return;
+  const uint32_t u = sorted_u[j];
+  const uint4 w = u_w[u];
+  const uint32_t len = u_len[u], ref = u_ref[u];
+  uint8_t* o = out + boff[j];
+  for (uint32_t i = 0; i < len; ++i) o[i] = (uint8_t)ubyte(w, text, ref, i);
+  o[len] = ' ';
+}
+
+__global__ void k_tok_owner(const uint32_t* slot, uint64_t n, const uint32_t* slot_uid, const uint32_t* u_owner,
+                            uint32_t* tkey, uint32_t* tidx, uint32_t* tok_cnt) {
+  const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= n) return;
+  const uint32_t o = u_owner[slot_uid[slot[t]]];
+  tkey[t] = o;
+  tidx[t] = (uint32_t)t;
+  atomicAdd(&tok_cnt[o], 1u);
+}
+
+__global__ void k_pack_tok(const uint32_t* sorted_t, uint64_t n, const uint32_t* slot, const uint32_t* doc,
+                           const uint32_t* slot_uid, const uint32_t* xid, uint2* rec) {
+  const uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= n) return;
+  const uint32_t t = sorted_t[j];
+  rec[j] = make_uint2(xid[slot_uid[slot[t]]], doc[t]);
+}
+
+// owner side: record j from source s -> term index term_base[s] + xid of the received term text,
+// whose (synthetic) token stream gives its table slot
+__global__ void k_map_recv(const uint2* rec, uint64_t n, const uint64_t* rec_off, const uint64_t* term_base, uint32_t K,
+                           const uint32_t* syn_slot, uint32_t* out_slot, uint32_t* out_doc) {
+  const uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= n) return;
+  uint32_t s = 0;
+  while (s + 1 < K && rec_off[s + 1] <= j) ++s;
+  const uint2 r = rec[j];
+  out_slot[j] = syn_slot[term_base[s] + r.x];
+  out_doc[j] = r.y;
+}
+
+}  // namespace wj

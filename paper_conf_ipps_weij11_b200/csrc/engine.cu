@@ -9,6 +9,8 @@
 #include "../../include/wjindex.h"
 #include "common.cuh"
 #include "dict.cuh"
+#include "dist.cuh"
+#include "exchange.h"
 #include "postings.cuh"
 #include "radix.cuh"
 #include "scan.cuh"
@@ -99,7 +101,11 @@ struct wj_index {
   uint64_t arena_used = 0;
   uint64_t table_est = 0;
   uint64_t P = 0, TB = 0;
+  uint64_t exchange_bytes = 0;
 
+  Transport* xport = nullptr;  // world > 1
+  DevBuf x_owner, x_iota, x_sorted, x_sorted2, x_owner2, x_xid, x_cnt, x_toff, x_boff, x_send, x_tkey, x_tidx, x_tkey2,
+      x_tidx2, x_rec, x_recv_terms, x_recv_rec, x_loc_slot, x_loc_doc, x_syn_slot, x_syn_doc, x_syn_off, x_roff, x_tbase;
   // persistent dictionary
   DevBuf nodes, coll_root, coll_n, coll_base, coll_base2, e_tid, e_bkt, e_tid2, e_bkt2, arena, t_arena, t_cache,
       t_bucket;
@@ -175,6 +181,10 @@ struct wj_index {
       b->p = nullptr;
       b->cap = 0;
     }
+    DevBuf* xs[] = {&x_owner, &x_iota, &x_sorted, &x_sorted2, &x_owner2, &x_xid, &x_cnt, &x_toff, &x_boff, &x_send,
+                    &x_tkey, &x_tidx, &x_tkey2, &x_tidx2, &x_rec, &x_recv_terms, &x_recv_rec, &x_loc_slot,
+                    &x_loc_doc, &x_syn_slot, &x_syn_doc, &x_syn_off, &x_roff, &x_tbase};
+    for (DevBuf* b : xs) { if (b->p) cudaFree(b->p); *b = DevBuf{}; }
     for (auto& b : chunk_map) if (b.p) cudaFree(b.p);
     chunk_map.clear();
     for (DevBuf* b : {&rle_look, &rle_p0, &rle_lead}) { if (b->p) cudaFree(b->p); *b = DevBuf{}; }
@@ -275,6 +285,7 @@ struct wj_index {
     chunk_C.clear();
     n_docs = n_tokens = n_dropped = n_chunks = 0;
     unique_last = new_last = n_nodes = height_max = 0;
+    exchange_bytes = 0;
     V = 0;
     arena_used = 0;
     P = TB = 0;
@@ -412,41 +423,27 @@ struct wj_index {
   }
 
   // ---------------------------------------------------------------- one chunk
-  void add_chunk(const void* bytes, uint64_t n_bytes, const uint64_t* doc_off_in, uint64_t nd) {
-    if (n_docs + nd > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 documents"};
-    const uint8_t* text = nullptr;
-    const uint64_t* off = nullptr;
-    stage(bytes, n_bytes, doc_off_in, nd, &text, &off);
-    const uint32_t doc_base = (uint32_t)n_docs;
-    ++n_chunks;
-    if (nd == 0 || n_bytes == 0) {
-      n_docs += nd;
-      phase(-1);
-      return;
-    }
-    ChunkView cv{text, n_bytes, off, nd};
-    const uint64_t n_segs = (n_bytes + kSegBytes - 1) / kSegBytes;
-
+  // K1 (count + emit + dedup): tokens of cv into (slot, docID) arrays given by out_alloc(Nc); unique
+  // terms of the chunk into the u_* arrays.  Returns Nc; sets C (table capacity), U.
+  template <class F>
+  uint64_t tokenize_dedup(const ChunkView& cv, uint32_t doc_base, F&& out_alloc, uint64_t& C, uint64_t& U,
+                          uint32_t*& slot_out, uint32_t*& doc_out) {
+    const uint64_t n_segs = (cv.n_bytes + kSegBytes - 1) / kSegBytes;
+    C = 0;
+    U = 0;
     phase(WJ_PHASE_TOKENIZE);
     const uint64_t Nc = count_tokens(cv, n_segs);
     n_dropped += h_scal[1];
-    if (n_tokens + Nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 tokens in one index"};
-    uint32_t* gt = buf_keep<uint32_t>(g_tid, n_tokens + Nc + 16, n_tokens);  // +16: TMA round-up reads
-    uint32_t* gd = buf_keep<uint32_t>(g_doc, n_tokens + Nc + 16, n_tokens);
-    if (Nc == 0) {
-      n_docs += nd;
-      phase(-1);
-      return;
-    }
+    out_alloc(Nc, slot_out, doc_out);
+    if (Nc == 0) return 0;
     // capacity ~1.5-3x the expected unique terms (U/N ~ 1/30 on Zipf text; the next chunk uses
     // the last U); a probe-sequence overflow retries with a doubled table
     uint64_t est = std::max<uint64_t>({table_est, Nc / 32, 4096});
     est = std::min<uint64_t>(est, Nc + 16);
-    uint64_t C = pow2_at_least(est + est / 2);
+    C = pow2_at_least(est + est / 2);
     uint32_t* slot_uid = nullptr;
-    uint64_t U = 0;
     for (;;) {
-      emit_tokens(cv, n_segs, gt + n_tokens, gd + n_tokens, doc_base, C, nullptr, nullptr);
+      emit_tokens(cv, n_segs, slot_out, doc_out, doc_base, C, nullptr, nullptr);
       phase(WJ_PHASE_UNIQUE);
       slot_uid = buf<uint32_t>(uid, C);
       scan<uint32_t>(NonZeroSlot{(const Slot*)table.p}, C, slot_uid, (uint32_t*)(dscal() + 2));
@@ -459,25 +456,28 @@ struct wj_index {
     }
     unique_last = U;
     table_est = (U * 5) / 4;
-
-    // unique terms: first occurrence, Table I bucket, stripped-suffix cache, sort key
+    // unique terms: first occurrence, folded bytes, Table I bucket, stripped-suffix cache, sort key
     uint4* uw = buf<uint4>(u_w, U);
     uint32_t* ur = buf<uint32_t>(u_ref, U);
     uint32_t* ul = buf<uint32_t>(u_len, U);
     uint32_t* ub = buf<uint32_t>(u_bucket, U);
     uint32_t* uc = buf<uint32_t>(u_cache, U);
     uint64_t* uk = buf<uint64_t>(u_key, U);
+    k_unique_gather<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, (const uint32_t*)slotref.p, (uint32_t)C,
+                                                      slot_uid, cv.text, uw, ur, ul, ub, uc, uk);
+    launched();
+    return Nc;
+  }
+
+  // K3 probe + K4 insert/rebuild of the chunk's unique terms (u_* arrays) -> u_tid
+  void dictionary_update(const uint8_t* text, uint64_t U) {
     uint32_t* ut = buf<uint32_t>(u_tid, U);
     uint32_t* urk = buf<uint32_t>(u_rank, U);
-    k_unique_gather<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, (const uint32_t*)slotref.p, (uint32_t)C, slot_uid, text, uw, ur, ul, ub,
-                                                      uc, uk);
-    launched();
-
-    // K3 probe
     phase(WJ_PHASE_PROBE);
     DictView dv{(const Node*)nodes.p, (const uint32_t*)coll_root.p, (const uint32_t*)coll_n.p, (const uint8_t*)arena.p};
     if (V > 0) {
-      UniqueView uv{text, uw, ur, ul, ub, uc};
+      UniqueView uv{text, (const uint4*)u_w.p, (const uint32_t*)u_ref.p, (const uint32_t*)u_len.p,
+                    (const uint32_t*)u_bucket.p, (const uint32_t*)u_cache.p};
       const unsigned blocks = (unsigned)std::min<uint64_t>((U + 7) / 8, 148ull * 64);
       ktime(WJ_KERNEL_PROBE, [&] {
         k_probe<<<blocks, 256, 0, st>>>(dv, uv, (uint32_t)U, ut, urk);
@@ -488,8 +488,6 @@ struct wj_index {
       k_fill<uint32_t><<<grid_for(U, 256), 256, 0, st>>>(urk, U, 0u);
       launched(2);
     }
-
-    // K4 insert
     phase(WJ_PHASE_INSERT);
     uint32_t* mi = buf<uint32_t>(midx, U);
     scan<uint32_t>(IsMiss{ut}, U, mi, (uint32_t*)(dscal() + 3));
@@ -503,21 +501,199 @@ struct wj_index {
       phase(WJ_PHASE_REBUILD);
       rebuild();
     }
+  }
 
-    // the chunk's (slot, docID) stream is the postings input; keep its slot -> termID map
+  // the chunk's (slot, docID) stream is the postings input; keep its slot -> termID map
+  void register_chunk_map(uint64_t C, uint64_t tok_start) {
     phase(WJ_PHASE_STREAM);
     const size_t ci = chunk_tok.size();
     if (chunk_map.size() <= ci) chunk_map.emplace_back();
     uint32_t* cmap = buf<uint32_t>(chunk_map[ci], C);
     ktime(WJ_KERNEL_SLOT_TO_TID, [&] {
-      k_slot_map<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, slot_uid, ut, (uint32_t)C, cmap);
+      k_slot_map<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, (const uint32_t*)uid.p,
+                                                    (const uint32_t*)u_tid.p, (uint32_t)C, cmap);
       launched();
     });
-    chunk_tok.push_back(n_tokens);
+    chunk_tok.push_back(tok_start);
     chunk_C.push_back((uint32_t)C);
-    n_tokens += Nc;
+  }
+
+  void add_chunk(const void* bytes, uint64_t n_bytes, const uint64_t* doc_off_in, uint64_t nd) {
+    const uint8_t* text = nullptr;
+    const uint64_t* off = nullptr;
+    stage(bytes, n_bytes, doc_off_in, nd, &text, &off);
+    ++n_chunks;
+    if (world > 1) {
+      add_chunk_dist(text, nd ? n_bytes : 0, off, nd);
+      phase(-1);
+      return;
+    }
+    if (n_docs + nd > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 documents"};
+    const uint32_t doc_base = (uint32_t)n_docs;
+    if (nd == 0 || n_bytes == 0) {
+      n_docs += nd;
+      phase(-1);
+      return;
+    }
+    ChunkView cv{text, n_bytes, off, nd};
+    uint64_t C = 0, U = 0;
+    uint32_t *so = nullptr, *dout = nullptr;
+    const uint64_t Nc = tokenize_dedup(cv, doc_base, [&](uint64_t nc, uint32_t*& sp, uint32_t*& dp) {
+      if (n_tokens + nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 tokens in one index"};
+      sp = buf_keep<uint32_t>(g_tid, n_tokens + nc + 16, n_tokens) + n_tokens;  // +16: TMA round-up reads
+      dp = buf_keep<uint32_t>(g_doc, n_tokens + nc + 16, n_tokens) + n_tokens;
+    }, C, U, so, dout);
+    if (Nc > 0) {
+      dictionary_update(text, U);
+      register_chunk_map(C, n_tokens);
+      n_tokens += Nc;
+    }
     n_docs += nd;
     phase(-1);
+  }
+
+  // ---------------------------------------------------------------- one chunk, world > 1
+  void add_chunk_dist(const uint8_t* text, uint64_t n_bytes, const uint64_t* off, uint64_t nd) {
+    const int K = world;
+    // DocID base = documents of earlier chunks + of lower ranks in this chunk
+    std::vector<uint64_t> ndall(K);
+    const uint64_t mine = nd;
+    phase(WJ_PHASE_EXCHANGE);
+    xport->allgather(&mine, 1, ndall.data(), st);
+    uint64_t base = n_docs, tot_docs = 0;
+    for (int r = 0; r < K; ++r) {
+      if (r < rank) base += ndall[r];
+      tot_docs += ndall[r];
+    }
+    if (n_docs + tot_docs > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 documents"};
+    // 1. local tokenize + dedup of this rank's documents
+    uint64_t C = 0, U = 0, Nc = 0;
+    uint32_t *lslot = nullptr, *ldoc = nullptr;
+    if (nd > 0 && n_bytes > 0) {
+      ChunkView cv{text, n_bytes, off, nd};
+      Nc = tokenize_dedup(cv, (uint32_t)base, [&](uint64_t nc, uint32_t*& sp, uint32_t*& dp) {
+        sp = buf<uint32_t>(x_loc_slot, nc + 16);
+        dp = buf<uint32_t>(x_loc_doc, nc + 16);
+      }, C, U, lslot, ldoc);
+    }
+    // 2. pack per owner (collection b -> rank b mod K)
+    phase(WJ_PHASE_EXCHANGE);
+    std::vector<uint64_t> cnt(3 * K, 0);  // [terms to o | term bytes to o | records to o]
+    uint64_t* toff_d = buf<uint64_t>(x_toff, K + 1);
+    std::vector<uint64_t> t_off(K + 1, 0), b_off(K + 1, 0), r_off(K + 1, 0);
+    uint8_t* send_terms = nullptr;
+    uint2* send_rec = nullptr;
+    if (U > 0) {
+      uint32_t* own = buf<uint32_t>(x_owner, U + 16);
+      uint32_t* iota = buf<uint32_t>(x_iota, U + 16);
+      uint32_t* own2 = buf<uint32_t>(x_owner2, U + 16);
+      uint32_t* srt2 = buf<uint32_t>(x_sorted2, U + 16);
+      uint32_t* oc = buf<uint32_t>(x_cnt, 2 * K);
+      WJ_CUDA_CHECK(cudaMemsetAsync(oc, 0, 2 * K * 4, st));
+      k_owner<<<grid_for(U, 256), 256, 0, st>>>((const uint32_t*)u_bucket.p, (uint32_t)U, (uint32_t)K, own, iota, oc);
+      launched();
+      // keep u_owner intact for the token pass: sort a copy
+      WJ_CUDA_CHECK(cudaMemcpyAsync(own2, own, U * 4, cudaMemcpyDeviceToDevice, st));
+      int bits = 0;
+      while ((1 << bits) < K) ++bits;
+      uint32_t* srt1 = (uint32_t*)grow(x_sorted, (U + 16) * 4);
+      const bool in1 = sort_pairs<uint32_t>(own2, iota, srt1, srt2, U, 0, bits, nullptr, false);
+      const uint32_t* sorted_u = in1 ? srt2 : iota;
+      std::vector<uint32_t> oc_h(K);
+      WJ_CUDA_CHECK(cudaMemcpyAsync(oc_h.data(), oc, K * 4, cudaMemcpyDeviceToHost, st));
+      sync();
+      for (int o = 0; o < K; ++o) t_off[o + 1] = t_off[o] + oc_h[o];
+      WJ_CUDA_CHECK(cudaMemcpyAsync(toff_d, t_off.data(), (K + 1) * 8, cudaMemcpyHostToDevice, st));
+      uint32_t* xid = buf<uint32_t>(x_xid, U);
+      k_xid<<<grid_for(U, 256), 256, 0, st>>>(sorted_u, (uint32_t)U, own, toff_d, xid);
+      launched();
+      uint64_t* boff = buf<uint64_t>(x_boff, U + 1);
+      scan<uint64_t>(PackTermSize{sorted_u, (const uint32_t*)u_len.p}, U, boff, boff + U);
+      // byte offsets at owner boundaries
+      for (int o = 0; o <= K; ++o)
+        WJ_CUDA_CHECK(cudaMemcpyAsync(&b_off[o], boff + t_off[o], 8, cudaMemcpyDeviceToHost, st));
+      sync();
+      send_terms = (uint8_t*)grow(x_send, b_off[K] + 16);
+      k_pack_terms<<<grid_for(U, 256), 256, 0, st>>>(sorted_u, (uint32_t)U, boff, (const uint4*)u_w.p, text,
+                                                    (const uint32_t*)u_ref.p, (const uint32_t*)u_len.p, send_terms);
+      launched();
+      // token records by owner, stream order kept (stable)
+      uint32_t* tk = buf<uint32_t>(x_tkey, Nc + 16);
+      uint32_t* ti = buf<uint32_t>(x_tidx, Nc + 16);
+      uint32_t* tk2 = buf<uint32_t>(x_tkey2, Nc + 16);
+      uint32_t* ti2 = buf<uint32_t>(x_tidx2, Nc + 16);
+      k_tok_owner<<<grid_for(Nc, 256), 256, 0, st>>>(lslot, Nc, (const uint32_t*)uid.p, own, tk, ti, oc + K);
+      launched();
+      const bool in2 = sort_pairs<uint32_t>(tk, ti, tk2, ti2, Nc, 0, bits, nullptr, false);
+      const uint32_t* sorted_t = in2 ? ti2 : ti;
+      send_rec = (uint2*)grow(x_rec, (Nc + 2) * sizeof(uint2));
+      k_pack_tok<<<grid_for(Nc, 256), 256, 0, st>>>(sorted_t, Nc, lslot, ldoc, (const uint32_t*)uid.p, xid, send_rec);
+      launched();
+      WJ_CUDA_CHECK(cudaMemcpyAsync(oc_h.data(), oc + K, K * 4, cudaMemcpyDeviceToHost, st));
+      sync();
+      for (int o = 0; o < K; ++o) r_off[o + 1] = r_off[o] + oc_h[o];
+      for (int o = 0; o < K; ++o) {
+        cnt[o] = t_off[o + 1] - t_off[o];
+        cnt[K + o] = b_off[o + 1] - b_off[o];
+        cnt[2 * K + o] = r_off[o + 1] - r_off[o];
+      }
+    }
+    // 3. exchange: counts, then the term text and the token records
+    std::vector<uint64_t> all(3 * K * K);
+    xport->allgather(cnt.data(), 3 * K, all.data(), st);
+    std::vector<uint64_t> rt_off(K + 1, 0), rb_off(K + 1, 0), rr_off(K + 1, 0);
+    for (int s = 0; s < K; ++s) {
+      const uint64_t* c = all.data() + (size_t)s * 3 * K;
+      rt_off[s + 1] = rt_off[s] + c[rank];
+      rb_off[s + 1] = rb_off[s] + c[K + rank];
+      rr_off[s + 1] = rr_off[s] + c[2 * K + rank];
+    }
+    uint8_t* recv_terms = (uint8_t*)grow(x_recv_terms, rb_off[K] + 32);
+    uint2* recv_rec = (uint2*)grow(x_recv_rec, (rr_off[K] + 2) * sizeof(uint2));
+    std::vector<uint64_t> rec_soff(K + 1), rec_roff(K + 1);
+    for (int o = 0; o <= K; ++o) { rec_soff[o] = r_off[o] * sizeof(uint2); rec_roff[o] = rr_off[o] * sizeof(uint2); }
+    const uint64_t t0 = xport->sent;
+    try {
+      xport->alltoallv(send_terms, b_off.data(), recv_terms, rb_off.data(), st);
+      xport->alltoallv(send_rec, rec_soff.data(), recv_rec, rec_roff.data(), st);
+    } catch (const ExchangeError& e) {
+      throw StatusError{WJ_ERR_NCCL, e.msg};
+    }
+    exchange_bytes += xport->sent - t0;
+    // 4. owner side: the received term text goes through the same tokenizer / dedup / dictionary
+    const uint64_t R = rr_off[K];
+    if (rt_off[K] > 0) {
+      uint64_t* so = buf<uint64_t>(x_syn_off, 2);
+      const uint64_t h2[2] = {0, rb_off[K]};
+      WJ_CUDA_CHECK(cudaMemcpyAsync(so, h2, 16, cudaMemcpyHostToDevice, st));
+      ChunkView sv{recv_terms, rb_off[K], so, 1};
+      uint64_t C2 = 0, U2 = 0;
+      uint32_t *sslot = nullptr, *sdoc = nullptr;
+      const uint64_t dropped0 = n_dropped;
+      const uint64_t Ns = tokenize_dedup(sv, 0, [&](uint64_t nc, uint32_t*& sp, uint32_t*& dp) {
+        sp = buf<uint32_t>(x_syn_slot, nc + 16);
+        dp = buf<uint32_t>(x_syn_doc, nc + 16);
+      }, C2, U2, sslot, sdoc);
+      n_dropped = dropped0;
+      if (Ns != rt_off[K]) throw StatusError{WJ_ERR_CUDA, "received term text: token count mismatch (internal)"};
+      dictionary_update(recv_terms, U2);
+      if (n_tokens + R > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 tokens in one index"};
+      uint32_t* gt = buf_keep<uint32_t>(g_tid, n_tokens + R + 16, n_tokens);
+      uint32_t* gd = buf_keep<uint32_t>(g_doc, n_tokens + R + 16, n_tokens);
+      uint64_t* ro = buf<uint64_t>(x_roff, K + 1);
+      uint64_t* tb = buf<uint64_t>(x_tbase, K + 1);
+      WJ_CUDA_CHECK(cudaMemcpyAsync(ro, rr_off.data(), (K + 1) * 8, cudaMemcpyHostToDevice, st));
+      WJ_CUDA_CHECK(cudaMemcpyAsync(tb, rt_off.data(), (K + 1) * 8, cudaMemcpyHostToDevice, st));
+      phase(WJ_PHASE_STREAM);
+      if (R > 0) {
+        k_map_recv<<<grid_for(R, 256), 256, 0, st>>>(recv_rec, R, ro, tb, (uint32_t)K, sslot, gt + n_tokens, gd + n_tokens);
+        launched();
+      }
+      register_chunk_map(C2, n_tokens);
+      n_tokens += R;
+    }
+    n_docs += tot_docs;
+    sync();  // exchange buffers are reused by the next chunk
   }
 
   void insert_new(const uint8_t* text, uint64_t U, uint64_t Nn) {
@@ -844,12 +1020,12 @@ extern "C" {
 int index_init(wj_index** out, const wj_config* cfg) {
   if (!out || !cfg) return WJ_ERR_INVALID_ARG;
   *out = nullptr;
-  if (cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~WJ_FLAG_PROFILE) || cfg->reserved) {
+  if (cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~(WJ_FLAG_PROFILE | WJ_FLAG_LOOPBACK)) || cfg->reserved) {
     g_init_err = "invalid config";
     return WJ_ERR_INVALID_ARG;
   }
-  if (cfg->world > 1) {
-    g_init_err = "world > 1 is not supported by this build";
+  if (cfg->world > 1 && !cfg->nccl_unique_id) {
+    g_init_err = "world > 1 needs nccl_unique_id (NCCL) or a loopback hub (WJ_FLAG_LOOPBACK)";
     return WJ_ERR_INVALID_ARG;
   }
   int ndev = 0;
@@ -876,6 +1052,16 @@ int index_init(wj_index** out, const wj_config* cfg) {
       ix->own_stream = true;
     }
     WJ_CUDA_CHECK(cudaHostAlloc(&ix->h_scal, 16 * sizeof(uint64_t), cudaHostAllocDefault));
+    if (cfg->world > 1) {
+      try {
+        if (cfg->flags & WJ_FLAG_LOOPBACK)
+          ix->xport = new LoopbackTransport((LoopbackHub*)cfg->nccl_unique_id, cfg->rank);
+        else
+          ix->xport = new NcclTransport(cfg->nccl_unique_id, cfg->rank, cfg->world);
+      } catch (const ExchangeError& e) {
+        throw StatusError{WJ_ERR_NCCL, e.msg};
+      }
+    }
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_os_pass<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)os_smem_bytes<uint64_t>()));
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_os_pass<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -995,7 +1181,7 @@ int index_stats(wj_index* ix, wj_stats* out) {
     out->new_terms_last = ix->new_last;
     out->btree_nodes = ix->n_nodes;
     out->btree_height_max = ix->height_max;
-    out->exchange_bytes = 0;
+    out->exchange_bytes = ix->exchange_bytes;
     out->device_bytes = ix->device_bytes;
     for (int i = 0; i < WJ_PHASE_COUNT; ++i) {
       out->phase_ms[i] = ix->phase_ms[i];
@@ -1085,11 +1271,104 @@ int index_debug_btree(wj_index* ix, void* nodes, uint64_t node_cap, uint64_t* n_
 
 const char* index_last_error(const wj_index* ix) { return ix ? ix->err.c_str() : g_init_err.c_str(); }
 
+int index_nccl_unique_id(void* out128) {
+  if (!out128) return WJ_ERR_INVALID_ARG;
+  try {
+    NcclApi& a = NcclApi::get();
+    ncclUniqueId id;
+    if (!a.GetUniqueId || a.GetUniqueId(&id) != ncclSuccess) {
+      g_init_err = "ncclGetUniqueId failed";
+      return WJ_ERR_NCCL;
+    }
+    memcpy(out128, &id, sizeof(id));
+    return WJ_OK;
+  } catch (const ExchangeError& e) {
+    g_init_err = e.msg;
+    return WJ_ERR_NCCL;
+  }
+}
+
+int index_loopback_create(int32_t world, void** hub) {
+  if (!hub || world < 1) return WJ_ERR_INVALID_ARG;
+  *hub = new (std::nothrow) LoopbackHub(world);
+  return *hub ? WJ_OK : WJ_ERR_OOM;
+}
+
+void index_loopback_destroy(void* hub) { delete (LoopbackHub*)hub; }
+
+int index_merge_serialized(int32_t k, const uint8_t* const* slices, const uint64_t* sizes, uint8_t* out, uint64_t cap,
+                           uint64_t* n_out) {
+  if (k < 1 || !slices || !sizes || !n_out) return WJ_ERR_INVALID_ARG;
+  std::vector<SliceView> v(k);
+  uint64_t nt = 0, np = 0, ntb = 0, ntok = 0, ndrop = 0;
+  for (int i = 0; i < k; ++i) {
+    if (!slices[i] || !parse_slice(slices[i], sizes[i], v[i])) {
+      g_init_err = "index_merge_serialized: slice " + std::to_string(i) + " is not a serialized index";
+      return WJ_ERR_INVALID_ARG;
+    }
+    if (v[i].n_docs != v[0].n_docs) {
+      g_init_err = "index_merge_serialized: slices disagree on n_docs";
+      return WJ_ERR_INVALID_ARG;
+    }
+    nt += v[i].n_terms; np += v[i].n_postings; ntb += v[i].n_tb; ntok += v[i].n_tokens; ndrop += v[i].n_dropped;
+  }
+  const uint64_t size = 64 + 8 * (nt + 1) + pad8(ntb) + pad8(4 * nt) + 8 * nt + 8 * (nt + 1) + 2 * pad8(4 * np);
+  *n_out = size;
+  if (!out) return WJ_OK;
+  if (cap < size) return WJ_ERR_BUFFER_TOO_SMALL;
+  memset(out, 0, size);
+  uint64_t h[8];
+  memcpy(h, "WJINV001", 8);
+  h[1] = v[0].n_docs; h[2] = ntok; h[3] = ndrop; h[4] = nt; h[5] = np; h[6] = ntb; h[7] = 0;
+  memcpy(out, h, 64);
+  uint64_t p = 64;
+  uint64_t* term_off = (uint64_t*)(out + p); p += 8 * (nt + 1);
+  uint8_t* tb = out + p; p += pad8(ntb);
+  uint32_t* df = (uint32_t*)(out + p); p += pad8(4 * nt);
+  uint64_t* cf = (uint64_t*)(out + p); p += 8 * nt;
+  uint64_t* post_off = (uint64_t*)(out + p); p += 8 * (nt + 1);
+  uint32_t* docid = (uint32_t*)(out + p); p += pad8(4 * np);
+  uint32_t* tf = (uint32_t*)(out + p);
+  std::vector<uint64_t> cur(k, 0);
+  auto term_less = [&](int a, int b) {
+    const SliceView &x = v[a], &y = v[b];
+    const uint8_t* s1 = x.term_bytes + x.term_off[cur[a]];
+    const uint64_t l1 = x.term_off[cur[a] + 1] - x.term_off[cur[a]];
+    const uint8_t* s2 = y.term_bytes + y.term_off[cur[b]];
+    const uint64_t l2 = y.term_off[cur[b] + 1] - y.term_off[cur[b]];
+    const int c = memcmp(s1, s2, l1 < l2 ? l1 : l2);
+    return c != 0 ? c < 0 : l1 < l2;
+  };
+  uint64_t to = 0, po = 0;
+  for (uint64_t t = 0; t < nt; ++t) {
+    int best = -1;
+    for (int i = 0; i < k; ++i)
+      if (cur[i] < v[i].n_terms && (best < 0 || term_less(i, best))) best = i;
+    SliceView& x = v[best];
+    const uint64_t j = cur[best]++;
+    const uint64_t l = x.term_off[j + 1] - x.term_off[j];
+    term_off[t] = to;
+    memcpy(tb + to, x.term_bytes + x.term_off[j], l);
+    to += l;
+    df[t] = x.df[j];
+    cf[t] = x.cf[j];
+    post_off[t] = po;
+    const uint64_t a = x.post_off[j], b = x.post_off[j + 1];
+    memcpy(docid + po, x.docid + a, 4 * (b - a));
+    memcpy(tf + po, x.tf + a, 4 * (b - a));
+    po += b - a;
+  }
+  term_off[nt] = to;
+  post_off[nt] = po;
+  return WJ_OK;
+}
+
 void index_destroy(wj_index* ix) {
   if (!ix) return;
   cudaSetDevice(ix->device);
   if (ix->st) cudaStreamSynchronize(ix->st);
   ix->free_all();
+  delete ix->xport;
   for (auto e : ix->ev_pool) cudaEventDestroy(e);
   if (ix->h_scal) cudaFreeHost(ix->h_scal);
   if (ix->own_stream && ix->st) cudaStreamDestroy(ix->st);

@@ -1,0 +1,109 @@
+"""Multi-rank indexing through the C ABI on one GPU (loopback transport, one host thread per rank).
+
+Each rank indexes its own contiguous document range of every chunk; terms are routed to the rank
+owning their trie collection (b mod K) with the same pack / all-to-all-v / unpack code
+the NCCL transport uses.  Parity: the merge of the K slices is byte-identical to the CPU oracle, and
+every slice holds only owned collections.
+"""
+import threading
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+import wjformat
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("no CUDA device", allow_module_level=True)
+
+import paper_conf_ipps_weij11_b200 as wj  # noqa: E402
+
+
+def dist_index(text, doc_off, K, cuts=None, queries=()):
+    off = np.asarray(doc_off, dtype=np.uint64)
+    text = np.asarray(text, dtype=np.uint8)
+    n = len(off) - 1
+    cuts = cuts or [0, n]
+    hub = wj.LoopbackHub(K)
+    slices = [None] * K
+    answers = [dict() for _ in range(K)]
+    errors = []
+
+    def run(r):
+        try:
+            with wj.Index(device=0, rank=r, world=K, hub=hub, own_stream=True) as ix:
+                for a, b in zip(cuts, cuts[1:]):
+                    # rank r's contiguous document range of this chunk (rank order = DocID order)
+                    bounds = [a + (b - a) * i // K for i in range(K + 1)]
+                    lo, hi = bounds[r], bounds[r + 1]
+                    t = text[int(off[lo]):int(off[hi])]
+                    o = off[lo:hi + 1] - off[lo]
+                    ix.add_stream(t, o)
+                ix.finalize()
+                slices[r] = ix.serialize()
+                for q in queries:
+                    answers[r][q] = ix.read_postings(q)
+        except Exception as e:  # pragma: no cover
+            errors.append((r, e))
+            raise
+
+    th = [threading.Thread(target=run, args=(r,)) for r in range(K)]
+    for x in th:
+        x.start()
+    for x in th:
+        x.join(timeout=600)
+    hub.close()
+    assert not errors, errors
+    return slices, answers
+
+
+@pytest.mark.parametrize("K", [2, 3, 4])
+def test_loopback_config1(K):
+    text, off = gen.generate(gen.CONFIGS[1])
+    want = oracle.index_bytes(text, off)
+    slices, _ = dist_index(text, off, K, cuts=[0, 400, 1000])
+    for r, sl in enumerate(slices):
+        ix = wjformat.parse(sl)
+        assert all(oracle.bucket(t) % K == r for t in ix.terms()), "slice holds a non-owned collection"
+        assert ix.n_docs == 1000
+    assert wj.merge_serialized(slices) == want
+
+
+def test_loopback_edges_and_queries():
+    docs = [b"", b"a", b"b", b"Apple apple APPLE", b"x" * 300 + b" zoo 01 0195 954", b"", b"aaat aabomycin zzzy",
+            b"application lication"] * 5
+    text, off = gen.from_docs(docs)
+    want = oracle.index_bytes(text, off)
+    o = oracle.Oracle()
+    o.add(text, off)
+    qs = [b"apple", b"zoo", b"application", b"01", b"nothere"]
+    slices, ans = dist_index(text, off, 3, cuts=[0, 7, 8, 40], queries=qs)
+    assert wj.merge_serialized(slices) == want
+    for q in qs:
+        owner = oracle.bucket(q) % 3
+        for r in range(3):
+            got = ans[r][q]
+            ref = o.postings(q)
+            if r == owner and ref is not None:
+                assert got is not None and np.array_equal(got[0], ref[0]) and np.array_equal(got[1], ref[1])
+            else:
+                assert got is None
+
+
+def test_loopback_many_chunks_new_terms():
+    cfg = gen.CONFIGS[1].scaled(vocab=80_000)
+    text, off = gen.generate(cfg)
+    want = oracle.index_bytes(text, off)
+    slices, _ = dist_index(text, off, 2, cuts=[0, 3, 100, 101, 500, 1000])
+    assert wj.merge_serialized(slices) == want
+
+
+def test_loopback_rank_with_no_documents():
+    text, off = gen.from_docs([b"one two three", b"two three four"])
+    want = oracle.index_bytes(text, off)
+    slices, _ = dist_index(text, off, 4)  # 2 documents over 4 ranks: two ranks send nothing
+    assert wj.merge_serialized(slices) == want

@@ -1,0 +1,83 @@
+"""Multi-GPU host-side logic on CPU (no GPU): the owner map, the K-way merge of
+per-rank dictionary slices done by the C ABI (index_merge_serialized), and the torch.distributed
+(gloo, world_size 2) gather + merge protocol that bench.py uses for N > 1."""
+import os
+import socket
+
+import pytest
+import torch.multiprocessing as mp
+
+import gen
+import oracle
+import paper_conf_ipps_weij11_b200 as wj
+import wjformat
+
+
+def test_owner_map_paper_example():
+    # "if unpopular trie collections have indices (0, 13, 27, 175, 384, 5810, 10041, 17316) and there
+    # are two GPU, then (0, 384, 5810, 17316) are assigned to GPU indexer 0 and (13, 27, 175, 10041) to GPU 1"
+    idx = [0, 13, 27, 175, 384, 5810, 10041, 17316]
+    assert [i for i in idx if wj.owner_of(i, 2) == 0] == [0, 384, 5810, 17316]
+    assert [i for i in idx if wj.owner_of(i, 2) == 1] == [13, 27, 175, 10041]
+
+
+def test_serialize_helper_roundtrip():
+    text, off = gen.generate(gen.CONFIGS[1].scaled(vocab=500))
+    b = oracle.index_bytes(text, off)
+    ix = wjformat.parse(b)
+    d = ix.as_dict()
+    assert wjformat.serialize(ix.n_docs, ix.n_tokens, ix.n_dropped, ix.terms(), [d[t] for t in ix.terms()]) == b
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 4, 8])
+def test_merge_of_owner_slices_is_the_global_index(world):
+    text, off = gen.generate(gen.CONFIGS[1])
+    full = oracle.index_bytes(text, off)
+    slices = wjformat.split_by_owner(full, world, oracle.bucket)
+    assert wj.merge_serialized(slices) == full
+
+
+def test_merge_rejects_bad_input():
+    text, off = gen.from_docs([b"a b", b"c"])
+    good = oracle.index_bytes(text, off)
+    with pytest.raises(wj.WJError):
+        wj.merge_serialized([good, b"not an index"])
+    t2, o2 = gen.from_docs([b"a b"])
+    with pytest.raises(wj.WJError):  # slices must agree on n_docs
+        wj.merge_serialized([good, oracle.index_bytes(t2, o2)])
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _gloo_worker(rank, world, port, q):
+    import torch.distributed as dist
+
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    text, off = gen.generate(gen.CONFIGS[1])
+    full = oracle.index_bytes(text, off)
+    mine = wjformat.split_by_owner(full, world, oracle.bucket)[rank]  # this rank's dictionary slice
+    got = [None] * world
+    dist.all_gather_object(got, mine)
+    if rank == 0:
+        q.put(wj.merge_serialized(got) == full)
+    dist.destroy_process_group()
+
+
+def test_gloo_world2_gather_and_merge():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_gloo_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    ok = q.get(timeout=120)
+    for p in ps:
+        p.join(timeout=60)
+    assert ok

@@ -105,3 +105,46 @@ def check_invariants(ix: Index) -> None:
         assert a < b, f"dictionary not strictly increasing: {a!r} >= {b!r}"
     for t in terms:
         assert all(not (65 <= c <= 90) for c in t), "unfolded upper-case byte"
+
+
+def serialize(n_docs, n_tokens, n_dropped, terms, postings):
+    """Canonical bytes from python lists (test helper): terms = [bytes], postings = [[(doc, tf)]]."""
+    import struct
+
+    out = bytearray(b"WJINV001")
+    n_post = sum(len(p) for p in postings)
+    tb = b"".join(terms)
+    out += struct.pack("<7Q", n_docs, n_tokens, n_dropped, len(terms), n_post, len(tb), 0)
+    off = 0
+    for t in terms:
+        out += struct.pack("<Q", off)
+        off += len(t)
+    out += struct.pack("<Q", off)
+    out += tb + b"\0" * (_pad8(len(tb)) - len(tb))
+    df = b"".join(struct.pack("<I", len(p)) for p in postings)
+    out += df + b"\0" * (_pad8(len(df)) - len(df))
+    for p in postings:
+        out += struct.pack("<Q", sum(f for _, f in p))
+    off = 0
+    for p in postings:
+        out += struct.pack("<Q", off)
+        off += len(p)
+    out += struct.pack("<Q", off)
+    d = b"".join(struct.pack("<I", x) for p in postings for x, _ in p)
+    out += d + b"\0" * (_pad8(len(d)) - len(d))
+    f = b"".join(struct.pack("<I", y) for p in postings for _, y in p)
+    out += f + b"\0" * (_pad8(len(f)) - len(f))
+    return bytes(out)
+
+
+def split_by_owner(buf: bytes, world: int, bucket_fn):
+    """Slices of a serialized index: rank r keeps the terms of trie collections b with b % world == r."""
+    ix = parse(buf)
+    d = ix.as_dict()
+    out = []
+    for r in range(world):
+        terms = [t for t in ix.terms() if bucket_fn(t) % world == r]
+        posts = [d[t] for t in terms]
+        ntok = sum(f for p in posts for _, f in p)
+        out.append(serialize(ix.n_docs, ntok, ix.n_dropped if r == 0 else 0, terms, posts))
+    return out
