@@ -172,10 +172,21 @@ def run_reference(args, rank, world):
                          "sample": f"first {nd} documents ({len(text)} B) per step, std::map oracle, 1 thread"},
         "e2e": {"value": val, "unit": "MB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
-    print(json.dumps(line), flush=True)
+    print_json(line)
+
+
+def print_json(obj):  # replaced in main() by a writer bound to the real stdout
+    print(json.dumps(obj), flush=True)
 
 
 def main():
+    # The driver parses exactly one JSON line from stdout: keep the real stdout for it and send
+    # everything else (NCCL's version banner, library prints) to stderr.
+    json_out = os.fdopen(os.dup(1), "w")
+    sys.stdout.flush()
+    os.dup2(2, 1)
+    global print_json
+    print_json = lambda obj: (json_out.write(json.dumps(obj) + "\n"), json_out.flush())  # noqa: E731
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=30)
@@ -211,9 +222,11 @@ def main():
     off_d = off_h.cuda()
     torch.cuda.synchronize()
 
-    if world > 1:
+    force_dist = os.environ.get("WJ_BENCH_FORCE_DIST") == "1"  # exercise the NCCL path at N=1
+    if world > 1 or force_dist:
         nid = [wj.nccl_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(nid, src=0)
+        if world > 1:
+            dist.broadcast_object_list(nid, src=0)
         ix = wj.Index(device=local, profile=True, rank=rank, world=world, nccl_id=nid[0])
     else:
         ix = wj.Index(device=local, profile=True)
@@ -342,7 +355,7 @@ def main():
             "kernels": kernels,
             "paper_context": "262.76 MB/s end-to-end on ClueWeb09 (2x X5560 + 2x C1060, Table VI); not this workload",
         }
-        print(json.dumps(line), flush=True)
+        print_json(line)
     ix.close()
     if world > 1:
         dist.destroy_process_group()

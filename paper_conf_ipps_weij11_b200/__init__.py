@@ -62,12 +62,27 @@ assert NODE_DTYPE.itemsize == 512
 _lib = None
 
 
+def _nccl_hint():
+    """Point the library's dlopen at the NCCL torch ships (only used when world > 1)."""
+    if "WJ_NCCL_LIB" in os.environ:
+        return
+    try:
+        import nvidia.nccl
+        base = list(nvidia.nccl.__path__)[0]
+        cand = os.path.join(base, "lib", "libnccl.so.2")
+        if os.path.exists(cand):
+            os.environ["WJ_NCCL_LIB"] = cand
+    except Exception:
+        pass
+
+
 def load_library():
     """Load libwjindex.so (in-tree).  Raises if it is missing: there is no fallback."""
     global _lib
     if _lib is None:
         if not os.path.exists(LIB_PATH):
             raise ImportError(f"{LIB_PATH} is missing: run __graft_entry__.build() (nvcc sm_100a)")
+        _nccl_hint()
         lib = ctypes.CDLL(LIB_PATH)
         vp, u64, u32, i32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int
         P64 = ctypes.POINTER(ctypes.c_uint64)

@@ -17,14 +17,24 @@
 
 namespace wj {
 
+// per-owner counts: block histogram in shared memory, one global atomic per (block, owner)
+constexpr int kMaxRanks = 1024;
+
 __global__ void k_owner(const uint32_t* u_bucket, uint32_t U, uint32_t K, uint32_t* owner, uint32_t* iota,
                         uint32_t* owner_cnt) {
+  __shared__ uint32_t h[kMaxRanks];
+  for (uint32_t i = threadIdx.x; i < K; i += blockDim.x) h[i] = 0;
+  __syncthreads();
   const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
-  if (u >= U) return;
-  const uint32_t o = u_bucket[u] % K;
-  owner[u] = o;
-  iota[u] = u;
-  atomicAdd(&owner_cnt[o], 1u);
+  if (u < U) {
+    const uint32_t o = u_bucket[u] % K;
+    owner[u] = o;
+    iota[u] = u;
+    atomicAdd(&h[o], 1u);
+  }
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < K; i += blockDim.x)
+    if (h[i]) atomicAdd(&owner_cnt[i], h[i]);
 }
 
 // xid = index of the unique term in the list sent to its owner (terms sorted stably by owner)
@@ -55,13 +65,20 @@ __global__ void k_pack_terms(const uint32_t* sorted_u, uint32_t U, const uint64_
 }
 
 __global__ void k_tok_owner(const uint32_t* slot, uint64_t n, const uint32_t* slot_uid, const uint32_t* u_owner,
-                            uint32_t* tkey, uint32_t* tidx, uint32_t* tok_cnt) {
+                            uint32_t K, uint32_t* tkey, uint32_t* tidx, uint32_t* tok_cnt) {
+  __shared__ uint32_t h[kMaxRanks];
+  for (uint32_t i = threadIdx.x; i < K; i += blockDim.x) h[i] = 0;
+  __syncthreads();
   const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (t >= n) return;
-  const uint32_t o = u_owner[slot_uid[slot[t]]];
-  tkey[t] = o;
-  tidx[t] = (uint32_t)t;
-  atomicAdd(&tok_cnt[o], 1u);
+  if (t < n) {
+    const uint32_t o = u_owner[slot_uid[slot[t]]];
+    tkey[t] = o;
+    tidx[t] = (uint32_t)t;
+    atomicAdd(&h[o], 1u);
+  }
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < K; i += blockDim.x)
+    if (h[i]) atomicAdd(&tok_cnt[i], h[i]);
 }
 
 __global__ void k_pack_tok(const uint32_t* sorted_t, uint64_t n, const uint32_t* slot, const uint32_t* doc,

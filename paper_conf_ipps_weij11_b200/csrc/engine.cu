@@ -523,7 +523,7 @@ struct wj_index {
     const uint64_t* off = nullptr;
     stage(bytes, n_bytes, doc_off_in, nd, &text, &off);
     ++n_chunks;
-    if (world > 1) {
+    if (xport) {
       add_chunk_dist(text, nd ? n_bytes : 0, off, nd);
       phase(-1);
       return;
@@ -622,7 +622,7 @@ struct wj_index {
       uint32_t* ti = buf<uint32_t>(x_tidx, Nc + 16);
       uint32_t* tk2 = buf<uint32_t>(x_tkey2, Nc + 16);
       uint32_t* ti2 = buf<uint32_t>(x_tidx2, Nc + 16);
-      k_tok_owner<<<grid_for(Nc, 256), 256, 0, st>>>(lslot, Nc, (const uint32_t*)uid.p, own, tk, ti, oc + K);
+      k_tok_owner<<<grid_for(Nc, 256), 256, 0, st>>>(lslot, Nc, (const uint32_t*)uid.p, own, (uint32_t)K, tk, ti, oc + K);
       launched();
       const bool in2 = sort_pairs<uint32_t>(tk, ti, tk2, ti2, Nc, 0, bits, nullptr, false);
       const uint32_t* sorted_t = in2 ? ti2 : ti;
@@ -1020,7 +1020,7 @@ extern "C" {
 int index_init(wj_index** out, const wj_config* cfg) {
   if (!out || !cfg) return WJ_ERR_INVALID_ARG;
   *out = nullptr;
-  if (cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~(WJ_FLAG_PROFILE | WJ_FLAG_LOOPBACK)) || cfg->reserved) {
+  if (cfg->world < 1 || cfg->world > 1024 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~(WJ_FLAG_PROFILE | WJ_FLAG_LOOPBACK)) || cfg->reserved) {
     g_init_err = "invalid config";
     return WJ_ERR_INVALID_ARG;
   }
@@ -1052,7 +1052,7 @@ int index_init(wj_index** out, const wj_config* cfg) {
       ix->own_stream = true;
     }
     WJ_CUDA_CHECK(cudaHostAlloc(&ix->h_scal, 16 * sizeof(uint64_t), cudaHostAllocDefault));
-    if (cfg->world > 1) {
+    if (cfg->world > 1 || cfg->nccl_unique_id) {  // a transport at world 1 runs the same distributed path
       try {
         if (cfg->flags & WJ_FLAG_LOOPBACK)
           ix->xport = new LoopbackTransport((LoopbackHub*)cfg->nccl_unique_id, cfg->rank);

@@ -163,8 +163,15 @@ struct NcclTransport : Transport {
   }
   void alltoallv(const void* send, const uint64_t* soff, void* recv, const uint64_t* roff, cudaStream_t st) override {
     NcclApi& a = NcclApi::get();
+    // the rank's own segment never leaves the GPU: a device copy, not an NCCL self send/recv
+    const uint64_t own = soff[rank + 1] - soff[rank];
+    if (own != roff[rank + 1] - roff[rank]) throw ExchangeError{"alltoallv: self size mismatch"};
+    if (own && cudaMemcpyAsync((char*)recv + roff[rank], (const char*)send + soff[rank], own, cudaMemcpyDeviceToDevice,
+                               st) != cudaSuccess)
+      throw ExchangeError{"alltoallv: self copy failed"};
     nccl_check(a.GroupStart(), "ncclGroupStart");
     for (int p = 0; p < world; ++p) {
+      if (p == rank) continue;
       const uint64_t sb = soff[p + 1] - soff[p], rb = roff[p + 1] - roff[p];
       if (sb) nccl_check(a.Send((const char*)send + soff[p], sb, ncclChar, p, comm, st), "ncclSend");
       if (rb) nccl_check(a.Recv((char*)recv + roff[p], rb, ncclChar, p, comm, st), "ncclRecv");

@@ -107,3 +107,24 @@ def test_loopback_rank_with_no_documents():
     want = oracle.index_bytes(text, off)
     slices, _ = dist_index(text, off, 4)  # 2 documents over 4 ranks: two ranks send nothing
     assert wj.merge_serialized(slices) == want
+
+
+def test_nccl_transport_single_rank():
+    # world 1 with an NCCL communicator runs the distributed path (comm init, all-gather, self send/recv)
+    text, off = gen.generate(gen.CONFIGS[1])
+    want = oracle.index_bytes(text, off)
+    nid = wj.nccl_unique_id()
+    with wj.Index(device=0, rank=0, world=1, nccl_id=nid) as ix:
+        ix.add_stream(text[: int(off[300])], off[:301])
+        ix.add_stream(text[int(off[300]):], off[300:] - off[300])
+        ix.finalize()
+        got = ix.serialize()
+        st = ix.stats()
+    assert got == want
+    assert st["exchange_bytes"] == 0  # nothing leaves a single rank
+
+
+def test_loopback_single_rank():
+    text, off = gen.generate(gen.CONFIGS[1].scaled(vocab=3000))
+    slices, _ = dist_index(text, off, 1, cuts=[0, 500, 1000])
+    assert slices[0] == oracle.index_bytes(text, off)
