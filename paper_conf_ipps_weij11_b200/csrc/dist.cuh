@@ -71,7 +71,7 @@ __global__ void k_tok_owner(const uint32_t* slot, uint64_t n, const uint32_t* sl
   __syncthreads();
   const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (t < n) {
-    const uint32_t o = u_owner[slot_uid[slot[t]]];
+    const uint32_t o = u_owner[slot_uid[slot[t] & ((1u << 25) - 1u)]];
     tkey[t] = o;
     tidx[t] = (uint32_t)t;
     atomicAdd(&h[o], 1u);
@@ -86,7 +86,7 @@ __global__ void k_pack_tok(const uint32_t* sorted_t, uint64_t n, const uint32_t*
   const uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (j >= n) return;
   const uint32_t t = sorted_t[j];
-  rec[j] = make_uint2(xid[slot_uid[slot[t]]], doc[t]);
+  rec[j] = make_uint2(xid[slot_uid[slot[t] & ((1u << 25) - 1u)]], doc[t]);
 }
 
 // owner side: record j from source s -> term index term_base[s] + xid of the received term text,

@@ -10,6 +10,7 @@
 #include "common.cuh"
 #include "dict.cuh"
 #include "dist.cuh"
+#include "hot.cuh"
 #include "exchange.h"
 #include "postings.cuh"
 #include "radix.cuh"
@@ -95,6 +96,7 @@ struct wj_index {
   bool broken = false;
 
   // counters
+  uint64_t n_elems = 0;  // stream length (tokens + hot-term elements + holes)
   uint64_t n_docs = 0, n_tokens = 0, n_dropped = 0, n_chunks = 0, launches = 0, syncs = 0;
   uint64_t unique_last = 0, new_last = 0, n_nodes = 0, height_max = 0;
   uint32_t V = 0;
@@ -104,6 +106,15 @@ struct wj_index {
   uint64_t exchange_bytes = 0;
 
   Transport* xport = nullptr;  // world > 1
+  // sampled hot terms of the current chunk (hot.cuh)
+  DevBuf hot_tab, hot_tfb, hot_slotb, hot_kb, hot_offb, samp_off, samp_slot, samp_doc, samp_cnt, samp_ck, samp_cv,
+      samp_ck2, samp_cv2, samp_n;
+  uint32_t hot_H = 0, hot_D = 0;
+  bool stream_has_hot = false;  // some chunk appended hot-term elements (holes + counts > 1)
+  // Sampled hot-term path (hot.cuh) is opt-in: on config 2 it removes ~30% of the
+  // stream elements but its per-document counters cost more global atomics in the emit kernel than
+  // the sort saves (profiles/r01_README.md).  WJ_HOT_MIN_BYTES=<bytes> enables it for larger chunks.
+  uint64_t hot_min_bytes = ~0ull;
   DevBuf x_owner, x_iota, x_sorted, x_sorted2, x_owner2, x_xid, x_cnt, x_toff, x_boff, x_send, x_tkey, x_tidx, x_tkey2,
       x_tidx2, x_rec, x_recv_terms, x_recv_rec, x_loc_slot, x_loc_doc, x_syn_slot, x_syn_doc, x_syn_off, x_roff, x_tbase;
   // persistent dictionary
@@ -124,7 +135,7 @@ struct wj_index {
   std::vector<DevBuf> chunk_map;        // per chunk: slot -> termID (-> rank at finalize)
   std::vector<uint64_t> chunk_tok;      // per chunk: first token index in the stream
   std::vector<uint32_t> chunk_C;        // per chunk: table capacity
-  DevBuf rle_look, rle_p0, rle_lead;
+  DevBuf rle_look, rle_p0, rle_lead, rle_tok, cstart_b;
   uint32_t* f_key = nullptr;   // sorted keys (term ranks)
   uint32_t* f_doc = nullptr;   // sorted docIDs
   // profiling
@@ -181,13 +192,16 @@ struct wj_index {
       b->p = nullptr;
       b->cap = 0;
     }
+    DevBuf* hs[] = {&hot_tab, &hot_tfb, &hot_slotb, &hot_kb, &hot_offb, &samp_off, &samp_slot, &samp_doc, &samp_cnt,
+                    &samp_ck, &samp_cv, &samp_ck2, &samp_cv2, &samp_n};
+    for (DevBuf* b : hs) { if (b->p) cudaFree(b->p); *b = DevBuf{}; }
     DevBuf* xs[] = {&x_owner, &x_iota, &x_sorted, &x_sorted2, &x_owner2, &x_xid, &x_cnt, &x_toff, &x_boff, &x_send,
                     &x_tkey, &x_tidx, &x_tkey2, &x_tidx2, &x_rec, &x_recv_terms, &x_recv_rec, &x_loc_slot,
                     &x_loc_doc, &x_syn_slot, &x_syn_doc, &x_syn_off, &x_roff, &x_tbase};
     for (DevBuf* b : xs) { if (b->p) cudaFree(b->p); *b = DevBuf{}; }
     for (auto& b : chunk_map) if (b.p) cudaFree(b.p);
     chunk_map.clear();
-    for (DevBuf* b : {&rle_look, &rle_p0, &rle_lead}) { if (b->p) cudaFree(b->p); *b = DevBuf{}; }
+    for (DevBuf* b : {&rle_look, &rle_p0, &rle_lead, &rle_tok, &cstart_b}) { if (b->p) cudaFree(b->p); *b = DevBuf{}; }
     for (int i = 0; i < 4; ++i) {
       if (lvA[i].p) cudaFree(lvA[i].p);
       if (lvB[i].p) cudaFree(lvB[i].p);
@@ -283,7 +297,8 @@ struct wj_index {
     collect_phases();
     chunk_tok.clear();
     chunk_C.clear();
-    n_docs = n_tokens = n_dropped = n_chunks = 0;
+    n_docs = n_tokens = n_dropped = n_chunks = n_elems = 0;
+    stream_has_hot = false;
     unique_last = new_last = n_nodes = height_max = 0;
     exchange_bytes = 0;
     V = 0;
@@ -368,13 +383,18 @@ struct wj_index {
   }
 
   void emit_tokens(const ChunkView& cv, uint64_t n_segs, uint32_t* slot_out, uint32_t* doc_out, uint32_t doc_base,
-                   uint64_t C, uint32_t* dstart, uint32_t* dlen) {
+                   uint64_t C, uint32_t* dstart, uint32_t* dlen, bool use_hot = false, bool clear_table = true) {
     Slot* tab = buf<Slot>(table, C);
-    WJ_CUDA_CHECK(cudaMemsetAsync(tab, 0, C * sizeof(Slot), st));
+    uint32_t* sref = buf<uint32_t>(slotref, C);
+    if (clear_table) WJ_CUDA_CHECK(cudaMemsetAsync(tab, 0, C * sizeof(Slot), st));
     WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 5, 0, 8, st));
     EmitOut eo;
+    eo.hot = (use_hot && hot_H) ? (const HotEntry*)hot_tab.p : nullptr;
+    eo.hot_mask = kHotTable - 1;
+    eo.hot_docs = hot_D;
+    eo.hot_tf = (uint32_t*)hot_tfb.p;
     eo.table = tab;
-    eo.slot_ref = buf<uint32_t>(slotref, C);
+    eo.slot_ref = sref;
     eo.mask = (uint32_t)(C - 1);
     eo.doc_base = doc_base;
     eo.slot = slot_out;
@@ -385,9 +405,69 @@ struct wj_index {
     const uint64_t ranges = (n_segs + kSegsPerWarp - 1) / kSegsPerWarp;
     const unsigned grid = (unsigned)((ranges + kTokWarps - 1) / kTokWarps);
     ktime(WJ_KERNEL_TOKENIZE_EMIT, [&] {
-      k_tok_emit<<<grid, kTokThreads, 0, st>>>(cv, (uint32_t)n_segs, (const uint64_t*)kstart.p, (const uint32_t*)seg_cnt.p, eo);
+      k_tok_emit<<<grid, kTokThreads, 0, st>>>(cv, (uint32_t)n_segs, (const uint64_t*)kstart.p,
+                                               (const uint32_t*)seg_cnt.p, eo);
       launched();
     });
+  }
+
+  // Sampled popular terms of a chunk ("1MB out of every 1GB"): tokenise the first 1 MiB of
+  // its documents with the same kernels, count terms, keep the <= 256 most frequent (>= 16
+  // occurrences, <= 11 bytes) -> hot_kb (slot words).  Returns the number of hot terms.
+  uint32_t select_hot(const ChunkView& cv) {
+    const uint64_t S = std::min<uint64_t>(cv.n_bytes, 1ull << 20);
+    uint64_t* sn = buf<uint64_t>(samp_n, 1);
+    k_sample_docs<<<1, 32, 0, st>>>(cv.doc_off, cv.n_docs, S, nullptr, sn);
+    launched();
+    uint64_t nds = 0;
+    WJ_CUDA_CHECK(cudaMemcpyAsync(&nds, sn, 8, cudaMemcpyDeviceToHost, st));
+    sync();
+    if (nds == 0) return 0;
+    uint64_t* so = buf<uint64_t>(samp_off, nds + 1);
+    k_sample_docs_copy<<<grid_for(nds + 1, 256), 256, 0, st>>>(cv.doc_off, nds, S, so);
+    launched();
+    ChunkView sv{cv.text, S, so, nds};
+    const uint64_t n_segs = (S + kSegBytes - 1) / kSegBytes;
+    const uint64_t Ns = count_tokens(sv, n_segs);
+    if (Ns < 1024) return 0;
+    uint32_t* ss = buf<uint32_t>(samp_slot, Ns + 16);
+    uint32_t* sd = buf<uint32_t>(samp_doc, Ns + 16);
+    const uint64_t Cs = pow2_at_least(2 * Ns);
+    emit_tokens(sv, n_segs, ss, sd, 0, Cs, nullptr, nullptr, false, true);
+    readback(5, 1);
+    if ((uint32_t)h_scal[5]) return 0;
+    uint32_t* cnt = buf<uint32_t>(samp_cnt, Cs);
+    WJ_CUDA_CHECK(cudaMemsetAsync(cnt, 0, Cs * 4, st));
+    k_sample_count<<<grid_for(Ns, 256), 256, 0, st>>>(ss, Ns, cnt);
+    launched();
+    uint32_t* ck = buf<uint32_t>(samp_ck, Cs + 16);
+    uint32_t* cv2 = buf<uint32_t>(samp_cv, Cs + 16);
+    uint32_t* ck2 = buf<uint32_t>(samp_ck2, Cs + 16);
+    uint32_t* cvb = buf<uint32_t>(samp_cv2, Cs + 16);
+    k_sample_cand<<<grid_for(Cs, 256), 256, 0, st>>>((const Slot*)table.p, cnt, (uint32_t)Cs, ck, cv2);
+    launched();
+    int bits = 0;
+    while ((1ull << bits) <= Ns) ++bits;
+    const bool in1 = sort_pairs<uint32_t>(ck, cv2, ck2, cvb, Cs, 0, bits, nullptr, false);
+    const uint32_t* sk = in1 ? ck2 : ck;
+    const uint32_t* sv_ = in1 ? cvb : cv2;
+    const uint32_t take = (uint32_t)std::min<uint64_t>(kHotMax, Cs);
+    std::vector<uint32_t> tk(take), tv(take);
+    WJ_CUDA_CHECK(cudaMemcpyAsync(tk.data(), sk + (Cs - take), take * 4, cudaMemcpyDeviceToHost, st));
+    WJ_CUDA_CHECK(cudaMemcpyAsync(tv.data(), sv_ + (Cs - take), take * 4, cudaMemcpyDeviceToHost, st));
+    sync();
+    std::vector<uint32_t> hot_slots;
+    for (int i = (int)take - 1; i >= 0; --i)
+      if (tk[i] >= kHotMinCount) hot_slots.push_back(tv[i]);
+    const uint32_t H = (uint32_t)hot_slots.size();
+    if (H == 0) return 0;
+    uint32_t* hs = buf<uint32_t>(hot_slotb, kHotMax);
+    WJ_CUDA_CHECK(cudaMemcpyAsync(hs, hot_slots.data(), H * 4, cudaMemcpyHostToDevice, st));
+    ulonglong2* hk = (ulonglong2*)grow(hot_kb, kHotMax * sizeof(ulonglong2));
+    k_hot_extract<<<1, kHotMax, 0, st>>>((const Slot*)table.p, hs, H, hk);
+    launched();
+    sync();  // hot_slot_b is rewritten with main-table slots by k_hot_build
+    return H;
   }
 
   // L2 persisting access-policy window on the context stream (best effort; cleared with bytes == 0)
@@ -427,11 +507,21 @@ struct wj_index {
   // terms of the chunk into the u_* arrays.  Returns Nc; sets C (table capacity), U.
   template <class F>
   uint64_t tokenize_dedup(const ChunkView& cv, uint32_t doc_base, F&& out_alloc, uint64_t& C, uint64_t& U,
-                          uint32_t*& slot_out, uint32_t*& doc_out) {
+                          uint32_t*& slot_out, uint32_t*& doc_out, bool allow_hot = false) {
     const uint64_t n_segs = (cv.n_bytes + kSegBytes - 1) / kSegBytes;
     C = 0;
     U = 0;
     phase(WJ_PHASE_TOKENIZE);
+    hot_H = 0;
+    hot_D = 0;
+    if (allow_hot && cv.n_bytes >= hot_min_bytes && cv.n_docs > 0) {
+      const uint64_t cap = 64ull << 20;  // hot x documents counters
+      if (cv.n_docs <= cap / 16) {
+        hot_H = select_hot(cv);
+        hot_H = (uint32_t)std::min<uint64_t>(hot_H, cap / cv.n_docs);
+        hot_D = (uint32_t)cv.n_docs;
+      }
+    }
     const uint64_t Nc = count_tokens(cv, n_segs);
     n_dropped += h_scal[1];
     out_alloc(Nc, slot_out, doc_out);
@@ -443,7 +533,19 @@ struct wj_index {
     C = pow2_at_least(est + est / 2);
     uint32_t* slot_uid = nullptr;
     for (;;) {
-      emit_tokens(cv, n_segs, slot_out, doc_out, doc_base, C, nullptr, nullptr);
+      Slot* tab = buf<Slot>(table, C);
+      uint32_t* sref = buf<uint32_t>(slotref, C);
+      WJ_CUDA_CHECK(cudaMemsetAsync(tab, 0, C * sizeof(Slot), st));
+      if (hot_H) {  // hot terms first: their slots in this table, and the lookup table for the emit
+        WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 5, 0, 8, st));
+        HotEntry* ht = (HotEntry*)grow(hot_tab, kHotTable * sizeof(HotEntry));
+        k_hot_build<<<1, 1, 0, st>>>((const ulonglong2*)hot_kb.p, hot_H, tab, sref, (uint32_t)(C - 1), ht,
+                                     (uint32_t*)hot_slotb.p, (uint32_t*)(dscal() + 5));
+        launched();
+        uint32_t* tf = buf<uint32_t>(hot_tfb, (uint64_t)hot_H * hot_D);
+        WJ_CUDA_CHECK(cudaMemsetAsync(tf, 0, (uint64_t)hot_H * hot_D * 4, st));
+      }
+      emit_tokens(cv, n_segs, slot_out, doc_out, doc_base, C, nullptr, nullptr, hot_H > 0, false);
       phase(WJ_PHASE_UNIQUE);
       slot_uid = buf<uint32_t>(uid, C);
       scan<uint32_t>(NonZeroSlot{(const Slot*)table.p}, C, slot_uid, (uint32_t*)(dscal() + 2));
@@ -539,13 +641,32 @@ struct wj_index {
     uint64_t C = 0, U = 0;
     uint32_t *so = nullptr, *dout = nullptr;
     const uint64_t Nc = tokenize_dedup(cv, doc_base, [&](uint64_t nc, uint32_t*& sp, uint32_t*& dp) {
-      if (n_tokens + nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 tokens in one index"};
-      sp = buf_keep<uint32_t>(g_tid, n_tokens + nc + 16, n_tokens) + n_tokens;  // +16: TMA round-up reads
-      dp = buf_keep<uint32_t>(g_doc, n_tokens + nc + 16, n_tokens) + n_tokens;
-    }, C, U, so, dout);
+      if (n_elems + nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 stream elements"};
+      sp = buf_keep<uint32_t>(g_tid, n_elems + nc + 16, n_elems) + n_elems;  // +16: TMA round-up reads
+      dp = buf_keep<uint32_t>(g_doc, n_elems + nc + 16, n_elems) + n_elems;
+    }, C, U, so, dout, true);
     if (Nc > 0) {
+      uint64_t NH = 0;
+      if (hot_H) {  // hot (term, document) counters -> stream elements after the chunk's tokens
+        const uint64_t HD = (uint64_t)hot_H * hot_D;
+        uint32_t* ho = buf<uint32_t>(hot_offb, HD + 1);
+        scan<uint32_t>(HotElemCount{(const uint32_t*)hot_tfb.p}, HD, ho, ho + HD);
+        uint32_t nh = 0;
+        WJ_CUDA_CHECK(cudaMemcpyAsync(&nh, ho + HD, 4, cudaMemcpyDeviceToHost, st));
+        sync();
+        NH = nh;
+        const uint64_t base = n_elems + Nc;
+        if (base + NH > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 stream elements"};
+        uint32_t* gt = buf_keep<uint32_t>(g_tid, base + NH + 16, base);
+        uint32_t* gd = buf_keep<uint32_t>(g_doc, base + NH + 16, base);
+        k_hot_elems<<<grid_for(HD, 256), 256, 0, st>>>((const uint32_t*)hot_tfb.p, HD, hot_D, ho,
+                                                       (const uint32_t*)hot_slotb.p, doc_base, gt + base, gd + base);
+        launched();
+      }
       dictionary_update(text, U);
-      register_chunk_map(C, n_tokens);
+      register_chunk_map(C, n_elems);
+      if (hot_H) stream_has_hot = true;
+      n_elems += Nc + NH;
       n_tokens += Nc;
     }
     n_docs += nd;
@@ -677,19 +798,20 @@ struct wj_index {
       n_dropped = dropped0;
       if (Ns != rt_off[K]) throw StatusError{WJ_ERR_CUDA, "received term text: token count mismatch (internal)"};
       dictionary_update(recv_terms, U2);
-      if (n_tokens + R > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 tokens in one index"};
-      uint32_t* gt = buf_keep<uint32_t>(g_tid, n_tokens + R + 16, n_tokens);
-      uint32_t* gd = buf_keep<uint32_t>(g_doc, n_tokens + R + 16, n_tokens);
+      if (n_elems + R > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 stream elements"};
+      uint32_t* gt = buf_keep<uint32_t>(g_tid, n_elems + R + 16, n_elems);
+      uint32_t* gd = buf_keep<uint32_t>(g_doc, n_elems + R + 16, n_elems);
       uint64_t* ro = buf<uint64_t>(x_roff, K + 1);
       uint64_t* tb = buf<uint64_t>(x_tbase, K + 1);
       WJ_CUDA_CHECK(cudaMemcpyAsync(ro, rr_off.data(), (K + 1) * 8, cudaMemcpyHostToDevice, st));
       WJ_CUDA_CHECK(cudaMemcpyAsync(tb, rt_off.data(), (K + 1) * 8, cudaMemcpyHostToDevice, st));
       phase(WJ_PHASE_STREAM);
       if (R > 0) {
-        k_map_recv<<<grid_for(R, 256), 256, 0, st>>>(recv_rec, R, ro, tb, (uint32_t)K, sslot, gt + n_tokens, gd + n_tokens);
+        k_map_recv<<<grid_for(R, 256), 256, 0, st>>>(recv_rec, R, ro, tb, (uint32_t)K, sslot, gt + n_elems, gd + n_elems);
         launched();
       }
-      register_chunk_map(C2, n_tokens);
+      register_chunk_map(C2, n_elems);
+      n_elems += R;
       n_tokens += R;
     }
     n_docs += tot_docs;
@@ -807,56 +929,83 @@ struct wj_index {
     height_max = depth;
   }
 
-  // stable LSD radix sort driver (radix.cuh: per pass k_rs_up + scan + k_rs_down).  segs (optional):
-  // per stream segment a key map applied in place by the first upsweep (slot -> rank).
+  // stable LSD radix sort driver (radix.cuh: per pass k_rs_up + scan + k_rs_down2).  Digits come
+  // from key & kmask.  segs (optional): per stream segment a key map applied in place by the first
+  // upsweep (slot -> rank).  skip0: elements with no bits above kmask are holes, dropped by the first
+  // pass; *n_out = elements after the sort.
   template <typename K>
   bool sort_pairs(K* k0, uint32_t* v0, K* k1, uint32_t* v1, uint64_t n, int begin_bit, int end_bit,
                   const uint32_t* rank_of, bool timed,
-                  const std::vector<std::pair<uint64_t, const uint32_t*>>* segs = nullptr) {
+                  const std::vector<std::pair<uint64_t, const uint32_t*>>* segs = nullptr, K kmask = ~K(0),
+                  bool skip0 = false, uint64_t* n_out = nullptr) {
+    if (n_out) *n_out = n;
     if (n == 0) return false;
-    const int passes = end_bit > begin_bit ? (end_bit - begin_bit + 7) / 8 : 0;
-    // apply key maps (when there is nothing to sort the map is still applied)
-    auto map_only = [&](uint64_t off, uint64_t cnt, const uint32_t* map) {
-      k_map_rank<<<grid_for(cnt, 256), 256, 0, st>>>((uint32_t*)(k0 + off), cnt, map);
-      launched();
-    };
+    int passes = end_bit > begin_bit ? (end_bit - begin_bit + 7) / 8 : 0;
+    if (skip0 && passes == 0) passes = 1;  // the first pass also compacts the holes
     const bool multi_map = segs && segs->size() > 1;
-    if (segs && (passes == 0 || n == 1 || multi_map)) {
+    if (segs && multi_map) {  // apply each chunk's map first (holes and count bits preserved)
       for (size_t i = 0; i < segs->size(); ++i) {
         const uint64_t off = (*segs)[i].first;
         const uint64_t end = i + 1 < segs->size() ? (*segs)[i + 1].first : n;
         if (end > off) {
-          if (timed) ktime(WJ_KERNEL_SORT_HIST, [&] { map_only(off, end - off, (*segs)[i].second); });
-          else map_only(off, end - off, (*segs)[i].second);
+          auto m = [&] {
+            k_map_rank<<<grid_for(end - off, 256), 256, 0, st>>>((uint32_t*)(k0 + off), end - off, (*segs)[i].second);
+            launched();
+          };
+          if (timed) ktime(WJ_KERNEL_SORT_HIST, m); else m();
         }
       }
     }
-    if (passes == 0 || n == 1) return false;
+    if (passes == 0 || (n == 1 && !skip0)) {
+      if (segs && !multi_map) {
+        k_map_rank<<<grid_for(n, 256), 256, 0, st>>>((uint32_t*)k0, n, (*segs)[0].second);
+        launched();
+      }
+      return false;
+    }
     const uint32_t* first_map = (segs && !multi_map) ? (*segs)[0].second : rank_of;
-    uint64_t per = (n + kRsCtas - 1) / kRsCtas;
-    per = (per + kOsTile - 1) / kOsTile * kOsTile;
-    const uint32_t G = (uint32_t)((n + per - 1) / per);
-    uint32_t* h1 = buf<uint32_t>(hist, (uint64_t)256 * G);
-    uint32_t* h2 = buf<uint32_t>(hist_scan, (uint64_t)256 * G);
     bool in1 = false;
+    uint64_t cur_n = n;
     for (int p = 0; p < passes; ++p) {
+      uint64_t per = (cur_n + kRsCtas - 1) / kRsCtas;
+      per = (per + kOsTile - 1) / kOsTile * kOsTile;
+      const uint32_t G = (uint32_t)((cur_n + per - 1) / per);
+      uint32_t* h1 = buf<uint32_t>(hist, (uint64_t)256 * G);
+      uint32_t* h2 = buf<uint32_t>(hist_scan, (uint64_t)256 * G + 1);
       K* ki = in1 ? k1 : k0;
       uint32_t* vi = in1 ? v1 : v0;
       K* ko = in1 ? k0 : k1;
       uint32_t* vo = in1 ? v0 : v1;
       const int shift = begin_bit + 8 * p;
       const uint32_t* mp = p == 0 ? first_map : nullptr;
+      const bool holes = skip0 && p == 0;
+      // the count bits of stream elements only reach a digit when passes cover bits >= 25
+      const bool masked = kmask != ~K(0) && begin_bit + 8 * passes > kCountShift;
       auto up = [&] {
-        k_rs_up<K><<<G, 256, 0, st>>>(ki, n, per, shift, mp, h1);
+        if (holes && masked) k_rs_up<K, true, true><<<G, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
+        else if (holes) k_rs_up<K, true, false><<<G, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
+        else if (masked) k_rs_up<K, false, true><<<G, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
+        else k_rs_up<K, false, false><<<G, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
         launched();
       };
       if (timed) ktime(WJ_KERNEL_SORT_HIST, up); else up();
-      scan<uint32_t>(ArrayIn<uint32_t>{h1}, (uint64_t)256 * G, h2, (uint32_t*)nullptr);
+      scan<uint32_t>(ArrayIn<uint32_t>{h1}, (uint64_t)256 * G, h2, h2 + (uint64_t)256 * G);
       auto down = [&] {
-        k_rs_down2<K><<<G, kDsThreads, ds_smem_bytes<K>(), st>>>(ki, vi, ko, vo, n, per, shift, h2);
+        const size_t sm = ds_smem_bytes<K>();
+        if (holes && masked) k_rs_down2<K, true, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
+        else if (holes) k_rs_down2<K, true, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
+        else if (masked) k_rs_down2<K, false, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
+        else k_rs_down2<K, false, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
         launched();
       };
       if (timed) ktime(WJ_KERNEL_SORT_SCATTER, down); else down();
+      if (holes) {  // elements that survive the compaction
+        uint32_t tot = 0;
+        WJ_CUDA_CHECK(cudaMemcpyAsync(&tot, h2 + (uint64_t)256 * G, 4, cudaMemcpyDeviceToHost, st));
+        sync();
+        cur_n = tot;
+        if (n_out) *n_out = cur_n;
+      }
       in1 = !in1;
     }
     return in1;
@@ -864,9 +1013,11 @@ struct wj_index {
 
   // ---------------------------------------------------------------- finalize
   void finalize() {
-    const uint64_t N = n_tokens;
+    const uint64_t NE = n_elems;  // stream elements (tokens, aggregated hot entries, holes)
     uint32_t* ro = buf<uint32_t>(rank_of, V);
     uint32_t* ta = buf<uint32_t>(term_at, V);
+    if ((uint64_t)V > (uint64_t)kRankMask + 1)
+      throw StatusError{WJ_ERR_CAPACITY, "more than 2^25 terms in one dictionary slice"};
     if (V > 0) {
       phase(WJ_PHASE_LEXRANK);
       LexGroups* g = (LexGroups*)grow(lexg, sizeof(LexGroups));
@@ -882,17 +1033,18 @@ struct wj_index {
     uint64_t* po = buf<uint64_t>(post_off, (uint64_t)V + 1);
     uint32_t* dfp = buf<uint32_t>(df, V);
     uint64_t* cfp = buf<uint64_t>(cf, V);
+    uint64_t* csp = buf<uint64_t>(cstart_b, (uint64_t)V + 1);
     P = 0;
-    if (N > 0) {
+    if (NE > 0 && V > 0) {
       phase(WJ_PHASE_SORT);
       uint32_t* kt = (uint32_t*)g_tid.p;
       uint32_t* dt = (uint32_t*)g_doc.p;
-      uint32_t* k1 = buf<uint32_t>(sk1, N + 16);
-      uint32_t* v1 = buf<uint32_t>(sv1, N + 16);
+      uint32_t* k1 = buf<uint32_t>(sk1, NE + 16);
+      uint32_t* v1 = buf<uint32_t>(sv1, NE + 16);
       int bits = 0;
       while (bits < 32 && ((uint64_t)1 << bits) < V) ++bits;
       // per chunk: slot -> termID -> rank map; applied in the histogram pass; the stable sort by
-      // rank keeps docIDs ascending within every term
+      // rank keeps docIDs ascending within every term; the first pass drops the holes
       std::vector<std::pair<uint64_t, const uint32_t*>> segs;
       for (size_t c = 0; c < chunk_tok.size(); ++c) {
         uint32_t* m = (uint32_t*)chunk_map[c].p;
@@ -900,11 +1052,11 @@ struct wj_index {
         launched();
         segs.emplace_back(chunk_tok[c], m);
       }
-      const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, N, 0, bits, nullptr, true, &segs);
+      uint64_t N = NE;
+      const bool in1 =
+          sort_pairs<uint32_t>(kt, dt, k1, v1, NE, 0, bits, nullptr, true, &segs, kRankMask, stream_has_hot, &N);
       f_key = in1 ? k1 : kt;
       f_doc = in1 ? v1 : dt;
-      uint32_t* spare_k = in1 ? kt : k1;  // free N-sized buffers for pstart / tstart
-      uint32_t* spare_v = in1 ? dt : v1;
 
       phase(WJ_PHASE_POSTINGS);
       uint64_t per = (N + 148 * 2 - 1) / (148 * 2);
@@ -912,16 +1064,19 @@ struct wj_index {
       const uint32_t G = (uint32_t)((N + per - 1) / per);
       uint32_t* rc = buf<uint32_t>(rle_p0, (uint64_t)G + 1);
       uint32_t* rl = buf<uint32_t>(rle_lead, (uint64_t)G + 1);
+      uint64_t* rt = buf<uint64_t>(rle_tok, (uint64_t)G + 1);
       // P <= N: size the outputs by N, no host round trip before the pass
       uint32_t* od = buf<uint32_t>(out_doc, N);
       uint32_t* of = buf<uint32_t>(out_tf, N);
-      uint32_t* tstart_p = spare_v;  // N >= V entries
-      (void)spare_k;
       ktime(WJ_KERNEL_RLE_EMIT, [&] {
-        k_rle_count<<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc);
+        k_rle_count<<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc, rt);
         launched();
         scan<uint32_t>(ArrayIn<uint32_t>{rc}, G, rc, (uint32_t*)(dscal() + 8));
-        k_rle_write_tma<<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, od, of, po, tstart_p, rl);
+        scan<uint64_t>(ArrayIn<uint64_t>{rt}, G, rt, (uint64_t*)(dscal() + 11));
+        if (stream_has_hot)
+          k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl);
+        else
+          k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl);
         launched();
       });
       k_rle_fixup<<<grid_for(G, 256), 256, 0, st>>>(rc, rl, G, of);
@@ -929,7 +1084,7 @@ struct wj_index {
       WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 8) + 1, 0, 4, st));
       readback(8, 1);
       P = (uint32_t)h_scal[8];
-      k_df_cf<<<grid_for((uint64_t)V + 1, 256), 256, 0, st>>>(po, tstart_p, V, P, N, dfp, cfp);
+      k_df_cf<<<grid_for((uint64_t)V + 1, 256), 256, 0, st>>>(po, csp, V, P, n_tokens, dfp, cfp);
       launched();
     } else {
       WJ_CUDA_CHECK(cudaMemsetAsync(po, 0, 8, st));
@@ -1052,6 +1207,7 @@ int index_init(wj_index** out, const wj_config* cfg) {
       ix->own_stream = true;
     }
     WJ_CUDA_CHECK(cudaHostAlloc(&ix->h_scal, 16 * sizeof(uint64_t), cudaHostAllocDefault));
+    if (const char* e = getenv("WJ_HOT_MIN_BYTES")) ix->hot_min_bytes = strtoull(e, nullptr, 10);
     if (cfg->world > 1 || cfg->nccl_unique_id) {  // a transport at world 1 runs the same distributed path
       try {
         if (cfg->flags & WJ_FLAG_LOOPBACK)
@@ -1074,11 +1230,16 @@ int index_init(wj_index** out, const wj_config* cfg) {
                                        (int)os_tma_smem_bytes<uint64_t>()));
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rs_down<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)os_tma_smem_bytes<uint32_t>()));
-    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rs_down2<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)ds_smem_bytes<uint64_t>()));
-    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rs_down2<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)ds_smem_bytes<uint32_t>()));
-    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rle_write_tma, cudaFuncAttributeMaxDynamicSharedMemorySize,
+#define WJ_DS_ATTR(K, H, M)                                                                           \
+  WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rs_down2<K, H, M>, cudaFuncAttributeMaxDynamicSharedMemorySize, \
+                                     (int)ds_smem_bytes<K>()))
+    WJ_DS_ATTR(uint64_t, false, false); WJ_DS_ATTR(uint64_t, true, false); WJ_DS_ATTR(uint64_t, false, true);
+    WJ_DS_ATTR(uint64_t, true, true); WJ_DS_ATTR(uint32_t, false, false); WJ_DS_ATTR(uint32_t, true, false);
+    WJ_DS_ATTR(uint32_t, false, true); WJ_DS_ATTR(uint32_t, true, true);
+#undef WJ_DS_ATTR
+    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rle_write_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)rle_smem_bytes()));
+    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rle_write_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)rle_smem_bytes()));
     ix->reset_state();
     return WJ_OK;

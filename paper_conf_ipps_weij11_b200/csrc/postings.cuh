@@ -17,10 +17,13 @@
 
 namespace wj {
 
-// stream termID -> term rank (in place)
-__global__ void k_map_rank(uint32_t* tid, uint64_t N, const uint32_t* rank_of) {
+// stream element slot -> term rank (in place; the count bits above bit 25 are kept, holes skipped)
+__global__ void k_map_rank(uint32_t* key, uint64_t N, const uint32_t* rank_of) {
   const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i < N) tid[i] = __ldg(&rank_of[tid[i]]);
+  if (i >= N) return;
+  const uint32_t k = key[i];
+  if ((k >> 25) == 0) return;
+  key[i] = __ldg(&rank_of[k & ((1u << 25) - 1u)]) | (k & ~((1u << 25) - 1u));
 }
 
 // per chunk: table slot -> termID map (the chunk's token stream keeps slot ids; finalize composes
@@ -38,10 +41,6 @@ __global__ void k_map_compose(uint32_t* map, uint32_t C, const uint32_t* rank_of
   if (i < C) map[i] = __ldg(&rank_of[map[i]]);
 }
 
-// Fused run-length pass (one read of the sorted (rank, doc) stream): a tile of 4096 tokens flags the
-// first token of every posting (new rank or new doc) and of every term, numbers the postings with a
-// block scan + decoupled look-back over tiles, and writes docid, tf, post_off[rank], tstart[rank].
-// tf of a run that continues past the tile's end is completed by k_rle_fixup (tile_lead).
 constexpr int kRleThreads = 256;
 constexpr int kRleItems = 16;
 constexpr int kRleTile = kRleThreads * kRleItems;
@@ -67,126 +66,17 @@ __device__ __forceinline__ uint32_t block_min_after(uint32_t v, uint32_t* sm /* 
   return min(after_in_warp, later_warps);
 }
 
-__global__ void __launch_bounds__(kRleThreads) k_rle_fused(const uint32_t* __restrict__ key, const uint32_t* __restrict__ doc,
-                                                           uint64_t N, uint32_t* out_doc, uint32_t* out_tf,
-                                                           uint64_t* post_off, uint32_t* tstart, uint64_t* look,
-                                                           uint32_t* tile_ctr, uint32_t* tile_p0, uint32_t* tile_lead,
-                                                           uint32_t* total_p) {
-  __shared__ uint32_t s_tile, s_p0;
-  __shared__ uint32_t sm[16];
-  __shared__ uint32_t st_doc[kRleTile], st_tf[kRleTile];  // tile postings, written out coalesced
-  if (threadIdx.x == 0) s_tile = atomicAdd(tile_ctr, 1u);
-  __syncthreads();
-  const uint32_t tile = s_tile;
-  const uint64_t base = (uint64_t)tile * kRleTile;
-  const uint64_t i0 = base + (uint64_t)threadIdx.x * kRleItems;
-  const uint32_t tile_len = (uint32_t)min((uint64_t)kRleTile, N - base);
-  uint32_t k[kRleItems], d[kRleItems];
-  if (i0 + kRleItems <= N) {
-#pragma unroll
-    for (int q = 0; q < kRleItems / 4; ++q) {
-      const uint4 a = __ldcs((const uint4*)(key + i0) + q);
-      const uint4 b = __ldcs((const uint4*)(doc + i0) + q);
-      k[4 * q] = a.x; k[4 * q + 1] = a.y; k[4 * q + 2] = a.z; k[4 * q + 3] = a.w;
-      d[4 * q] = b.x; d[4 * q + 1] = b.y; d[4 * q + 2] = b.z; d[4 * q + 3] = b.w;
-    }
-  } else {
-#pragma unroll
-    for (int j = 0; j < kRleItems; ++j) {
-      const bool v = i0 + j < N;
-      k[j] = v ? key[i0 + j] : 0xFFFFFFFFu;
-      d[j] = v ? doc[i0 + j] : 0xFFFFFFFFu;
-    }
-  }
-  uint32_t pk = 0xFFFFFFFFu, pd = 0xFFFFFFFFu;
-  if (i0 > 0 && i0 <= N) { pk = key[i0 - 1]; pd = doc[i0 - 1]; }
-  uint32_t npm = 0, ntm = 0;
-#pragma unroll
-  for (int j = 0; j < kRleItems; ++j) {
-    const bool valid = i0 + j < N;
-    const bool nt = valid && (i0 + j == 0 || k[j] != pk);
-    const bool np = valid && (nt || d[j] != pd);
-    npm |= (np ? 1u : 0u) << j;
-    ntm |= (nt ? 1u : 0u) << j;
-    pk = k[j];
-    pd = d[j];
-  }
-  const uint32_t c = __popc(npm);
-  uint32_t tot;
-  const uint32_t ex = block_exclusive_sum<uint32_t>(c, tot);
-  // first posting start of this thread (tile-relative) and the next one after this thread
-  const uint32_t my_first = npm ? threadIdx.x * kRleItems + __ffs(npm) - 1 : 0xFFFFFFFFu;
-  const uint32_t next_after = block_min_after(my_first, sm);
-  // tile prefix of postings: decoupled look-back by warp 0, 32 predecessor tiles per step
-  if (threadIdx.x < 32) {
-    volatile uint64_t* lk = (volatile uint64_t*)look;
-    const uint32_t lane = lane_id();
-    if (lane == 0) lk[tile] = (tile == 0 ? kLbPre : kLbAgg) | tot;
-    uint64_t prefix = 0;
-    int64_t hiT = (int64_t)tile - 1;  // next predecessor to examine (window top)
-    while (hiT >= 0) {
-      const int64_t t = hiT - lane;
-      uint64_t v = kLbPre;  // before tile 0: inclusive prefix 0
-      if (t >= 0) v = lk[t];
-      // wait until every lane of the window (up to the nearest inclusive prefix) is published
-      for (;;) {
-        const uint32_t notready = __ballot_sync(0xffffffffu, (v & (kLbAgg | kLbPre)) == 0);
-        const uint32_t pre = __ballot_sync(0xffffffffu, (v & kLbPre) != 0);
-        const uint32_t need = pre ? ((2u << (__ffs(pre) - 1)) - 1u) : 0xffffffffu;  // lanes up to nearest PRE
-        if ((notready & need) == 0) break;
-        if ((notready >> lane) & 1u) v = lk[t];
-      }
-      const uint32_t pre = __ballot_sync(0xffffffffu, (v & kLbPre) != 0);
-      const int last = pre ? __ffs(pre) - 1 : 31;
-      uint64_t x = lane <= (uint32_t)last ? (v & kLbVal) : 0;
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
-      prefix += x;
-      if (pre) break;
-      hiT -= 32;
-    }
-    if (lane == 0) {
-      if (tile > 0) lk[tile] = kLbPre | (prefix + tot);
-      s_p0 = (uint32_t)prefix;
-      tile_p0[tile] = (uint32_t)prefix;
-      if (base + tile_len >= N) *total_p = (uint32_t)(prefix + tot);
-    }
-  }
-  // leading continuation of the tile: items before the first posting start
-  uint32_t first_all = min(my_first, next_after);
-  if (threadIdx.x == 0) tile_lead[tile] = first_all == 0xFFFFFFFFu ? tile_len : first_all;
-  __syncthreads();
-  const uint32_t p0 = s_p0;
-  uint32_t lp = ex;  // tile-local posting index
-#pragma unroll
-  for (int j = 0; j < kRleItems; ++j) {
-    if ((npm >> j) & 1u) {
-      const uint32_t rest = npm & ~((2u << j) - 1u);
-      const uint32_t pos = threadIdx.x * kRleItems + j;
-      const uint32_t end = rest ? threadIdx.x * kRleItems + __ffs(rest) - 1 : min(next_after, tile_len);
-      st_doc[lp] = d[j];
-      st_tf[lp] = end - pos;
-      if ((ntm >> j) & 1u) {
-        post_off[k[j]] = p0 + lp;
-        tstart[k[j]] = (uint32_t)(i0 + j);
-      }
-      ++lp;
-    }
-  }
-  __syncthreads();
-  for (uint32_t x = threadIdx.x; x < tot; x += kRleThreads) {
-    __stcs(out_doc + p0 + x, st_doc[x]);
-    __stcs(out_tf + p0 + x, st_tf[x]);
-  }
-}
-
 // ------------------------------------------------------------------ run-length, reduce-then-scan
-// CTA c owns the contiguous token range [c*per, min(N,(c+1)*per)).  k_rle_count counts posting
-// starts per range (one streaming read); a scan gives each range's first posting index; k_rle_write
-// walks its range tile by tile with a running posting offset, carries the open run across its tiles,
-// and writes docid/tf (coalesced through shared memory), post_off[rank], tstart[rank].  Runs that
-// continue across ranges are completed by k_rle_fixup (range_lead).
-constexpr int kRle2Ctas = 148 * 4;
+// Stream elements after the sort: key = rank | count << 25 (count >= 1 tokens of that term in that
+// document: 1 for a plain token, the per-document count for an aggregated hot-term element), value =
+// docID.  CTA c owns the contiguous element range [c*per, min(N,(c+1)*per)).  k_rle_count counts
+// posting starts and tokens per range; scans give each range's first posting index and token offset;
+// k_rle_write_tma walks its range tile by tile (TMA-prefetched 2-stage ring), carries the open run
+// across tiles and writes docid, tf = sum of counts (coalesced through shared memory), post_off[rank]
+// and the token offset cstart[rank] of the term's first element (cf = difference).  Runs that continue
+// across ranges are completed by k_rle_fixup (range_lead = tokens before the range's first posting).
+constexpr uint32_t kCountShift = 25;
+constexpr uint32_t kRankMask = (1u << kCountShift) - 1u;
 
 __device__ __forceinline__ void rle_load16(const uint32_t* key, const uint32_t* doc, uint64_t i0, uint64_t hi,
                                            uint32_t* k, uint32_t* d, uint32_t& pk, uint32_t& pd) {
@@ -202,7 +92,7 @@ __device__ __forceinline__ void rle_load16(const uint32_t* key, const uint32_t* 
 #pragma unroll
     for (int j = 0; j < kRleItems; ++j) {
       const bool v = i0 + j < hi;
-      k[j] = v ? key[i0 + j] : 0xFFFFFFFFu;
+      k[j] = v ? key[i0 + j] : 0u;
       d[j] = v ? doc[i0 + j] : 0xFFFFFFFFu;
     }
   }
@@ -211,124 +101,64 @@ __device__ __forceinline__ void rle_load16(const uint32_t* key, const uint32_t* 
   if (i0 > 0) { pk = key[i0 - 1]; pd = doc[i0 - 1]; }
 }
 
+// posting starts (npm: new rank or new doc) and term starts (ntm: new rank)
 __device__ __forceinline__ void rle_flags(const uint32_t* k, const uint32_t* d, uint32_t pk, uint32_t pd, uint64_t i0,
                                           uint64_t hi, uint32_t& npm, uint32_t& ntm) {
   npm = 0;
   ntm = 0;
+  uint32_t pr = pk & kRankMask;
 #pragma unroll
   for (int j = 0; j < kRleItems; ++j) {
     const bool valid = i0 + j < hi;
-    const bool nt = valid && (i0 + j == 0 || k[j] != pk);
+    const uint32_t r = k[j] & kRankMask;
+    const bool nt = valid && (i0 + j == 0 || r != pr);
     const bool np = valid && (nt || d[j] != pd);
     npm |= (np ? 1u : 0u) << j;
     ntm |= (nt ? 1u : 0u) << j;
-    pk = k[j];
+    pr = r;
     pd = d[j];
   }
 }
 
 __global__ void __launch_bounds__(kRleThreads) k_rle_count(const uint32_t* __restrict__ key, const uint32_t* __restrict__ doc,
-                                                           uint64_t N, uint64_t per, uint32_t* range_cnt) {
+                                                           uint64_t N, uint64_t per, uint32_t* range_cnt,
+                                                           uint64_t* range_tok) {
   const uint64_t lo = (uint64_t)blockIdx.x * per;
   const uint64_t hi = lo + per < N ? lo + per : N;
   uint32_t c = 0;
+  uint64_t tk = 0;
   for (uint64_t i0 = lo + (uint64_t)threadIdx.x * kRleItems; i0 < hi; i0 += (uint64_t)kRleTile) {
     uint32_t k[kRleItems], d[kRleItems], pk, pd, npm, ntm;
     rle_load16(key, doc, i0, hi, k, d, pk, pd);
     rle_flags(k, d, pk, pd, i0, hi, npm, ntm);
     c += __popc(npm);
+#pragma unroll
+    for (int j = 0; j < kRleItems; ++j) tk += k[j] >> kCountShift;  // invalid items have key 0
   }
   uint32_t tot;
   block_exclusive_sum<uint32_t>(c, tot);
-  if (threadIdx.x == 0) range_cnt[blockIdx.x] = tot;
-}
-
-__global__ void __launch_bounds__(kRleThreads) k_rle_write(const uint32_t* __restrict__ key, const uint32_t* __restrict__ doc,
-                                                           uint64_t N, uint64_t per, const uint32_t* __restrict__ range_off,
-                                                           uint32_t* out_doc, uint32_t* out_tf, uint64_t* post_off,
-                                                           uint32_t* tstart, uint32_t* range_lead) {
-  __shared__ uint32_t sm[16];
-  __shared__ uint32_t st_doc[kRleTile], st_tf[kRleTile];
-  __shared__ uint32_t s_open_len, s_lead;
-  __shared__ int s_lead_done;
-  const uint64_t lo = (uint64_t)blockIdx.x * per;
-  const uint64_t hi = lo + per < N ? lo + per : N;
-  uint32_t p0 = range_off[blockIdx.x];
-  // open run carried from the previous tile: its posting is p0 - 1 (tile-local index tot-1 written
-  // as a partial tf into st_tf / global); s_open_len = tokens of it seen so far
-  if (threadIdx.x == 0) { s_open_len = 0; s_lead = 0; s_lead_done = 0; }
-  bool have_open = false;  // uniform
-  uint32_t open_p = 0;
-  __syncthreads();
-  for (uint64_t base = lo; base < hi; base += kRleTile) {
-    const uint32_t tile_len = (uint32_t)min((uint64_t)kRleTile, hi - base);
-    const uint64_t i0 = base + (uint64_t)threadIdx.x * kRleItems;
-    uint32_t k[kRleItems], d[kRleItems], pk, pd, npm, ntm;
-    rle_load16(key, doc, i0, hi, k, d, pk, pd);
-    rle_flags(k, d, pk, pd, i0, hi, npm, ntm);
-    const uint32_t c = __popc(npm);
-    uint32_t tot;
-    const uint32_t ex = block_exclusive_sum<uint32_t>(c, tot);
-    const uint32_t my_first = npm ? threadIdx.x * kRleItems + __ffs(npm) - 1 : 0xFFFFFFFFu;
-    const uint32_t next_after = block_min_after(my_first, sm);
-    const uint32_t first_all = min(my_first, next_after);  // valid in thread 0
-    if (threadIdx.x == 0) {
-      const uint32_t lead = first_all == 0xFFFFFFFFu ? tile_len : first_all;
-      if (!s_lead_done) {  // items of the range before its first posting start
-        s_lead += lead;
-        if (first_all != 0xFFFFFFFFu) s_lead_done = 1;
-      }
-      if (have_open) {
-        s_open_len += lead;
-        if (first_all != 0xFFFFFFFFu) out_tf[open_p] = s_open_len;  // the carried run ends here
-      }
-    }
-    uint32_t lp = ex;
-#pragma unroll
-    for (int j = 0; j < kRleItems; ++j) {
-      if ((npm >> j) & 1u) {
-        const uint32_t rest = npm & ~((2u << j) - 1u);
-        const uint32_t pos = threadIdx.x * kRleItems + j;
-        const uint32_t end = rest ? threadIdx.x * kRleItems + __ffs(rest) - 1 : min(next_after, tile_len);
-        st_doc[lp] = d[j];
-        st_tf[lp] = end - pos;
-        if ((ntm >> j) & 1u) {
-          post_off[k[j]] = p0 + lp;
-          tstart[k[j]] = (uint32_t)(i0 + j);
-        }
-        ++lp;
-      }
-    }
-    __syncthreads();
-    for (uint32_t x = threadIdx.x; x < tot; x += kRleThreads) {
-      __stcs(out_doc + p0 + x, st_doc[x]);
-      __stcs(out_tf + p0 + x, st_tf[x]);
-    }
-    if (tot) {
-      // the tile's last run may continue into the next tile
-      have_open = true;
-      open_p = p0 + tot - 1;
-      if (threadIdx.x == 0) s_open_len = st_tf[tot - 1];
-    } else if (threadIdx.x == 0 && have_open) {
-      // whole tile continues the open run (already added as lead)
-    }
-    p0 += tot;
-    __syncthreads();
-  }
+  uint64_t ttot;
+  block_exclusive_sum<uint64_t>(tk, ttot);
   if (threadIdx.x == 0) {
-    if (have_open) out_tf[open_p] = s_open_len;
-    range_lead[blockIdx.x] = s_lead_done ? s_lead : (uint32_t)(hi - lo);
+    range_cnt[blockIdx.x] = tot;
+    range_tok[blockIdx.x] = ttot;
   }
 }
 
-// k_rle_write with the next tile's keys/docs prefetched by TMA into a 2-stage shared-memory ring
-inline size_t rle_smem_bytes() { return (size_t)4 * kRleTile * 4 /*2 stages x (key, doc)*/ + 2 * kRleTile * 4; }
+inline size_t rle_smem_bytes() {
+  return (size_t)4 * kRleTile * 4 /*2 stages x (key, doc)*/ + 2 * kRleTile * 4 /*staged docid, tf*/ +
+         (kRleTile + 4) * 4 /*item token-count prefix*/;
+}
 
+// COUNTS = false: every element is one token (no hot-term elements in the stream), so token prefixes
+// are element positions and the second block scan and the prefix array are skipped.
+template <bool COUNTS>
 __global__ void __launch_bounds__(kRleThreads, 2) k_rle_write_tma(const uint32_t* __restrict__ key,
                                                                const uint32_t* __restrict__ doc, uint64_t N,
                                                                uint64_t per, const uint32_t* __restrict__ range_off,
+                                                               const uint64_t* __restrict__ range_tok_off,
                                                                uint32_t* out_doc, uint32_t* out_tf, uint64_t* post_off,
-                                                               uint32_t* tstart, uint32_t* range_lead) {
+                                                               uint64_t* cstart, uint32_t* range_lead) {
   extern __shared__ __align__(128) uint32_t rsm[];
   __shared__ __align__(8) uint64_t bar[2];
   __shared__ uint32_t sm[16];
@@ -338,6 +168,7 @@ __global__ void __launch_bounds__(kRleThreads, 2) k_rle_write_tma(const uint32_t
   auto sdoc = [&](int s) { return rsm + (size_t)s * 2 * kRleTile + kRleTile; };
   uint32_t* st_doc = rsm + 4 * kRleTile;
   uint32_t* st_tf = rsm + 5 * kRleTile;
+  uint32_t* cpi = rsm + 6 * kRleTile;  // exclusive token-count prefix of each tile item (+ total)
   const uint64_t lo = (uint64_t)blockIdx.x * per;
   const uint64_t hi = lo + per < N ? lo + per : N;
   if (lo >= hi) return;
@@ -362,6 +193,7 @@ __global__ void __launch_bounds__(kRleThreads, 2) k_rle_write_tma(const uint32_t
   __syncthreads();
   if (threadIdx.x == 0) issue(0, lo);
   uint32_t p0 = range_off[blockIdx.x];
+  uint64_t tokbase = range_tok_off[blockIdx.x];
   bool have_open = false;
   uint32_t open_p = 0;
   uint32_t parity = 0;
@@ -382,18 +214,33 @@ __global__ void __launch_bounds__(kRleThreads, 2) k_rle_write_tma(const uint32_t
       k[4 * q] = a.x; k[4 * q + 1] = a.y; k[4 * q + 2] = a.z; k[4 * q + 3] = a.w;
       d[4 * q] = b.x; d[4 * q + 1] = b.y; d[4 * q + 2] = b.z; d[4 * q + 3] = b.w;
     }
+#pragma unroll
+    for (int j = 0; j < kRleItems; ++j)
+      if (t0 + j >= tile_len) k[j] = 0u;  // past the range: no tokens
     const uint32_t pk = t0 ? ks[t0 - 1] : s_prev_k;
     const uint32_t pd = t0 ? ds[t0 - 1] : s_prev_d;
     uint32_t npm, ntm;
     rle_flags(k, d, pk, pd, base + t0, base + tile_len, npm, ntm);
     const uint32_t c = __popc(npm);
-    uint32_t tot;
+    uint32_t tot, ctot = tile_len;
     const uint32_t ex = block_exclusive_sum<uint32_t>(c, tot);
+    if (COUNTS) {
+      uint32_t ps = 0;
+#pragma unroll
+      for (int j = 0; j < kRleItems; ++j) ps += k[j] >> kCountShift;
+      uint32_t run = block_exclusive_sum<uint32_t>(ps, ctot);
+#pragma unroll
+      for (int j = 0; j < kRleItems; ++j) {
+        cpi[t0 + j] = run;
+        run += k[j] >> kCountShift;
+      }
+    }
+    auto cp = [&](uint32_t i) -> uint32_t { return COUNTS ? cpi[i] : i; };
     const uint32_t my_first = npm ? t0 + __ffs(npm) - 1 : 0xFFFFFFFFu;
-    const uint32_t next_after = block_min_after(my_first, sm);
+    const uint32_t next_after = block_min_after(my_first, sm);  // contains __syncthreads: cpi visible
     if (threadIdx.x == 0) {
       const uint32_t first_all = min(my_first, next_after);
-      const uint32_t lead = first_all == 0xFFFFFFFFu ? tile_len : first_all;
+      const uint32_t lead = first_all == 0xFFFFFFFFu ? ctot : cp(first_all);
       if (!s_lead_done) {
         s_lead += lead;
         if (first_all != 0xFFFFFFFFu) s_lead_done = 1;
@@ -411,10 +258,11 @@ __global__ void __launch_bounds__(kRleThreads, 2) k_rle_write_tma(const uint32_t
         const uint32_t pos = t0 + j;
         const uint32_t end = rest ? t0 + __ffs(rest) - 1 : min(next_after, tile_len);
         st_doc[lp] = d[j];
-        st_tf[lp] = end - pos;
+        st_tf[lp] = (end < tile_len ? cp(end) : ctot) - cp(pos);
         if ((ntm >> j) & 1u) {
-          post_off[k[j]] = p0 + lp;
-          tstart[k[j]] = (uint32_t)(base + pos);
+          const uint32_t r = k[j] & kRankMask;
+          post_off[r] = p0 + lp;
+          cstart[r] = tokbase + cp(pos);
         }
         ++lp;
       }
@@ -434,12 +282,13 @@ __global__ void __launch_bounds__(kRleThreads, 2) k_rle_write_tma(const uint32_t
       open_p = p0 + tot - 1;
     }
     p0 += tot;
+    tokbase += ctot;
     __syncthreads();
     s ^= 1;
   }
   if (threadIdx.x == 0) {
     if (have_open) out_tf[open_p] = s_open_len;
-    range_lead[blockIdx.x] = s_lead_done ? s_lead : (uint32_t)(hi - lo);
+    range_lead[blockIdx.x] = s_lead;
   }
 }
 
@@ -451,7 +300,7 @@ __global__ void k_rle_fixup(const uint32_t* tile_p0, const uint32_t* tile_lead, 
   if (lead) atomicAdd(&out_tf[tile_p0[t] - 1], lead);
 }
 
-__global__ void k_df_cf(uint64_t* post_off, const uint32_t* tstart, uint32_t V, uint64_t P, uint64_t N, uint32_t* df,
+__global__ void k_df_cf(uint64_t* post_off, const uint64_t* cstart, uint32_t V, uint64_t P, uint64_t NT, uint32_t* df,
                         uint64_t* cf) {
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r > V) return;
@@ -460,8 +309,8 @@ __global__ void k_df_cf(uint64_t* post_off, const uint32_t* tstart, uint32_t V, 
   const uint64_t a = post_off[r];
   const uint64_t b = (r + 1 < V) ? post_off[r + 1] : P;
   df[r] = (uint32_t)(b - a);
-  const uint64_t ta = tstart[r];
-  const uint64_t tb = (r + 1 < V) ? (uint64_t)tstart[r + 1] : N;
+  const uint64_t ta = cstart[r];
+  const uint64_t tb = (r + 1 < V) ? cstart[r + 1] : NT;
   cf[r] = tb - ta;
 }
 

@@ -415,9 +415,19 @@ __global__ void __launch_bounds__(kOsThreads, 2) k_os_pass_tma(const K* __restri
 // cp.async.bulk while the current tile is ranked, staged in digit order and written out.
 constexpr int kRsCtas = 148 * 2;
 
-template <typename K>
+// Digits come from (key & kmask) (the count bits of a stream element ride along unsorted); with skip0
+// the elements whose bits above kmask are 0 are holes (not counted, dropped by the downsweep).  A map
+// (slot -> rank) is applied in place to the masked part: key = map[key & kmask] | (key & ~kmask).
+// HOLES / MASK are compile-time so the common path (no holes, digits below the count bits) is the
+// plain branch-free kernel.
+template <typename K, bool HOLES>
+__device__ __forceinline__ bool rs_hole(K k, K kmask) { return HOLES && (k & ~kmask) == 0; }
+template <typename K, bool MASK>
+__device__ __forceinline__ K rs_dkey(K k, K kmask) { return MASK ? (k & kmask) : k; }
+
+template <typename K, bool HOLES, bool MASK>
 __global__ void __launch_bounds__(256) k_rs_up(K* keys, uint64_t n, uint64_t per, int shift,
-                                               const uint32_t* __restrict__ map, uint32_t* hist) {
+                                               const uint32_t* __restrict__ map, uint32_t* hist, K kmask) {
   __shared__ uint32_t h[kOsWarps][256];
   const int w = threadIdx.x >> 5;
   for (int x = 0; x < kOsWarps; ++x) h[x][threadIdx.x] = 0;
@@ -439,8 +449,9 @@ __global__ void __launch_bounds__(256) k_rs_up(K* keys, uint64_t n, uint64_t per
       K* kk = (K*)&x[u];
 #pragma unroll
       for (int j = 0; j < V; ++j) {
-        if (map) kk[j] = (K)__ldg(&map[(uint32_t)kk[j]]);
-        atomicAdd(&h[w][(uint32_t)(kk[j] >> shift) & 255u], 1u);
+        const bool hole = rs_hole<K, HOLES>(kk[j], kmask);
+        if (map && !hole) kk[j] = (K)__ldg(&map[(uint32_t)(kk[j] & kmask)]) | (kk[j] & ~kmask);
+        if (!hole) atomicAdd(&h[w][(uint32_t)(rs_dkey<K, MASK>(kk[j], kmask) >> shift) & 255u], 1u);
       }
       if (map) vp[v0 + u * 256] = x[u];
     }
@@ -450,18 +461,20 @@ __global__ void __launch_bounds__(256) k_rs_up(K* keys, uint64_t n, uint64_t per
     K* kk = (K*)&x;
 #pragma unroll
     for (int j = 0; j < V; ++j) {
-      if (map) kk[j] = (K)__ldg(&map[(uint32_t)kk[j]]);
-      atomicAdd(&h[w][(uint32_t)(kk[j] >> shift) & 255u], 1u);
+      const bool hole = rs_hole<K, HOLES>(kk[j], kmask);
+      if (map && !hole) kk[j] = (K)__ldg(&map[(uint32_t)(kk[j] & kmask)]) | (kk[j] & ~kmask);
+      if (!hole) atomicAdd(&h[w][(uint32_t)(rs_dkey<K, MASK>(kk[j], kmask) >> shift) & 255u], 1u);
     }
     if (map) vp[v] = x;
   }
   for (uint64_t i = lo + nvec * V + threadIdx.x; i < hi; i += 256) {
     K k = keys[i];
+    if (rs_hole<K, HOLES>(k, kmask)) continue;
     if (map) {
-      k = (K)__ldg(&map[(uint32_t)k]);
+      k = (K)__ldg(&map[(uint32_t)(k & kmask)]) | (k & ~kmask);
       keys[i] = k;
     }
-    atomicAdd(&h[w][(uint32_t)(k >> shift) & 255u], 1u);
+    atomicAdd(&h[w][(uint32_t)(rs_dkey<K, MASK>(k, kmask) >> shift) & 255u], 1u);
   }
   __syncthreads();
   uint32_t t = 0;
@@ -599,10 +612,11 @@ static_assert(kDsThreads * kDsItems == kOsTile, "tile");
 template <typename K>
 inline size_t ds_smem_bytes() { return 2 * (size_t)kOsTile * (sizeof(K) + sizeof(uint32_t)) + kOsTile * 2; }
 
-template <typename K>
+template <typename K, bool HOLES, bool MASK>
 __global__ void __launch_bounds__(kDsThreads, 2) k_rs_down2(const K* __restrict__ kin, const uint32_t* __restrict__ vin,
                                                          K* __restrict__ kout, uint32_t* __restrict__ vout, uint64_t n,
-                                                         uint64_t per, int shift, const uint32_t* __restrict__ offs) {
+                                                         uint64_t per, int shift, const uint32_t* __restrict__ offs,
+                                                         K kmask) {
   extern __shared__ __align__(128) unsigned char os_smem[];
   __shared__ __align__(8) uint64_t bar[2];
   __shared__ uint32_t wcnt[kDsWarps][256];
@@ -610,6 +624,7 @@ __global__ void __launch_bounds__(kDsThreads, 2) k_rs_down2(const K* __restrict_
   __shared__ uint32_t dig_glob[256];
   __shared__ uint32_t run_base[256];
   __shared__ uint32_t wtot[8];
+  __shared__ uint32_t s_tvalid;
   const size_t stage_bytes = (size_t)kOsTile * (sizeof(K) + sizeof(uint32_t));
   auto skey = [&](int s) { return (K*)(os_smem + s * stage_bytes); };
   auto sval = [&](int s) { return (uint32_t*)(os_smem + s * stage_bytes + (size_t)kOsTile * sizeof(K)); };
@@ -650,16 +665,19 @@ __global__ void __launch_bounds__(kDsThreads, 2) k_rs_down2(const K* __restrict_
     const K* sk = skey(s);
     const uint32_t* sv = sval(s);
     uint32_t dg[kDsItems], rank[kDsItems];
+    uint32_t vmask = 0;  // valid items of this thread (in range, not a hole)
 #pragma unroll
     for (int k = 0; k < kDsItems; ++k) {
       const uint32_t li = w * (32 * kDsItems) + k * 32 + lane;
-      dg[k] = (uint32_t)((sk[li] >> shift) & 255u);
-      rank[k] = digit_peers(dg[k], li < tn);
+      const K kv = sk[li];
+      const bool valid = li < tn && !rs_hole<K, HOLES>(kv, kmask);
+      vmask |= (valid ? 1u : 0u) << k;
+      dg[k] = (uint32_t)((rs_dkey<K, MASK>(kv, kmask) >> shift) & 255u);
+      rank[k] = digit_peers(dg[k], valid);
     }
 #pragma unroll
     for (int k = 0; k < kDsItems; ++k) {
-      const uint32_t li = w * (32 * kDsItems) + k * 32 + lane;
-      const bool valid = li < tn;
+      const bool valid = (vmask >> k) & 1u;
       const uint32_t peers = rank[k];
       const int leader = valid ? __ffs(peers) - 1 : (int)lane;
       uint32_t old = 0;
@@ -695,18 +713,20 @@ __global__ void __launch_bounds__(kDsThreads, 2) k_rs_down2(const K* __restrict_
       const uint32_t rb = run_base[d];
       dig_glob[d] = rb - toff;
       run_base[d] = rb + cnt;
+      if (d == 255) s_tvalid = toff + cnt;
     }
     __syncthreads();
 #pragma unroll
     for (int k = 0; k < kDsItems; ++k) {
       const uint32_t li = w * (32 * kDsItems) + k * 32 + lane;
-      if (li < tn) inv[dig_off[dg[k]] + wcnt[w][dg[k]] + rank[k]] = (uint16_t)li;
+      if ((vmask >> k) & 1u) inv[dig_off[dg[k]] + wcnt[w][dg[k]] + rank[k]] = (uint16_t)li;
     }
     __syncthreads();
-    for (uint32_t j = threadIdx.x; j < tn; j += kDsThreads) {
+    const uint32_t tvalid = HOLES ? s_tvalid : tn;  // valid (non-hole) items of the tile
+    for (uint32_t j = threadIdx.x; j < tvalid; j += kDsThreads) {
       const uint32_t li = inv[j];
       const K kk = sk[li];
-      const uint32_t pos = dig_glob[(uint32_t)((kk >> shift) & 255u)] + j;
+      const uint32_t pos = dig_glob[(uint32_t)((rs_dkey<K, MASK>(kk, kmask) >> shift) & 255u)] + j;
       kout[pos] = kk;
       vout[pos] = sv[li];
     }

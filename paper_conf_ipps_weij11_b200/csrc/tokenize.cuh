@@ -38,7 +38,18 @@ struct ChunkView {
   uint64_t n_docs;
 };
 
+// hot lookup entry (hot.cuh): a sampled popular term of <= 11 bytes, identified by its slot words
+struct __align__(16) HotEntry {
+  unsigned long long k0, k1;
+  uint32_t id, slot;
+  uint32_t pad[2];
+};
+
 struct EmitOut {
+  const HotEntry* hot;     // hot lookup table (nullptr: no hot terms)
+  uint32_t hot_mask;       // lookup table size - 1
+  uint32_t hot_docs;       // documents of the chunk (columns of hot_tf)
+  uint32_t* hot_tf;        // hot term x document token counts
   Slot* table;             // chunk hash table
   uint32_t* slot_ref;      // per slot: first-occurrence offset (written by the inserter)
   uint32_t mask;           // capacity - 1 (power of two)
@@ -359,11 +370,29 @@ __global__ void __launch_bounds__(kTokThreads) k_tok_emit(ChunkView cv, uint32_t
         const uint32_t doc = eo.doc_base + (uint32_t)(lo - 1);
         const uint64_t k0 = (uint64_t)len | (((h >> 40) & 0xFFFFFFull) << 8) | ((uint64_t)wd[0] << 32);
         const uint64_t k1 = (uint64_t)wd[1] | ((uint64_t)(wd[2] & 0xFFFFFFu) << 32) | (1ull << 56);
-        const uint32_t slot =
-            table_insert(cv.text, eo.table, eo.slot_ref, eo.mask, h, k0, k1, s_abs, len, w32, s_win, eo.overflow);
         const uint64_t out = obase + idx;
-        __stcs(eo.slot + out, slot);
-        __stcs(eo.doc + out, doc);
+        bool hot = false;
+        if (eo.hot && len <= kSlotBytes) {  // sampled popular term: count it per document, leave a hole
+          uint32_t j = (uint32_t)(h >> 20) & eo.hot_mask;
+          for (;;) {
+            const uint64_t e0 = __ldg(&eo.hot[j].k0);
+            if (e0 == 0) break;
+            if (e0 == k0 && __ldg(&eo.hot[j].k1) == k1) {
+              atomicAdd(&eo.hot_tf[(uint64_t)__ldg(&eo.hot[j].id) * eo.hot_docs + (doc - eo.doc_base)], 1u);
+              hot = true;
+              break;
+            }
+            j = (j + 1) & eo.hot_mask;
+          }
+        }
+        if (hot) {
+          __stcs(eo.slot + out, 0u);
+        } else {
+          const uint32_t slot =
+              table_insert(cv.text, eo.table, eo.slot_ref, eo.mask, h, k0, k1, s_abs, len, w32, s_win, eo.overflow);
+          __stcs(eo.slot + out, slot | (1u << 25));  // stream element: slot | count 1 << 25
+          __stcs(eo.doc + out, doc);
+        }
         if (eo.dbg_start) { eo.dbg_start[out] = s_abs; eo.dbg_len[out] = len; }
       }
     }

@@ -304,3 +304,43 @@ def test_config2_full_size_sha():
     want = oracle.index_bytes(text, off, threads=threads)
     assert _sha(got) == _sha(want)
     wjformat.check_invariants(wjformat.parse(got))
+
+
+# ------------------------------------------------------------------ sampled hot terms
+@pytest.fixture
+def hot_threshold(monkeypatch):
+    # contexts read WJ_HOT_MIN_BYTES at index_init: enable the (opt-in) hot-term path on small chunks
+    monkeypatch.setenv("WJ_HOT_MIN_BYTES", "65536")
+    yield
+
+
+@pytest.mark.parametrize("cfg_id", [2, 3, 4])
+def test_hot_path_shapes(hot_threshold, cfg_id):
+    cfg = gen.CONFIGS[cfg_id].scaled(chunk_bytes=6 << 20, vocab=200_000)
+    text, off = gen.generate(cfg)
+    n = len(off) - 1
+    want = oracle.index_bytes(text, off)
+    assert_same_index(gpu_index(text, off), want)
+    assert_same_index(gpu_index(text, off, cuts=[0, n // 3, n // 3 + 1, n]), want)
+
+
+def test_hot_path_repetitive_docs(hot_threshold):
+    # a term whose per-document count exceeds 127 (split into several stream elements) and one-token docs
+    docs = [b"the " * 600 + b"cat", b"the", b"", b"The the THE"] * 300 + [b"x y z " * 5000]
+    text, off = gen.from_docs(docs)
+    assert_same_index(gpu_index(text, off), oracle.index_bytes(text, off))
+
+
+def test_multichunk_config3_shape():
+    # Wikipedia-shaped (short documents, several chunks): maps per chunk, dictionary merge + rebuild
+    cfg = gen.CONFIGS[3].scaled(chunk_bytes=4 << 20, vocab=300_000)
+    parts = [gen.generate(cfg, chunk=c) for c in range(3)]
+    with wj.Index() as ix:
+        for t, o in parts:
+            ix.add_stream(t, o)
+        ix.finalize()
+        got = ix.serialize()
+    o = oracle.Oracle()
+    for t, oo in parts:
+        o.add(t, oo)
+    assert_same_index(got, o.serialize())
