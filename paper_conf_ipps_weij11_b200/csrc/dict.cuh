@@ -294,26 +294,26 @@ __global__ void k_tie_fix(const uint64_t* key, uint32_t* val, uint32_t N, const 
   }
 }
 
-// New terms in sorted order: termIDs by warp-aggregated atomics (the paper's GPU indexer assigns
-// postings pointers as it inserts), arena append <len><suffix> (Fig. 6), per-term columns.
-__global__ void k_new_terms(const uint32_t* sorted_u, uint32_t N, const uint32_t* aoff, uint64_t arena_base,
-                            const uint8_t* text, const uint4* u_w, const uint32_t* u_ref, const uint32_t* u_len,
-                            const uint32_t* u_bucket, const uint32_t* u_cache, const uint32_t* u_rank,
-                            uint32_t* u_tid, uint32_t* tid_counter, uint8_t* arena, uint32_t* t_arena,
-                            uint32_t* t_cache, uint32_t* t_bucket, uint32_t* ns_tid, uint32_t* ns_bucket,
-                            uint32_t* ns_rank) {
-  const uint32_t k = blockIdx.x * blockDim.x + threadIdx.x;
-  const bool active = k < N;
+// New terms, in unique order (coalesced column reads): termIDs by warp-aggregated atomics (the
+// paper's GPU indexer assigns postings pointers as it inserts), arena append <len><suffix>
+// (Fig. 6) at the scanned offset, per-term columns.  The sorted-order lists for the merge are filled
+// afterwards by k_ns_fill.
+__global__ void k_new_terms(uint32_t U, const uint32_t* aoff, uint64_t arena_base, const uint8_t* text,
+                            const uint4* u_w, const uint32_t* u_ref, const uint32_t* u_len, const uint32_t* u_bucket,
+                            const uint32_t* u_cache, uint32_t* u_tid, uint32_t* tid_counter, uint8_t* arena,
+                            uint32_t* t_arena, uint32_t* t_cache, uint32_t* t_bucket) {
+  const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
+  const bool active = u < U && u_tid[u] == kMiss;
   const uint32_t lane = lane_id();
   const uint32_t am = __ballot_sync(0xffffffffu, active);
+  if (!am) return;
   uint32_t base = 0;
-  if (lane == 0 && am) base = atomicAdd(tid_counter, (uint32_t)__popc(am));
+  if (lane == 0) base = atomicAdd(tid_counter, (uint32_t)__popc(am));
   base = __shfl_sync(0xffffffffu, base, 0);
   if (!active) return;
   const uint32_t tid = base + __popc(am & ((1u << lane) - 1u));
-  const uint32_t u = sorted_u[k];
   const uint32_t b = u_bucket[u], plen = bucket_plen(b), ref = u_ref[u], slen = u_len[u] - plen;
-  const uint64_t off = arena_base + aoff[k];
+  const uint64_t off = arena_base + aoff[u];
   arena[off] = (uint8_t)slen;
   const uint4 w = u_w[u];
   for (uint32_t i = 0; i < slen; ++i) arena[off + 1 + i] = (uint8_t)ubyte(w, text, ref, plen + i);
@@ -321,8 +321,15 @@ __global__ void k_new_terms(const uint32_t* sorted_u, uint32_t N, const uint32_t
   t_cache[tid] = u_cache[u];
   t_bucket[tid] = b;
   u_tid[u] = tid;
-  ns_tid[k] = tid;
-  ns_bucket[k] = b;
+}
+
+__global__ void k_ns_fill(const uint32_t* sorted_u, uint32_t N, const uint32_t* u_tid, const uint32_t* u_bucket,
+                          const uint32_t* u_rank, uint32_t* ns_tid, uint32_t* ns_bucket, uint32_t* ns_rank) {
+  const uint32_t k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= N) return;
+  const uint32_t u = sorted_u[k];
+  ns_tid[k] = u_tid[u];
+  ns_bucket[k] = u_bucket[u];
   ns_rank[k] = u_rank[u];
 }
 
@@ -472,9 +479,10 @@ struct LexGroups {
 
 __global__ void k_lex_groups(const uint32_t* e_tid, const uint32_t* coll_base, const uint32_t* coll_n,
                              const uint32_t* t_cache, LexGroups* g) {
-  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  // lanes 0..10: first bucket-0 index whose first byte is >= '0'+k (k = 10: >= 0x80), in parallel
+  const uint32_t k = threadIdx.x;
   const uint32_t b0 = coll_base[0], n0 = coll_n[0];
-  for (int k = 0; k <= 10; ++k) {
+  if (k <= 10) {
     const uint32_t target = k < 10 ? '0' + k : 0x80;
     uint32_t lo = 0, hi = n0;
     while (lo < hi) {
@@ -483,17 +491,19 @@ __global__ void k_lex_groups(const uint32_t* e_tid, const uint32_t* coll_base, c
     }
     g->zlo[k] = lo;
   }
+  __syncwarp();
+  if (k != 0) return;
   uint32_t acc = 0;
-  for (int k = 0; k < 10; ++k) {
-    g->gbase[k] = acc;
-    const uint32_t zhi = k < 9 ? g->zlo[k + 1] : g->zlo[10];
-    acc += coll_n[1 + k] + (zhi - g->zlo[k]);
+  for (int q = 0; q < 10; ++q) {
+    g->gbase[q] = acc;
+    const uint32_t zhi = q < 9 ? g->zlo[q + 1] : g->zlo[10];
+    acc += coll_n[1 + q] + (zhi - g->zlo[q]);
   }
-  for (int k = 0; k < 26; ++k) {
-    g->gbase[10 + k] = acc;
-    const uint32_t s = coll_base[37 + 676 * k];
-    const uint32_t e = (k == 25) ? coll_base[kCollections - 1] + coll_n[kCollections - 1] : coll_base[37 + 676 * (k + 1)];
-    acc += coll_n[11 + k] + (e - s);
+  for (int q = 0; q < 26; ++q) {
+    g->gbase[10 + q] = acc;
+    const uint32_t s = coll_base[37 + 676 * q];
+    const uint32_t e = (q == 25) ? coll_base[kCollections - 1] + coll_n[kCollections - 1] : coll_base[37 + 676 * (q + 1)];
+    acc += coll_n[11 + q] + (e - s);
   }
   g->gbase[36] = acc;
 }

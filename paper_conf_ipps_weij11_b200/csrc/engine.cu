@@ -71,13 +71,12 @@ struct IsMiss {
   const uint32_t* t;
   __device__ __forceinline__ uint32_t operator()(uint64_t i) const { return t[i] == kMiss ? 1u : 0u; }
 };
-struct ArenaSize {
-  const uint32_t* sorted_u;
+struct ArenaSizeU {
+  const uint32_t* u_tid;
   const uint32_t* u_len;
   const uint32_t* u_bucket;
-  __device__ __forceinline__ uint32_t operator()(uint64_t k) const {
-    const uint32_t u = sorted_u[k];
-    return 1u + u_len[u] - bucket_plen(u_bucket[u]);
+  __device__ __forceinline__ uint32_t operator()(uint64_t u) const {
+    return u_tid[u] == kMiss ? 1u + u_len[u] - bucket_plen(u_bucket[u]) : 0u;
   }
 };
 
@@ -833,9 +832,9 @@ struct wj_index {
     k_tie_fix<<<grid_for(Nn, 256), 256, 0, st>>>(sk, sv, (uint32_t)Nn, text, (const uint4*)u_w.p, (const uint32_t*)u_ref.p,
                                                  (const uint32_t*)u_len.p);
     launched();
-    // arena offsets
-    uint32_t* ao = buf<uint32_t>(aoff, Nn);
-    scan<uint32_t>(ArenaSize{sv, (const uint32_t*)u_len.p, (const uint32_t*)u_bucket.p}, Nn, ao,
+    // arena offsets, in unique order (only misses take space)
+    uint32_t* ao = buf<uint32_t>(aoff, U);
+    scan<uint32_t>(ArenaSizeU{(const uint32_t*)u_tid.p, (const uint32_t*)u_len.p, (const uint32_t*)u_bucket.p}, U, ao,
                    (uint32_t*)(dscal() + 4));
     WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 4) + 1, 0, 4, st));
     readback(4, 1);
@@ -852,11 +851,13 @@ struct wj_index {
     uint32_t* counter = (uint32_t*)(dscal() + 6);
     k_fill<uint32_t><<<1, 1, 0, st>>>(counter, 1, V);
     launched();
-    k_new_terms<<<grid_for(Nn, 256), 256, 0, st>>>(sv, (uint32_t)Nn, ao, arena_used, text, (const uint4*)u_w.p,
-                                                   (const uint32_t*)u_ref.p,
-                                                   (const uint32_t*)u_len.p, (const uint32_t*)u_bucket.p,
-                                                   (const uint32_t*)u_cache.p, (const uint32_t*)u_rank.p,
-                                                   (uint32_t*)u_tid.p, counter, ar, ta, tc, tb, nt, nb, nr);
+    k_new_terms<<<grid_for(U, 256), 256, 0, st>>>((uint32_t)U, ao, arena_used, text, (const uint4*)u_w.p,
+                                                  (const uint32_t*)u_ref.p, (const uint32_t*)u_len.p,
+                                                  (const uint32_t*)u_bucket.p, (const uint32_t*)u_cache.p,
+                                                  (uint32_t*)u_tid.p, counter, ar, ta, tc, tb);
+    launched();
+    k_ns_fill<<<grid_for(Nn, 256), 256, 0, st>>>(sv, (uint32_t)Nn, (const uint32_t*)u_tid.p,
+                                                 (const uint32_t*)u_bucket.p, (const uint32_t*)u_rank.p, nt, nb, nr);
     launched();
     arena_used += A;
     // merge into the sorted key order E of every collection
