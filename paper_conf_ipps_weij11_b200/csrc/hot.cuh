@@ -18,10 +18,12 @@ constexpr uint32_t kHotMinCount = 16;
 
 // hash of a term of <= 16 bytes from its folded words: identical to k_tok_emit's
 __device__ __forceinline__ uint64_t term_hash16(uint32_t w0, uint32_t w1, uint32_t w2, uint32_t w3, uint32_t len) {
-  uint64_t h = 0x9E3779B97F4A7C15ull ^ ((uint64_t)len * 0xA0761D6478BD642Full);
-  h = mix_hash(h, (uint64_t)w0 | ((uint64_t)w1 << 32));
-  h = mix_hash(h, (uint64_t)w2 | ((uint64_t)w3 << 32));
-  return fmix64(h);
+  uint32_t h = hash_init(len);
+  h = hash_mix(h, w0);
+  h = hash_mix(h, w1);
+  h = hash_mix(h, w2);
+  h = hash_mix(h, w3);
+  return hash_fin(h);
 }
 
 // sample documents: doc_off prefix with the last document clipped at S

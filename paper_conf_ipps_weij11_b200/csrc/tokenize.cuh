@@ -265,10 +265,19 @@ __device__ __forceinline__ uint32_t win_word(const uint32_t* win32, uint32_t s, 
   return w;  // the window is staged already folded (reading S2)
 }
 
-__device__ __forceinline__ uint64_t mix_hash(uint64_t h, uint64_t x) {
-  h = (h ^ x) * 0xff51afd7ed558ccdull;
-  return h ^ (h >> 29);
+// 32-bit term hash over the folded, zero-padded little-endian words (cheap integer ops: the emit
+// kernel is instruction-bound).  Slot index = h & mask; the slot tag is a second mix of h.
+__device__ __forceinline__ uint32_t hash_init(uint32_t len) { return len * 0x9E3779B1u + 0x7F4A7C15u; }
+__device__ __forceinline__ uint32_t hash_mix(uint32_t h, uint32_t w) {
+  h = (h ^ w) * 0x85EBCA77u;
+  return h ^ (h >> 15);
 }
+__device__ __forceinline__ uint32_t hash_fin(uint32_t h) {
+  h ^= h >> 13;
+  h *= 0xC2B2AE3Du;
+  return h ^ (h >> 16);
+}
+__device__ __forceinline__ uint32_t hash_tag(uint32_t h) { return (h * 0x9E3779B1u) >> 8; }
 
 __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* table, uint32_t* slot_ref, uint32_t mask,
                                                  uint64_t h, uint64_t k0, uint64_t k1, uint32_t s_abs, uint32_t len,
@@ -349,18 +358,25 @@ __global__ void __launch_bounds__(kTokThreads) k_tok_emit(ChunkView cv, uint32_t
         const uint32_t e = q[idx];
         const uint32_t s_win = e >> 8, len = e & 255u;
         const uint32_t s_abs = B0 + s_win;
+        // first 16 folded bytes: 5 window words, 4 funnel shifts, length masks
         uint32_t wd[4];
+        {
+          const uint32_t a = s_win >> 2, sh = (s_win & 3) * 8;
+          uint32_t x[5];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) wd[k] = (4u * k < len) ? win_word(w32, s_win, len, k) : 0u;
-        uint64_t h = 0x9E3779B97F4A7C15ull ^ ((uint64_t)len * 0xA0761D6478BD642Full);
-        h = mix_hash(h, (uint64_t)wd[0] | ((uint64_t)wd[1] << 32));
-        h = mix_hash(h, (uint64_t)wd[2] | ((uint64_t)wd[3] << 32));
-        for (uint32_t k = 4; k * 4 < len; k += 2) {
-          const uint32_t a = win_word(w32, s_win, len, k);
-          const uint32_t b = ((k + 1) * 4 < len) ? win_word(w32, s_win, len, k + 1) : 0u;
-          h = mix_hash(h, (uint64_t)a | ((uint64_t)b << 32));
+          for (int k = 0; k < 5; ++k) x[k] = w32[a + k];
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const uint32_t rem = min(max((int)len - 4 * k, 0), 4);
+            wd[k] = __funnelshift_r(x[k], x[k + 1], sh) & __funnelshift_lc(0xFFFFFFFFu, 0u, rem * 8);
+          }
         }
-        h = fmix64(h);
+        uint32_t h32 = hash_init(len);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) h32 = hash_mix(h32, wd[k]);
+        for (uint32_t k = 4; k * 4 < len; ++k) h32 = hash_mix(h32, win_word(w32, s_win, len, k));
+        h32 = hash_fin(h32);
+        const uint64_t h = h32;
         // DocID = (number of doc_off[k] <= s, k < n_docs) - 1 (readings S9, S16)
         uint64_t lo = k_range_lo, hi = k_range_hi;
         while (lo < hi) {
@@ -368,7 +384,7 @@ __global__ void __launch_bounds__(kTokThreads) k_tok_emit(ChunkView cv, uint32_t
           if (cv.doc_off[mid] <= s_abs) lo = mid + 1; else hi = mid;
         }
         const uint32_t doc = eo.doc_base + (uint32_t)(lo - 1);
-        const uint64_t k0 = (uint64_t)len | (((h >> 40) & 0xFFFFFFull) << 8) | ((uint64_t)wd[0] << 32);
+        const uint64_t k0 = (uint64_t)len | ((uint64_t)hash_tag(h32) << 8) | ((uint64_t)wd[0] << 32);
         const uint64_t k1 = (uint64_t)wd[1] | ((uint64_t)(wd[2] & 0xFFFFFFu) << 32) | (1ull << 56);
         const uint64_t out = obase + idx;
         bool hot = false;
@@ -420,12 +436,16 @@ __global__ void __launch_bounds__(kTokThreads) k_tok_emit(ChunkView cv, uint32_t
     }
     if (seg == se) break;
     k_range_hi = kcur;
-    uint32_t c = 0;
-    for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
-      const int jb = __ffs(sm) - 1;
-      const uint32_t pos = 16 * lane + jb;
-      if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
-      c += (tok_end_rel(sb, tk, jb) - pos <= kMaxTermLen) ? 1u : 0u;
+    // kept tokens starting in this lane (a > 255-byte token needs a lane of 16 token bytes)
+    uint32_t c = __popc(sb.startm) - ((int)lane == tk.open_lane ? 1u : 0u);
+    if (__ballot_sync(0xffffffffu, sb.tm == 0xFFFFu)) {
+      c = 0;
+      for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
+        const int jb = __ffs(sm) - 1;
+        const uint32_t pos = 16 * lane + jb;
+        if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
+        c += (tok_end_rel(sb, tk, jb) - pos <= kMaxTermLen) ? 1u : 0u;
+      }
     }
     uint32_t inc = c;
 #pragma unroll
