@@ -97,14 +97,18 @@ struct SegBits {
   uint32_t termm;   // terminators: non-token byte or document start
 };
 
-// Classifies one segment; kcur = first boundary index (k >= 1) with doc_off[k] >= segment start
-// (advanced past the segment); prev = token bit of the byte before the segment.
-__device__ __forceinline__ SegBits seg_bits(const ChunkView& cv, uint32_t s0, uint4 v, uint32_t prev,
-                                            uint64_t& kcur, uint32_t* bnd_smem) {
-  const uint32_t lane = lane_id();
-  const uint64_t p0 = (uint64_t)s0 + 16 * lane;
+// 16-bit token-byte mask of the lane's 16 bytes of the segment starting at s0
+__device__ __forceinline__ uint32_t lane_tm(const ChunkView& cv, uint32_t s0, uint4 v) {
+  const uint64_t p0 = (uint64_t)s0 + 16 * lane_id();
   uint32_t tm = tokmask4(v.x) | (tokmask4(v.y) << 4) | (tokmask4(v.z) << 8) | (tokmask4(v.w) << 12);
   if (p0 + 16 > cv.n_bytes) tm = p0 >= cv.n_bytes ? 0u : tm & ((1u << (uint32_t)(cv.n_bytes - p0)) - 1u);
+  return tm;
+}
+
+// Document starts inside the segment [s0, s0 + 512) as the lane's 16-bit mask; kcur = first
+// boundary index (k >= 1) with doc_off[k] >= s0, advanced past the segment.
+__device__ __forceinline__ uint32_t seg_bounds(const ChunkView& cv, uint32_t s0, uint64_t& kcur, uint32_t* bnd_smem) {
+  const uint32_t lane = lane_id();
   const uint64_t s1 = (uint64_t)s0 + kSegBytes;
   uint32_t bm = 0;
   const uint64_t nb = (kcur < cv.n_docs) ? cv.doc_off[kcur] : ~0ull;  // warp-uniform
@@ -124,11 +128,24 @@ __device__ __forceinline__ SegBits seg_bits(const ChunkView& cv, uint32_t s0, ui
     bm = bnd_smem[lane];
     __syncwarp();
   }
+  return bm;
+}
+
+// token starts of the lane: token byte whose predecessor is not one, or a document start
+__device__ __forceinline__ uint32_t start_mask(uint32_t tm, uint32_t bm, uint32_t prev) {
   uint32_t pv = __shfl_up_sync(0xffffffffu, tm >> 15, 1) & 1u;
-  if (lane == 0) pv = prev;
+  if (lane_id() == 0) pv = prev;
+  return tm & (~((tm << 1) | pv) | bm) & 0xFFFFu;
+}
+
+// Classifies one segment; prev = token bit of the byte before the segment.
+__device__ __forceinline__ SegBits seg_bits(const ChunkView& cv, uint32_t s0, uint4 v, uint32_t prev,
+                                            uint64_t& kcur, uint32_t* bnd_smem) {
+  const uint32_t tm = lane_tm(cv, s0, v);
+  const uint32_t bm = seg_bounds(cv, s0, kcur, bnd_smem);
   SegBits sb;
   sb.tm = tm;
-  sb.startm = tm & (~((tm << 1) | pv) | bm) & 0xFFFFu;
+  sb.startm = start_mask(tm, bm, prev);
   sb.termm = (~tm | bm) & 0xFFFFu;
   return sb;
 }
@@ -211,6 +228,28 @@ __global__ void __launch_bounds__(kTokThreads) k_tok_count(ChunkView cv, uint32_
   uint4 vr[kSegsPerWarp + 1];
 #pragma unroll
   for (int j = 0; j <= kSegsPerWarp; ++j) vr[j] = (sb0 + j <= last) ? load_lane16(cv, sb0 + j) : make_uint4(0, 0, 0, 0);
+  // Fast path: no lane of the range or the look-ahead segment holds 16 token bytes, so every token
+  // starting in the range is <= 30 bytes long and is kept: the count is the number of token starts.
+  uint32_t tmv[kSegsPerWarp + 1];
+  bool full = false;
+#pragma unroll
+  for (int j = 0; j <= kSegsPerWarp; ++j) {
+    tmv[j] = (sb0 + j <= last) ? lane_tm(cv, (sb0 + j) * kSegBytes, vr[j]) : 0u;
+    full |= tmv[j] == 0xFFFFu;
+  }
+  if (!__any_sync(0xffffffffu, full)) {
+#pragma unroll
+    for (int j = 0; j < kSegsPerWarp; ++j) {
+      if (sb0 + j >= se) break;
+      const uint32_t bm = seg_bounds(cv, (sb0 + j) * kSegBytes, kcur, bnd[w]);
+      cnt += __popc(start_mask(tmv[j], bm, prev));
+      prev = __shfl_sync(0xffffffffu, tmv[j], 31) >> 15;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
+    if (lane == 0) range_count[gw] = cnt;
+    return;
+  }
 #pragma unroll
   for (int jj = 0; jj <= kSegsPerWarp; ++jj) {
     const uint32_t seg = sb0 + jj;
