@@ -45,6 +45,10 @@ def _load():
         lib.oracle_add_mt.restype = ctypes.c_int
         lib.oracle_serialize.argtypes = [vp, vp, u64, P64]
         lib.oracle_serialize.restype = ctypes.c_int
+        lib.oracle_serialize_vbyte.argtypes = [vp, vp, u64, P64]
+        lib.oracle_serialize_vbyte.restype = ctypes.c_int
+        lib.oracle_vbyte.argtypes = [vp, u64, vp]
+        lib.oracle_vbyte.restype = u64
         lib.oracle_postings.argtypes = [vp, ctypes.c_char_p, u32, vp, vp, u64, P64]
         lib.oracle_postings.restype = ctypes.c_int
         lib.oracle_dump_tokens.argtypes = [vp, vp, u64, u32, vp, u64, P64]
@@ -84,11 +88,13 @@ class Oracle:
         if rc != 0:
             raise RuntimeError(f"oracle_add failed: {rc}")
 
-    def serialize(self) -> bytes:
+    def serialize(self, vbyte: bool = False) -> bytes:
+        """Canonical index bytes: WJINV001, or WJINV002 (d-gap + variable-byte postings) if vbyte."""
+        f = self._lib.oracle_serialize_vbyte if vbyte else self._lib.oracle_serialize
         n = ctypes.c_uint64()
-        self._lib.oracle_serialize(self._h, None, 0, ctypes.byref(n))
+        f(self._h, None, 0, ctypes.byref(n))
         buf = ctypes.create_string_buffer(n.value)
-        rc = self._lib.oracle_serialize(self._h, buf, n.value, ctypes.byref(n))
+        rc = f(self._h, buf, n.value, ctypes.byref(n))
         if rc != 0:
             raise RuntimeError(f"oracle_serialize failed: {rc}")
         return buf.raw[: n.value]
@@ -105,11 +111,20 @@ class Oracle:
         return d, t
 
 
-def index_bytes(text, doc_off, threads: int = 1) -> bytes:
+def index_bytes(text, doc_off, threads: int = 1, vbyte: bool = False) -> bytes:
     """Serialized oracle index of one batch of documents."""
     o = Oracle()
     o.add(text, doc_off, threads)
-    return o.serialize()
+    return o.serialize(vbyte)
+
+
+def vbyte(values) -> bytes:
+    """Variable-byte code of a sequence of u32 values (reading S19)."""
+    v = np.ascontiguousarray(values, dtype=np.uint32)
+    lib = _load()
+    out = ctypes.create_string_buffer(5 * max(len(v), 1))
+    n = lib.oracle_vbyte(v.ctypes.data, len(v), out)
+    return out.raw[:n]
 
 
 def dump_tokens(text, doc_off, doc_base: int = 0):

@@ -187,3 +187,57 @@ def test_invariants_config1():
     ix = wjformat.parse(oracle.index_bytes(text, off))
     wjformat.check_invariants(ix)
     assert ix.n_docs == 1000 and ix.n_terms > 1000
+
+
+# ---------------------------------------------------------------- f1: d-gap + variable-byte code
+# Layout fixed by SURVEY.md §8(f1) ("7-bit groups, LSB-first, high bit = continuation"), the
+# d-gaps by P:49, the encoding step by P:216; reading S19 in DESIGN.md.
+VBYTE_TEXTBOOK = [(0, "00"), (1, "01"), (5, "05"), (127, "7f"), (128, "8001"), (300, "ac02"), (16383, "ff7f"),
+                  (16384, "808001"), (2 ** 21, "80808001"), (2 ** 32 - 1, "ffffffff0f")]
+
+
+@pytest.mark.parametrize("value,hexcode", VBYTE_TEXTBOOK)
+def test_vbyte_hand_values(value, hexcode):
+    assert oracle.vbyte([value]).hex() == hexcode
+
+
+def test_vbyte_matches_protobuf_varint():
+    # the same byte code is the protocol-buffers base-128 varint (library routine)
+    enc = pytest.importorskip("google.protobuf.internal.encoder")
+    rng = np.random.default_rng(7)
+    vals = np.concatenate([rng.integers(0, 2 ** 32, 2000, dtype=np.uint64),
+                           2 ** np.arange(32, dtype=np.uint64), 2 ** np.arange(1, 33, dtype=np.uint64) - 1])
+    assert oracle.vbyte(vals.astype(np.uint32)) == b"".join(enc._VarintBytes(int(v)) for v in vals)
+
+
+def test_vbyte_hand_counted_survey_corpus():
+    # docs ["The cat sat.", "the CAT, the hat!", ""]: cat (0,1),(1,1); hat (1,1); sat (0,1);
+    # the (0,1),(1,2) -> (gap, tf) bytes 00 01 01 01 | 01 01 | 00 01 | 00 01 01 02
+    text, off = gen.from_docs([b"The cat sat.", b"the CAT, the hat!", b""])
+    buf = oracle.index_bytes(text, off, vbyte=True)
+    assert buf[:8] == b"WJINV002"
+    hdr = np.frombuffer(buf, dtype="<u8", count=8)
+    assert hdr[7] == 12
+    assert buf[-16:-4] == bytes.fromhex("000101010101000100010102") and buf[-4:] == b"\0" * 4
+    assert np.frombuffer(buf, dtype="<u8", count=5, offset=len(buf) - 16 - 40).tolist() == [0, 4, 6, 8, 12]
+
+
+@pytest.mark.parametrize("which", ["config1", "edges", "bruteforce"])
+def test_vbyte_decodes_to_pinned_index(which):
+    if which == "config1":
+        text, off = gen.generate(gen.CONFIGS[1])
+    elif which == "edges":
+        docs, _, _ = load_corpus("corpus_edges.txt")
+        text, off = gen.from_docs(docs)
+    else:
+        rng = np.random.default_rng(3)
+        docs = [bytes(rng.choice(BYTE_POOL, size=int(rng.integers(0, 80)))) for _ in range(300)]
+        text, off = gen.from_docs(docs)
+    plain = oracle.index_bytes(text, off)
+    comp = oracle.index_bytes(text, off, vbyte=True)
+    a, b = wjformat.parse(plain), wjformat.parse(comp)
+    wjformat.check_invariants(b)
+    for f in ("n_docs", "n_tokens", "n_dropped", "n_terms", "n_postings", "n_term_bytes"):
+        assert getattr(a, f) == getattr(b, f)
+    assert a.as_dict() == b.as_dict()
+    assert len(comp) < len(plain) or a.n_postings == 0

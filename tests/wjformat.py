@@ -4,6 +4,12 @@ Layout (little-endian):  64-B header {char magic[8]="WJINV001"; u64 n_docs, n_to
 n_dropped, n_terms, n_postings, n_term_bytes, reserved}; u64 term_off[n_terms+1];
 u8 term_bytes[] (pad 8); u32 df[] (pad 8); u64 cf[]; u64 post_off[n_terms+1];
 u32 docid[] (pad 8); u32 tf[] (pad 8).
+
+Compressed layout "WJINV002" (reading S19): same header with word 7 =
+n_post_bytes, same dictionary / df / cf; then u64 post_off[n_terms+1] as BYTE offsets and the
+postings bytes (pad 8): per posting vbyte(d-gap) then vbyte(tf); vbyte = 7-bit groups, least
+significant first, high bit set iff more bytes follow; the first gap of a list is the docID.
+`parse` accepts both and returns the decoded (uncompressed) index.
 """
 from __future__ import annotations
 
@@ -12,6 +18,7 @@ from dataclasses import dataclass
 import numpy as np
 
 MAGIC = b"WJINV001"
+MAGIC_VB = b"WJINV002"
 
 
 def _pad8(n: int) -> int:
@@ -52,12 +59,30 @@ class Index:
         return out
 
 
+def vbyte_decode(code: bytes, n_values: int):
+    """Decode n_values variable-byte values from code; returns (values, bytes consumed)."""
+    out = []
+    p = 0
+    for _ in range(n_values):
+        v = shift = 0
+        while True:
+            c = code[p]
+            p += 1
+            v |= (c & 0x7F) << shift
+            shift += 7
+            if not c & 0x80:
+                break
+        out.append(v)
+    return out, p
+
+
 def parse(buf: bytes) -> Index:
-    if buf[:8] != MAGIC:
+    vb = buf[:8] == MAGIC_VB
+    if buf[:8] != MAGIC and not vb:
         raise ValueError("bad magic")
     hdr = np.frombuffer(buf, dtype="<u8", count=8)
     n_docs, n_tokens, n_dropped, n_terms, n_post, n_tb, reserved = (int(x) for x in hdr[1:8])
-    if reserved != 0:
+    if reserved != 0 and not vb:
         raise ValueError("reserved != 0")
     p = 64
     term_off = np.frombuffer(buf, dtype="<u8", count=n_terms + 1, offset=p); p += 8 * (n_terms + 1)
@@ -68,6 +93,33 @@ def parse(buf: bytes) -> Index:
     df = np.frombuffer(buf, dtype="<u4", count=n_terms, offset=p); p += _pad8(4 * n_terms)
     cf = np.frombuffer(buf, dtype="<u8", count=n_terms, offset=p); p += 8 * n_terms
     post_off = np.frombuffer(buf, dtype="<u8", count=n_terms + 1, offset=p); p += 8 * (n_terms + 1)
+    if vb:
+        n_pb = reserved
+        code = buf[p:p + n_pb]
+        if any(buf[p + n_pb:p + _pad8(n_pb)]):
+            raise ValueError("nonzero padding after postings bytes")
+        p += _pad8(n_pb)
+        if p != len(buf):
+            raise ValueError(f"trailing bytes: parsed {p} of {len(buf)}")
+        if post_off[0] != 0 or post_off[-1] != n_pb:
+            raise ValueError("postings byte offsets do not span the code")
+        docid = np.empty(n_post, dtype=np.uint32)
+        tf = np.empty(n_post, dtype=np.uint32)
+        k = 0
+        for i in range(n_terms):
+            a, b = int(post_off[i]), int(post_off[i + 1])
+            vals, used = vbyte_decode(code[a:b], 2 * int(df[i]))
+            if used != b - a:
+                raise ValueError(f"term {i}: postings bytes not consumed exactly")
+            gaps = np.array(vals[0::2], dtype=np.int64)
+            docid[k:k + int(df[i])] = np.cumsum(gaps)
+            tf[k:k + int(df[i])] = vals[1::2]
+            k += int(df[i])
+        if k != n_post:
+            raise ValueError("sum df != n_postings")
+        post_off = np.concatenate([[0], np.cumsum(df.astype(np.uint64))]).astype(np.uint64)
+        return Index(n_docs, n_tokens, n_dropped, n_terms, n_post, n_tb, term_off, term_bytes, df, cf,
+                     post_off, docid, tf)
     docid = np.frombuffer(buf, dtype="<u4", count=n_post, offset=p); p += _pad8(4 * n_post)
     tf = np.frombuffer(buf, dtype="<u4", count=n_post, offset=p); p += _pad8(4 * n_post)
     if p != len(buf):
