@@ -196,6 +196,8 @@ def main():
     ap.add_argument("--chunk-bytes", type=int, default=None, help="override bytes per GPU (debug)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--vbyte", action="store_true",
+                    help="also encode the postings as d-gaps + variable-byte code (SURVEY 8(f1), WJINV002)")
     args = ap.parse_args()
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
@@ -227,9 +229,9 @@ def main():
         nid = [wj.nccl_unique_id() if rank == 0 else None]
         if world > 1:
             dist.broadcast_object_list(nid, src=0)
-        ix = wj.Index(device=local, profile=True, rank=rank, world=world, nccl_id=nid[0])
+        ix = wj.Index(device=local, profile=True, rank=rank, world=world, nccl_id=nid[0], vbyte=args.vbyte)
     else:
-        ix = wj.Index(device=local, profile=True)
+        ix = wj.Index(device=local, profile=True, vbyte=args.vbyte)
 
     def step(t, o):
         ix.reset()
@@ -286,7 +288,11 @@ def main():
         except Exception:
             traffic = None
     # whole-step compulsory bytes: T + 8P + sum(len + 28) over terms
-    b_min = T + 8 * P + s1["n_term_bytes"] + 28 * V
+    post_bytes = 8 * P
+    if args.vbyte:  # compressed postings: the code bytes replace the (docid, tf) arrays
+        pad8 = lambda x: (x + 7) & ~7  # noqa: E731
+        post_bytes = ix.serialized_size() - (64 + 16 * (V + 1) + pad8(s1["n_term_bytes"]) + pad8(4 * V) + 8 * V)
+    b_min = T + post_bytes + s1["n_term_bytes"] + 28 * V
     step_gbs = b_min * world / (ms / 1e3) / 1e9
 
     phases = {k: (s1["phase_ms"][k] - s0["phase_ms"][k]) / args.steps for k in wj.PHASES}
@@ -334,6 +340,7 @@ def main():
             "config": {"workload": WORKLOAD.get(args.config, str(args.config)), "bytes_per_gpu": T,
                        "docs_per_gpu": len(doc_off) - 1, "tokens_per_gpu": N, "terms_per_gpu": V,
                        "postings_per_gpu": P, "l2": "no flush: 1 GiB input per step > 126 MB L2",
+                       "postings_format": "vbyte d-gaps (WJINV002)" if args.vbyte else "u32 docid + u32 tf (WJINV001)",
                        "parallelism": "single GPU" if world == 1 else
                        f"{world} ranks: document ranges, trie collections b mod {world}, NCCL all-to-all-v"},
             "exchange_bytes_per_step": (s1["exchange_bytes"]),
@@ -345,7 +352,7 @@ def main():
                          "launches_per_step": launches_per_step},
             "roofline_step": {"bytes_min": b_min, "achieved": step_gbs, "peak": peak * world, "unit": "GB/s",
                               "frac": step_gbs / (peak * world),
-                              "def": "B_min = T + 8P + sum(len+28) over terms (SURVEY 8(d)) / step time"},
+                              "def": ("B_min = T + (vbyte code bytes if --vbyte else 8P) + sum(len+28) over terms (SURVEY 8(d)) / step time")},
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": int(round(launches * args.steps)),

@@ -1,6 +1,6 @@
 /* wjindex.h — C ABI of the B200-native inverted-file indexer (Wei & JaJa, IPDPS 2011).
  *
- * PAPER.md = /root/reference/PAPER.md; "P:n" is its line n.  Readings S1..S18 of the paper are
+ * PAPER.md = /root/reference/PAPER.md; "P:n" is its line n.  Readings S1..S19 of the paper are
  * listed in DESIGN.md §3.
  *
  * What the library computes (the paper's problem statement):
@@ -50,6 +50,9 @@ typedef enum {
 #define WJ_FLAG_PROFILE 0x1u   /* record CUDA events per phase (index_stats.phase_ms)               */
 #define WJ_FLAG_LOOPBACK 0x2u  /* world > 1 inside one process: nccl_unique_id is a hub from        */
                                /* index_loopback_create; one host thread per rank context (tests)   */
+#define WJ_FLAG_VBYTE 0x4u     /* finalize also encodes every postings list as d-gaps + variable-   */
+                               /* byte code (reading S19) and            */
+                               /* index_serialize writes the compressed file "WJINV002"             */
 
 typedef struct wj_index wj_index; /* opaque; all index state is owned by the library */
 
@@ -77,6 +80,7 @@ enum {
   WJ_PHASE_POSTINGS,     /* finalize: run-length (docID, tf), df, cf, post_off                     */
   WJ_PHASE_DICT,         /* finalize: term_off + term bytes of the final dictionary                */
   WJ_PHASE_EXCHANGE,     /* world > 1: all-to-all of the routed stream                             */
+  WJ_PHASE_VBYTE,        /* finalize (WJ_FLAG_VBYTE): d-gap + variable-byte postings code  */
   WJ_PHASE_COUNT = 16
 };
 
@@ -146,7 +150,9 @@ int index_read_postings(wj_index* ix, const uint8_t* term, uint32_t len, uint32_
                         uint32_t* tfs, uint64_t cap, uint64_t* n_out);
 
 /* Canonical serialized inverted file (identical to the oracle's bytes), written to a
- * host buffer.  buf may be NULL (sizing call).  Requires finalize.  Errors: WJ_ERR_STATE,
+ * host buffer: "WJINV001", or with WJ_FLAG_VBYTE the compressed "WJINV002" (same header with
+ * word 7 = code bytes, dictionary, df, cf; then u64 post_off[n_terms+1] in bytes and the code:
+ * per posting vbyte(d-gap) then vbyte(tf), the first gap of a list = its docID; reading S19).  buf may be NULL (sizing call).  Requires finalize.  Errors: WJ_ERR_STATE,
  * WJ_ERR_BUFFER_TOO_SMALL (*n_out = size needed), WJ_ERR_CUDA. */
 int index_serialize(wj_index* ix, uint8_t* buf, uint64_t cap, uint64_t* n_out);
 

@@ -22,7 +22,7 @@ ERRORS = {-1: "WJ_ERR_INVALID_ARG", -2: "WJ_ERR_STATE", -3: "WJ_ERR_CUDA", -4: "
           -6: "WJ_ERR_CAPACITY", -7: "WJ_ERR_BUFFER_TOO_SMALL"}
 WJ_FLAG_PROFILE = 1
 PHASES = ["h2d", "tokenize", "unique", "probe", "insert", "rebuild", "stream", "lexrank", "sort", "postings",
-          "dict", "exchange"]
+          "dict", "exchange", "vbyte"]
 KERNELS = ["tokenize_count", "tokenize_emit", "probe", "slot_to_tid", "map_rank", "sort_hist", "sort_scatter",
            "rle_emit"]
 N_COLLECTIONS = 17613
@@ -32,6 +32,7 @@ EXPORTS = ["index_init", "index_add_stream", "index_finalize", "index_read_posti
            "index_loopback_create", "index_loopback_destroy", "index_merge_serialized", "index_last_error",
            "index_destroy"]
 WJ_FLAG_LOOPBACK = 2
+WJ_FLAG_VBYTE = 4
 
 
 class WJError(RuntimeError):
@@ -140,11 +141,15 @@ class Index:
     """One indexing context on one GPU (index_init .. index_destroy)."""
 
     def __init__(self, device: int = 0, stream=None, profile: bool = False, rank: int = 0, world: int = 1,
-                 nccl_id: bytes | None = None, hub: "LoopbackHub | None" = None, own_stream: bool = False):
+                 nccl_id: bytes | None = None, hub: "LoopbackHub | None" = None, own_stream: bool = False,
+                 vbyte: bool = False):
         """world > 1: pass nccl_id (128 bytes from nccl_unique_id(), broadcast by the caller) or a
-        LoopbackHub shared by `world` contexts of this process (one host thread each)."""
+        LoopbackHub shared by `world` contexts of this process (one host thread each).
+        vbyte: finalize also builds the d-gap + variable-byte postings code; serialize() then
+        returns the compressed file WJINV002."""
         self._lib = load_library()
-        flags = (WJ_FLAG_PROFILE if profile else 0) | (WJ_FLAG_LOOPBACK if hub is not None else 0)
+        flags = (WJ_FLAG_PROFILE if profile else 0) | (WJ_FLAG_LOOPBACK if hub is not None else 0) | (
+            WJ_FLAG_VBYTE if vbyte else 0)
         self._nid = ctypes.create_string_buffer(bytes(nccl_id), 128) if nccl_id is not None else None
         uid = hub._h if hub is not None else (ctypes.cast(self._nid, ctypes.c_void_p) if self._nid is not None else None)
         if own_stream:

@@ -16,6 +16,7 @@
 #include "radix.cuh"
 #include "scan.cuh"
 #include "tokenize.cuh"
+#include "vbyte.cuh"
 
 using namespace wj;
 
@@ -101,7 +102,8 @@ struct wj_index {
   uint32_t V = 0;
   uint64_t arena_used = 0;
   uint64_t table_est = 0;
-  uint64_t P = 0, TB = 0;
+  uint64_t P = 0, TB = 0, PB = 0;  // postings, term bytes, vbyte code bytes
+  bool vbyte = false;              // WJ_FLAG_VBYTE
   uint64_t exchange_bytes = 0;
 
   Transport* xport = nullptr;  // world > 1
@@ -131,6 +133,7 @@ struct wj_index {
       scan_scr, hist, hist_scan, os_hist, os_look, os_ctr, kstart, slotref, dbg_start, dbg_len, dbg_off, dbg_out, dbg_slot, dbg_doc, lexg, qbuf, qres;
   // finalize
   DevBuf rank_of, term_at, sk1, sv1, pidx, out_doc, out_tf, post_off, df, cf, term_off, term_bytes;
+  DevBuf vb_first, vb_tiles, vb_code, vb_boff;  // f1 (WJ_FLAG_VBYTE)
   std::vector<DevBuf> chunk_map;        // per chunk: slot -> termID (-> rank at finalize)
   std::vector<uint64_t> chunk_tok;      // per chunk: first token index in the stream
   std::vector<uint32_t> chunk_C;        // per chunk: table capacity
@@ -185,7 +188,7 @@ struct wj_index {
                      &nk_key2, &nk_val2, &aoff, &ns_tid, &ns_bucket, &ns_rank, &nlo, &nhi, &nbase, &child_off,
                      &root_idx, &scan_scr, &hist, &hist_scan, &os_hist, &os_look, &os_ctr, &kstart, &slotref, &dbg_start, &dbg_len, &dbg_off, &dbg_out, &dbg_slot,
                      &dbg_doc, &lexg, &qbuf, &qres, &rank_of, &term_at, &sk1, &sv1, &pidx, &out_doc, &out_tf,
-                     &post_off, &df, &cf, &term_off, &term_bytes};
+                     &post_off, &df, &cf, &term_off, &term_bytes, &vb_first, &vb_tiles, &vb_code, &vb_boff};
     for (DevBuf* b : all) {
       if (b->p) cudaFree(b->p);
       b->p = nullptr;
@@ -302,7 +305,7 @@ struct wj_index {
     exchange_bytes = 0;
     V = 0;
     arena_used = 0;
-    P = TB = 0;
+    P = TB = PB = 0;
     finalized = false;
     f_key = f_doc = nullptr;
     cur_phase = -1;
@@ -1090,6 +1093,8 @@ struct wj_index {
     } else {
       WJ_CUDA_CHECK(cudaMemsetAsync(po, 0, 8, st));
     }
+    PB = 0;
+    if (vbyte) encode_vbyte();
     phase(WJ_PHASE_DICT);
     uint64_t* to = buf<uint64_t>(term_off, (uint64_t)V + 1);
     TB = 0;
@@ -1111,17 +1116,47 @@ struct wj_index {
     finalized = true;
   }
 
+  // f1: d-gap + variable-byte code of the postings (vbyte.cuh, reading S19) ->
+  // vb_code[PB], vb_boff[V+1] (byte offset of every list)
+  void encode_vbyte() {
+    phase(WJ_PHASE_VBYTE);
+    uint64_t* pbo = buf<uint64_t>(vb_boff, (uint64_t)V + 1);
+    if (P == 0) {
+      WJ_CUDA_CHECK(cudaMemsetAsync(pbo, 0, 8 * ((uint64_t)V + 1), st));
+      return;
+    }
+    uint32_t* fb = buf<uint32_t>(vb_first, P / 32 + 1);
+    WJ_CUDA_CHECK(cudaMemsetAsync(fb, 0, 4 * (P / 32 + 1), st));
+    k_vb_first<<<grid_for(V, 256), 256, 0, st>>>((const uint64_t*)post_off.p, V, fb);
+    launched();
+    const uint64_t G = (P + kVbTile - 1) / kVbTile;
+    uint64_t* tb = buf<uint64_t>(vb_tiles, G + 1);
+    const uint32_t* od = (const uint32_t*)out_doc.p;
+    const uint32_t* of = (const uint32_t*)out_tf.p;
+    k_vb_tile<<<(unsigned)G, kVbThreads, 0, st>>>(od, of, fb, P, tb);
+    launched();
+    scan<uint64_t>(ArrayIn<uint64_t>{tb}, G, tb, tb + G);
+    WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 13, tb + G, 8, cudaMemcpyDeviceToHost, st));
+    sync();
+    PB = h_scal[13];
+    uint8_t* code = buf<uint8_t>(vb_code, PB + 16);
+    k_vb_encode<<<(unsigned)G, kVbThreads, kVbMaxTileBytes, st>>>(od, of, fb, P, (const uint64_t*)post_off.p, V, tb,
+                                                                  code, pbo);
+    launched();
+    WJ_CUDA_CHECK(cudaMemcpyAsync(pbo + V, tb + G, 8, cudaMemcpyDeviceToDevice, st));
+  }
+
   // ---------------------------------------------------------------- serialize
   uint64_t serialized_size() const {
     auto pad8 = [](uint64_t x) { return (x + 7) & ~7ull; };
-    return 64 + 8 * ((uint64_t)V + 1) + pad8(TB) + pad8(4ull * V) + 8ull * V + 8 * ((uint64_t)V + 1) + pad8(4 * P) +
-           pad8(4 * P);
+    return 64 + 8 * ((uint64_t)V + 1) + pad8(TB) + pad8(4ull * V) + 8ull * V + 8 * ((uint64_t)V + 1) +
+           (vbyte ? pad8(PB) : pad8(4 * P) + pad8(4 * P));
   }
   void serialize(uint8_t* out) {
     auto pad8 = [](uint64_t x) { return (x + 7) & ~7ull; };
     uint64_t hdr[8];
-    memcpy(hdr, "WJINV001", 8);
-    hdr[1] = n_docs; hdr[2] = n_tokens; hdr[3] = n_dropped; hdr[4] = V; hdr[5] = P; hdr[6] = TB; hdr[7] = 0;
+    memcpy(hdr, vbyte ? "WJINV002" : "WJINV001", 8);
+    hdr[1] = n_docs; hdr[2] = n_tokens; hdr[3] = n_dropped; hdr[4] = V; hdr[5] = P; hdr[6] = TB; hdr[7] = vbyte ? PB : 0;
     memcpy(out, hdr, 64);
     uint64_t p = 64;
     auto d2h = [&](const void* src, uint64_t bytes, uint64_t padded) {
@@ -1133,9 +1168,14 @@ struct wj_index {
     d2h(term_bytes.p, TB, pad8(TB));
     d2h(df.p, 4ull * V, pad8(4ull * V));
     d2h(cf.p, 8ull * V, 8ull * V);
-    d2h(post_off.p, 8 * ((uint64_t)V + 1), 8 * ((uint64_t)V + 1));
-    d2h(out_doc.p, 4 * P, pad8(4 * P));
-    d2h(out_tf.p, 4 * P, pad8(4 * P));
+    if (vbyte) {
+      d2h(vb_boff.p, 8 * ((uint64_t)V + 1), 8 * ((uint64_t)V + 1));
+      d2h(vb_code.p, PB, pad8(PB));
+    } else {
+      d2h(post_off.p, 8 * ((uint64_t)V + 1), 8 * ((uint64_t)V + 1));
+      d2h(out_doc.p, 4 * P, pad8(4 * P));
+      d2h(out_tf.p, 4 * P, pad8(4 * P));
+    }
     sync();
   }
 };
@@ -1176,7 +1216,7 @@ extern "C" {
 int index_init(wj_index** out, const wj_config* cfg) {
   if (!out || !cfg) return WJ_ERR_INVALID_ARG;
   *out = nullptr;
-  if (cfg->world < 1 || cfg->world > 1024 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~(WJ_FLAG_PROFILE | WJ_FLAG_LOOPBACK)) || cfg->reserved) {
+  if (cfg->world < 1 || cfg->world > 1024 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~(WJ_FLAG_PROFILE | WJ_FLAG_LOOPBACK | WJ_FLAG_VBYTE)) || cfg->reserved) {
     g_init_err = "invalid config";
     return WJ_ERR_INVALID_ARG;
   }
@@ -1200,6 +1240,7 @@ int index_init(wj_index** out, const wj_config* cfg) {
   ix->rank = cfg->rank;
   ix->world = cfg->world;
   ix->flags = cfg->flags;
+  ix->vbyte = (cfg->flags & WJ_FLAG_VBYTE) != 0;
   int rc = guarded(ix, [&]() {
     if (cfg->stream) {
       ix->st = (cudaStream_t)cfg->stream;
@@ -1462,26 +1503,29 @@ int index_merge_serialized(int32_t k, const uint8_t* const* slices, const uint64
                            uint64_t* n_out) {
   if (k < 1 || !slices || !sizes || !n_out) return WJ_ERR_INVALID_ARG;
   std::vector<SliceView> v(k);
-  uint64_t nt = 0, np = 0, ntb = 0, ntok = 0, ndrop = 0;
+  uint64_t nt = 0, np = 0, ntb = 0, ntok = 0, ndrop = 0, npb = 0;
   for (int i = 0; i < k; ++i) {
     if (!slices[i] || !parse_slice(slices[i], sizes[i], v[i])) {
       g_init_err = "index_merge_serialized: slice " + std::to_string(i) + " is not a serialized index";
       return WJ_ERR_INVALID_ARG;
     }
-    if (v[i].n_docs != v[0].n_docs) {
-      g_init_err = "index_merge_serialized: slices disagree on n_docs";
+    if (v[i].n_docs != v[0].n_docs || v[i].vb != v[0].vb) {
+      g_init_err = "index_merge_serialized: slices disagree on n_docs or format";
       return WJ_ERR_INVALID_ARG;
     }
     nt += v[i].n_terms; np += v[i].n_postings; ntb += v[i].n_tb; ntok += v[i].n_tokens; ndrop += v[i].n_dropped;
+    npb += v[i].n_pb;
   }
-  const uint64_t size = 64 + 8 * (nt + 1) + pad8(ntb) + pad8(4 * nt) + 8 * nt + 8 * (nt + 1) + 2 * pad8(4 * np);
+  const bool vb = v[0].vb;
+  const uint64_t size = 64 + 8 * (nt + 1) + pad8(ntb) + pad8(4 * nt) + 8 * nt + 8 * (nt + 1) +
+                        (vb ? pad8(npb) : 2 * pad8(4 * np));
   *n_out = size;
   if (!out) return WJ_OK;
   if (cap < size) return WJ_ERR_BUFFER_TOO_SMALL;
   memset(out, 0, size);
   uint64_t h[8];
-  memcpy(h, "WJINV001", 8);
-  h[1] = v[0].n_docs; h[2] = ntok; h[3] = ndrop; h[4] = nt; h[5] = np; h[6] = ntb; h[7] = 0;
+  memcpy(h, vb ? "WJINV002" : "WJINV001", 8);
+  h[1] = v[0].n_docs; h[2] = ntok; h[3] = ndrop; h[4] = nt; h[5] = np; h[6] = ntb; h[7] = vb ? npb : 0;
   memcpy(out, h, 64);
   uint64_t p = 64;
   uint64_t* term_off = (uint64_t*)(out + p); p += 8 * (nt + 1);
@@ -1489,8 +1533,15 @@ int index_merge_serialized(int32_t k, const uint8_t* const* slices, const uint64
   uint32_t* df = (uint32_t*)(out + p); p += pad8(4 * nt);
   uint64_t* cf = (uint64_t*)(out + p); p += 8 * nt;
   uint64_t* post_off = (uint64_t*)(out + p); p += 8 * (nt + 1);
-  uint32_t* docid = (uint32_t*)(out + p); p += pad8(4 * np);
-  uint32_t* tf = (uint32_t*)(out + p);
+  uint32_t* docid = nullptr;
+  uint32_t* tf = nullptr;
+  uint8_t* code = nullptr;
+  if (vb) {
+    code = out + p;
+  } else {
+    docid = (uint32_t*)(out + p); p += pad8(4 * np);
+    tf = (uint32_t*)(out + p);
+  }
   std::vector<uint64_t> cur(k, 0);
   auto term_less = [&](int a, int b) {
     const SliceView &x = v[a], &y = v[b];
@@ -1516,8 +1567,12 @@ int index_merge_serialized(int32_t k, const uint8_t* const* slices, const uint64
     cf[t] = x.cf[j];
     post_off[t] = po;
     const uint64_t a = x.post_off[j], b = x.post_off[j + 1];
-    memcpy(docid + po, x.docid + a, 4 * (b - a));
-    memcpy(tf + po, x.tf + a, 4 * (b - a));
+    if (vb) {  // a list's code is self-contained (its first gap is the docID): copy it
+      memcpy(code + po, x.code + a, b - a);
+    } else {
+      memcpy(docid + po, x.docid + a, 4 * (b - a));
+      memcpy(tf + po, x.tf + a, 4 * (b - a));
+    }
     po += b - a;
   }
   term_off[nt] = to;

@@ -187,7 +187,8 @@ struct NcclTransport : Transport {
 // n_docs (global in every slice).
 struct SliceView {
   const uint8_t* base;
-  uint64_t n_docs, n_tokens, n_dropped, n_terms, n_postings, n_tb;
+  bool vb;  // WJINV002: post_off in bytes into `code` (reading S19)
+  uint64_t n_docs, n_tokens, n_dropped, n_terms, n_postings, n_tb, n_pb;
   const uint64_t* term_off;
   const uint8_t* term_bytes;
   const uint32_t* df;
@@ -195,23 +196,33 @@ struct SliceView {
   const uint64_t* post_off;
   const uint32_t* docid;
   const uint32_t* tf;
+  const uint8_t* code;
 };
 
 inline uint64_t pad8(uint64_t x) { return (x + 7) & ~7ull; }
 
 inline bool parse_slice(const uint8_t* b, uint64_t size, SliceView& v) {
-  if (size < 64 || memcmp(b, "WJINV001", 8) != 0) return false;
+  if (size < 64) return false;
+  v.vb = memcmp(b, "WJINV002", 8) == 0;
+  if (!v.vb && memcmp(b, "WJINV001", 8) != 0) return false;
   const uint64_t* h = (const uint64_t*)b;
   v.base = b;
   v.n_docs = h[1]; v.n_tokens = h[2]; v.n_dropped = h[3]; v.n_terms = h[4]; v.n_postings = h[5]; v.n_tb = h[6];
+  v.n_pb = v.vb ? h[7] : 0;
   uint64_t p = 64;
   v.term_off = (const uint64_t*)(b + p); p += 8 * (v.n_terms + 1);
   v.term_bytes = b + p; p += pad8(v.n_tb);
   v.df = (const uint32_t*)(b + p); p += pad8(4 * v.n_terms);
   v.cf = (const uint64_t*)(b + p); p += 8 * v.n_terms;
   v.post_off = (const uint64_t*)(b + p); p += 8 * (v.n_terms + 1);
-  v.docid = (const uint32_t*)(b + p); p += pad8(4 * v.n_postings);
-  v.tf = (const uint32_t*)(b + p); p += pad8(4 * v.n_postings);
+  v.docid = v.tf = nullptr;
+  v.code = nullptr;
+  if (v.vb) {
+    v.code = b + p; p += pad8(v.n_pb);
+  } else {
+    v.docid = (const uint32_t*)(b + p); p += pad8(4 * v.n_postings);
+    v.tf = (const uint32_t*)(b + p); p += pad8(4 * v.n_postings);
+  }
   return p == size;
 }
 

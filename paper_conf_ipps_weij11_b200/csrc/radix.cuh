@@ -170,6 +170,19 @@ __device__ __forceinline__ uint32_t digit_peers(uint32_t d, bool valid) {
   return peers;
 }
 
+// Same result through a per-warp table of 256 lane masks in shared memory (all zero on entry and
+// on exit): one shared atomic OR per lane instead of 8 ballots.
+__device__ __forceinline__ uint32_t digit_peers_smem(uint32_t* bins, uint32_t d, bool valid) {
+  const uint32_t lane = lane_id();
+  if (valid) atomicOr(&bins[d], 1u << lane);
+  __syncwarp();
+  const uint32_t peers = valid ? bins[d] : 0u;
+  __syncwarp();
+  if (valid && (peers & ((1u << lane) - 1u)) == 0) bins[d] = 0u;  // the lowest peer clears
+  __syncwarp();
+  return peers;
+}
+
 template <typename K>
 __global__ void __launch_bounds__(kOsThreads, 4) k_os_pass(const K* __restrict__ kin, const uint32_t* __restrict__ vin,
                                                         K* __restrict__ kout, uint32_t* __restrict__ vout, uint64_t n,
@@ -620,6 +633,7 @@ __global__ void __launch_bounds__(kDsThreads, 2) k_rs_down2(const K* __restrict_
   extern __shared__ __align__(128) unsigned char os_smem[];
   __shared__ __align__(8) uint64_t bar[2];
   __shared__ uint32_t wcnt[kDsWarps][256];
+  __shared__ uint32_t wbins[kDsWarps][256];
   __shared__ uint32_t dig_off[256];
   __shared__ uint32_t dig_glob[256];
   __shared__ uint32_t run_base[256];
@@ -651,7 +665,7 @@ __global__ void __launch_bounds__(kDsThreads, 2) k_rs_down2(const K* __restrict_
     mbar_init(&bar[1], 1);
     fence_mbar_init();
   }
-  for (int i = threadIdx.x; i < kDsWarps * 256; i += kDsThreads) (&wcnt[0][0])[i] = 0;
+  for (int i = threadIdx.x; i < kDsWarps * 256; i += kDsThreads) (&wcnt[0][0])[i] = (&wbins[0][0])[i] = 0;
   if (threadIdx.x < 256) run_base[threadIdx.x] = offs[(uint64_t)threadIdx.x * gridDim.x + blockIdx.x];
   __syncthreads();
   if (threadIdx.x == 0) issue(0, lo);
@@ -673,7 +687,9 @@ __global__ void __launch_bounds__(kDsThreads, 2) k_rs_down2(const K* __restrict_
       const bool valid = li < tn && !rs_hole<K, HOLES>(kv, kmask);
       vmask |= (valid ? 1u : 0u) << k;
       dg[k] = (uint32_t)((rs_dkey<K, MASK>(kv, kmask) >> shift) & 255u);
-      rank[k] = digit_peers(dg[k], valid);
+      // 64-bit keys (all distinct: new-term sort): shared-memory masks; 32-bit keys (Zipf-skewed
+      // ranks, many equal digits per warp -> atomic conflicts): ballots
+      rank[k] = sizeof(K) == 8 ? digit_peers_smem(wbins[w], dg[k], valid) : digit_peers(dg[k], valid);
     }
 #pragma unroll
     for (int k = 0; k < kDsItems; ++k) {

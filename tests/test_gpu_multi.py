@@ -23,7 +23,7 @@ if not torch.cuda.is_available():  # pragma: no cover
 import paper_conf_ipps_weij11_b200 as wj  # noqa: E402
 
 
-def dist_index(text, doc_off, K, cuts=None, queries=()):
+def dist_index(text, doc_off, K, cuts=None, queries=(), vbyte=False):
     off = np.asarray(doc_off, dtype=np.uint64)
     text = np.asarray(text, dtype=np.uint8)
     n = len(off) - 1
@@ -35,7 +35,7 @@ def dist_index(text, doc_off, K, cuts=None, queries=()):
 
     def run(r):
         try:
-            with wj.Index(device=0, rank=r, world=K, hub=hub, own_stream=True) as ix:
+            with wj.Index(device=0, rank=r, world=K, hub=hub, own_stream=True, vbyte=vbyte) as ix:
                 for a, b in zip(cuts, cuts[1:]):
                     # rank r's contiguous document range of this chunk (rank order = DocID order)
                     bounds = [a + (b - a) * i // K for i in range(K + 1)]
@@ -128,3 +128,11 @@ def test_loopback_single_rank():
     text, off = gen.generate(gen.CONFIGS[1].scaled(vocab=3000))
     slices, _ = dist_index(text, off, 1, cuts=[0, 500, 1000])
     assert slices[0] == oracle.index_bytes(text, off)
+
+
+@pytest.mark.parametrize("K", [2, 3])
+def test_loopback_vbyte_merge(K):
+    # compressed slices (WJINV002) merge by concatenating each list's self-contained code
+    text, off = gen.generate(gen.CONFIGS[1])
+    slices, _ = dist_index(text, off, K, cuts=[0, 500, 1000], vbyte=True)
+    assert wj.merge_serialized(slices) == oracle.index_bytes(text, off, vbyte=True)

@@ -23,8 +23,8 @@ if not torch.cuda.is_available():  # pragma: no cover
 import paper_conf_ipps_weij11_b200 as wj  # noqa: E402
 
 
-def gpu_index(text, doc_off, cuts=None, device_input=False):
-    with wj.Index(device=0) as ix:
+def gpu_index(text, doc_off, cuts=None, device_input=False, vbyte=False):
+    with wj.Index(device=0, vbyte=vbyte) as ix:
         off = np.asarray(doc_off, dtype=np.uint64)
         text = np.asarray(text, dtype=np.uint8)
         cuts = cuts or [0, len(off) - 1]
@@ -344,3 +344,63 @@ def test_multichunk_config3_shape():
     for t, oo in parts:
         o.add(t, oo)
     assert_same_index(got, o.serialize())
+
+
+# ------------------------------------------------------------------ f1: d-gap + vbyte code
+def test_vbyte_golden_and_config1():
+    docs, _, _ = load_corpus("corpus_edges.txt")
+    text, off = gen.from_docs(docs)
+    assert gpu_index(text, off, vbyte=True) == oracle.index_bytes(text, off, vbyte=True)
+    text, off = gen.generate(gen.CONFIGS[1])
+    want = oracle.index_bytes(text, off, vbyte=True)
+    assert gpu_index(text, off, vbyte=True) == want
+    assert gpu_index(text, off, cuts=[0, 1, 333, 334, 1000], vbyte=True) == want
+
+
+@pytest.mark.parametrize("seed", [0, 1])
+def test_vbyte_multi_tile_large_gaps(seed):
+    # > 4096 postings (several encode tiles), lists spanning tiles, gaps of 1..5 bytes, big tf
+    rng = np.random.default_rng(seed)
+    docs = []
+    for d in range(30000):
+        words = [b"w%d" % int(x) for x in rng.zipf(1.3, size=int(rng.integers(0, 12))) if x < 10 ** 6]
+        if d % 997 == 0:
+            words += [b"many"] * int(rng.integers(100, 400))
+        docs.append(b" ".join(words))
+    text, off = gen.from_docs(docs)
+    want = oracle.index_bytes(text, off, vbyte=True)
+    got = gpu_index(text, off, vbyte=True)
+    if got != want:
+        assert wjformat.parse(got).as_dict() == wjformat.parse(want).as_dict()
+    assert got == want
+
+
+def test_vbyte_config_shapes_and_read_postings():
+    cfg = gen.CONFIGS[4].scaled(chunk_bytes=8 << 20, vocab=300_000)
+    text, off = gen.generate(cfg)
+    o = oracle.Oracle()
+    o.add(text, off)
+    with wj.Index(vbyte=True) as ix:
+        ix.add_stream(text, off)
+        ix.finalize()
+        got = ix.serialize()
+        for q in (b"the", b"zzzzzzzz", b"a"):
+            ref = o.postings(q)
+            ans = ix.read_postings(q)
+            assert (ans is None) == (ref is None)
+            if ref is not None:
+                assert np.array_equal(ans[0], ref[0]) and np.array_equal(ans[1], ref[1])
+    assert got == o.serialize(vbyte=True)
+
+
+def test_vbyte_empty_index():
+    text, off = gen.from_docs([b"", b"...", b""])
+    assert gpu_index(text, off, vbyte=True) == oracle.index_bytes(text, off, vbyte=True)
+
+
+def test_vbyte_four_byte_gaps():
+    # 2.7 M empty documents between two postings: 4-byte gap and first-posting codes
+    docs = [b"a b"] + [b""] * 2_700_000 + [b"a c", b"c"]
+    text, off = gen.from_docs(docs)
+    want = oracle.index_bytes(text, off, vbyte=True)
+    assert gpu_index(text, off, vbyte=True) == want
