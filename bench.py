@@ -196,6 +196,8 @@ def main():
     ap.add_argument("--chunk-bytes", type=int, default=None, help="override bytes per GPU (debug)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--e2e-chunks", type=int, default=4,
+                    help="e2e: feed the step as this many pinned host chunks through the host pipeline")
     ap.add_argument("--vbyte", action="store_true",
                     help="also encode the postings as d-gaps + variable-byte code (SURVEY 8(f1), WJINV002)")
     args = ap.parse_args()
@@ -298,13 +300,35 @@ def main():
     phases = {k: (s1["phase_ms"][k] - s0["phase_ms"][k]) / args.steps for k in wj.PHASES}
     kernels = {k: {"ms_per_step": kms[k] / args.steps, "launches_per_step": kcnt[k] / args.steps} for k in wj.KERNELS}
 
-    # e2e through the public API with host buffers: H2D of the chunk inside, D2H of the whole index
+    # e2e through the public API with host buffers: H2D of the chunk inside, D2H of the whole index.
+    # --e2e-chunks S > 1 feeds the step's text as S pinned host chunks to a context with the host
+    # pipeline (Fig. 9: the copy of chunk c+1 overlaps the indexing of chunk c).
     e2e = None
     if args.e2e_steps > 0:
-        ix.reset()
-        ix.add_stream(text_h, off_h)
-        ix.finalize()
-        out_bytes = ix.serialized_size()
+        S = max(1, args.e2e_chunks)
+        ixe = ix
+        if S > 1:
+            nid2 = [None]
+            if world > 1 or force_dist:  # a fresh communicator for the second context
+                nid2 = [wj.nccl_unique_id() if rank == 0 else None]
+                if world > 1:
+                    dist.broadcast_object_list(nid2, src=0)
+            ixe = wj.Index(device=local, rank=rank, world=world, vbyte=args.vbyte, pipeline=True, nccl_id=nid2[0])
+        nd = len(doc_off) - 1
+        cuts = sorted({0, nd} | {int(np.searchsorted(doc_off, T * k // S)) for k in range(1, S)})
+        parts = []
+        for a, b in zip(cuts, cuts[1:]):
+            o = torch.from_numpy((doc_off[a:b + 1] - doc_off[a]).astype(np.int64)).pin_memory()
+            parts.append((text_h[int(doc_off[a]):int(doc_off[b])], o))
+
+        def e2e_step():
+            ixe.reset()
+            for t, o in parts:
+                ixe.add_stream(t, o)
+            ixe.finalize()
+
+        e2e_step()
+        out_bytes = ixe.serialized_size()
         out_h = torch.empty(out_bytes, dtype=torch.uint8, pin_memory=True)
         torch.cuda.synchronize()
         if world > 1:
@@ -313,10 +337,8 @@ def main():
         f1 = torch.cuda.Event(enable_timing=True)
         f0.record()
         for _ in range(args.e2e_steps):
-            ix.reset()
-            ix.add_stream(text_h, off_h)
-            ix.finalize()
-            ix.serialize_into(out_h.data_ptr(), out_bytes)
+            e2e_step()
+            ixe.serialize_into(out_h.data_ptr(), out_bytes)
         f1.record()
         torch.cuda.synchronize()
         ems = f0.elapsed_time(f1) / args.e2e_steps
@@ -325,8 +347,12 @@ def main():
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ems = float(t.item())
         e2e = {"value": total_bytes / (ems / 1e3) / 1e6, "unit": "MB/s", "ms_per_step": ems,
-               "h2d_bytes_per_step": T + 8 * len(doc_off), "d2h_bytes_per_step": out_bytes,
-               "what": "index_add_stream(pinned host text + doc_off) + index_finalize + index_serialize to pinned host"}
+               "h2d_bytes_per_step": T + 8 * (nd + len(parts)), "d2h_bytes_per_step": out_bytes,
+               "host_chunks": len(parts),
+               "what": ("index_add_stream(pinned host text + doc_off%s) + index_finalize + index_serialize to pinned host"
+                        % (f", {len(parts)} chunks, WJ_FLAG_HOST_PIPELINE" if len(parts) > 1 else ""))}
+        if ixe is not ix:
+            ixe.close()
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

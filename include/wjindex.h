@@ -53,6 +53,12 @@ typedef enum {
 #define WJ_FLAG_VBYTE 0x4u     /* finalize also encodes every postings list as d-gaps + variable-   */
                                /* byte code (reading S19) and            */
                                /* index_serialize writes the compressed file "WJINV002"             */
+#define WJ_FLAG_HOST_PIPELINE 0x8u /* host-memory chunks are double-buffered: index_add_stream      */
+                               /* enqueues the chunk's copy on a copy stream and indexes the        */
+                               /* PREVIOUS host chunk meanwhile (Fig. 9 pipeline);       */
+                               /* finalize (or a device-memory chunk) drains the pending chunk;     */
+                               /* index_reset drops it.  Errors of a chunk may surface one call     */
+                               /* late.  Use pinned host memory for the copy to overlap.            */
 
 typedef struct wj_index wj_index; /* opaque; all index state is owned by the library */
 

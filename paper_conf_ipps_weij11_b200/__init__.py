@@ -33,6 +33,7 @@ EXPORTS = ["index_init", "index_add_stream", "index_finalize", "index_read_posti
            "index_destroy"]
 WJ_FLAG_LOOPBACK = 2
 WJ_FLAG_VBYTE = 4
+WJ_FLAG_HOST_PIPELINE = 8
 
 
 class WJError(RuntimeError):
@@ -142,14 +143,16 @@ class Index:
 
     def __init__(self, device: int = 0, stream=None, profile: bool = False, rank: int = 0, world: int = 1,
                  nccl_id: bytes | None = None, hub: "LoopbackHub | None" = None, own_stream: bool = False,
-                 vbyte: bool = False):
+                 vbyte: bool = False, pipeline: bool = False):
         """world > 1: pass nccl_id (128 bytes from nccl_unique_id(), broadcast by the caller) or a
         LoopbackHub shared by `world` contexts of this process (one host thread each).
         vbyte: finalize also builds the d-gap + variable-byte postings code; serialize() then
-        returns the compressed file WJINV002."""
+        returns the compressed file WJINV002.
+        pipeline: host chunks are copied on a copy stream while the previous one is indexed
+        (Fig. 9); keep each host buffer unchanged until the next call returns."""
         self._lib = load_library()
         flags = (WJ_FLAG_PROFILE if profile else 0) | (WJ_FLAG_LOOPBACK if hub is not None else 0) | (
-            WJ_FLAG_VBYTE if vbyte else 0)
+            WJ_FLAG_VBYTE if vbyte else 0) | (WJ_FLAG_HOST_PIPELINE if pipeline else 0)
         self._nid = ctypes.create_string_buffer(bytes(nccl_id), 128) if nccl_id is not None else None
         uid = hub._h if hub is not None else (ctypes.cast(self._nid, ctypes.c_void_p) if self._nid is not None else None)
         if own_stream:
@@ -188,7 +191,9 @@ class Index:
         """Append one chunk: text (u8) and doc_off (u64, n_docs+1); host or device buffers."""
         tp, tn, tk = _ptr_len(text, np.uint8)
         dp, dn, dk = _ptr_len(doc_off, np.uint64)
-        self._keep = [tk, dk]  # buffers must stay alive until the next call (stream-ordered)
+        # buffers must stay alive until the next call returns (stream-ordered; with pipeline=True
+        # a host chunk is read by the copy engine until the following call has indexed it)
+        self._keep = (self._keep + [tk, dk])[-4:]
         self._check(self._lib.index_add_stream(self._h, tp, tn, dp, dn - 1))
 
     def finalize(self):

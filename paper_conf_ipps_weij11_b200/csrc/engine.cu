@@ -90,6 +90,16 @@ struct wj_index {
   int rank = 0, world = 1;
   cudaStream_t st = nullptr;
   bool own_stream = false;
+  // f3 host-streamed pipelining (WJ_FLAG_HOST_PIPELINE; Fig. 9): a host chunk is copied
+  // on the copy stream `cs` into one of two staging slots while the previous chunk is indexed
+  bool pipeline = false;
+  cudaStream_t cs = nullptr;
+  DevBuf pipe_text[2], pipe_off[2];
+  cudaEvent_t pipe_copied[2] = {nullptr, nullptr}, pipe_done[2] = {nullptr, nullptr};
+  bool pipe_used[2] = {false, false};
+  bool pend = false;
+  int pend_slot = 0, next_slot = 0;
+  uint64_t pend_bytes = 0, pend_nd = 0;
   uint32_t flags = 0;
   std::string err;
   bool finalized = false;
@@ -296,6 +306,8 @@ struct wj_index {
 
   // ---------------------------------------------------------------- init / reset
   void reset_state() {
+    if (cs) WJ_CUDA_CHECK(cudaStreamSynchronize(cs));
+    pend = false;  // a pending (copied, not yet indexed) host chunk is dropped
     collect_phases();
     chunk_tok.clear();
     chunk_C.clear();
@@ -620,6 +632,48 @@ struct wj_index {
     });
     chunk_tok.push_back(tok_start);
     chunk_C.push_back((uint32_t)C);
+  }
+
+  // ---------------------------------------------------------------- f3: host pipeline
+  // Index the pending host chunk (its copy was enqueued by the previous call).
+  void drain() {
+    if (!pend) return;
+    pend = false;
+    const int s = pend_slot;
+    WJ_CUDA_CHECK(cudaStreamWaitEvent(st, pipe_copied[s], 0));
+    add_chunk(pipe_text[s].p, pend_bytes, (const uint64_t*)pipe_off[s].p, pend_nd);
+    WJ_CUDA_CHECK(cudaEventRecord(pipe_done[s], st));
+    pipe_used[s] = true;
+  }
+
+  // Host chunk with WJ_FLAG_HOST_PIPELINE: validate doc_off, enqueue its copy on the copy stream,
+  // then index the previous chunk on the context stream while the copy engine moves this one.
+  void add_stream_pipelined(const void* bytes, uint64_t n_bytes, const uint64_t* doc_off, uint64_t nd) {
+    if (doc_off[0] != 0 || doc_off[nd] != n_bytes) throw StatusError{WJ_ERR_INVALID_ARG, "doc_off[0] must be 0 and doc_off[n_docs] == n_bytes"};
+    for (uint64_t i = 0; i < nd; ++i)
+      if (doc_off[i] > doc_off[i + 1]) throw StatusError{WJ_ERR_INVALID_ARG, "doc_off must be non-decreasing"};
+    const int s = next_slot;
+    if (pipe_used[s]) WJ_CUDA_CHECK(cudaStreamWaitEvent(cs, pipe_done[s], 0));  // slot consumed (chunk c-2)
+    uint8_t* t = buf<uint8_t>(pipe_text[s], n_bytes + 16);
+    uint64_t* o = buf<uint64_t>(pipe_off[s], nd + 1);
+    if (n_bytes) WJ_CUDA_CHECK(cudaMemcpyAsync(t, bytes, n_bytes, cudaMemcpyHostToDevice, cs));
+    WJ_CUDA_CHECK(cudaMemcpyAsync(o, doc_off, (nd + 1) * 8, cudaMemcpyHostToDevice, cs));
+    WJ_CUDA_CHECK(cudaEventRecord(pipe_copied[s], cs));
+    next_slot ^= 1;
+    drain();
+    pend = true;
+    pend_slot = s;
+    pend_bytes = n_bytes;
+    pend_nd = nd;
+  }
+
+  void add_stream(const void* bytes, uint64_t n_bytes, const uint64_t* doc_off, uint64_t nd) {
+    if (pipeline && !is_device_ptr(doc_off) && (n_bytes == 0 || !is_device_ptr(bytes))) {
+      add_stream_pipelined(bytes, n_bytes, doc_off, nd);
+      return;
+    }
+    drain();
+    add_chunk(bytes, n_bytes, doc_off, nd);
   }
 
   void add_chunk(const void* bytes, uint64_t n_bytes, const uint64_t* doc_off_in, uint64_t nd) {
@@ -1017,6 +1071,7 @@ struct wj_index {
 
   // ---------------------------------------------------------------- finalize
   void finalize() {
+    drain();
     const uint64_t NE = n_elems;  // stream elements (tokens, aggregated hot entries, holes)
     uint32_t* ro = buf<uint32_t>(rank_of, V);
     uint32_t* ta = buf<uint32_t>(term_at, V);
@@ -1216,7 +1271,7 @@ extern "C" {
 int index_init(wj_index** out, const wj_config* cfg) {
   if (!out || !cfg) return WJ_ERR_INVALID_ARG;
   *out = nullptr;
-  if (cfg->world < 1 || cfg->world > 1024 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~(WJ_FLAG_PROFILE | WJ_FLAG_LOOPBACK | WJ_FLAG_VBYTE)) || cfg->reserved) {
+  if (cfg->world < 1 || cfg->world > 1024 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~(WJ_FLAG_PROFILE | WJ_FLAG_LOOPBACK | WJ_FLAG_VBYTE | WJ_FLAG_HOST_PIPELINE)) || cfg->reserved) {
     g_init_err = "invalid config";
     return WJ_ERR_INVALID_ARG;
   }
@@ -1241,6 +1296,7 @@ int index_init(wj_index** out, const wj_config* cfg) {
   ix->world = cfg->world;
   ix->flags = cfg->flags;
   ix->vbyte = (cfg->flags & WJ_FLAG_VBYTE) != 0;
+  ix->pipeline = (cfg->flags & WJ_FLAG_HOST_PIPELINE) != 0;
   int rc = guarded(ix, [&]() {
     if (cfg->stream) {
       ix->st = (cudaStream_t)cfg->stream;
@@ -1249,6 +1305,13 @@ int index_init(wj_index** out, const wj_config* cfg) {
       ix->own_stream = true;
     }
     WJ_CUDA_CHECK(cudaHostAlloc(&ix->h_scal, 16 * sizeof(uint64_t), cudaHostAllocDefault));
+    if (ix->pipeline) {
+      WJ_CUDA_CHECK(cudaStreamCreateWithFlags(&ix->cs, cudaStreamNonBlocking));
+      for (int i = 0; i < 2; ++i) {
+        WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->pipe_copied[i], cudaEventDisableTiming));
+        WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->pipe_done[i], cudaEventDisableTiming));
+      }
+    }
     if (const char* e = getenv("WJ_HOT_MIN_BYTES")) ix->hot_min_bytes = strtoull(e, nullptr, 10);
     if (cfg->world > 1 || cfg->nccl_unique_id) {  // a transport at world 1 runs the same distributed path
       try {
@@ -1302,7 +1365,7 @@ int index_add_stream(wj_index* ix, const void* bytes, uint64_t n_bytes, const ui
     if (!doc_off || (n_bytes && !bytes)) throw StatusError{WJ_ERR_INVALID_ARG, "NULL bytes or doc_off"};
     if (n_bytes >= 0xFFFFFFFFull) throw StatusError{WJ_ERR_INVALID_ARG, "n_bytes must be < 2^32 per call"};
     if (n_docs == 0 && n_bytes != 0) throw StatusError{WJ_ERR_INVALID_ARG, "n_bytes > 0 with no documents"};
-    ix->add_chunk(bytes, n_bytes, doc_off, n_docs);
+    ix->add_stream(bytes, n_bytes, doc_off, n_docs);
     return WJ_OK;
   });
 }
@@ -1584,7 +1647,15 @@ void index_destroy(wj_index* ix) {
   if (!ix) return;
   cudaSetDevice(ix->device);
   if (ix->st) cudaStreamSynchronize(ix->st);
+  if (ix->cs) cudaStreamSynchronize(ix->cs);
   ix->free_all();
+  for (int i = 0; i < 2; ++i) {
+    for (DevBuf* b : {&ix->pipe_text[i], &ix->pipe_off[i]})
+      if (b->p) cudaFree(b->p);
+    if (ix->pipe_copied[i]) cudaEventDestroy(ix->pipe_copied[i]);
+    if (ix->pipe_done[i]) cudaEventDestroy(ix->pipe_done[i]);
+  }
+  if (ix->cs) cudaStreamDestroy(ix->cs);
   delete ix->xport;
   for (auto e : ix->ev_pool) cudaEventDestroy(e);
   if (ix->h_scal) cudaFreeHost(ix->h_scal);

@@ -136,3 +136,35 @@ def test_loopback_vbyte_merge(K):
     text, off = gen.generate(gen.CONFIGS[1])
     slices, _ = dist_index(text, off, K, cuts=[0, 500, 1000], vbyte=True)
     assert wj.merge_serialized(slices) == oracle.index_bytes(text, off, vbyte=True)
+
+
+def test_loopback_host_pipeline():
+    # every rank defers its host chunks by one call; collectives still pair up in chunk order
+    text, off = gen.generate(gen.CONFIGS[1])
+    off = np.asarray(off, dtype=np.uint64)
+    K = 2
+    hub = wj.LoopbackHub(K)
+    slices = [None] * K
+    errors = []
+
+    def run(r):
+        try:
+            with wj.Index(device=0, rank=r, world=K, hub=hub, own_stream=True, pipeline=True) as ix:
+                for a, b in zip([0, 300, 700], [300, 700, 1000]):
+                    bounds = [a + (b - a) * i // K for i in range(K + 1)]
+                    lo, hi = bounds[r], bounds[r + 1]
+                    ix.add_stream(text[int(off[lo]):int(off[hi])].copy(), off[lo:hi + 1] - off[lo])
+                ix.finalize()
+                slices[r] = ix.serialize()
+        except Exception as e:  # pragma: no cover
+            errors.append((r, e))
+            raise
+
+    th = [threading.Thread(target=run, args=(r,)) for r in range(K)]
+    for x in th:
+        x.start()
+    for x in th:
+        x.join(timeout=600)
+    hub.close()
+    assert not errors, errors
+    assert wj.merge_serialized(slices) == oracle.index_bytes(text, off)

@@ -404,3 +404,58 @@ def test_vbyte_four_byte_gaps():
     text, off = gen.from_docs(docs)
     want = oracle.index_bytes(text, off, vbyte=True)
     assert gpu_index(text, off, vbyte=True) == want
+
+
+# ------------------------------------------------------------------ f3: host-streamed pipeline
+def _chunks(text, off, cuts):
+    off = np.asarray(off, dtype=np.uint64)
+    for a, b in zip(cuts, cuts[1:]):
+        yield text[int(off[a]):int(off[b])], off[a:b + 1] - off[a]
+
+
+@pytest.mark.parametrize("pinned", [True, False])
+def test_pipeline_host_chunks(pinned):
+    text, off = gen.generate(gen.CONFIGS[1])
+    want = oracle.index_bytes(text, off)
+    cuts = [0, 100, 100, 101, 400, 999, 1000]  # includes a chunk with no documents
+    with wj.Index(pipeline=True) as ix:
+        for t, o in _chunks(text, off, cuts):
+            if pinned:
+                t = torch.from_numpy(t.copy()).pin_memory()
+                o = torch.from_numpy(o.astype(np.int64)).pin_memory()
+            ix.add_stream(t, o)
+        ix.finalize()
+        got = ix.serialize()
+        assert ix.stats()["n_docs"] == 1000
+    assert_same_index(got, want)
+
+
+def test_pipeline_mixed_host_device_and_vbyte():
+    text, off = gen.generate(gen.CONFIGS[1].scaled(vocab=50_000))
+    cuts = [0, 250, 500, 750, 1000]
+    with wj.Index(pipeline=True, vbyte=True) as ix:
+        for i, (t, o) in enumerate(_chunks(text, off, cuts)):
+            if i == 2:  # a device chunk drains the pending host chunk first (DocID order)
+                t = torch.from_numpy(t.copy()).cuda()
+                o = torch.from_numpy(o.astype(np.int64)).cuda()
+            ix.add_stream(t, o)
+        ix.finalize()
+        got = ix.serialize()
+    assert got == oracle.index_bytes(text, off, vbyte=True)
+
+
+def test_pipeline_reset_drops_pending_and_errors_at_call():
+    text, off = gen.generate(gen.CONFIGS[1])
+    with wj.Index(pipeline=True) as ix:
+        t, o = next(_chunks(text, off, [0, 300]))
+        ix.add_stream(t, o)  # copied, not yet indexed
+        ix.reset()           # dropped
+        bad = o.copy()
+        bad[5], bad[6] = bad[6], bad[5] + 1
+        with pytest.raises(wj.WJError):
+            ix.add_stream(t, bad)  # doc_off validated at the call
+        for t, o in _chunks(text, off, [0, 500, 1000]):
+            ix.add_stream(t, o)
+        ix.finalize()
+        got = ix.serialize()
+    assert_same_index(got, oracle.index_bytes(text, off))
