@@ -231,7 +231,8 @@ def main():
         nid = [wj.nccl_unique_id() if rank == 0 else None]
         if world > 1:
             dist.broadcast_object_list(nid, src=0)
-        ix = wj.Index(device=local, profile=True, rank=rank, world=world, nccl_id=nid[0], vbyte=args.vbyte)
+        ix = wj.Index(device=local, profile=True, rank=rank, world=world, nccl_id=nid[0], vbyte=args.vbyte,
+                      balanced=world > 1)
     else:
         ix = wj.Index(device=local, profile=True, vbyte=args.vbyte)
 
@@ -313,7 +314,8 @@ def main():
                 nid2 = [wj.nccl_unique_id() if rank == 0 else None]
                 if world > 1:
                     dist.broadcast_object_list(nid2, src=0)
-            ixe = wj.Index(device=local, rank=rank, world=world, vbyte=args.vbyte, pipeline=True, nccl_id=nid2[0])
+            ixe = wj.Index(device=local, rank=rank, world=world, vbyte=args.vbyte, pipeline=True, nccl_id=nid2[0],
+                           balanced=world > 1)
         nd = len(doc_off) - 1
         cuts = sorted({0, nd} | {int(np.searchsorted(doc_off, T * k // S)) for k in range(1, S)})
         parts = []
@@ -368,7 +370,7 @@ def main():
                        "postings_per_gpu": P, "l2": "no flush: 1 GiB input per step > 126 MB L2",
                        "postings_format": "vbyte d-gaps (WJINV002)" if args.vbyte else "u32 docid + u32 tf (WJINV001)",
                        "parallelism": "single GPU" if world == 1 else
-                       f"{world} ranks: document ranges, trie collections b mod {world}, NCCL all-to-all-v"},
+                       f"{world} ranks: document ranges, trie collections bin-packed by sampled load (P:212), NCCL all-to-all-v"},
             "exchange_bytes_per_step": (s1["exchange_bytes"]),
             "mib_per_s": total_bytes / (ms / 1e3) / 2**20,
             "tokens_per_s": N * world / (ms / 1e3),

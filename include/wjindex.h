@@ -59,6 +59,10 @@ typedef enum {
                                /* finalize (or a device-memory chunk) drains the pending chunk;     */
                                /* index_reset drops it.  Errors of a chunk may surface one call     */
                                /* late.  Use pinned host memory for the copy to overlap.            */
+#define WJ_FLAG_BALANCED_OWNERS 0x10u /* world > 1: instead of b mod K, the first chunk's   */
+                               /* 1 MiB samples are all-gathered and every rank bin-packs   */
+                               /* the trie collections by sampled token count; the map is  */
+                               /* kept for the context's lifetime, also across reset       */
 
 typedef struct wj_index wj_index; /* opaque; all index state is owned by the library */
 
@@ -202,6 +206,15 @@ void index_loopback_destroy(void* hub);
  * index_serialize.  WJ_ERR_INVALID_ARG if a slice does not parse or n_docs differ. */
 int index_merge_serialized(int32_t k, const uint8_t* const* slices, const uint64_t* sizes, uint8_t* out, uint64_t cap,
                            uint64_t* n_out);
+
+/* Host helper (no device): the balanced owner map's bin packing, exposed for tests.  Items (trie
+ * collections) by count desc, index asc on ties, each to the least-loaded rank (lowest on ties);
+ * count-0 items keep i mod world.  WJ_ERR_INVALID_ARG on NULL or world < 1. */
+int index_balance_owners(const uint64_t* counts, uint32_t n, int32_t world, uint32_t* owner);
+
+/* Owner rank of every trie collection (out: n >= 17613 entries): b mod world, or the balanced map
+ * once the first chunk has built it (WJ_FLAG_BALANCED_OWNERS).  WJ_ERR_INVALID_ARG if n is small. */
+int index_owner_map(wj_index* ix, uint32_t* out, uint32_t n);
 
 const char* index_last_error(const wj_index* ix);
 void index_destroy(wj_index* ix);

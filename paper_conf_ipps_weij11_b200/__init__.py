@@ -29,11 +29,13 @@ N_COLLECTIONS = 17613
 
 EXPORTS = ["index_init", "index_add_stream", "index_finalize", "index_read_postings", "index_serialize",
            "index_stats", "index_reset", "index_debug_tokens", "index_debug_btree", "index_nccl_unique_id",
-           "index_loopback_create", "index_loopback_destroy", "index_merge_serialized", "index_last_error",
-           "index_destroy"]
+           "index_loopback_create", "index_loopback_destroy", "index_merge_serialized", "index_owner_map",
+           "index_balance_owners",
+           "index_last_error", "index_destroy"]
 WJ_FLAG_LOOPBACK = 2
 WJ_FLAG_VBYTE = 4
 WJ_FLAG_HOST_PIPELINE = 8
+WJ_FLAG_BALANCED_OWNERS = 16
 
 
 class WJError(RuntimeError):
@@ -108,6 +110,8 @@ def load_library():
         for f in EXPORTS:
             if f not in ("index_last_error", "index_destroy", "index_loopback_destroy"):
                 getattr(lib, f).restype = i32
+        lib.index_owner_map.argtypes = [vp, vp, u32]
+        lib.index_balance_owners.argtypes = [vp, u32, ctypes.c_int32, vp]
         lib.index_destroy.restype = None
         lib.index_loopback_destroy.restype = None
         _lib = lib
@@ -143,16 +147,18 @@ class Index:
 
     def __init__(self, device: int = 0, stream=None, profile: bool = False, rank: int = 0, world: int = 1,
                  nccl_id: bytes | None = None, hub: "LoopbackHub | None" = None, own_stream: bool = False,
-                 vbyte: bool = False, pipeline: bool = False):
+                 vbyte: bool = False, pipeline: bool = False, balanced: bool = False):
         """world > 1: pass nccl_id (128 bytes from nccl_unique_id(), broadcast by the caller) or a
         LoopbackHub shared by `world` contexts of this process (one host thread each).
         vbyte: finalize also builds the d-gap + variable-byte postings code; serialize() then
         returns the compressed file WJINV002.
         pipeline: host chunks are copied on a copy stream while the previous one is indexed
-        (Fig. 9); keep each host buffer unchanged until the next call returns."""
+        (Fig. 9); keep each host buffer unchanged until the next call returns.
+        balanced: world > 1, owners of the trie collections from a sampled bin-packing."""
         self._lib = load_library()
         flags = (WJ_FLAG_PROFILE if profile else 0) | (WJ_FLAG_LOOPBACK if hub is not None else 0) | (
-            WJ_FLAG_VBYTE if vbyte else 0) | (WJ_FLAG_HOST_PIPELINE if pipeline else 0)
+            WJ_FLAG_VBYTE if vbyte else 0) | (WJ_FLAG_HOST_PIPELINE if pipeline else 0) | (
+            WJ_FLAG_BALANCED_OWNERS if balanced else 0)
         self._nid = ctypes.create_string_buffer(bytes(nccl_id), 128) if nccl_id is not None else None
         uid = hub._h if hub is not None else (ctypes.cast(self._nid, ctypes.c_void_p) if self._nid is not None else None)
         if own_stream:
@@ -220,6 +226,12 @@ class Index:
         buf = np.empty(n.value, dtype=np.uint8)
         self._check(self._lib.index_serialize(self._h, buf.ctypes.data, n.value, ctypes.byref(n)))
         return buf.tobytes()
+
+    def owner_map(self) -> np.ndarray:
+        """Owner rank of every trie collection (b mod world, or the balanced map once built)."""
+        out = np.empty(N_COLLECTIONS, dtype=np.uint32)
+        self._check(self._lib.index_owner_map(self._h, out.ctypes.data, N_COLLECTIONS))
+        return out
 
     def serialized_size(self) -> int:
         n = ctypes.c_uint64()
@@ -322,6 +334,16 @@ def merge_serialized(slices) -> bytes:
     if rc != WJ_OK:
         raise WJError(rc, lib.index_last_error(None).decode())
     return out.tobytes()
+
+
+def balance_owners(counts, world: int) -> np.ndarray:
+    """The balanced owner map's bin packing (host) for per-collection token counts."""
+    c = np.ascontiguousarray(counts, dtype=np.uint64)
+    out = np.empty(len(c), dtype=np.uint32)
+    rc = load_library().index_balance_owners(c.ctypes.data, len(c), world, out.ctypes.data)
+    if rc != WJ_OK:
+        raise WJError(rc, "index_balance_owners")
+    return out
 
 
 def owner_of(collection: int, world: int) -> int:

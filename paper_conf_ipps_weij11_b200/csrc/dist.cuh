@@ -2,7 +2,9 @@
 //
 // Ownership: trie collection b belongs to rank b mod K — the paper's static split of collections
 // over GPUs, "assigning the trie collection TC_i with index i to the GPU whose index is given by
-// i mod N_2".  Each rank owns an exclusive slice of the dictionary.
+// i mod N_2" — or, with WJ_FLAG_BALANCED_OWNERS, to the rank a sampled
+// bin-packing picked (engine.cu build_owner_map).  Each rank owns an exclusive slice of the
+// dictionary.
 //
 // Per chunk, rank r has tokenised its own document range into a chunk table (unique terms) and a
 // (slot, docID) stream.  For every owner o it sends
@@ -20,14 +22,15 @@ namespace wj {
 // per-owner counts: block histogram in shared memory, one global atomic per (block, owner)
 constexpr int kMaxRanks = 1024;
 
-__global__ void k_owner(const uint32_t* u_bucket, uint32_t U, uint32_t K, uint32_t* owner, uint32_t* iota,
-                        uint32_t* owner_cnt) {
+__global__ void k_owner(const uint32_t* u_bucket, uint32_t U, uint32_t K, const uint32_t* owner_tab, uint32_t* owner,
+                        uint32_t* iota, uint32_t* owner_cnt) {
   __shared__ uint32_t h[kMaxRanks];
   for (uint32_t i = threadIdx.x; i < K; i += blockDim.x) h[i] = 0;
   __syncthreads();
   const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
   if (u < U) {
-    const uint32_t o = u_bucket[u] % K;
+    const uint32_t b = u_bucket[u];
+    const uint32_t o = owner_tab ? owner_tab[b] : b % K;
     owner[u] = o;
     iota[u] = u;
     atomicAdd(&h[o], 1u);

@@ -85,6 +85,26 @@ inline unsigned grid_for(uint64_t n, unsigned block) { return (unsigned)((n + bl
 
 }  // namespace
 
+// Greedy longest-processing-time bin packing (host): items by count desc (index asc on ties), each
+// to the least-loaded rank (lowest rank on ties); items with count 0 keep i mod K.
+static void lpt_owner_map(const uint64_t* count, uint32_t n, int K, uint32_t* owner) {
+  std::vector<uint32_t> order(n);
+  for (uint32_t b = 0; b < n; ++b) {
+    order[b] = b;
+    owner[b] = b % (uint32_t)K;
+  }
+  std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) { return count[a] > count[b]; });
+  std::vector<uint64_t> load(K, 0);
+  for (uint32_t b : order) {
+    if (count[b] == 0) break;
+    int best = 0;
+    for (int r = 1; r < K; ++r)
+      if (load[r] < load[best]) best = r;
+    owner[b] = (uint32_t)best;
+    load[best] += count[b];
+  }
+}
+
 struct wj_index {
   int device = 0;
   int rank = 0, world = 1;
@@ -114,6 +134,9 @@ struct wj_index {
   uint64_t table_est = 0;
   uint64_t P = 0, TB = 0, PB = 0;  // postings, term bytes, vbyte code bytes
   bool vbyte = false;              // WJ_FLAG_VBYTE
+  bool balanced = false;           // WJ_FLAG_BALANCED_OWNERS
+  bool owner_ready = false;        // owner_tab built (kept across index_reset: bound for the lifetime)
+  std::vector<uint32_t> owner_h;   // collection -> rank (host copy)
   uint64_t exchange_bytes = 0;
 
   Transport* xport = nullptr;  // world > 1
@@ -144,6 +167,7 @@ struct wj_index {
   // finalize
   DevBuf rank_of, term_at, sk1, sv1, pidx, out_doc, out_tf, post_off, df, cf, term_off, term_bytes;
   DevBuf vb_first, vb_tiles, vb_code, vb_boff;  // f1 (WJ_FLAG_VBYTE)
+  DevBuf samp_hist, owner_tab;                  // f2(i) (WJ_FLAG_BALANCED_OWNERS)
   std::vector<DevBuf> chunk_map;        // per chunk: slot -> termID (-> rank at finalize)
   std::vector<uint64_t> chunk_tok;      // per chunk: first token index in the stream
   std::vector<uint32_t> chunk_C;        // per chunk: table capacity
@@ -198,7 +222,7 @@ struct wj_index {
                      &nk_key2, &nk_val2, &aoff, &ns_tid, &ns_bucket, &ns_rank, &nlo, &nhi, &nbase, &child_off,
                      &root_idx, &scan_scr, &hist, &hist_scan, &os_hist, &os_look, &os_ctr, &kstart, &slotref, &dbg_start, &dbg_len, &dbg_off, &dbg_out, &dbg_slot,
                      &dbg_doc, &lexg, &qbuf, &qres, &rank_of, &term_at, &sk1, &sv1, &pidx, &out_doc, &out_tf,
-                     &post_off, &df, &cf, &term_off, &term_bytes, &vb_first, &vb_tiles, &vb_code, &vb_boff};
+                     &post_off, &df, &cf, &term_off, &term_bytes, &vb_first, &vb_tiles, &vb_code, &vb_boff, &samp_hist, &owner_tab};
     for (DevBuf* b : all) {
       if (b->p) cudaFree(b->p);
       b->p = nullptr;
@@ -428,8 +452,13 @@ struct wj_index {
   // Sampled popular terms of a chunk ("1MB out of every 1GB"): tokenise the first 1 MiB of
   // its documents with the same kernels, count terms, keep the <= 256 most frequent (>= 16
   // occurrences, <= 11 bytes) -> hot_kb (slot words).  Returns the number of hot terms.
-  uint32_t select_hot(const ChunkView& cv) {
+  // The paper's sample, "1MB out of every 1GB": tokenise the first 1 MiB of the chunk's
+  // documents into the chunk table and count tokens per slot (samp_cnt).  Returns the sample's
+  // kept tokens (0: no usable sample); Cs = table capacity used.
+  uint64_t sample_counts(const ChunkView& cv, uint64_t& Cs, uint64_t min_tokens) {
+    Cs = 0;
     const uint64_t S = std::min<uint64_t>(cv.n_bytes, 1ull << 20);
+    if (S == 0 || cv.n_docs == 0) return 0;
     uint64_t* sn = buf<uint64_t>(samp_n, 1);
     k_sample_docs<<<1, 32, 0, st>>>(cv.doc_off, cv.n_docs, S, nullptr, sn);
     launched();
@@ -443,10 +472,10 @@ struct wj_index {
     ChunkView sv{cv.text, S, so, nds};
     const uint64_t n_segs = (S + kSegBytes - 1) / kSegBytes;
     const uint64_t Ns = count_tokens(sv, n_segs);
-    if (Ns < 1024) return 0;
+    if (Ns < std::max<uint64_t>(min_tokens, 1)) return 0;
     uint32_t* ss = buf<uint32_t>(samp_slot, Ns + 16);
     uint32_t* sd = buf<uint32_t>(samp_doc, Ns + 16);
-    const uint64_t Cs = pow2_at_least(2 * Ns);
+    Cs = pow2_at_least(2 * Ns);
     emit_tokens(sv, n_segs, ss, sd, 0, Cs, nullptr, nullptr, false, true);
     readback(5, 1);
     if ((uint32_t)h_scal[5]) return 0;
@@ -454,6 +483,45 @@ struct wj_index {
     WJ_CUDA_CHECK(cudaMemsetAsync(cnt, 0, Cs * 4, st));
     k_sample_count<<<grid_for(Ns, 256), 256, 0, st>>>(ss, Ns, cnt);
     launched();
+    return Ns;
+  }
+
+  // f2(i): balanced owner map ("split these trie collections into N_I independent sets such
+  // that each contains almost the same number of tokens"; bound for the lifetime).  Every
+  // rank samples its first chunk, the per-collection token counts are all-gathered, and every rank
+  // runs the same greedy longest-processing-time assignment (collections by count desc, then index;
+  // each to the least-loaded rank, lowest rank on ties); unsampled collections keep b mod K.
+  void build_owner_map(const ChunkView* cv) {
+    const int K = world;
+    std::vector<uint64_t> mine(kCollections, 0), all((size_t)kCollections * K);
+    uint64_t Cs = 0;
+    if (cv && sample_counts(*cv, Cs, 1) > 0) {
+      uint64_t* h = buf<uint64_t>(samp_hist, kCollections);
+      WJ_CUDA_CHECK(cudaMemsetAsync(h, 0, kCollections * 8, st));
+      k_sample_buckets<<<grid_for(Cs, 256), 256, 0, st>>>((const Slot*)table.p, (const uint32_t*)slotref.p,
+                                                          (const uint32_t*)samp_cnt.p, (uint32_t)Cs, cv->text,
+                                                          (unsigned long long*)h);
+      launched();
+      WJ_CUDA_CHECK(cudaMemcpyAsync(mine.data(), h, kCollections * 8, cudaMemcpyDeviceToHost, st));
+      sync();
+    }
+    xport->allgather(mine.data(), kCollections, all.data(), st);
+    std::vector<uint64_t> tot(kCollections, 0);
+    for (int r = 0; r < K; ++r)
+      for (uint32_t b = 0; b < kCollections; ++b) tot[b] += all[(size_t)r * kCollections + b];
+    owner_h.assign(kCollections, 0);
+    lpt_owner_map(tot.data(), kCollections, K, owner_h.data());
+    uint32_t* d = buf<uint32_t>(owner_tab, kCollections);
+    WJ_CUDA_CHECK(cudaMemcpyAsync(d, owner_h.data(), kCollections * 4, cudaMemcpyHostToDevice, st));
+    sync();
+    owner_ready = true;
+  }
+
+  uint32_t select_hot(const ChunkView& cv) {
+    uint64_t Cs = 0;
+    const uint64_t Ns = sample_counts(cv, Cs, 1024);
+    if (Ns == 0) return 0;
+    const uint32_t* cnt = (const uint32_t*)samp_cnt.p;
     uint32_t* ck = buf<uint32_t>(samp_ck, Cs + 16);
     uint32_t* cv2 = buf<uint32_t>(samp_cv, Cs + 16);
     uint32_t* ck2 = buf<uint32_t>(samp_ck2, Cs + 16);
@@ -743,6 +811,11 @@ struct wj_index {
       tot_docs += ndall[r];
     }
     if (n_docs + tot_docs > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 documents"};
+    if (balanced && !owner_ready) {  // first chunk: sampled, bin-packed owner map (collective)
+      ChunkView cv0{text, n_bytes, off, nd};
+      build_owner_map(nd > 0 && n_bytes > 0 ? &cv0 : nullptr);
+      phase(WJ_PHASE_EXCHANGE);
+    }
     // 1. local tokenize + dedup of this rank's documents
     uint64_t C = 0, U = 0, Nc = 0;
     uint32_t *lslot = nullptr, *ldoc = nullptr;
@@ -753,7 +826,7 @@ struct wj_index {
         dp = buf<uint32_t>(x_loc_doc, nc + 16);
       }, C, U, lslot, ldoc);
     }
-    // 2. pack per owner (collection b -> rank b mod K)
+    // 2. pack per owner (collection b -> rank b mod K, or the balanced map)
     phase(WJ_PHASE_EXCHANGE);
     std::vector<uint64_t> cnt(3 * K, 0);  // [terms to o | term bytes to o | records to o]
     uint64_t* toff_d = buf<uint64_t>(x_toff, K + 1);
@@ -767,7 +840,8 @@ struct wj_index {
       uint32_t* srt2 = buf<uint32_t>(x_sorted2, U + 16);
       uint32_t* oc = buf<uint32_t>(x_cnt, 2 * K);
       WJ_CUDA_CHECK(cudaMemsetAsync(oc, 0, 2 * K * 4, st));
-      k_owner<<<grid_for(U, 256), 256, 0, st>>>((const uint32_t*)u_bucket.p, (uint32_t)U, (uint32_t)K, own, iota, oc);
+      k_owner<<<grid_for(U, 256), 256, 0, st>>>((const uint32_t*)u_bucket.p, (uint32_t)U, (uint32_t)K,
+                                                owner_ready ? (const uint32_t*)owner_tab.p : nullptr, own, iota, oc);
       launched();
       // keep u_owner intact for the token pass: sort a copy
       WJ_CUDA_CHECK(cudaMemcpyAsync(own2, own, U * 4, cudaMemcpyDeviceToDevice, st));
@@ -1271,7 +1345,7 @@ extern "C" {
 int index_init(wj_index** out, const wj_config* cfg) {
   if (!out || !cfg) return WJ_ERR_INVALID_ARG;
   *out = nullptr;
-  if (cfg->world < 1 || cfg->world > 1024 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~(WJ_FLAG_PROFILE | WJ_FLAG_LOOPBACK | WJ_FLAG_VBYTE | WJ_FLAG_HOST_PIPELINE)) || cfg->reserved) {
+  if (cfg->world < 1 || cfg->world > 1024 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~(WJ_FLAG_PROFILE | WJ_FLAG_LOOPBACK | WJ_FLAG_VBYTE | WJ_FLAG_HOST_PIPELINE | WJ_FLAG_BALANCED_OWNERS)) || cfg->reserved) {
     g_init_err = "invalid config";
     return WJ_ERR_INVALID_ARG;
   }
@@ -1297,6 +1371,7 @@ int index_init(wj_index** out, const wj_config* cfg) {
   ix->flags = cfg->flags;
   ix->vbyte = (cfg->flags & WJ_FLAG_VBYTE) != 0;
   ix->pipeline = (cfg->flags & WJ_FLAG_HOST_PIPELINE) != 0;
+  ix->balanced = (cfg->flags & WJ_FLAG_BALANCED_OWNERS) != 0;
   int rc = guarded(ix, [&]() {
     if (cfg->stream) {
       ix->st = (cudaStream_t)cfg->stream;
@@ -1533,6 +1608,19 @@ int index_debug_btree(wj_index* ix, void* nodes, uint64_t node_cap, uint64_t* n_
     }
     return (int)WJ_OK;
   });
+}
+
+int index_balance_owners(const uint64_t* counts, uint32_t n, int32_t world, uint32_t* owner) {
+  if (!counts || !owner || world < 1) return WJ_ERR_INVALID_ARG;
+  lpt_owner_map(counts, n, world, owner);
+  return WJ_OK;
+}
+
+int index_owner_map(wj_index* ix, uint32_t* out, uint32_t n) {
+  if (!ix || !out || n < kCollections) return WJ_ERR_INVALID_ARG;
+  for (uint32_t b = 0; b < kCollections; ++b)
+    out[b] = ix->owner_ready ? ix->owner_h[b] : b % (uint32_t)ix->world;
+  return WJ_OK;
 }
 
 const char* index_last_error(const wj_index* ix) { return ix ? ix->err.c_str() : g_init_err.c_str(); }

@@ -9,6 +9,7 @@
 #pragma once
 #include "common.cuh"
 #include "tokenize.cuh"
+#include "dict.cuh"
 
 namespace wj {
 
@@ -46,6 +47,16 @@ __global__ void k_sample_docs_copy(const uint64_t* doc_off, uint64_t nd, uint64_
 __global__ void k_sample_count(const uint32_t* key, uint64_t n, uint32_t* cnt) {
   const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) atomicAdd(&cnt[key[i] & ((1u << 25) - 1u)], 1u);
+}
+
+// sampled tokens per trie collection (balanced owner map): hist[bucket(slot term)] += count
+__global__ void k_sample_buckets(const Slot* table, const uint32_t* slot_ref, const uint32_t* cnt, uint32_t C,
+                                 const uint8_t* text, unsigned long long* hist) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= C || cnt[i] == 0) return;
+  const uint32_t len = (uint32_t)table[i].k0 & 0xFFu;
+  const TermInfo ti = term_info(text, slot_ref[i], len);
+  atomicAdd(&hist[ti.bucket], (unsigned long long)cnt[i]);
 }
 
 // candidates: count if the term is short enough to be identified by its slot bytes, else 0

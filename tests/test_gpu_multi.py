@@ -23,7 +23,7 @@ if not torch.cuda.is_available():  # pragma: no cover
 import paper_conf_ipps_weij11_b200 as wj  # noqa: E402
 
 
-def dist_index(text, doc_off, K, cuts=None, queries=(), vbyte=False):
+def dist_index(text, doc_off, K, cuts=None, queries=(), vbyte=False, balanced=False, maps=None):
     off = np.asarray(doc_off, dtype=np.uint64)
     text = np.asarray(text, dtype=np.uint8)
     n = len(off) - 1
@@ -35,7 +35,7 @@ def dist_index(text, doc_off, K, cuts=None, queries=(), vbyte=False):
 
     def run(r):
         try:
-            with wj.Index(device=0, rank=r, world=K, hub=hub, own_stream=True, vbyte=vbyte) as ix:
+            with wj.Index(device=0, rank=r, world=K, hub=hub, own_stream=True, vbyte=vbyte, balanced=balanced) as ix:
                 for a, b in zip(cuts, cuts[1:]):
                     # rank r's contiguous document range of this chunk (rank order = DocID order)
                     bounds = [a + (b - a) * i // K for i in range(K + 1)]
@@ -45,6 +45,8 @@ def dist_index(text, doc_off, K, cuts=None, queries=(), vbyte=False):
                     ix.add_stream(t, o)
                 ix.finalize()
                 slices[r] = ix.serialize()
+                if maps is not None:
+                    maps[r] = ix.owner_map()
                 for q in queries:
                     answers[r][q] = ix.read_postings(q)
         except Exception as e:  # pragma: no cover
@@ -168,3 +170,28 @@ def test_loopback_host_pipeline():
     hub.close()
     assert not errors, errors
     assert wj.merge_serialized(slices) == oracle.index_bytes(text, off)
+
+
+@pytest.mark.parametrize("K", [3, 4])
+def test_loopback_balanced_owner_map(K):
+    # sampled bin-packing of the trie collections: same map on every rank, every slice
+    # holds exactly its collections, the merge is the oracle's file, and the sampled-token load of
+    # the busiest rank is close to the mean
+    cfg = gen.CONFIGS[2].scaled(chunk_bytes=12 << 20, vocab=300_000)
+    text, off = gen.generate(cfg)
+    n = len(off) - 1
+    maps = [None] * K
+    slices, _ = dist_index(text, off, K, cuts=[0, n // 2, n], balanced=True, maps=maps)
+    assert all(np.array_equal(maps[0], m) for m in maps)
+    assert not np.array_equal(maps[0], np.arange(wj.N_COLLECTIONS) % K)
+    for r, sl in enumerate(slices):
+        ix = wjformat.parse(sl)
+        assert all(maps[0][oracle.bucket(t)] == r for t in ix.terms())
+    assert wj.merge_serialized(slices) == oracle.index_bytes(text, off)
+    load = np.array([int(wjformat.parse(sl).n_tokens) for sl in slices], dtype=np.float64)
+    mod = np.zeros(K)
+    full = wjformat.parse(oracle.index_bytes(text, off))
+    for t, c in zip(full.terms(), full.cf):
+        mod[oracle.bucket(t) % K] += int(c)
+    assert load.max() / load.mean() < 1.10
+    assert load.max() / load.mean() <= mod.max() / mod.mean() + 1e-9

@@ -4,6 +4,7 @@ per-rank dictionary slices done by the C ABI (index_merge_serialized), and the t
 import os
 import socket
 
+import numpy as np
 import pytest
 import torch.multiprocessing as mp
 
@@ -81,3 +82,25 @@ def test_gloo_world2_gather_and_merge():
     for p in ps:
         p.join(timeout=60)
     assert ok
+
+
+# ---------------------------------------------------------------- balanced owner map (host)
+def test_balance_owners_lpt_properties():
+    wj = pytest.importorskip("paper_conf_ipps_weij11_b200")
+    rng = np.random.default_rng(5)
+    counts = np.zeros(17613, dtype=np.uint64)
+    nz = rng.choice(17613, 6000, replace=False)
+    counts[nz] = (1e6 / np.arange(1, 6001) ** 1.1).astype(np.uint64) + 1  # Zipf-like collection sizes
+    for K in (2, 3, 4, 8):
+        own = wj.balance_owners(counts, K)
+        assert own.max() < K
+        zero = counts == 0
+        assert np.array_equal(own[zero], np.arange(17613)[zero] % K)  # unsampled: b mod K
+        load = np.bincount(own, weights=counts.astype(np.float64), minlength=K)
+        # greedy LPT: the busiest rank exceeds the mean by at most the largest single item
+        assert load.max() <= load.sum() / K + counts.max()
+        mod = np.bincount(np.arange(17613) % K, weights=counts.astype(np.float64), minlength=K)
+        assert load.max() <= mod.max()
+    # hand example: counts 5,4,3,3,3 over 2 ranks -> 5->r0, 4->r1, 3->r1 (4<5), 3->r0 (8>7? r0=5<7), 3->r1
+    own = wj.balance_owners(np.array([5, 4, 3, 3, 3], dtype=np.uint64), 2)
+    assert own.tolist() == [0, 1, 1, 0, 1]
