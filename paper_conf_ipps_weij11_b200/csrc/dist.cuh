@@ -84,25 +84,43 @@ __global__ void k_tok_owner(const uint32_t* slot, uint64_t n, const uint32_t* sl
     if (h[i]) atomicAdd(&tok_cnt[i], h[i]);
 }
 
+// K > 64 path: records gathered in owner order from the sorted token indices
 __global__ void k_pack_tok(const uint32_t* sorted_t, uint64_t n, const uint32_t* slot, const uint32_t* doc,
-                           const uint32_t* slot_uid, const uint32_t* xid, uint2* rec) {
+                           const uint32_t* slot_uid, const uint32_t* xid, uint32_t* rkey, uint32_t* rdoc) {
   const uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (j >= n) return;
   const uint32_t t = sorted_t[j];
-  rec[j] = make_uint2(xid[slot_uid[slot[t] & ((1u << 25) - 1u)]], doc[t]);
+  rkey[j] = xid[slot_uid[slot[t] & ((1u << 25) - 1u)]];
+  rdoc[j] = doc[t];
+}
+
+// K <= 64 path: per table slot, the token's record key owner << 26 | xid (bit 25 stays the stream
+// element's count flag); one radix pass over the (slot, docID) stream with this map applied in the
+// histogram pass partitions the records by owner, stably (docID order kept per owner).
+constexpr uint32_t kXidMask = (1u << 25) - 1u;
+constexpr int kOwnerShift = 26;
+__global__ void k_slot_xkey(const Slot* table, uint32_t C, const uint32_t* slot_uid, const uint32_t* u_owner,
+                            const uint32_t* xid, uint32_t* km) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= C || table[i].k0 == 0) return;
+  const uint32_t u = slot_uid[i];
+  km[i] = (u_owner[u] << kOwnerShift) | xid[u];
 }
 
 // owner side: record j from source s -> term index term_base[s] + xid of the received term text,
 // whose (synthetic) token stream gives its table slot
-__global__ void k_map_recv(const uint2* rec, uint64_t n, const uint64_t* rec_off, const uint64_t* term_base, uint32_t K,
-                           const uint32_t* syn_slot, uint32_t* out_slot, uint32_t* out_doc) {
+__global__ void k_map_recv(const uint32_t* rkey, const uint32_t* rdoc, uint64_t n, const uint64_t* rec_off,
+                           const uint64_t* term_base, uint32_t K, const uint32_t* syn_slot, uint32_t* out_slot,
+                           uint32_t* out_doc) {
   const uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (j >= n) return;
-  uint32_t s = 0;
-  while (s + 1 < K && rec_off[s + 1] <= j) ++s;
-  const uint2 r = rec[j];
-  out_slot[j] = syn_slot[term_base[s] + r.x];
-  out_doc[j] = r.y;
+  uint32_t lo = 0, hi = K - 1;  // source rank: last s with rec_off[s] <= j
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi + 1) >> 1;
+    if (rec_off[mid] <= j) lo = mid; else hi = mid - 1;
+  }
+  out_slot[j] = syn_slot[term_base[lo] + (rkey[j] & kXidMask)];
+  out_doc[j] = rdoc[j];
 }
 
 }  // namespace wj

@@ -150,7 +150,7 @@ struct wj_index {
   // the sort saves (profiles/r01_README.md).  WJ_HOT_MIN_BYTES=<bytes> enables it for larger chunks.
   uint64_t hot_min_bytes = ~0ull;
   DevBuf x_owner, x_iota, x_sorted, x_sorted2, x_owner2, x_xid, x_cnt, x_toff, x_boff, x_send, x_tkey, x_tidx, x_tkey2,
-      x_tidx2, x_rec, x_recv_terms, x_recv_rec, x_loc_slot, x_loc_doc, x_syn_slot, x_syn_doc, x_syn_off, x_roff, x_tbase;
+      x_tidx2, x_rkey, x_rdoc, x_keymap, x_recv_terms, x_recv_key, x_recv_doc, x_loc_slot, x_loc_doc, x_syn_slot, x_syn_doc, x_syn_off, x_roff, x_tbase;
   // persistent dictionary
   DevBuf nodes, coll_root, coll_n, coll_base, coll_base2, e_tid, e_bkt, e_tid2, e_bkt2, arena, t_arena, t_cache,
       t_bucket;
@@ -232,7 +232,7 @@ struct wj_index {
                     &samp_ck, &samp_cv, &samp_ck2, &samp_cv2, &samp_n};
     for (DevBuf* b : hs) { if (b->p) cudaFree(b->p); *b = DevBuf{}; }
     DevBuf* xs[] = {&x_owner, &x_iota, &x_sorted, &x_sorted2, &x_owner2, &x_xid, &x_cnt, &x_toff, &x_boff, &x_send,
-                    &x_tkey, &x_tidx, &x_tkey2, &x_tidx2, &x_rec, &x_recv_terms, &x_recv_rec, &x_loc_slot,
+                    &x_tkey, &x_tidx, &x_tkey2, &x_tidx2, &x_rkey, &x_rdoc, &x_keymap, &x_recv_terms, &x_recv_key, &x_recv_doc, &x_loc_slot,
                     &x_loc_doc, &x_syn_slot, &x_syn_doc, &x_syn_off, &x_roff, &x_tbase};
     for (DevBuf* b : xs) { if (b->p) cudaFree(b->p); *b = DevBuf{}; }
     for (auto& b : chunk_map) if (b.p) cudaFree(b.p);
@@ -832,7 +832,7 @@ struct wj_index {
     uint64_t* toff_d = buf<uint64_t>(x_toff, K + 1);
     std::vector<uint64_t> t_off(K + 1, 0), b_off(K + 1, 0), r_off(K + 1, 0);
     uint8_t* send_terms = nullptr;
-    uint2* send_rec = nullptr;
+    uint32_t *send_key = nullptr, *send_doc = nullptr;
     if (U > 0) {
       uint32_t* own = buf<uint32_t>(x_owner, U + 16);
       uint32_t* iota = buf<uint32_t>(x_iota, U + 16);
@@ -868,21 +868,52 @@ struct wj_index {
       k_pack_terms<<<grid_for(U, 256), 256, 0, st>>>(sorted_u, (uint32_t)U, boff, (const uint4*)u_w.p, text,
                                                     (const uint32_t*)u_ref.p, (const uint32_t*)u_len.p, send_terms);
       launched();
-      // token records by owner, stream order kept (stable)
-      uint32_t* tk = buf<uint32_t>(x_tkey, Nc + 16);
-      uint32_t* ti = buf<uint32_t>(x_tidx, Nc + 16);
-      uint32_t* tk2 = buf<uint32_t>(x_tkey2, Nc + 16);
-      uint32_t* ti2 = buf<uint32_t>(x_tidx2, Nc + 16);
-      k_tok_owner<<<grid_for(Nc, 256), 256, 0, st>>>(lslot, Nc, (const uint32_t*)uid.p, own, (uint32_t)K, tk, ti, oc + K);
-      launched();
-      const bool in2 = sort_pairs<uint32_t>(tk, ti, tk2, ti2, Nc, 0, bits, nullptr, false);
-      const uint32_t* sorted_t = in2 ? ti2 : ti;
-      send_rec = (uint2*)grow(x_rec, (Nc + 2) * sizeof(uint2));
-      k_pack_tok<<<grid_for(Nc, 256), 256, 0, st>>>(sorted_t, Nc, lslot, ldoc, (const uint32_t*)uid.p, xid, send_rec);
-      launched();
-      WJ_CUDA_CHECK(cudaMemcpyAsync(oc_h.data(), oc + K, K * 4, cudaMemcpyDeviceToHost, st));
-      sync();
-      for (int o = 0; o < K; ++o) r_off[o + 1] = r_off[o] + oc_h[o];
+      // token records (key with xid, docID) partitioned by owner, stream (= docID) order kept
+      uint32_t* rk = buf<uint32_t>(x_rkey, Nc + 16);
+      uint32_t* rd = buf<uint32_t>(x_rdoc, Nc + 16);
+      if (K <= 64) {  // one radix pass on the owner bits of the mapped key
+        uint32_t* km = buf<uint32_t>(x_keymap, C);
+        k_slot_xkey<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, (uint32_t)C, (const uint32_t*)uid.p, own,
+                                                      xid, km);
+        launched();
+        std::vector<std::pair<uint64_t, const uint32_t*>> segs{{0, km}};
+        std::vector<uint64_t> ds;
+        const bool in2 = sort_pairs<uint32_t>(lslot, ldoc, rk, rd, Nc, kOwnerShift, kOwnerShift + bits, nullptr, false,
+                                              &segs, kXidMask, false, nullptr, false, &ds);
+        if (!in2) {  // K == 1 or a single token: no pass, the map was applied in place
+          rk = lslot;
+          rd = ldoc;
+        }
+        if (ds.size() == 257) {
+          for (int o = 0; o < K; ++o) r_off[o] = ds[o];
+          r_off[K] = Nc;
+        } else {
+          uint32_t o1 = 0;  // owner of the single record (Nc == 1)
+          if (K > 1) {
+            uint32_t v = 0;
+            WJ_CUDA_CHECK(cudaMemcpyAsync(&v, rk, 4, cudaMemcpyDeviceToHost, st));
+            sync();
+            o1 = v >> kOwnerShift;
+          }
+          for (int o = 0; o <= K; ++o) r_off[o] = (uint32_t)o > o1 ? Nc : 0;
+        }
+      } else {
+        uint32_t* tk = buf<uint32_t>(x_tkey, Nc + 16);
+        uint32_t* ti = buf<uint32_t>(x_tidx, Nc + 16);
+        uint32_t* tk2 = buf<uint32_t>(x_tkey2, Nc + 16);
+        uint32_t* ti2 = buf<uint32_t>(x_tidx2, Nc + 16);
+        k_tok_owner<<<grid_for(Nc, 256), 256, 0, st>>>(lslot, Nc, (const uint32_t*)uid.p, own, (uint32_t)K, tk, ti, oc + K);
+        launched();
+        const bool in2 = sort_pairs<uint32_t>(tk, ti, tk2, ti2, Nc, 0, bits, nullptr, false);
+        const uint32_t* sorted_t = in2 ? ti2 : ti;
+        k_pack_tok<<<grid_for(Nc, 256), 256, 0, st>>>(sorted_t, Nc, lslot, ldoc, (const uint32_t*)uid.p, xid, rk, rd);
+        launched();
+        WJ_CUDA_CHECK(cudaMemcpyAsync(oc_h.data(), oc + K, K * 4, cudaMemcpyDeviceToHost, st));
+        sync();
+        for (int o = 0; o < K; ++o) r_off[o + 1] = r_off[o] + oc_h[o];
+      }
+      send_key = rk;
+      send_doc = rd;
       for (int o = 0; o < K; ++o) {
         cnt[o] = t_off[o + 1] - t_off[o];
         cnt[K + o] = b_off[o + 1] - b_off[o];
@@ -900,13 +931,15 @@ struct wj_index {
       rr_off[s + 1] = rr_off[s] + c[2 * K + rank];
     }
     uint8_t* recv_terms = (uint8_t*)grow(x_recv_terms, rb_off[K] + 32);
-    uint2* recv_rec = (uint2*)grow(x_recv_rec, (rr_off[K] + 2) * sizeof(uint2));
+    uint32_t* recv_key = buf<uint32_t>(x_recv_key, rr_off[K] + 16);
+    uint32_t* recv_doc = buf<uint32_t>(x_recv_doc, rr_off[K] + 16);
     std::vector<uint64_t> rec_soff(K + 1), rec_roff(K + 1);
-    for (int o = 0; o <= K; ++o) { rec_soff[o] = r_off[o] * sizeof(uint2); rec_roff[o] = rr_off[o] * sizeof(uint2); }
+    for (int o = 0; o <= K; ++o) { rec_soff[o] = r_off[o] * 4; rec_roff[o] = rr_off[o] * 4; }
     const uint64_t t0 = xport->sent;
     try {
       xport->alltoallv(send_terms, b_off.data(), recv_terms, rb_off.data(), st);
-      xport->alltoallv(send_rec, rec_soff.data(), recv_rec, rec_roff.data(), st);
+      xport->alltoallv(send_key, rec_soff.data(), recv_key, rec_roff.data(), st);
+      xport->alltoallv(send_doc, rec_soff.data(), recv_doc, rec_roff.data(), st);
     } catch (const ExchangeError& e) {
       throw StatusError{WJ_ERR_NCCL, e.msg};
     }
@@ -937,7 +970,8 @@ struct wj_index {
       WJ_CUDA_CHECK(cudaMemcpyAsync(tb, rt_off.data(), (K + 1) * 8, cudaMemcpyHostToDevice, st));
       phase(WJ_PHASE_STREAM);
       if (R > 0) {
-        k_map_recv<<<grid_for(R, 256), 256, 0, st>>>(recv_rec, R, ro, tb, (uint32_t)K, sslot, gt + n_elems, gd + n_elems);
+        k_map_recv<<<grid_for(R, 256), 256, 0, st>>>(recv_key, recv_doc, R, ro, tb, (uint32_t)K, sslot, gt + n_elems,
+                                                     gd + n_elems);
         launched();
       }
       register_chunk_map(C2, n_elems);
@@ -1069,7 +1103,8 @@ struct wj_index {
   bool sort_pairs(K* k0, uint32_t* v0, K* k1, uint32_t* v1, uint64_t n, int begin_bit, int end_bit,
                   const uint32_t* rank_of, bool timed,
                   const std::vector<std::pair<uint64_t, const uint32_t*>>* segs = nullptr, K kmask = ~K(0),
-                  bool skip0 = false, uint64_t* n_out = nullptr) {
+                  bool skip0 = false, uint64_t* n_out = nullptr, bool mask_digits = true,
+                  std::vector<uint64_t>* digit_start = nullptr) {
     if (n_out) *n_out = n;
     if (n == 0) return false;
     int passes = end_bit > begin_bit ? (end_bit - begin_bit + 7) / 8 : 0;
@@ -1112,7 +1147,7 @@ struct wj_index {
       const uint32_t* mp = p == 0 ? first_map : nullptr;
       const bool holes = skip0 && p == 0;
       // the count bits of stream elements only reach a digit when passes cover bits >= 25
-      const bool masked = kmask != ~K(0) && begin_bit + 8 * passes > kCountShift;
+      const bool masked = mask_digits && kmask != ~K(0) && begin_bit + 8 * passes > kCountShift;
       auto up = [&] {
         if (holes && masked) k_rs_up<K, true, true><<<G, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
         else if (holes) k_rs_up<K, true, false><<<G, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
@@ -1131,6 +1166,13 @@ struct wj_index {
         launched();
       };
       if (timed) ktime(WJ_KERNEL_SORT_SCATTER, down); else down();
+      if (digit_start && passes == 1) {  // global start of every digit (single-pass partitions)
+        std::vector<uint32_t> ds(257);
+        WJ_CUDA_CHECK(cudaMemcpy2DAsync(ds.data(), 4, h2, (size_t)G * 4, 4, 256, cudaMemcpyDeviceToHost, st));
+        WJ_CUDA_CHECK(cudaMemcpyAsync(&ds[256], h2 + (uint64_t)256 * G, 4, cudaMemcpyDeviceToHost, st));
+        sync();
+        digit_start->assign(ds.begin(), ds.end());
+      }
       if (holes) {  // elements that survive the compaction
         uint32_t tot = 0;
         WJ_CUDA_CHECK(cudaMemcpyAsync(&tot, h2 + (uint64_t)256 * G, 4, cudaMemcpyDeviceToHost, st));
