@@ -107,20 +107,15 @@ __global__ void k_slot_xkey(const Slot* table, uint32_t C, const uint32_t* slot_
   km[i] = (u_owner[u] << kOwnerShift) | xid[u];
 }
 
-// owner side: record j from source s -> term index term_base[s] + xid of the received term text,
-// whose (synthetic) token stream gives its table slot
-__global__ void k_map_recv(const uint32_t* rkey, const uint32_t* rdoc, uint64_t n, const uint64_t* rec_off,
-                           const uint64_t* term_base, uint32_t K, const uint32_t* syn_slot, uint32_t* out_slot,
-                           uint32_t* out_doc) {
-  const uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (j >= n) return;
-  uint32_t lo = 0, hi = K - 1;  // source rank: last s with rec_off[s] <= j
-  while (lo < hi) {
-    const uint32_t mid = (lo + hi + 1) >> 1;
-    if (rec_off[mid] <= j) lo = mid; else hi = mid - 1;
-  }
-  out_slot[j] = syn_slot[term_base[lo] + (rkey[j] & kXidMask)];
-  out_doc[j] = rdoc[j];
+// owner side: the records of source s carry xid = index of the term in the text s sent; the
+// received text was tokenised as one synthetic document, so term j has token j and slot syn_slot[j].
+// map[xid] = termID of term (base + xid); registered as the stream segment's map.
+__global__ void k_xid_map(const uint32_t* syn_slot, uint32_t n, const Slot* table, const uint32_t* slot_uid,
+                          const uint32_t* u_tid, uint32_t* map) {
+  const uint32_t x = blockIdx.x * blockDim.x + threadIdx.x;
+  if (x >= n) return;
+  const uint32_t sl = syn_slot[x] & kXidMask;
+  map[x] = table[sl].k0 ? u_tid[slot_uid[sl]] : 0u;
 }
 
 }  // namespace wj

@@ -931,8 +931,12 @@ struct wj_index {
       rr_off[s + 1] = rr_off[s] + c[2 * K + rank];
     }
     uint8_t* recv_terms = (uint8_t*)grow(x_recv_terms, rb_off[K] + 32);
-    uint32_t* recv_key = buf<uint32_t>(x_recv_key, rr_off[K] + 16);
-    uint32_t* recv_doc = buf<uint32_t>(x_recv_doc, rr_off[K] + 16);
+    // records land directly in the (termID, docID) stream; per-source maps (xid -> termID) are
+    // registered below, so no per-record translation pass is needed
+    const uint64_t R = rr_off[K];
+    if (n_elems + R > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 stream elements"};
+    uint32_t* recv_key = buf_keep<uint32_t>(g_tid, n_elems + R + 16, n_elems) + n_elems;
+    uint32_t* recv_doc = buf_keep<uint32_t>(g_doc, n_elems + R + 16, n_elems) + n_elems;
     std::vector<uint64_t> rec_soff(K + 1), rec_roff(K + 1);
     for (int o = 0; o <= K; ++o) { rec_soff[o] = r_off[o] * 4; rec_roff[o] = rr_off[o] * 4; }
     const uint64_t t0 = xport->sent;
@@ -945,7 +949,6 @@ struct wj_index {
     }
     exchange_bytes += xport->sent - t0;
     // 4. owner side: the received term text goes through the same tokenizer / dedup / dictionary
-    const uint64_t R = rr_off[K];
     if (rt_off[K] > 0) {
       uint64_t* so = buf<uint64_t>(x_syn_off, 2);
       const uint64_t h2[2] = {0, rb_off[K]};
@@ -961,20 +964,20 @@ struct wj_index {
       n_dropped = dropped0;
       if (Ns != rt_off[K]) throw StatusError{WJ_ERR_CUDA, "received term text: token count mismatch (internal)"};
       dictionary_update(recv_terms, U2);
-      if (n_elems + R > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 stream elements"};
-      uint32_t* gt = buf_keep<uint32_t>(g_tid, n_elems + R + 16, n_elems);
-      uint32_t* gd = buf_keep<uint32_t>(g_doc, n_elems + R + 16, n_elems);
-      uint64_t* ro = buf<uint64_t>(x_roff, K + 1);
-      uint64_t* tb = buf<uint64_t>(x_tbase, K + 1);
-      WJ_CUDA_CHECK(cudaMemcpyAsync(ro, rr_off.data(), (K + 1) * 8, cudaMemcpyHostToDevice, st));
-      WJ_CUDA_CHECK(cudaMemcpyAsync(tb, rt_off.data(), (K + 1) * 8, cudaMemcpyHostToDevice, st));
       phase(WJ_PHASE_STREAM);
-      if (R > 0) {
-        k_map_recv<<<grid_for(R, 256), 256, 0, st>>>(recv_key, recv_doc, R, ro, tb, (uint32_t)K, sslot, gt + n_elems,
-                                                     gd + n_elems);
+      // source s's records: key & kRankMask = xid = index into the terms s sent; map xid -> termID
+      for (int src = 0; src < K; ++src) {
+        const uint64_t nr = rr_off[src + 1] - rr_off[src], nt = rt_off[src + 1] - rt_off[src];
+        if (nr == 0) continue;
+        const size_t ci = chunk_tok.size();
+        if (chunk_map.size() <= ci) chunk_map.emplace_back();
+        uint32_t* m = buf<uint32_t>(chunk_map[ci], nt);
+        k_xid_map<<<grid_for(nt, 256), 256, 0, st>>>(sslot + rt_off[src], (uint32_t)nt, (const Slot*)table.p,
+                                                     (const uint32_t*)uid.p, (const uint32_t*)u_tid.p, m);
         launched();
+        chunk_tok.push_back(n_elems + rr_off[src]);
+        chunk_C.push_back((uint32_t)nt);
       }
-      register_chunk_map(C2, n_elems);
       n_elems += R;
       n_tokens += R;
     }
@@ -1244,7 +1247,10 @@ struct wj_index {
       uint32_t* od = buf<uint32_t>(out_doc, N);
       uint32_t* of = buf<uint32_t>(out_tf, N);
       ktime(WJ_KERNEL_RLE_EMIT, [&] {
-        k_rle_count<<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc, rt);
+        if (stream_has_hot)
+          k_rle_count<true><<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc, rt);
+        else
+          k_rle_count<false><<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc, rt);
         launched();
         scan<uint32_t>(ArrayIn<uint32_t>{rc}, G, rc, (uint32_t*)(dscal() + 8));
         scan<uint64_t>(ArrayIn<uint64_t>{rt}, G, rt, (uint64_t*)(dscal() + 11));

@@ -120,6 +120,7 @@ __device__ __forceinline__ void rle_flags(const uint32_t* k, const uint32_t* d, 
   }
 }
 
+template <bool COUNTS>
 __global__ void __launch_bounds__(kRleThreads) k_rle_count(const uint32_t* __restrict__ key, const uint32_t* __restrict__ doc,
                                                            uint64_t N, uint64_t per, uint32_t* range_cnt,
                                                            uint64_t* range_tok) {
@@ -133,7 +134,8 @@ __global__ void __launch_bounds__(kRleThreads) k_rle_count(const uint32_t* __res
     rle_flags(k, d, pk, pd, i0, hi, npm, ntm);
     c += __popc(npm);
 #pragma unroll
-    for (int j = 0; j < kRleItems; ++j) tk += k[j] >> kCountShift;  // invalid items have key 0
+    for (int j = 0; j < kRleItems; ++j)  // invalid items have key 0; without counts every element is 1 token
+      tk += COUNTS ? (k[j] >> kCountShift) : (k[j] != 0u ? 1u : 0u);
   }
   uint32_t tot;
   block_exclusive_sum<uint32_t>(c, tot);
