@@ -49,6 +49,11 @@ def _load():
         lib.oracle_serialize_vbyte.restype = ctypes.c_int
         lib.oracle_vbyte.argtypes = [vp, u64, vp]
         lib.oracle_vbyte.restype = u64
+        lib.oracle_set_options.argtypes = [vp, ctypes.c_int, ctypes.c_int]
+        lib.oracle_set_options.restype = ctypes.c_int
+        lib.oracle_porter.argtypes = [ctypes.c_char_p, u32, ctypes.c_int, vp]
+        lib.oracle_porter.restype = ctypes.c_int
+        lib.oracle_stop_words.restype = ctypes.c_char_p
         lib.oracle_postings.argtypes = [vp, ctypes.c_char_p, u32, vp, vp, u64, P64]
         lib.oracle_postings.restype = ctypes.c_int
         lib.oracle_dump_tokens.argtypes = [vp, vp, u64, u32, vp, u64, P64]
@@ -65,9 +70,12 @@ def bucket(term: bytes) -> int:
 class Oracle:
     """Incremental oracle: add() chunks of documents in submission order, then serialize()."""
 
-    def __init__(self):
+    def __init__(self, stem: bool = False, stop: bool = False):
+        """stem / stop: the parser's Steps 3-4 (reading S20)."""
         self._lib = _load()
         self._h = self._lib.oracle_new()
+        if stem or stop:
+            self._lib.oracle_set_options(self._h, int(stem), int(stop))
 
     def close(self):
         if self._h:
@@ -111,11 +119,24 @@ class Oracle:
         return d, t
 
 
-def index_bytes(text, doc_off, threads: int = 1, vbyte: bool = False) -> bytes:
+def index_bytes(text, doc_off, threads: int = 1, vbyte: bool = False, stem: bool = False,
+                stop: bool = False) -> bytes:
     """Serialized oracle index of one batch of documents."""
-    o = Oracle()
+    o = Oracle(stem, stop)
     o.add(text, doc_off, threads)
     return o.serialize(vbyte)
+
+
+def porter(term: bytes, step: int = -1) -> bytes:
+    """Porter (1980) stem of a folded term; step 0..7 applies only step 1a,1b,1c,2,3,4,5a,5b."""
+    out = ctypes.create_string_buffer(len(term) + 1)
+    n = _load().oracle_porter(term, len(term), step, out)
+    return out.raw[:n]
+
+
+def stop_words() -> list:
+    """The oracle's stop list (parser Step 4)."""
+    return _load().oracle_stop_words().decode().split()
 
 
 def vbyte(values) -> bytes:

@@ -241,3 +241,86 @@ def test_vbyte_decodes_to_pinned_index(which):
         assert getattr(a, f) == getattr(b, f)
     assert a.as_dict() == b.as_dict()
     assert len(comp) < len(plain) or a.n_postings == 0
+
+
+# ---------------------------------------------------------------- f4: parser Steps 3-4
+# Porter stemmer: the per-step examples printed in M.F. Porter, "An algorithm for suffix stripping"
+# (Program 14(3), 1980), each applied to that step alone (step index 0..7 = 1a,1b,1c,2,3,4,5a,5b).
+PORTER_STEP_EXAMPLES = {
+    0: [("caresses", "caress"), ("ponies", "poni"), ("ties", "ti"), ("caress", "caress"), ("cats", "cat")],
+    1: [("feed", "feed"), ("agreed", "agree"), ("plastered", "plaster"), ("bled", "bled"), ("motoring", "motor"),
+        ("sing", "sing"), ("conflated", "conflate"), ("troubled", "trouble"), ("sized", "size"),
+        ("hopping", "hop"), ("tanned", "tan"), ("falling", "fall"), ("hissing", "hiss"), ("fizzed", "fizz"),
+        ("failing", "fail"), ("filing", "file")],
+    2: [("happy", "happi"), ("sky", "sky")],
+    3: [("relational", "relate"), ("conditional", "condition"), ("rational", "rational"), ("valenci", "valence"),
+        ("hesitanci", "hesitance"), ("digitizer", "digitize"), ("conformabli", "conformable"),
+        ("radicalli", "radical"), ("differentli", "different"), ("vileli", "vile"), ("analogousli", "analogous"),
+        ("vietnamization", "vietnamize"), ("predication", "predicate"), ("operator", "operate"),
+        ("feudalism", "feudal"), ("decisiveness", "decisive"), ("hopefulness", "hopeful"),
+        ("callousness", "callous"), ("formaliti", "formal"), ("sensitiviti", "sensitive"),
+        ("sensibiliti", "sensible")],
+    4: [("triplicate", "triplic"), ("formative", "form"), ("formalize", "formal"), ("electriciti", "electric"),
+        ("electrical", "electric"), ("hopeful", "hope"), ("goodness", "good")],
+    5: [("revival", "reviv"), ("allowance", "allow"), ("inference", "infer"), ("airliner", "airlin"),
+        ("gyroscopic", "gyroscop"), ("adjustable", "adjust"), ("defensible", "defens"), ("irritant", "irrit"),
+        ("replacement", "replac"), ("adjustment", "adjust"), ("dependent", "depend"), ("adoption", "adopt"),
+        ("homologou", "homolog"), ("communism", "commun"), ("activate", "activ"), ("angulariti", "angular"),
+        ("homologous", "homolog"), ("effective", "effect"), ("bowdlerize", "bowdler")],
+    6: [("probate", "probat"), ("rate", "rate"), ("cease", "ceas")],
+    7: [("controll", "control"), ("roll", "roll")],
+}
+
+
+@pytest.mark.parametrize("step", sorted(PORTER_STEP_EXAMPLES))
+def test_porter_paper_step_examples(step):
+    for word, want in PORTER_STEP_EXAMPLES[step]:
+        assert oracle.porter(word.encode(), step) == want.encode(), (step, word)
+
+
+def test_porter_paper_whole_word_examples():
+    # Porter's worked chains (GENERALIZATIONS -> ... -> GENER, OSCILLATORS -> ... -> OSCIL) and words
+    # whose full result follows from the step examples above
+    cases = {"generalizations": "gener", "oscillators": "oscil", "caresses": "caress", "ponies": "poni",
+             "agreed": "agre", "relational": "relat", "rational": "ration", "conditional": "condit",
+             "hopeful": "hope", "goodness": "good", "motoring": "motor", "plastered": "plaster",
+             "replacement": "replac", "probate": "probat", "rate": "rate", "cease": "ceas", "controll": "control"}
+    for word, want in cases.items():
+        assert oracle.porter(word.encode()) == want.encode(), word
+    # reading S20: fewer than 3 bytes, digits or bytes >= 0x80 -> unchanged
+    for w in (b"is", b"as", b"3d", b"a\xc3\xb1os", b"abc1"):
+        assert oracle.porter(w) == w
+
+
+def test_stop_list_is_sklearn_english():
+    text = pytest.importorskip("sklearn.feature_extraction.text")
+    assert sorted(oracle.stop_words()) == sorted(text.ENGLISH_STOP_WORDS)
+
+
+def test_stem_stop_hand_counted():
+    # docs ["The cats sat.", "cat catS, the hat!", ""]; "the" is a stop word; cats -> cat
+    text, off = gen.from_docs([b"The cats sat.", b"cat catS, the hat!", b""])
+    ix = wjformat.parse(oracle.index_bytes(text, off, stem=True, stop=True))
+    assert ix.as_dict() == {b"cat": [(0, 1), (1, 2)], b"hat": [(1, 1)], b"sat": [(0, 1)]}
+    assert (ix.n_docs, ix.n_tokens, ix.n_dropped) == (3, 5, 0)
+    # stop only: surface forms kept, "the" removed
+    ix = wjformat.parse(oracle.index_bytes(text, off, stop=True))
+    assert ix.as_dict() == {b"cat": [(1, 1)], b"cats": [(0, 1), (1, 1)], b"hat": [(1, 1)], b"sat": [(0, 1)]}
+
+
+def test_stem_stop_invariants_and_chunking():
+    text, off = gen.generate(gen.CONFIGS[1])
+    one = oracle.index_bytes(text, off, stem=True, stop=True)
+    ix = wjformat.parse(one)
+    wjformat.check_invariants(ix)
+    stems = set(ix.terms())
+    o = oracle.Oracle(stem=True, stop=True)
+    o.add(text[: int(off[500])], off[:501])
+    o.add(text[int(off[500]):], off[500:] - off[500])
+    assert o.serialize() == one
+    assert oracle.index_bytes(text, off, threads=4, stem=True, stop=True) == one
+    # every dictionary term is the stem of some token and none is a (stemmed) stop word
+    stop = {oracle.porter(w.encode()) for w in oracle.stop_words()}
+    assert not (stems & stop)
+    surface = wjformat.parse(oracle.index_bytes(text, off))
+    assert stems <= {oracle.porter(t) for t in surface.terms()}
