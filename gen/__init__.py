@@ -181,3 +181,71 @@ def from_docs(docs) -> tuple[np.ndarray, np.ndarray]:
     np.cumsum([len(d) for d in docs], out=doc_off[1:]) if docs else None
     text = np.frombuffer(b"".join(docs), dtype=np.uint8).copy()
     return text, doc_off
+
+
+# English-like words for the parser Steps 3-4 tests: stems joined with the suffixes
+# Porter's rules act on, plus the stop list's words, so stemming and stop-word removal fire often.
+# Input generation only: nothing here stems or tests a word.
+SUFFIXES = ["", "s", "es", "ies", "sses", "ss", "ed", "eed", "ing", "y", "ational", "tional", "enci", "anci",
+            "izer", "abli", "alli", "entli", "eli", "ousli", "ization", "ation", "ator", "alism", "iveness",
+            "fulness", "ousness", "aliti", "iviti", "biliti", "icate", "ative", "alize", "iciti", "ical", "ful",
+            "ness", "al", "ance", "ence", "er", "ic", "able", "ible", "ant", "ement", "ment", "ent", "ion", "sion",
+            "tion", "ou", "ism", "ate", "iti", "ous", "ive", "ize", "e", "ll", "led", "ling", "ings", "ers",
+            "ations", "izing", "ally", "fully", "lessness", "ying", "yed"]
+STEMS = ["relat", "condit", "ration", "valen", "hesit", "digit", "conform", "radic", "differ", "vil", "analog",
+         "vietnam", "predic", "oper", "feud", "decis", "hope", "callous", "form", "sensit", "sensib", "trip",
+         "electr", "good", "reviv", "allow", "infer", "airlin", "gyroscop", "adjust", "defens", "irrit",
+         "replac", "depend", "adopt", "homolog", "commun", "activ", "angular", "effect", "bowdler", "prob",
+         "rat", "ceas", "control", "rol", "cat", "pony", "ti", "caress", "feed", "agre", "plaster", "bl",
+         "motor", "s", "conflat", "troubl", "siz", "hop", "tann", "fall", "hiss", "fizz", "fail", "fil",
+         "happ", "sk", "gener", "oscill", "y", "by", "sy", "ay", "oy", "boy", "tr", "fl", "abc", "xyz",
+         "book", "run", "sit", "lov", "mak", "nation", "organ", "class", "car", "ward", "quiet", "stud"]
+
+
+def suffix_rich_docs(seed: int, n_docs: int, words_per_doc=(0, 120), stop_words=None) -> list:
+    """Seeded documents of stem+suffix words, stop words (if given), numbers and a few non-ASCII
+    words, with random capitalisation and punctuation."""
+    rng = np.random.default_rng(seed)
+    stop_words = list(stop_words or [])
+    docs = []
+    for _ in range(n_docs):
+        n = int(rng.integers(words_per_doc[0], words_per_doc[1] + 1))
+        out = []
+        for _ in range(n):
+            r = rng.random()
+            if r < 0.25 and stop_words:
+                w = stop_words[int(rng.integers(len(stop_words)))]
+            elif r < 0.90:
+                w = STEMS[int(rng.integers(len(STEMS)))] + SUFFIXES[int(rng.integers(len(SUFFIXES)))]
+            elif r < 0.95:
+                w = str(int(rng.integers(0, 10 ** int(rng.integers(1, 6)))))
+            else:
+                w = "año" + SUFFIXES[int(rng.integers(len(SUFFIXES)))]
+            c = rng.random()
+            if c < 0.08:
+                w = w[:1].upper() + w[1:]
+            elif c < 0.1:
+                w = w.upper()
+            out.append(w + [" ", " ", " ", ", ", ". ", "\n"][int(rng.integers(6))])
+        docs.append("".join(out).encode("utf-8"))
+    return docs
+
+
+def suffix_rich_words(seed: int, n: int) -> list:
+    """n seeded lowercase stem+suffix words (plus short words, digits and non-ASCII ones)."""
+    rng = np.random.default_rng(seed)
+    out = []
+    for _ in range(n):
+        r = rng.random()
+        if r < 0.8:
+            w = STEMS[int(rng.integers(len(STEMS)))] + SUFFIXES[int(rng.integers(len(SUFFIXES)))]
+            if rng.random() < 0.3:
+                w = SUFFIXES[int(rng.integers(len(SUFFIXES)))] + w
+        elif r < 0.9:
+            w = "".join(chr(97 + int(x)) for x in rng.integers(0, 26, size=int(rng.integers(1, 14))))
+        elif r < 0.95:
+            w = "".join("aeiouy"[int(x)] if x < 6 else chr(97 + int(x)) for x in rng.integers(0, 26, size=int(rng.integers(1, 9))))
+        else:
+            w = str(int(rng.integers(0, 99999))) + ("x" if rng.random() < 0.5 else "")
+        out.append(w.encode())
+    return out

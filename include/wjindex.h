@@ -63,6 +63,13 @@ typedef enum {
                                /* 1 MiB samples are all-gathered and every rank bin-packs   */
                                /* the trie collections by sampled token count; the map is  */
                                /* kept for the context's lifetime, also across reset       */
+#define WJ_FLAG_STEM 0x20u     /* parser Step 3 (reading S20): every term of   */
+                               /* >= 3 bytes made only of a-z is replaced by its Porter (1980) stem */
+                               /* before indexing; the dictionary holds stems (query by the stem)  */
+#define WJ_FLAG_STOPWORDS 0x40u /* parser Step 4 (reading S20): tokens whose (stemmed, with */
+                               /* WJ_FLAG_STEM) term equals the (stemmed) form of a word of the     */
+                               /* built-in 318-word English stop list are dropped; they count in    */
+                               /* neither n_tokens nor n_dropped (index_stop_words lists the words) */
 
 typedef struct wj_index wj_index; /* opaque; all index state is owned by the library */
 
@@ -91,6 +98,8 @@ enum {
   WJ_PHASE_DICT,         /* finalize: term_off + term bytes of the final dictionary                */
   WJ_PHASE_EXCHANGE,     /* world > 1: all-to-all of the routed stream                             */
   WJ_PHASE_VBYTE,        /* finalize (WJ_FLAG_VBYTE): d-gap + variable-byte postings code  */
+  WJ_PHASE_STEM,         /* WJ_FLAG_STEM/STOPWORDS: stem + stop-word test of the unique terms,     */
+                         /* stem dedup, stop-word token compaction                     */
   WJ_PHASE_COUNT = 16
 };
 
@@ -211,6 +220,19 @@ int index_merge_serialized(int32_t k, const uint8_t* const* slices, const uint64
  * collections) by count desc, index asc on ties, each to the least-loaded rank (lowest on ties);
  * count-0 items keep i mod world.  WJ_ERR_INVALID_ARG on NULL or world < 1. */
 int index_balance_owners(const uint64_t* counts, uint32_t n, int32_t world, uint32_t* owner);
+
+/* The built-in stop list of WJ_FLAG_STOPWORDS (parser Step 4; reading S20): 318 lowercase
+ * words separated by single spaces, NUL-terminated, owned by the library (static storage). */
+const char* index_stop_words(void);
+
+/* Debug (tests): the device Porter stemmer (parser Step 3) on n host words.  Word i is
+ * words[word_off[i] .. word_off[i+1]) (folded bytes, <= 255 each); its stem (reading S20: only
+ * words of >= 3 bytes of a-z change) is written to out[word_off[i] ..] (a stem is never longer
+ * than its word) with its length in out_len[i].  All pointers are host memory owned by the caller.
+ * Runs on `device` with a temporary stream.  WJ_ERR_INVALID_ARG on NULL or a word > 255 bytes,
+ * WJ_ERR_CUDA without a device. */
+int index_debug_stem(int32_t device, const uint8_t* words, const uint32_t* word_off, uint32_t n, uint8_t* out,
+                     uint32_t* out_len);
 
 /* Owner rank of every trie collection (out: n >= 17613 entries): b mod world, or the balanced map
  * once the first chunk has built it (WJ_FLAG_BALANCED_OWNERS).  WJ_ERR_INVALID_ARG if n is small. */

@@ -22,7 +22,7 @@ ERRORS = {-1: "WJ_ERR_INVALID_ARG", -2: "WJ_ERR_STATE", -3: "WJ_ERR_CUDA", -4: "
           -6: "WJ_ERR_CAPACITY", -7: "WJ_ERR_BUFFER_TOO_SMALL"}
 WJ_FLAG_PROFILE = 1
 PHASES = ["h2d", "tokenize", "unique", "probe", "insert", "rebuild", "stream", "lexrank", "sort", "postings",
-          "dict", "exchange", "vbyte"]
+          "dict", "exchange", "vbyte", "stem"]
 KERNELS = ["tokenize_count", "tokenize_emit", "probe", "slot_to_tid", "map_rank", "sort_hist", "sort_scatter",
            "rle_emit"]
 N_COLLECTIONS = 17613
@@ -30,12 +30,14 @@ N_COLLECTIONS = 17613
 EXPORTS = ["index_init", "index_add_stream", "index_finalize", "index_read_postings", "index_serialize",
            "index_stats", "index_reset", "index_debug_tokens", "index_debug_btree", "index_nccl_unique_id",
            "index_loopback_create", "index_loopback_destroy", "index_merge_serialized", "index_owner_map",
-           "index_balance_owners",
+           "index_balance_owners", "index_stop_words", "index_debug_stem",
            "index_last_error", "index_destroy"]
 WJ_FLAG_LOOPBACK = 2
 WJ_FLAG_VBYTE = 4
 WJ_FLAG_HOST_PIPELINE = 8
 WJ_FLAG_BALANCED_OWNERS = 16
+WJ_FLAG_STEM = 32
+WJ_FLAG_STOPWORDS = 64
 
 
 class WJError(RuntimeError):
@@ -108,11 +110,14 @@ def load_library():
         lib.index_merge_serialized.argtypes = [ctypes.c_int32, ctypes.POINTER(ctypes.c_void_p), ctypes.POINTER(ctypes.c_uint64),
                                                vp, u64, P64]
         for f in EXPORTS:
-            if f not in ("index_last_error", "index_destroy", "index_loopback_destroy"):
+            if f not in ("index_last_error", "index_destroy", "index_loopback_destroy", "index_stop_words"):
                 getattr(lib, f).restype = i32
         lib.index_owner_map.argtypes = [vp, vp, u32]
         lib.index_balance_owners.argtypes = [vp, u32, ctypes.c_int32, vp]
         lib.index_destroy.restype = None
+        lib.index_stop_words.argtypes = []
+        lib.index_stop_words.restype = ctypes.c_char_p
+        lib.index_debug_stem.argtypes = [ctypes.c_int32, vp, vp, u32, vp, vp]
         lib.index_loopback_destroy.restype = None
         _lib = lib
     return _lib
@@ -147,18 +152,22 @@ class Index:
 
     def __init__(self, device: int = 0, stream=None, profile: bool = False, rank: int = 0, world: int = 1,
                  nccl_id: bytes | None = None, hub: "LoopbackHub | None" = None, own_stream: bool = False,
-                 vbyte: bool = False, pipeline: bool = False, balanced: bool = False):
+                 vbyte: bool = False, pipeline: bool = False, balanced: bool = False, stem: bool = False,
+                 stop: bool = False):
         """world > 1: pass nccl_id (128 bytes from nccl_unique_id(), broadcast by the caller) or a
         LoopbackHub shared by `world` contexts of this process (one host thread each).
         vbyte: finalize also builds the d-gap + variable-byte postings code; serialize() then
         returns the compressed file WJINV002.
         pipeline: host chunks are copied on a copy stream while the previous one is indexed
         (Fig. 9); keep each host buffer unchanged until the next call returns.
-        balanced: world > 1, owners of the trie collections from a sampled bin-packing."""
+        balanced: world > 1, owners of the trie collections from a sampled bin-packing.
+        stem / stop: the parser's Steps 3-4 (reading S20): Porter (1980)
+        stems and removal of the built-in stop words (stop_words())."""
         self._lib = load_library()
         flags = (WJ_FLAG_PROFILE if profile else 0) | (WJ_FLAG_LOOPBACK if hub is not None else 0) | (
             WJ_FLAG_VBYTE if vbyte else 0) | (WJ_FLAG_HOST_PIPELINE if pipeline else 0) | (
-            WJ_FLAG_BALANCED_OWNERS if balanced else 0)
+            WJ_FLAG_BALANCED_OWNERS if balanced else 0) | (WJ_FLAG_STEM if stem else 0) | (
+            WJ_FLAG_STOPWORDS if stop else 0)
         self._nid = ctypes.create_string_buffer(bytes(nccl_id), 128) if nccl_id is not None else None
         uid = hub._h if hub is not None else (ctypes.cast(self._nid, ctypes.c_void_p) if self._nid is not None else None)
         if own_stream:
@@ -344,6 +353,27 @@ def balance_owners(counts, world: int) -> np.ndarray:
     if rc != WJ_OK:
         raise WJError(rc, "index_balance_owners")
     return out
+
+
+def stop_words() -> list:
+    """The library's built-in stop list (index_stop_words; parser Step 4)."""
+    return load_library().index_stop_words().decode().split()
+
+
+def debug_stem(words, device: int = 0) -> list:
+    """Porter stems of folded words computed by the device stemmer (index_debug_stem)."""
+    words = [bytes(w) for w in words]
+    off = np.zeros(len(words) + 1, dtype=np.uint32)
+    off[1:] = np.cumsum([len(w) for w in words])
+    packed = np.frombuffer(b"".join(words) + b"\0", dtype=np.uint8)
+    out = np.zeros(max(int(off[-1]), 1), dtype=np.uint8)
+    lens = np.zeros(max(len(words), 1), dtype=np.uint32)
+    rc = load_library().index_debug_stem(device, packed.ctypes.data, off.ctypes.data, len(words), out.ctypes.data,
+                                         lens.ctypes.data)
+    if rc != WJ_OK:
+        raise WJError(rc, "index_debug_stem")
+    raw = out.tobytes()
+    return [raw[int(off[i]):int(off[i]) + int(lens[i])] for i in range(len(words))]
 
 
 def owner_of(collection: int, world: int) -> int:

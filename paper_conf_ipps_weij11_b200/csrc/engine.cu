@@ -15,6 +15,7 @@
 #include "postings.cuh"
 #include "radix.cuh"
 #include "scan.cuh"
+#include "stem.cuh"
 #include "tokenize.cuh"
 #include "vbyte.cuh"
 
@@ -105,6 +106,30 @@ static void lpt_owner_map(const uint64_t* count, uint32_t n, int K, uint32_t* ow
   }
 }
 
+// Stop list of WJ_FLAG_STOPWORDS (parser Step 4; the paper names no list).  Reading S20:
+// the 318-word English list scikit-learn ships as ENGLISH_STOP_WORDS (Glasgow IR group), sorted.
+static const char kStopList[] =
+    "a about above across after afterwards again against all almost alone along already also although "
+    "always am among amongst amoungst amount an and another any anyhow anyone anything anyway anywhere are "
+    "around as at back be became because become becomes becoming been before beforehand behind being below "
+    "beside besides between beyond bill both bottom but by call can cannot cant co con could couldnt cry de "
+    "describe detail do done down due during each eg eight either eleven else elsewhere empty enough etc "
+    "even ever every everyone everything everywhere except few fifteen fifty fill find fire first five for "
+    "former formerly forty found four from front full further get give go had has hasnt have he hence her "
+    "here hereafter hereby herein hereupon hers herself him himself his how however hundred i ie if in inc "
+    "indeed interest into is it its itself keep last latter latterly least less ltd made many may me "
+    "meanwhile might mill mine more moreover most mostly move much must my myself name namely neither never "
+    "nevertheless next nine no nobody none noone nor not nothing now nowhere of off often on once one only "
+    "onto or other others otherwise our ours ourselves out over own part per perhaps please put rather re "
+    "same see seem seemed seeming seems serious several she should show side since sincere six sixty so "
+    "some somehow someone something sometime sometimes somewhere still such system take ten than that the "
+    "their them themselves then thence there thereafter thereby therefore therein thereupon these they "
+    "thick thin third this those though three through throughout thru thus to together too top toward "
+    "towards twelve twenty two un under until up upon us very via was we well were what whatever when "
+    "whence whenever where whereafter whereas whereby wherein whereupon wherever whether which while "
+    "whither who whoever whole whom whose why will with within without would yet you your yours yourself "
+    "yourselves";
+
 struct wj_index {
   int device = 0;
   int rank = 0, world = 1;
@@ -168,6 +193,11 @@ struct wj_index {
   DevBuf rank_of, term_at, sk1, sv1, pidx, out_doc, out_tf, post_off, df, cf, term_off, term_bytes;
   DevBuf vb_first, vb_tiles, vb_code, vb_boff;  // f1 (WJ_FLAG_VBYTE)
   DevBuf samp_hist, owner_tab;                  // f2(i) (WJ_FLAG_BALANCED_OWNERS)
+  // f4 parser Steps 3-4 (WJ_FLAG_STEM / WJ_FLAG_STOPWORDS; stem.cuh): the surface table is kept in
+  // table_s / uid_s while table / uid / u_* describe the chunk's unique stems over the stem text
+  bool stem_on = false, stop_on = false;
+  uint32_t n_stop = 0;
+  DevBuf table_s, uid_s, st_off, st_text, st_keep, st_tidx, st_m1, st_slot, st_doc, st_tiles, st_doff, stop_keys;
   std::vector<DevBuf> chunk_map;        // per chunk: slot -> termID (-> rank at finalize)
   std::vector<uint64_t> chunk_tok;      // per chunk: first token index in the stream
   std::vector<uint32_t> chunk_C;        // per chunk: table capacity
@@ -222,7 +252,9 @@ struct wj_index {
                      &nk_key2, &nk_val2, &aoff, &ns_tid, &ns_bucket, &ns_rank, &nlo, &nhi, &nbase, &child_off,
                      &root_idx, &scan_scr, &hist, &hist_scan, &os_hist, &os_look, &os_ctr, &kstart, &slotref, &dbg_start, &dbg_len, &dbg_off, &dbg_out, &dbg_slot,
                      &dbg_doc, &lexg, &qbuf, &qres, &rank_of, &term_at, &sk1, &sv1, &pidx, &out_doc, &out_tf,
-                     &post_off, &df, &cf, &term_off, &term_bytes, &vb_first, &vb_tiles, &vb_code, &vb_boff, &samp_hist, &owner_tab};
+                     &post_off, &df, &cf, &term_off, &term_bytes, &vb_first, &vb_tiles, &vb_code, &vb_boff, &samp_hist, &owner_tab,
+                     &table_s, &uid_s, &st_off, &st_text, &st_keep, &st_tidx, &st_m1, &st_slot, &st_doc, &st_tiles,
+                     &st_doff, &stop_keys};
     for (DevBuf* b : all) {
       if (b->p) cudaFree(b->p);
       b->p = nullptr;
@@ -653,6 +685,122 @@ struct wj_index {
     return Nc;
   }
 
+  // ---------------------------------------------------------------- f4: parser Steps 3-4
+  // WJ_FLAG_STEM / WJ_FLAG_STOPWORDS (stem.cuh).  In: the surface dedup of a chunk
+  // (table / uid / u_*: C1 slots, U1 unique terms over `text`) and its stream (slot, doc)[Nc].
+  // Out: table_s / uid_s hold the surface table; table / uid / u_* the U2 unique stems over
+  // `ntext`; st_m1[s] = unique-stem index of surface slot s; the stream is compacted in place
+  // (stop-word tokens removed).  Returns the kept token count.
+  uint64_t normalize(const uint8_t* text, uint64_t C1, uint64_t U1, uint32_t* slot, uint32_t* doc, uint64_t Nc,
+                     uint64_t& U2, const uint8_t*& ntext) {
+    phase(WJ_PHASE_STEM);
+    U2 = 0;
+    uint64_t* off = buf<uint64_t>(st_off, U1 + 1);
+    scan<uint64_t>(LenPlus1{(const uint32_t*)u_len.p}, U1, off, off + U1);
+    WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 12, off + U1, 8, cudaMemcpyDeviceToHost, st));
+    sync();
+    const uint64_t B = h_scal[12];
+    uint8_t* nt = (uint8_t*)grow(st_text, B + 32);
+    uint32_t* keep = buf<uint32_t>(st_keep, U1 + 1);
+    k_stem_terms<<<grid_for(U1, 256), 256, 0, st>>>((const uint4*)u_w.p, (const uint32_t*)u_ref.p,
+                                                    (const uint32_t*)u_len.p, text, (uint32_t)U1, off, nt, stem_on ? 1 : 0,
+                                                    stop_on ? (const ulonglong2*)stop_keys.p : nullptr, n_stop, keep);
+    launched();
+    uint32_t* tidx = buf<uint32_t>(st_tidx, U1 + 1);
+    scan<uint32_t>(ArrayIn<uint32_t>{keep}, U1, tidx, tidx + U1);
+    WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 13, tidx + U1, 4, cudaMemcpyDeviceToHost, st));
+    sync();
+    const uint64_t Kk = (uint32_t)h_scal[13];
+    std::swap(table, table_s);  // keep the surface table; the stem dedup reuses the scratch set
+    std::swap(uid, uid_s);
+    uint32_t* sslot = nullptr;
+    if (Kk > 0) {
+      uint64_t* so = buf<uint64_t>(st_doff, 2);
+      const uint64_t h2[2] = {0, B};
+      WJ_CUDA_CHECK(cudaMemcpyAsync(so, h2, 16, cudaMemcpyHostToDevice, st));
+      ChunkView sv{nt, B, so, 1};
+      const uint64_t est0 = table_est, dropped0 = n_dropped;
+      uint64_t C2 = 0;
+      uint32_t* sdoc = nullptr;
+      const uint64_t Ns = tokenize_dedup(sv, 0, [&](uint64_t nc, uint32_t*& sp, uint32_t*& dp) {
+        sp = buf<uint32_t>(st_slot, nc + 16);
+        dp = buf<uint32_t>(st_doc, nc + 16);
+      }, C2, U2, sslot, sdoc);
+      table_est = est0;
+      n_dropped = dropped0;
+      unique_last = U1;
+      if (Ns != Kk) throw StatusError{WJ_ERR_CUDA, "stem text: token count mismatch (internal)"};
+      phase(WJ_PHASE_STEM);
+    }
+    uint32_t* m1 = buf<uint32_t>(st_m1, C1);
+    k_norm_map<<<grid_for(C1, 256), 256, 0, st>>>((const Slot*)table_s.p, (const uint32_t*)uid_s.p, (uint32_t)C1, keep,
+                                                  tidx, sslot, (const uint32_t*)uid.p, m1);
+    launched();
+    uint64_t kept = Nc;
+    if (Kk < U1) {
+      kept = drop_tokens(slot, doc, Nc, m1);
+      k_clear_drop<<<grid_for(C1, 256), 256, 0, st>>>(m1, (uint32_t)C1);
+      launched();
+    }
+    ntext = nt;
+    return kept;
+  }
+
+  // stable in-place compaction of a (slot, doc) stream: drops elements whose m1[slot] has kDropBit
+  uint64_t drop_tokens(uint32_t* slot, uint32_t* doc, uint64_t n, const uint32_t* m1) {
+    if (n == 0) return 0;
+    const uint64_t T = (n + kDropTile - 1) / kDropTile;
+    uint32_t* tk = buf<uint32_t>(st_tiles, T + 1);
+    k_drop_count<<<(unsigned)T, kDropThreads, 0, st>>>(slot, n, m1, tk);
+    launched();
+    scan<uint32_t>(ArrayIn<uint32_t>{tk}, T, tk, tk + T);
+    WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 14, tk + T, 4, cudaMemcpyDeviceToHost, st));
+    uint32_t* s2 = buf<uint32_t>(sk1, n + 16);
+    uint32_t* d2 = buf<uint32_t>(sv1, n + 16);
+    k_drop_write<<<(unsigned)T, kDropThreads, 0, st>>>(slot, doc, n, m1, tk, s2, d2);
+    launched();
+    sync();
+    const uint64_t kept = (uint32_t)h_scal[14];
+    if (kept) {
+      WJ_CUDA_CHECK(cudaMemcpyAsync(slot, s2, kept * 4, cudaMemcpyDeviceToDevice, st));
+      WJ_CUDA_CHECK(cudaMemcpyAsync(doc, d2, kept * 4, cudaMemcpyDeviceToDevice, st));
+    }
+    return kept;
+  }
+
+  // stop keys (index_init, WJ_FLAG_STOPWORDS): the built-in list, stemmed on the device when
+  // WJ_FLAG_STEM (Step 4 follows Step 3, S20), sorted and deduplicated on the host
+  void build_stop_keys() {
+    std::vector<uint8_t> words;
+    std::vector<uint32_t> woff{0};
+    for (const char* p = kStopList;; ++p) {
+      if (*p == ' ' || *p == 0) {
+        if (words.size() > woff.back()) woff.push_back((uint32_t)words.size());
+        if (*p == 0) break;
+      } else {
+        words.push_back((uint8_t)*p);
+      }
+    }
+    const uint32_t nw = (uint32_t)woff.size() - 1;
+    uint8_t* dw = (uint8_t*)grow(st_text, words.size() + 32);
+    uint32_t* doff = buf<uint32_t>(st_tidx, nw + 1);
+    ulonglong2* dk = (ulonglong2*)grow(stop_keys, (size_t)nw * sizeof(ulonglong2));
+    WJ_CUDA_CHECK(cudaMemcpyAsync(dw, words.data(), words.size(), cudaMemcpyHostToDevice, st));
+    WJ_CUDA_CHECK(cudaMemcpyAsync(doff, woff.data(), woff.size() * 4, cudaMemcpyHostToDevice, st));
+    k_stop_keys<<<grid_for(nw, 128), 128, 0, st>>>(dw, doff, nw, stem_on ? 1 : 0, dk);
+    launched();
+    std::vector<ulonglong2> hk(nw);
+    WJ_CUDA_CHECK(cudaMemcpyAsync(hk.data(), dk, (size_t)nw * sizeof(ulonglong2), cudaMemcpyDeviceToHost, st));
+    sync();
+    auto less = [](const ulonglong2& a, const ulonglong2& b) { return a.x < b.x || (a.x == b.x && a.y < b.y); };
+    std::sort(hk.begin(), hk.end(), less);
+    hk.erase(std::unique(hk.begin(), hk.end(), [](const ulonglong2& a, const ulonglong2& b) { return a.x == b.x && a.y == b.y; }),
+             hk.end());
+    n_stop = (uint32_t)hk.size();
+    WJ_CUDA_CHECK(cudaMemcpyAsync(dk, hk.data(), hk.size() * sizeof(ulonglong2), cudaMemcpyHostToDevice, st));
+    sync();
+  }
+
   // K3 probe + K4 insert/rebuild of the chunk's unique terms (u_* arrays) -> u_tid
   void dictionary_update(const uint8_t* text, uint64_t U) {
     uint32_t* ut = buf<uint32_t>(u_tid, U);
@@ -764,12 +912,31 @@ struct wj_index {
     ChunkView cv{text, n_bytes, off, nd};
     uint64_t C = 0, U = 0;
     uint32_t *so = nullptr, *dout = nullptr;
+    const bool norm = stem_on || stop_on;
     const uint64_t Nc = tokenize_dedup(cv, doc_base, [&](uint64_t nc, uint32_t*& sp, uint32_t*& dp) {
       if (n_elems + nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 stream elements"};
       sp = buf_keep<uint32_t>(g_tid, n_elems + nc + 16, n_elems) + n_elems;  // +16: TMA round-up reads
       dp = buf_keep<uint32_t>(g_doc, n_elems + nc + 16, n_elems) + n_elems;
-    }, C, U, so, dout, true);
-    if (Nc > 0) {
+    }, C, U, so, dout, !norm);
+    if (Nc > 0 && norm) {  // f4: stems / stop words
+      uint64_t U2 = 0;
+      const uint8_t* ntext = nullptr;
+      const uint64_t kept = normalize(text, C, U, so, dout, Nc, U2, ntext);
+      if (kept > 0) {
+        dictionary_update(ntext, U2);
+        phase(WJ_PHASE_STREAM);
+        const size_t ci = chunk_tok.size();
+        if (chunk_map.size() <= ci) chunk_map.emplace_back();
+        uint32_t* cmap = buf<uint32_t>(chunk_map[ci], C);
+        k_norm_tid_map<<<grid_for(C, 256), 256, 0, st>>>((const uint32_t*)st_m1.p, (uint32_t)C, (const uint32_t*)u_tid.p,
+                                                         cmap);
+        launched();
+        chunk_tok.push_back(n_elems);
+        chunk_C.push_back((uint32_t)C);
+        n_elems += kept;
+        n_tokens += kept;
+      }
+    } else if (Nc > 0) {
       uint64_t NH = 0;
       if (hot_H) {  // hot (term, document) counters -> stream elements after the chunk's tokens
         const uint64_t HD = (uint64_t)hot_H * hot_D;
@@ -824,7 +991,20 @@ struct wj_index {
       Nc = tokenize_dedup(cv, (uint32_t)base, [&](uint64_t nc, uint32_t*& sp, uint32_t*& dp) {
         sp = buf<uint32_t>(x_loc_slot, nc + 16);
         dp = buf<uint32_t>(x_loc_doc, nc + 16);
-      }, C, U, lslot, ldoc);
+      }, C, U, lslot, ldoc, false);
+    }
+    // f4: the unique stems (stop words removed) are the chunk's terms; tokens map to them via st_m1
+    const Slot* tok_table = (const Slot*)table.p;
+    const uint32_t* tok_uid = (const uint32_t*)uid.p;
+    const uint8_t* term_text = text;
+    if (Nc > 0 && (stem_on || stop_on)) {
+      uint64_t U2 = 0;
+      const uint8_t* ntext = nullptr;
+      Nc = normalize(text, C, U, lslot, ldoc, Nc, U2, ntext);
+      U = Nc > 0 ? U2 : 0;
+      tok_table = (const Slot*)table_s.p;
+      tok_uid = (const uint32_t*)st_m1.p;
+      term_text = ntext;
     }
     // 2. pack per owner (collection b -> rank b mod K, or the balanced map)
     phase(WJ_PHASE_EXCHANGE);
@@ -865,7 +1045,7 @@ struct wj_index {
         WJ_CUDA_CHECK(cudaMemcpyAsync(&b_off[o], boff + t_off[o], 8, cudaMemcpyDeviceToHost, st));
       sync();
       send_terms = (uint8_t*)grow(x_send, b_off[K] + 16);
-      k_pack_terms<<<grid_for(U, 256), 256, 0, st>>>(sorted_u, (uint32_t)U, boff, (const uint4*)u_w.p, text,
+      k_pack_terms<<<grid_for(U, 256), 256, 0, st>>>(sorted_u, (uint32_t)U, boff, (const uint4*)u_w.p, term_text,
                                                     (const uint32_t*)u_ref.p, (const uint32_t*)u_len.p, send_terms);
       launched();
       // token records (key with xid, docID) partitioned by owner, stream (= docID) order kept
@@ -873,8 +1053,7 @@ struct wj_index {
       uint32_t* rd = buf<uint32_t>(x_rdoc, Nc + 16);
       if (K <= 64) {  // one radix pass on the owner bits of the mapped key
         uint32_t* km = buf<uint32_t>(x_keymap, C);
-        k_slot_xkey<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, (uint32_t)C, (const uint32_t*)uid.p, own,
-                                                      xid, km);
+        k_slot_xkey<<<grid_for(C, 256), 256, 0, st>>>(tok_table, (uint32_t)C, tok_uid, own, xid, km);
         launched();
         std::vector<std::pair<uint64_t, const uint32_t*>> segs{{0, km}};
         std::vector<uint64_t> ds;
@@ -902,11 +1081,11 @@ struct wj_index {
         uint32_t* ti = buf<uint32_t>(x_tidx, Nc + 16);
         uint32_t* tk2 = buf<uint32_t>(x_tkey2, Nc + 16);
         uint32_t* ti2 = buf<uint32_t>(x_tidx2, Nc + 16);
-        k_tok_owner<<<grid_for(Nc, 256), 256, 0, st>>>(lslot, Nc, (const uint32_t*)uid.p, own, (uint32_t)K, tk, ti, oc + K);
+        k_tok_owner<<<grid_for(Nc, 256), 256, 0, st>>>(lslot, Nc, tok_uid, own, (uint32_t)K, tk, ti, oc + K);
         launched();
         const bool in2 = sort_pairs<uint32_t>(tk, ti, tk2, ti2, Nc, 0, bits, nullptr, false);
         const uint32_t* sorted_t = in2 ? ti2 : ti;
-        k_pack_tok<<<grid_for(Nc, 256), 256, 0, st>>>(sorted_t, Nc, lslot, ldoc, (const uint32_t*)uid.p, xid, rk, rd);
+        k_pack_tok<<<grid_for(Nc, 256), 256, 0, st>>>(sorted_t, Nc, lslot, ldoc, tok_uid, xid, rk, rd);
         launched();
         WJ_CUDA_CHECK(cudaMemcpyAsync(oc_h.data(), oc + K, K * 4, cudaMemcpyDeviceToHost, st));
         sync();
@@ -1393,7 +1572,7 @@ extern "C" {
 int index_init(wj_index** out, const wj_config* cfg) {
   if (!out || !cfg) return WJ_ERR_INVALID_ARG;
   *out = nullptr;
-  if (cfg->world < 1 || cfg->world > 1024 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~(WJ_FLAG_PROFILE | WJ_FLAG_LOOPBACK | WJ_FLAG_VBYTE | WJ_FLAG_HOST_PIPELINE | WJ_FLAG_BALANCED_OWNERS)) || cfg->reserved) {
+  if (cfg->world < 1 || cfg->world > 1024 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~(WJ_FLAG_PROFILE | WJ_FLAG_LOOPBACK | WJ_FLAG_VBYTE | WJ_FLAG_HOST_PIPELINE | WJ_FLAG_BALANCED_OWNERS | WJ_FLAG_STEM | WJ_FLAG_STOPWORDS)) || cfg->reserved) {
     g_init_err = "invalid config";
     return WJ_ERR_INVALID_ARG;
   }
@@ -1420,6 +1599,8 @@ int index_init(wj_index** out, const wj_config* cfg) {
   ix->vbyte = (cfg->flags & WJ_FLAG_VBYTE) != 0;
   ix->pipeline = (cfg->flags & WJ_FLAG_HOST_PIPELINE) != 0;
   ix->balanced = (cfg->flags & WJ_FLAG_BALANCED_OWNERS) != 0;
+  ix->stem_on = (cfg->flags & WJ_FLAG_STEM) != 0;
+  ix->stop_on = (cfg->flags & WJ_FLAG_STOPWORDS) != 0;
   int rc = guarded(ix, [&]() {
     if (cfg->stream) {
       ix->st = (cudaStream_t)cfg->stream;
@@ -1470,6 +1651,7 @@ int index_init(wj_index** out, const wj_config* cfg) {
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rle_write_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)rle_smem_bytes()));
     ix->reset_state();
+    if (ix->stop_on) ix->build_stop_keys();
     return WJ_OK;
   });
   if (rc != WJ_OK) {
@@ -1669,6 +1851,47 @@ int index_owner_map(wj_index* ix, uint32_t* out, uint32_t n) {
   for (uint32_t b = 0; b < kCollections; ++b)
     out[b] = ix->owner_ready ? ix->owner_h[b] : b % (uint32_t)ix->world;
   return WJ_OK;
+}
+
+const char* index_stop_words(void) { return kStopList; }
+
+int index_debug_stem(int32_t device, const uint8_t* words, const uint32_t* word_off, uint32_t n, uint8_t* out,
+                     uint32_t* out_len) {
+  if (!words || !word_off || !out || !out_len) return WJ_ERR_INVALID_ARG;
+  for (uint32_t i = 0; i < n; ++i)
+    if (word_off[i + 1] < word_off[i] || word_off[i + 1] - word_off[i] > kMaxTermLen) return WJ_ERR_INVALID_ARG;
+  if (n == 0) return WJ_OK;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0 || device < 0 || device >= ndev) {
+    cudaGetLastError();
+    return WJ_ERR_CUDA;
+  }
+  const uint64_t nb = word_off[n];
+  uint8_t *dw = nullptr, *dout = nullptr;
+  uint32_t *doff = nullptr, *dlen = nullptr;
+  cudaStream_t s = nullptr;
+  int prev = 0;
+  cudaGetDevice(&prev);
+  bool ok = cudaSetDevice(device) == cudaSuccess && cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) == cudaSuccess &&
+            cudaMalloc(&dw, nb + 1) == cudaSuccess && cudaMalloc(&dout, nb + 1) == cudaSuccess &&
+            cudaMalloc(&doff, (n + 1) * 4ull) == cudaSuccess && cudaMalloc(&dlen, n * 4ull) == cudaSuccess &&
+            cudaMemcpyAsync(dw, words, nb, cudaMemcpyHostToDevice, s) == cudaSuccess &&
+            cudaMemcpyAsync(doff, word_off, (n + 1) * 4ull, cudaMemcpyHostToDevice, s) == cudaSuccess;
+  if (ok) {
+    k_stem_words<<<(n + 127) / 128, 128, 0, s>>>(dw, doff, n, dout, dlen);
+    ok = cudaGetLastError() == cudaSuccess &&
+         cudaMemcpyAsync(out, dout, nb, cudaMemcpyDeviceToHost, s) == cudaSuccess &&
+         cudaMemcpyAsync(out_len, dlen, n * 4ull, cudaMemcpyDeviceToHost, s) == cudaSuccess &&
+         cudaStreamSynchronize(s) == cudaSuccess;
+  }
+  cudaFree(dw);
+  cudaFree(dout);
+  cudaFree(doff);
+  cudaFree(dlen);
+  if (s) cudaStreamDestroy(s);
+  cudaSetDevice(prev);
+  cudaGetLastError();
+  return ok ? WJ_OK : WJ_ERR_CUDA;
 }
 
 const char* index_last_error(const wj_index* ix) { return ix ? ix->err.c_str() : g_init_err.c_str(); }

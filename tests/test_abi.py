@@ -60,3 +60,20 @@ def test_product_package_does_not_import_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
                 txt = open(os.path.join(dirpath, f), errors="ignore").read()
                 assert "import oracle" not in txt and "oracle/" not in txt and "oracle.h" not in txt, f
+
+
+def test_library_stop_list_is_sklearn_english():
+    # the CUDA path's own copy of the stop list (reading S20), pinned independently of the oracle's
+    text = pytest.importorskip("sklearn.feature_extraction.text")
+    words = wj.stop_words()
+    assert len(words) == len(set(words)) == 318
+    assert sorted(words) == sorted(text.ENGLISH_STOP_WORDS)
+
+
+def test_debug_stem_validates_without_gpu():
+    torch = pytest.importorskip("torch")
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    with pytest.raises(wj.WJError) as e:
+        wj.debug_stem([b"cats"])
+    assert e.value.code == -3  # WJ_ERR_CUDA: no CPU fallback

@@ -23,7 +23,8 @@ if not torch.cuda.is_available():  # pragma: no cover
 import paper_conf_ipps_weij11_b200 as wj  # noqa: E402
 
 
-def dist_index(text, doc_off, K, cuts=None, queries=(), vbyte=False, balanced=False, maps=None):
+def dist_index(text, doc_off, K, cuts=None, queries=(), vbyte=False, balanced=False, maps=None, stem=False,
+               stop=False):
     off = np.asarray(doc_off, dtype=np.uint64)
     text = np.asarray(text, dtype=np.uint8)
     n = len(off) - 1
@@ -35,7 +36,8 @@ def dist_index(text, doc_off, K, cuts=None, queries=(), vbyte=False, balanced=Fa
 
     def run(r):
         try:
-            with wj.Index(device=0, rank=r, world=K, hub=hub, own_stream=True, vbyte=vbyte, balanced=balanced) as ix:
+            with wj.Index(device=0, rank=r, world=K, hub=hub, own_stream=True, vbyte=vbyte, balanced=balanced, stem=stem,
+                          stop=stop) as ix:
                 for a, b in zip(cuts, cuts[1:]):
                     # rank r's contiguous document range of this chunk (rank order = DocID order)
                     bounds = [a + (b - a) * i // K for i in range(K + 1)]
