@@ -157,6 +157,11 @@ struct wj_index {
   uint32_t V = 0;
   uint64_t arena_used = 0;
   uint64_t table_est = 0;
+  // chunk table capacity = pow2 >= table_pct% of the expected unique terms (WJ_TABLE_PCT).  150%
+  // (16M slots on config 2): the emit kernel's probes are shorter (load ~0.3), but the slot ->
+  // rank map gathered by the first sort pass spans 64 MB; 125% (8M slots, load ~0.6) measured
+  // 0.1 ms/step faster overall (profiles/r01_README.md)
+  uint64_t table_pct = 125;
   uint64_t P = 0, TB = 0, PB = 0;  // postings, term bytes, vbyte code bytes
   bool vbyte = false;              // WJ_FLAG_VBYTE
   bool balanced = false;           // WJ_FLAG_BALANCED_OWNERS
@@ -644,7 +649,7 @@ struct wj_index {
     // the last U); a probe-sequence overflow retries with a doubled table
     uint64_t est = std::max<uint64_t>({table_est, Nc / 32, 4096});
     est = std::min<uint64_t>(est, Nc + 16);
-    C = pow2_at_least(est + est / 2);
+    C = pow2_at_least(est * table_pct / 100);
     uint32_t* slot_uid = nullptr;
     for (;;) {
       Slot* tab = buf<Slot>(table, C);
@@ -1617,6 +1622,7 @@ int index_init(wj_index** out, const wj_config* cfg) {
       }
     }
     if (const char* e = getenv("WJ_HOT_MIN_BYTES")) ix->hot_min_bytes = strtoull(e, nullptr, 10);
+    if (const char* e = getenv("WJ_TABLE_PCT")) ix->table_pct = std::max<uint64_t>(strtoull(e, nullptr, 10), 110);
     if (cfg->world > 1 || cfg->nccl_unique_id) {  // a transport at world 1 runs the same distributed path
       try {
         if (cfg->flags & WJ_FLAG_LOOPBACK)

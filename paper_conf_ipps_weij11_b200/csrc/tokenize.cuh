@@ -355,7 +355,8 @@ __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* tabl
   return kMiss;
 }
 
-__global__ void __launch_bounds__(kTokThreads) k_tok_emit(ChunkView cv, uint32_t n_segs, const uint64_t* kstart,
+// 5 CTAs/SM (48 registers): 0.3 ms/step faster than 4 CTAs (64 registers) on config 2
+__global__ void __launch_bounds__(kTokThreads, 5) k_tok_emit(ChunkView cv, uint32_t n_segs, const uint64_t* kstart,
                                                           const uint32_t* range_off, EmitOut eo) {
   __shared__ __align__(16) uint32_t win[kTokWarps][kWinBytes / 4];
   __shared__ uint32_t queue[kTokWarps][kQueueCap + 1];
