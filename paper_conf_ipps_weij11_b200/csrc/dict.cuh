@@ -521,7 +521,7 @@ __device__ __forceinline__ uint32_t count_less(const uint32_t* e_tid, uint32_t l
 
 __global__ void k_lexrank(const uint32_t* e_tid, const uint32_t* e_bkt, uint32_t V, const uint32_t* coll_base,
                           const uint32_t* coll_n, const LexGroups* g, const uint8_t* arena, const uint32_t* t_arena,
-                          const uint32_t* t_bucket, const uint32_t* t_cache, uint32_t* rank_of, uint32_t* term_at) {
+                          const uint32_t* t_bucket, const uint32_t* t_cache, uint32_t* rank_of, uint2* rank_info) {
   const uint32_t p = blockIdx.x * blockDim.x + threadIdx.x;
   if (p >= V) return;
   const uint32_t tid = e_tid[p], b = e_bkt[p];
@@ -553,7 +553,9 @@ __global__ void k_lexrank(const uint32_t* e_tid, const uint32_t* e_bkt, uint32_t
            count_less(e_tid, coll_base[11 + k], coll_base[11 + k] + coll_n[11 + k], arena, t_arena, t_bucket, tid);
   }
   rank_of[tid] = rank;
-  term_at[rank] = tid;
+  // by rank, for the final dictionary bytes: arena offset, Table I index | full term length << 16
+  const uint32_t a = t_arena[tid];
+  rank_info[rank] = make_uint2(a, b | ((bucket_plen(b) + arena[a]) << 16));
 }
 
 }  // namespace wj

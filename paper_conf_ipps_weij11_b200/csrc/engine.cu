@@ -1377,7 +1377,7 @@ struct wj_index {
     drain();
     const uint64_t NE = n_elems;  // stream elements (tokens, aggregated hot entries, holes)
     uint32_t* ro = buf<uint32_t>(rank_of, V);
-    uint32_t* ta = buf<uint32_t>(term_at, V);
+    uint2* ta = buf<uint2>(term_at, V);  // rank_info
     if ((uint64_t)V > (uint64_t)kRankMask + 1)
       throw StatusError{WJ_ERR_CAPACITY, "more than 2^25 terms in one dictionary slice"};
     if (V > 0) {
@@ -1460,14 +1460,13 @@ struct wj_index {
     uint64_t* to = buf<uint64_t>(term_off, (uint64_t)V + 1);
     TB = 0;
     if (V > 0) {
-      scan<uint64_t>(TermFullLen{ta, (const uint32_t*)t_bucket.p, (const uint32_t*)t_arena.p, (const uint8_t*)arena.p},
+      scan<uint64_t>(TermFullLen{ta},
                      V, to, to + V);
       WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 9, to + V, 8, cudaMemcpyDeviceToHost, st));
       sync();
       TB = h_scal[9];
       uint8_t* tbp = buf<uint8_t>(term_bytes, TB);
-      k_term_bytes<<<grid_for(V, 256), 256, 0, st>>>(ta, V, (const uint32_t*)t_bucket.p, (const uint32_t*)t_arena.p,
-                                                     (const uint8_t*)arena.p, to, tbp);
+      k_term_bytes<<<grid_for(V, 256), 256, 0, st>>>(ta, V, (const uint8_t*)arena.p, to, tbp);
       launched();
     } else {
       WJ_CUDA_CHECK(cudaMemsetAsync(to, 0, 8, st));

@@ -316,24 +316,18 @@ __global__ void k_df_cf(uint64_t* post_off, const uint64_t* cstart, uint32_t V, 
   cf[r] = tb - ta;
 }
 
-struct TermFullLen {
-  const uint32_t* term_at;
-  const uint32_t* t_bucket;
-  const uint32_t* t_arena;
-  const uint8_t* arena;
-  __device__ __forceinline__ uint64_t operator()(uint64_t r) const {
-    const uint32_t tid = term_at[r];
-    return bucket_plen(t_bucket[tid]) + arena[t_arena[tid]];
-  }
+struct TermFullLen {  // full length of the term of rank r (rank_info written by k_lexrank)
+  const uint2* rank_info;
+  __device__ __forceinline__ uint64_t operator()(uint64_t r) const { return rank_info[r].y >> 16; }
 };
 
 // final dictionary bytes: trie prefix (restored) + stored suffix
-__global__ void k_term_bytes(const uint32_t* term_at, uint32_t V, const uint32_t* t_bucket, const uint32_t* t_arena,
-                             const uint8_t* arena, const uint64_t* term_off, uint8_t* out) {
+__global__ void k_term_bytes(const uint2* rank_info, uint32_t V, const uint8_t* arena, const uint64_t* term_off,
+                             uint8_t* out) {
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= V) return;
-  const uint32_t tid = term_at[r];
-  const uint32_t b = t_bucket[tid], plen = bucket_plen(b), a = t_arena[tid], slen = arena[a];
+  const uint2 ri = rank_info[r];
+  const uint32_t b = ri.y & 0xFFFFu, plen = bucket_plen(b), a = ri.x, slen = (ri.y >> 16) - plen;
   uint8_t* o = out + term_off[r];
   for (uint32_t i = 0; i < plen; ++i) o[i] = (uint8_t)prefix_byte(b, i);
   for (uint32_t i = 0; i < slen; ++i) o[plen + i] = arena[a + 1 + i];
