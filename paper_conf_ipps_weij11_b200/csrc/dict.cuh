@@ -25,9 +25,17 @@
 namespace wj {
 
 // ------------------------------------------------------------------ term info (Table I)
+// New terms are radix-sorted by (collection, first kSortSfxBytes suffix bytes); equal keys are
+// ordered by the rest of the suffix (k_tie_fix).  4 bytes = the node cache: 47-bit keys,
+// 6 passes; 6 bytes: 63-bit keys, 8 passes.
+#ifndef WJ_SORT_SFX_BYTES
+#define WJ_SORT_SFX_BYTES 4
+#endif
+constexpr uint32_t kSortSfxBytes = WJ_SORT_SFX_BYTES;
+constexpr int kSortKeyBits = 15 + 8 * kSortSfxBytes;  // 17,613 collections < 2^15
 struct TermInfo {
   uint32_t bucket, plen, slen, cache;
-  uint64_t key;  // bucket << 48 | first 6 suffix bytes (big-endian, zero-padded)
+  uint64_t key;  // bucket << (8 kSortSfxBytes) | first kSortSfxBytes suffix bytes (big-endian, zero-padded)
 };
 
 __device__ __forceinline__ bool is_letter(uint32_t c) { return c - 'a' < 26u; }
@@ -64,7 +72,7 @@ __device__ __forceinline__ TermInfo term_info(const uint8_t* text, uint64_t ref,
     k6 |= (uint64_t)b << (40 - 8 * i);
   }
   ti.cache = c;
-  ti.key = ((uint64_t)ti.bucket << 48) | k6;
+  ti.key = kSortSfxBytes == 6 ? (((uint64_t)ti.bucket << 48) | k6) : (((uint64_t)ti.bucket << 32) | c);
   return ti;
 }
 
@@ -110,7 +118,7 @@ __device__ __forceinline__ TermInfo term_info_w(const uint4& w, const uint8_t* t
     k6 |= (uint64_t)b << (40 - 8 * i);
   }
   ti.cache = c;
-  ti.key = ((uint64_t)ti.bucket << 48) | k6;
+  ti.key = kSortSfxBytes == 6 ? (((uint64_t)ti.bucket << 48) | k6) : (((uint64_t)ti.bucket << 32) | c);
   return ti;
 }
 
@@ -278,7 +286,7 @@ __global__ void k_tie_fix(const uint64_t* key, uint32_t* val, uint32_t N, const 
   if (i + 1 >= N || key[i + 1] != key[i]) return;
   uint32_t e = i + 1;
   while (e < N && key[e] == key[i]) ++e;
-  const uint32_t plen = bucket_plen((uint32_t)(key[i] >> 48));
+  const uint32_t plen = bucket_plen((uint32_t)(key[i] >> (8 * kSortSfxBytes)));
   for (uint32_t a = i + 1; a < e; ++a) {
     const uint32_t x = val[a];
     const uint4 wx = u_w[x];
@@ -286,7 +294,7 @@ __global__ void k_tie_fix(const uint64_t* key, uint32_t* val, uint32_t N, const 
     uint32_t b = a;
     while (b > i) {
       const uint32_t y = val[b - 1];
-      if (cmp_sfx_sfx(u_w[y], u_ref[y], u_len[y] - plen, wx, rx, lx, text, plen, 6) <= 0) break;
+      if (cmp_sfx_sfx(u_w[y], u_ref[y], u_len[y] - plen, wx, rx, lx, text, plen, kSortSfxBytes) <= 0) break;
       val[b] = y;
       --b;
     }

@@ -1177,8 +1177,8 @@ struct wj_index {
     k_miss_compact<<<grid_for(U, 256), 256, 0, st>>>((const uint32_t*)u_tid.p, (const uint32_t*)midx.p,
                                                      (const uint64_t*)u_key.p, (uint32_t)U, kk, kv);
     launched();
-    // sort new terms by (collection, suffix): 8-bit LSD over the 63-bit key, then tie runs
-    const bool in2 = sort_pairs<uint64_t>(kk, kv, kk2, kv2, Nn, 0, 63, nullptr, false);
+    // sort new terms by (collection, suffix): 8-bit LSD over the kSortKeyBits-bit key, then tie runs
+    const bool in2 = sort_pairs<uint64_t>(kk, kv, kk2, kv2, Nn, 0, kSortKeyBits, nullptr, false);
     uint64_t* sk = in2 ? kk2 : kk;
     uint32_t* sv = in2 ? kv2 : kv;
     k_tie_fix<<<grid_for(Nn, 256), 256, 0, st>>>(sk, sv, (uint32_t)Nn, text, (const uint4*)u_w.p, (const uint32_t*)u_ref.p,

@@ -459,3 +459,22 @@ def test_pipeline_reset_drops_pending_and_errors_at_call():
         ix.finalize()
         got = ix.serialize()
     assert_same_index(got, oracle.index_bytes(text, off))
+
+
+@pytest.mark.parametrize("seed", [0, 1])
+def test_new_terms_sharing_long_prefixes(seed):
+    # new-term sort: equal (collection, first cached suffix bytes) keys are ordered by the rest of
+    # the suffix (tie runs); terms that are prefixes of each other, and bytes >= 0x80 after the prefix
+    rng = np.random.default_rng(seed)
+    stems = [b"internation", b"abcdefgh", b"zzzzzzz", b"aaaa", b"qu\xc3\xa9bec", b"1234567"]
+    words = []
+    for st_ in stems:
+        for _ in range(700):
+            n = int(rng.integers(0, 9))
+            words.append(st_ + bytes(int(x) for x in rng.choice(list(b"abcxyz09\xc3\xa9"), size=n)))
+        words += [st_[:k] for k in range(1, len(st_) + 1)]
+    docs = [b" ".join(words[i::7]) for i in range(7)] + [b" ".join(sorted(set(words)))]
+    text, off = docs_to_corpus(docs)
+    want = oracle.index_bytes(text, off)
+    assert_same_index(gpu_index(text, off), want)
+    assert_same_index(gpu_index(text, off, cuts=[0, 3, 5, 8]), want)
