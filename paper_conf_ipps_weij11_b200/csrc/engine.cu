@@ -1336,10 +1336,12 @@ struct wj_index {
       // the count bits of stream elements only reach a digit when passes cover bits >= 25
       const bool masked = mask_digits && kmask != ~K(0) && begin_bit + 8 * passes > kCountShift;
       auto up = [&] {
-        if (holes && masked) k_rs_up<K, true, true><<<G, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
-        else if (holes) k_rs_up<K, true, false><<<G, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
-        else if (masked) k_rs_up<K, false, true><<<G, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
-        else k_rs_up<K, false, false><<<G, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
+        WJ_CUDA_CHECK(cudaMemsetAsync(h1, 0, (size_t)256 * G * 4, st));
+        const uint32_t GU = G * kRsUpSplit;
+        if (holes && masked) k_rs_up<K, true, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
+        else if (holes) k_rs_up<K, true, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
+        else if (masked) k_rs_up<K, false, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
+        else k_rs_up<K, false, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
         launched();
       };
       if (timed) ktime(WJ_KERNEL_SORT_HIST, up); else up();

@@ -438,6 +438,11 @@ __device__ __forceinline__ bool rs_hole(K k, K kmask) { return HOLES && (k & ~km
 template <typename K, bool MASK>
 __device__ __forceinline__ K rs_dkey(K k, K kmask) { return MASK ? (k & kmask) : k; }
 
+// kRsUpSplit CTAs share one downsweep range (each a contiguous quarter), adding their counts to the
+// range's histogram column with global atomics (hist zeroed by the caller): 4x the warps in flight for
+// the map gather of the first pass, which is L2-latency bound at 2 CTAs/SM.
+constexpr int kRsUpSplit = 4;
+
 template <typename K, bool HOLES, bool MASK>
 __global__ void __launch_bounds__(256) k_rs_up(K* keys, uint64_t n, uint64_t per, int shift,
                                                const uint32_t* __restrict__ map, uint32_t* hist, K kmask) {
@@ -445,8 +450,13 @@ __global__ void __launch_bounds__(256) k_rs_up(K* keys, uint64_t n, uint64_t per
   const int w = threadIdx.x >> 5;
   for (int x = 0; x < kOsWarps; ++x) h[x][threadIdx.x] = 0;
   __syncthreads();
-  const uint64_t lo = (uint64_t)blockIdx.x * per;  // multiple of the tile size: 16-byte aligned
-  const uint64_t hi = lo + per < n ? lo + per : n;
+  const uint32_t range = blockIdx.x / kRsUpSplit, part = blockIdx.x % kRsUpSplit;
+  const uint32_t n_ranges = gridDim.x / kRsUpSplit;
+  const uint64_t sub = per / kRsUpSplit;  // per is a multiple of the 4096-element tile
+  const uint64_t rhi = (uint64_t)range * per + per < n ? (uint64_t)range * per + per : n;
+  const uint64_t lo0 = (uint64_t)range * per + part * sub;  // 16-byte aligned
+  const uint64_t lo = lo0 < rhi ? lo0 : rhi;
+  const uint64_t hi = (part + 1 == kRsUpSplit) ? rhi : (lo0 + sub < rhi ? lo0 + sub : rhi);
   constexpr int V = 16 / sizeof(K);  // keys per 16-byte vector
   const uint64_t nvec = (hi - lo) / V;
   typedef typename std::conditional<sizeof(K) == 4, uint4, ulonglong2>::type Vec;
@@ -493,7 +503,7 @@ __global__ void __launch_bounds__(256) k_rs_up(K* keys, uint64_t n, uint64_t per
   uint32_t t = 0;
 #pragma unroll
   for (int x = 0; x < kOsWarps; ++x) t += h[x][threadIdx.x];
-  hist[(uint64_t)threadIdx.x * gridDim.x + blockIdx.x] = t;
+  if (t) atomicAdd(&hist[(uint64_t)threadIdx.x * n_ranges + range], t);
 }
 
 template <typename K>
