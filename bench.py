@@ -38,15 +38,16 @@ WORKLOAD = {2: "clueweb09-shaped synthetic, 1 GiB per GPU (BASELINE configs[1])"
 HBM_FALLBACK_GBS = 6650.0
 
 # Algorithmic bytes per launch of each timed kernel, given the chunk's
-# T (text bytes), N (kept tokens), P (postings).
+# T (text bytes), N (kept tokens), P (postings), E (stream elements after the per-document combine).
 KERNEL_BYTES = {
-    "tokenize_count": lambda T, N, P: T,                  # read the text once
-    "tokenize_emit": lambda T, N, P: T + 8 * N,           # read text, write (slot u32, doc u32) per token
-    "slot_to_tid": lambda T, N, P: 8 * N,                 # read + write u32 per token
-    "map_rank": lambda T, N, P: 8 * N,                    # read + write u32 per token
-    "sort_hist": lambda T, N, P: 4 * N,                   # read u32 keys
-    "sort_scatter": lambda T, N, P: 16 * N,               # read + write (u32 key, u32 doc) per token
-    "rle_emit": lambda T, N, P: 8 * N + 8 * P,            # read (key, doc), write (docid, tf)
+    "tokenize_count": lambda T, N, P, E: T,                 # read the text once
+    "tokenize_emit": lambda T, N, P, E: T + 8 * N,          # read text, write (slot u32, doc u32) per token
+    "slot_to_tid": lambda T, N, P, E: 8 * N,                # read + write u32 per token
+    "map_rank": lambda T, N, P, E: 8 * E,                   # read + write u32 per element
+    "doc_combine": lambda T, N, P, E: 8 * N + 8 * E,        # read (slot, doc) per token, write per element
+    "sort_hist": lambda T, N, P, E: 4 * E,                  # read u32 keys
+    "sort_scatter": lambda T, N, P, E: 16 * E,              # read + write (u32 key, u32 doc) per element
+    "rle_emit": lambda T, N, P, E: 8 * E + 8 * P,           # read (key, doc), write (docid, tf)
 }
 
 
@@ -281,7 +282,8 @@ def main():
     dom = max((k for k in KERNEL_BYTES if kcnt.get(k)), key=lambda k: kms[k])
     per_launch_ms = kms[dom] / kcnt[dom]
     launches_per_step = kcnt[dom] / args.steps
-    bytes_per_launch = KERNEL_BYTES[dom](T, N, P) if dom not in ("sort_hist", "sort_scatter") else KERNEL_BYTES[dom](T, N, P)
+    E = s1["stream_elems"]
+    bytes_per_launch = KERNEL_BYTES[dom](T, N, P, E)
     achieved = bytes_per_launch / (per_launch_ms / 1e3) / 1e9
     traffic = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -367,7 +369,7 @@ def main():
             "vs_baseline": None, "dtype": "u32", "data": "synthetic (gen/wjgen.cpp seeded generator)",
             "config": {"workload": WORKLOAD.get(args.config, str(args.config)), "bytes_per_gpu": T,
                        "docs_per_gpu": len(doc_off) - 1, "tokens_per_gpu": N, "terms_per_gpu": V,
-                       "postings_per_gpu": P, "l2": "no flush: 1 GiB input per step > 126 MB L2",
+                       "postings_per_gpu": P, "stream_elems_per_gpu": E, "l2": "no flush: 1 GiB input per step > 126 MB L2",
                        "postings_format": "vbyte d-gaps (WJINV002)" if args.vbyte else "u32 docid + u32 tf (WJINV001)",
                        "parallelism": "single GPU" if world == 1 else
                        f"{world} ranks: document ranges, trie collections bin-packed by sampled load (P:212), NCCL all-to-all-v"},

@@ -113,7 +113,8 @@ enum {
   WJ_KERNEL_SORT_HIST,          /* finalize: radix digit histogram (token stream)                  */
   WJ_KERNEL_SORT_SCATTER,       /* finalize: stable radix scatter (token stream)                   */
   WJ_KERNEL_RLE_EMIT,           /* finalize: run-length (docID, tf) emit                           */
-  WJ_KERNEL_COUNT = 8
+  WJ_KERNEL_DOC_COMBINE,        /* per-document pre-aggregation of a chunk's stream (combine.cuh)   */
+  WJ_KERNEL_COUNT = 9
 };
 
 typedef struct {
@@ -127,6 +128,8 @@ typedef struct {
   uint64_t btree_height_max;       /* tallest trie-collection B-tree                                 */
   uint64_t exchange_bytes;         /* world > 1: bytes this rank sent                                */
   uint64_t device_bytes;           /* device memory held by the context                              */
+  uint64_t stream_elems;           /* (term, docID) stream elements of the index so far: tokens after */
+                                   /* the per-document combine (elements the finalize sort moves)    */
   /* The fields below are cumulative since index_init (index_reset does not clear them).          */
   double phase_ms[WJ_PHASE_COUNT]; /* WJ_FLAG_PROFILE: accumulated CUDA-event time per phase        */
   uint64_t phase_launches[WJ_PHASE_COUNT];

@@ -7,6 +7,7 @@
 #include <vector>
 
 #include "../../include/wjindex.h"
+#include "combine.cuh"
 #include "common.cuh"
 #include "dict.cuh"
 #include "dist.cuh"
@@ -175,6 +176,12 @@ struct wj_index {
       samp_ck2, samp_cv2, samp_n;
   uint32_t hot_H = 0, hot_D = 0;
   bool stream_has_hot = false;  // some chunk appended hot-term elements (holes + counts > 1)
+  bool stream_counts = false;   // some chunk's elements carry counts > 1 (doc combine, combine.cuh)
+  // Per-document pre-aggregation of the stream (combine.cuh) is opt-in (WJ_DOC_COMBINE=1): it shrinks
+  // the sorted stream to 0.68 N on config 2 (sort 3.69 -> 2.67 ms) but its shared-memory hash costs two
+  // shared atomics per token (2 cycles/lane on sm_100a): 3.65 ms, a net loss (profiles/r01_README.md).
+  bool combine_on = false;
+  DevBuf dc_look;
   // Sampled hot-term path (hot.cuh) is opt-in: on config 2 it removes ~30% of the
   // stream elements but its per-document counters cost more global atomics in the emit kernel than
   // the sort saves (profiles/r01_README.md).  WJ_HOT_MIN_BYTES=<bytes> enables it for larger chunks.
@@ -185,7 +192,8 @@ struct wj_index {
   DevBuf nodes, coll_root, coll_n, coll_base, coll_base2, e_tid, e_bkt, e_tid2, e_bkt2, arena, t_arena, t_cache,
       t_bucket;
   // device scalars: [0] tokens, [1] dropped, [2] U, [3] Nnew, [4] arena total, [5] overflow|bad,
-  // [6] tid counter (u32 view), [7] level count, [8] P, [9] TB, [10] bad doc_off
+  // [6] tid counter (u32 view), [7] level count, [8] P, [9] TB, [10] bad doc_off, [11] rle tokens,
+  // [12] doc-combine output length
   DevBuf scal;
   uint64_t* h_scal = nullptr;  // pinned
   // token stream (termID, docID) of all chunks
@@ -374,6 +382,7 @@ struct wj_index {
     chunk_C.clear();
     n_docs = n_tokens = n_dropped = n_chunks = n_elems = 0;
     stream_has_hot = false;
+    stream_counts = false;
     unique_last = new_last = n_nodes = height_max = 0;
     exchange_bytes = 0;
     V = 0;
@@ -840,6 +849,26 @@ struct wj_index {
     }
   }
 
+  // Per-document pre-aggregation of a chunk's stream segment in place (combine.cuh): elements of
+  // one (slot, docID) pair merge into one count-carrying element.  Returns the new length.
+  uint64_t doc_combine(uint32_t* key, uint32_t* doc, uint64_t n) {
+    if (!combine_on || n < 2) return n;
+    phase(WJ_PHASE_STREAM);
+    const uint32_t ntiles = (uint32_t)((n + kDcTile - 1) / kDcTile);
+    uint64_t* lk = buf<uint64_t>(dc_look, (uint64_t)ntiles + 1);
+    WJ_CUDA_CHECK(cudaMemsetAsync(lk, 0, ((size_t)ntiles + 1) * 8, st));
+    ktime(WJ_KERNEL_DOC_COMBINE, [&] {
+      k_doc_combine<<<ntiles, kDcThreads, dc_smem_bytes(), st>>>(key, doc, n, ntiles, lk, (uint32_t*)(lk + ntiles),
+                                                                 (uint32_t*)(dscal() + 12));
+      launched();
+    });
+    WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 12, dscal() + 12, 8, cudaMemcpyDeviceToHost, st));
+    sync();
+    const uint64_t m = (uint32_t)h_scal[12];
+    if (m < n) stream_counts = true;
+    return m;
+  }
+
   // the chunk's (slot, docID) stream is the postings input; keep its slot -> termID map
   void register_chunk_map(uint64_t C, uint64_t tok_start) {
     phase(WJ_PHASE_STREAM);
@@ -927,6 +956,7 @@ struct wj_index {
       uint64_t U2 = 0;
       const uint8_t* ntext = nullptr;
       const uint64_t kept = normalize(text, C, U, so, dout, Nc, U2, ntext);
+      const uint64_t kept_el = doc_combine(so, dout, kept);
       if (kept > 0) {
         dictionary_update(ntext, U2);
         phase(WJ_PHASE_STREAM);
@@ -938,7 +968,7 @@ struct wj_index {
         launched();
         chunk_tok.push_back(n_elems);
         chunk_C.push_back((uint32_t)C);
-        n_elems += kept;
+        n_elems += kept_el;
         n_tokens += kept;
       }
     } else if (Nc > 0) {
@@ -959,10 +989,11 @@ struct wj_index {
                                                        (const uint32_t*)hot_slotb.p, doc_base, gt + base, gd + base);
         launched();
       }
+      const uint64_t Ne = hot_H ? Nc : doc_combine(so, dout, Nc);
       dictionary_update(text, U);
       register_chunk_map(C, n_elems);
       if (hot_H) stream_has_hot = true;
-      n_elems += Nc + NH;
+      n_elems += Ne + NH;
       n_tokens += Nc;
     }
     n_docs += nd;
@@ -1433,14 +1464,14 @@ struct wj_index {
       uint32_t* od = buf<uint32_t>(out_doc, N);
       uint32_t* of = buf<uint32_t>(out_tf, N);
       ktime(WJ_KERNEL_RLE_EMIT, [&] {
-        if (stream_has_hot)
+        if (stream_has_hot || stream_counts)
           k_rle_count<true><<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc, rt);
         else
           k_rle_count<false><<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc, rt);
         launched();
         scan<uint32_t>(ArrayIn<uint32_t>{rc}, G, rc, (uint32_t*)(dscal() + 8));
         scan<uint64_t>(ArrayIn<uint64_t>{rt}, G, rt, (uint64_t*)(dscal() + 11));
-        if (stream_has_hot)
+        if (stream_has_hot || stream_counts)
           k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl);
         else
           k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl);
@@ -1622,6 +1653,7 @@ int index_init(wj_index** out, const wj_config* cfg) {
         WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->pipe_done[i], cudaEventDisableTiming));
       }
     }
+    if (const char* e = getenv("WJ_DOC_COMBINE")) ix->combine_on = strtoull(e, nullptr, 10) != 0;
     if (const char* e = getenv("WJ_HOT_MIN_BYTES")) ix->hot_min_bytes = strtoull(e, nullptr, 10);
     if (const char* e = getenv("WJ_TABLE_PCT")) ix->table_pct = std::max<uint64_t>(strtoull(e, nullptr, 10), 110);
     if (cfg->world > 1 || cfg->nccl_unique_id) {  // a transport at world 1 runs the same distributed path
@@ -1653,6 +1685,8 @@ int index_init(wj_index** out, const wj_config* cfg) {
     WJ_DS_ATTR(uint64_t, true, true); WJ_DS_ATTR(uint32_t, false, false); WJ_DS_ATTR(uint32_t, true, false);
     WJ_DS_ATTR(uint32_t, false, true); WJ_DS_ATTR(uint32_t, true, true);
 #undef WJ_DS_ATTR
+    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_doc_combine, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)dc_smem_bytes()));
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rle_write_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)rle_smem_bytes()));
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rle_write_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1761,6 +1795,7 @@ int index_stats(wj_index* ix, wj_stats* out) {
     out->btree_height_max = ix->height_max;
     out->exchange_bytes = ix->exchange_bytes;
     out->device_bytes = ix->device_bytes;
+    out->stream_elems = ix->n_elems;
     for (int i = 0; i < WJ_PHASE_COUNT; ++i) {
       out->phase_ms[i] = ix->phase_ms[i];
       out->phase_launches[i] = ix->phase_launches[i];

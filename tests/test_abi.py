@@ -37,10 +37,20 @@ def test_library_is_sm100a():
     assert "sm_100a" in out
 
 
-def test_struct_sizes_match_header():
+def test_struct_sizes_match_header(tmp_path):
     # wj_config: 3 x i32 + pad + 2 pointers + u64 + 2 x u32 = 48 bytes on LP64
     assert ctypes.sizeof(wj.Config) == 48
-    assert ctypes.sizeof(wj.Stats) == 15 * 8 + 16 * 8 + 16 * 8 + 8 * 8 + 8 * 8
+    # the binding's structs against the C compiler's view of include/wjindex.h
+    src = tmp_path / "sz.c"
+    src.write_text('#include <stdio.h>\n#include "wjindex.h"\n'
+                   'int main(void){printf("%zu %zu %d %d\\n", sizeof(wj_config), sizeof(wj_stats),'
+                   ' (int)WJ_PHASE_COUNT, (int)WJ_KERNEL_COUNT); return 0;}\n')
+    exe = tmp_path / "sz"
+    subprocess.run(["gcc", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)], check=True)
+    cfg, sts, nph, nk = map(int, subprocess.run([str(exe)], check=True, capture_output=True, text=True).stdout.split())
+    assert ctypes.sizeof(wj.Config) == cfg
+    assert ctypes.sizeof(wj.Stats) == sts
+    assert len(wj.KERNELS) == nk and nph == 16
     assert wj.NODE_DTYPE.itemsize == 512  # Table II
 
 
