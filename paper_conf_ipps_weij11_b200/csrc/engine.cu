@@ -158,11 +158,11 @@ struct wj_index {
   uint32_t V = 0;
   uint64_t arena_used = 0;
   uint64_t table_est = 0;
-  // chunk table capacity = pow2 >= table_pct% of the expected unique terms (WJ_TABLE_PCT).  150%
-  // (16M slots on config 2): the emit kernel's probes are shorter (load ~0.3), but the slot ->
-  // rank map gathered by the first sort pass spans 64 MB; 125% (8M slots, load ~0.6) measured
-  // 0.1 ms/step faster overall (profiles/r01_README.md)
-  uint64_t table_pct = 125;
+  // chunk table capacity = table_pct% of the expected unique terms (WJ_TABLE_PCT), any multiple of
+  // 4096 slots (mulhi indexing).  On config 2 the emit kernel gets faster with capacity (2.82 / 2.45 /
+  // 2.36 ms at 125 / 190 / 320%: shorter probe runs) while the slot -> rank gather of the first sort
+  // pass and the slot scans get slower; 190-230% was the best step time (profiles/r01_README.md)
+  uint64_t table_pct = 200;
   uint64_t P = 0, TB = 0, PB = 0;  // postings, term bytes, vbyte code bytes
   bool vbyte = false;              // WJ_FLAG_VBYTE
   bool balanced = false;           // WJ_FLAG_BALANCED_OWNERS
@@ -176,12 +176,14 @@ struct wj_index {
       samp_ck2, samp_cv2, samp_n;
   uint32_t hot_H = 0, hot_D = 0;
   bool stream_has_hot = false;  // some chunk appended hot-term elements (holes + counts > 1)
-  bool stream_counts = false;   // some chunk's elements carry counts > 1 (doc combine, combine.cuh)
-  // Per-document pre-aggregation of the stream (combine.cuh) is opt-in (WJ_DOC_COMBINE=1): it shrinks
-  // the sorted stream to 0.68 N on config 2 (sort 3.69 -> 2.67 ms) but its shared-memory hash costs two
-  // shared atomics per token (2 cycles/lane on sm_100a): 3.65 ms, a net loss (profiles/r01_README.md).
+  // Per-document pre-aggregation of the stream before the finalize sort (combine.cuh) is opt-in
+  // (WJ_DOC_COMBINE=1): it shrinks the sorted stream to 0.68 N on config 2 (sort 3.76 -> 2.66 ms), but
+  // merging needs a shared hash table per tile and neither a CAS insert (returning shared atomics run
+  // at ~2 cycles/lane: 3.6 ms) nor a CAS-free round-based insert (5.8 ms) costs less than it saves
+  // (profiles/r01_README.md)
   bool combine_on = false;
-  DevBuf dc_look;
+  DevBuf dc_len;
+  uint64_t sorted_elems = 0;    // stream elements the last finalize sorted (after the combine)
   // Sampled hot-term path (hot.cuh) is opt-in: on config 2 it removes ~30% of the
   // stream elements but its per-document counters cost more global atomics in the emit kernel than
   // the sort saves (profiles/r01_README.md).  WJ_HOT_MIN_BYTES=<bytes> enables it for larger chunks.
@@ -382,7 +384,7 @@ struct wj_index {
     chunk_C.clear();
     n_docs = n_tokens = n_dropped = n_chunks = n_elems = 0;
     stream_has_hot = false;
-    stream_counts = false;
+    sorted_elems = 0;
     unique_last = new_last = n_nodes = height_max = 0;
     exchange_bytes = 0;
     V = 0;
@@ -479,7 +481,7 @@ struct wj_index {
     eo.hot_tf = (uint32_t*)hot_tfb.p;
     eo.table = tab;
     eo.slot_ref = sref;
-    eo.mask = (uint32_t)(C - 1);
+    eo.cap = (uint32_t)C;
     eo.doc_base = doc_base;
     eo.slot = slot_out;
     eo.doc = doc_out;
@@ -624,6 +626,13 @@ struct wj_index {
     if (!bytes && cudaCtxResetPersistingL2Cache() != cudaSuccess) cudaGetLastError();
   }
 
+  // chunk table capacity: WJ_TABLE_POW2=1 rounds to a power of two (the layout before mulhi indexing),
+  // else to a multiple of 4096 slots
+  bool table_pow2 = false;
+  uint64_t table_cap(uint64_t x) const {
+    if (table_pow2) return pow2_at_least(x);
+    return std::max<uint64_t>((x + 4095) / 4096 * 4096, 4096);
+  }
   static uint64_t pow2_at_least(uint64_t x) {
     uint64_t c = 1;
     while (c < x) c <<= 1;
@@ -658,7 +667,7 @@ struct wj_index {
     // the last U); a probe-sequence overflow retries with a doubled table
     uint64_t est = std::max<uint64_t>({table_est, Nc / 32, 4096});
     est = std::min<uint64_t>(est, Nc + 16);
-    C = pow2_at_least(est * table_pct / 100);
+    C = table_cap(est * table_pct / 100);
     uint32_t* slot_uid = nullptr;
     for (;;) {
       Slot* tab = buf<Slot>(table, C);
@@ -667,7 +676,7 @@ struct wj_index {
       if (hot_H) {  // hot terms first: their slots in this table, and the lookup table for the emit
         WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 5, 0, 8, st));
         HotEntry* ht = (HotEntry*)grow(hot_tab, kHotTable * sizeof(HotEntry));
-        k_hot_build<<<1, 1, 0, st>>>((const ulonglong2*)hot_kb.p, hot_H, tab, sref, (uint32_t)(C - 1), ht,
+        k_hot_build<<<1, 1, 0, st>>>((const ulonglong2*)hot_kb.p, hot_H, tab, sref, (uint32_t)C, ht,
                                      (uint32_t*)hot_slotb.p, (uint32_t*)(dscal() + 5));
         launched();
         uint32_t* tf = buf<uint32_t>(hot_tfb, (uint64_t)hot_H * hot_D);
@@ -849,26 +858,6 @@ struct wj_index {
     }
   }
 
-  // Per-document pre-aggregation of a chunk's stream segment in place (combine.cuh): elements of
-  // one (slot, docID) pair merge into one count-carrying element.  Returns the new length.
-  uint64_t doc_combine(uint32_t* key, uint32_t* doc, uint64_t n) {
-    if (!combine_on || n < 2) return n;
-    phase(WJ_PHASE_STREAM);
-    const uint32_t ntiles = (uint32_t)((n + kDcTile - 1) / kDcTile);
-    uint64_t* lk = buf<uint64_t>(dc_look, (uint64_t)ntiles + 1);
-    WJ_CUDA_CHECK(cudaMemsetAsync(lk, 0, ((size_t)ntiles + 1) * 8, st));
-    ktime(WJ_KERNEL_DOC_COMBINE, [&] {
-      k_doc_combine<<<ntiles, kDcThreads, dc_smem_bytes(), st>>>(key, doc, n, ntiles, lk, (uint32_t*)(lk + ntiles),
-                                                                 (uint32_t*)(dscal() + 12));
-      launched();
-    });
-    WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 12, dscal() + 12, 8, cudaMemcpyDeviceToHost, st));
-    sync();
-    const uint64_t m = (uint32_t)h_scal[12];
-    if (m < n) stream_counts = true;
-    return m;
-  }
-
   // the chunk's (slot, docID) stream is the postings input; keep its slot -> termID map
   void register_chunk_map(uint64_t C, uint64_t tok_start) {
     phase(WJ_PHASE_STREAM);
@@ -956,7 +945,6 @@ struct wj_index {
       uint64_t U2 = 0;
       const uint8_t* ntext = nullptr;
       const uint64_t kept = normalize(text, C, U, so, dout, Nc, U2, ntext);
-      const uint64_t kept_el = doc_combine(so, dout, kept);
       if (kept > 0) {
         dictionary_update(ntext, U2);
         phase(WJ_PHASE_STREAM);
@@ -968,7 +956,7 @@ struct wj_index {
         launched();
         chunk_tok.push_back(n_elems);
         chunk_C.push_back((uint32_t)C);
-        n_elems += kept_el;
+        n_elems += kept;
         n_tokens += kept;
       }
     } else if (Nc > 0) {
@@ -989,11 +977,10 @@ struct wj_index {
                                                        (const uint32_t*)hot_slotb.p, doc_base, gt + base, gd + base);
         launched();
       }
-      const uint64_t Ne = hot_H ? Nc : doc_combine(so, dout, Nc);
       dictionary_update(text, U);
       register_chunk_map(C, n_elems);
       if (hot_H) stream_has_hot = true;
-      n_elems += Ne + NH;
+      n_elems += Nc + NH;
       n_tokens += Nc;
     }
     n_docs += nd;
@@ -1322,7 +1309,7 @@ struct wj_index {
                   const uint32_t* rank_of, bool timed,
                   const std::vector<std::pair<uint64_t, const uint32_t*>>* segs = nullptr, K kmask = ~K(0),
                   bool skip0 = false, uint64_t* n_out = nullptr, bool mask_digits = true,
-                  std::vector<uint64_t>* digit_start = nullptr) {
+                  std::vector<uint64_t>* digit_start = nullptr, bool combine = false) {
     if (n_out) *n_out = n;
     if (n == 0) return false;
     int passes = end_bit > begin_bit ? (end_bit - begin_bit + 7) / 8 : 0;
@@ -1351,6 +1338,20 @@ struct wj_index {
     const uint32_t* first_map = (segs && !multi_map) ? (*segs)[0].second : rank_of;
     bool in1 = false;
     uint64_t cur_n = n;
+    // per-document combine (combine.cuh) on the first pass's ranges: range c keeps rlen[c] elements
+    const uint32_t* rlen = nullptr;
+    if (combine) {
+      uint64_t per = (n + kRsCtas - 1) / kRsCtas;
+      per = (per + kOsTile - 1) / kOsTile * kOsTile;
+      const uint32_t G = (uint32_t)((n + per - 1) / per);
+      uint32_t* rl = buf<uint32_t>(dc_len, G);
+      auto c = [&] {
+        k_doc_combine<<<G, kDcThreads, dc_smem_bytes(), st>>>((uint32_t*)k0, v0, n, per, rl);
+        launched();
+      };
+      if (timed) ktime(WJ_KERNEL_DOC_COMBINE, c); else c();
+      rlen = rl;
+    }
     for (int p = 0; p < passes; ++p) {
       uint64_t per = (cur_n + kRsCtas - 1) / kRsCtas;
       per = (per + kOsTile - 1) / kOsTile * kOsTile;
@@ -1364,25 +1365,26 @@ struct wj_index {
       const int shift = begin_bit + 8 * p;
       const uint32_t* mp = p == 0 ? first_map : nullptr;
       const bool holes = skip0 && p == 0;
+      const uint32_t* rl = p == 0 ? rlen : nullptr;
       // the count bits of stream elements only reach a digit when passes cover bits >= 25
       const bool masked = mask_digits && kmask != ~K(0) && begin_bit + 8 * passes > kCountShift;
       auto up = [&] {
         WJ_CUDA_CHECK(cudaMemsetAsync(h1, 0, (size_t)256 * G * 4, st));
         const uint32_t GU = G * kRsUpSplit;
-        if (holes && masked) k_rs_up<K, true, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
-        else if (holes) k_rs_up<K, true, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
-        else if (masked) k_rs_up<K, false, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
-        else k_rs_up<K, false, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
+        if (holes && masked) k_rs_up<K, true, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, rl);
+        else if (holes) k_rs_up<K, true, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, rl);
+        else if (masked) k_rs_up<K, false, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, rl);
+        else k_rs_up<K, false, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, rl);
         launched();
       };
       if (timed) ktime(WJ_KERNEL_SORT_HIST, up); else up();
       scan<uint32_t>(ArrayIn<uint32_t>{h1}, (uint64_t)256 * G, h2, h2 + (uint64_t)256 * G);
       auto down = [&] {
         const size_t sm = ds_smem_bytes<K>();
-        if (holes && masked) k_rs_down2<K, true, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
-        else if (holes) k_rs_down2<K, true, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
-        else if (masked) k_rs_down2<K, false, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
-        else k_rs_down2<K, false, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
+        if (holes && masked) k_rs_down2<K, true, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, rl);
+        else if (holes) k_rs_down2<K, true, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, rl);
+        else if (masked) k_rs_down2<K, false, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, rl);
+        else k_rs_down2<K, false, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, rl);
         launched();
       };
       if (timed) ktime(WJ_KERNEL_SORT_SCATTER, down); else down();
@@ -1393,7 +1395,7 @@ struct wj_index {
         sync();
         digit_start->assign(ds.begin(), ds.end());
       }
-      if (holes) {  // elements that survive the compaction
+      if (holes || rl) {  // elements that survive the compaction / the combine
         uint32_t tot = 0;
         WJ_CUDA_CHECK(cudaMemcpyAsync(&tot, h2 + (uint64_t)256 * G, 4, cudaMemcpyDeviceToHost, st));
         sync();
@@ -1448,8 +1450,12 @@ struct wj_index {
         segs.emplace_back(chunk_tok[c], m);
       }
       uint64_t N = NE;
+      // the combine needs single-token input elements (no hot-term count elements or holes)
+      const bool combine = combine_on && !stream_has_hot;
       const bool in1 =
-          sort_pairs<uint32_t>(kt, dt, k1, v1, NE, 0, bits, nullptr, true, &segs, kRankMask, stream_has_hot, &N);
+          sort_pairs<uint32_t>(kt, dt, k1, v1, NE, 0, bits, nullptr, true, &segs, kRankMask, stream_has_hot, &N, true,
+                               nullptr, combine);
+      sorted_elems = N;
       f_key = in1 ? k1 : kt;
       f_doc = in1 ? v1 : dt;
 
@@ -1464,14 +1470,14 @@ struct wj_index {
       uint32_t* od = buf<uint32_t>(out_doc, N);
       uint32_t* of = buf<uint32_t>(out_tf, N);
       ktime(WJ_KERNEL_RLE_EMIT, [&] {
-        if (stream_has_hot || stream_counts)
+        if (stream_has_hot || combine)
           k_rle_count<true><<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc, rt);
         else
           k_rle_count<false><<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc, rt);
         launched();
         scan<uint32_t>(ArrayIn<uint32_t>{rc}, G, rc, (uint32_t*)(dscal() + 8));
         scan<uint64_t>(ArrayIn<uint64_t>{rt}, G, rt, (uint64_t*)(dscal() + 11));
-        if (stream_has_hot || stream_counts)
+        if (stream_has_hot || combine)
           k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl);
         else
           k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl);
@@ -1655,6 +1661,7 @@ int index_init(wj_index** out, const wj_config* cfg) {
     }
     if (const char* e = getenv("WJ_DOC_COMBINE")) ix->combine_on = strtoull(e, nullptr, 10) != 0;
     if (const char* e = getenv("WJ_HOT_MIN_BYTES")) ix->hot_min_bytes = strtoull(e, nullptr, 10);
+    if (const char* e = getenv("WJ_TABLE_POW2")) ix->table_pow2 = strtoull(e, nullptr, 10) != 0;
     if (const char* e = getenv("WJ_TABLE_PCT")) ix->table_pct = std::max<uint64_t>(strtoull(e, nullptr, 10), 110);
     if (cfg->world > 1 || cfg->nccl_unique_id) {  // a transport at world 1 runs the same distributed path
       try {
@@ -1795,7 +1802,7 @@ int index_stats(wj_index* ix, wj_stats* out) {
     out->btree_height_max = ix->height_max;
     out->exchange_bytes = ix->exchange_bytes;
     out->device_bytes = ix->device_bytes;
-    out->stream_elems = ix->n_elems;
+    out->stream_elems = ix->finalized ? ix->sorted_elems : ix->n_elems;
     for (int i = 0; i < WJ_PHASE_COUNT; ++i) {
       out->phase_ms[i] = ix->phase_ms[i];
       out->phase_launches[i] = ix->phase_launches[i];

@@ -75,7 +75,7 @@ __global__ void k_hot_extract(const Slot* table, const uint32_t* slots, uint32_t
 }
 
 // one thread: insert the hot terms into the chunk table (their slots) and into the hot lookup table
-__global__ void k_hot_build(const ulonglong2* hk, uint32_t H, Slot* table, uint32_t* slot_ref, uint32_t mask,
+__global__ void k_hot_build(const ulonglong2* hk, uint32_t H, Slot* table, uint32_t* slot_ref, uint32_t cap,
                             HotEntry* hot, uint32_t* hot_slot, uint32_t* overflow) {
   if (threadIdx.x != 0 || blockIdx.x != 0) return;
   for (uint32_t i = 0; i < kHotTable; ++i) hot[i] = HotEntry{0ull, 0ull, 0u, 0u, {0u, 0u}};
@@ -84,7 +84,7 @@ __global__ void k_hot_build(const ulonglong2* hk, uint32_t H, Slot* table, uint3
     const uint32_t len = (uint32_t)k0 & 0xFFu;
     const uint32_t w0 = (uint32_t)(k0 >> 32), w1 = (uint32_t)k1, w2 = (uint32_t)(k1 >> 32) & 0xFFFFFFu;
     const uint64_t h = term_hash16(w0, w1, w2, 0u, len);
-    const uint32_t s = table_insert(nullptr, table, slot_ref, mask, h, k0, k1, 0u, len, nullptr, 0u, overflow);
+    const uint32_t s = table_insert(nullptr, table, slot_ref, cap, h, k0, k1, 0u, len, nullptr, 0u, overflow);
     hot_slot[id] = s;
     uint32_t j = (uint32_t)(h >> 20) & (kHotTable - 1);
     while (hot[j].k0 != 0) j = (j + 1) & (kHotTable - 1);

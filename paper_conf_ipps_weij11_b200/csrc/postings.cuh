@@ -42,7 +42,13 @@ __global__ void k_map_compose(uint32_t* map, uint32_t C, const uint32_t* rank_of
 }
 
 constexpr int kRleThreads = 256;
-constexpr int kRleItems = 16;
+#ifndef WJ_RLE_ITEMS
+#define WJ_RLE_ITEMS 16
+#endif
+#ifndef WJ_RLE_MINB
+#define WJ_RLE_MINB 2
+#endif
+constexpr int kRleItems = WJ_RLE_ITEMS;
 constexpr int kRleTile = kRleThreads * kRleItems;
 
 __device__ __forceinline__ uint32_t block_min_after(uint32_t v, uint32_t* sm /* >= 9 words */) {
@@ -155,7 +161,7 @@ inline size_t rle_smem_bytes() {
 // COUNTS = false: every element is one token (no hot-term elements in the stream), so token prefixes
 // are element positions and the second block scan and the prefix array are skipped.
 template <bool COUNTS>
-__global__ void __launch_bounds__(kRleThreads, 2) k_rle_write_tma(const uint32_t* __restrict__ key,
+__global__ void __launch_bounds__(kRleThreads, WJ_RLE_MINB) k_rle_write_tma(const uint32_t* __restrict__ key,
                                                                const uint32_t* __restrict__ doc, uint64_t N,
                                                                uint64_t per, const uint32_t* __restrict__ range_off,
                                                                const uint64_t* __restrict__ range_tok_off,

@@ -445,7 +445,8 @@ constexpr int kRsUpSplit = 4;
 
 template <typename K, bool HOLES, bool MASK>
 __global__ void __launch_bounds__(256) k_rs_up(K* keys, uint64_t n, uint64_t per, int shift,
-                                               const uint32_t* __restrict__ map, uint32_t* hist, K kmask) {
+                                               const uint32_t* __restrict__ map, uint32_t* hist, K kmask,
+                                               const uint32_t* __restrict__ rlen) {
   __shared__ uint32_t h[kOsWarps][256];
   const int w = threadIdx.x >> 5;
   for (int x = 0; x < kOsWarps; ++x) h[x][threadIdx.x] = 0;
@@ -453,7 +454,9 @@ __global__ void __launch_bounds__(256) k_rs_up(K* keys, uint64_t n, uint64_t per
   const uint32_t range = blockIdx.x / kRsUpSplit, part = blockIdx.x % kRsUpSplit;
   const uint32_t n_ranges = gridDim.x / kRsUpSplit;
   const uint64_t sub = per / kRsUpSplit;  // per is a multiple of the 4096-element tile
-  const uint64_t rhi = (uint64_t)range * per + per < n ? (uint64_t)range * per + per : n;
+  // rlen (optional): range r holds only its first rlen[r] elements (doc combine, combine.cuh)
+  const uint64_t rhi = rlen ? (uint64_t)range * per + rlen[range]
+                            : ((uint64_t)range * per + per < n ? (uint64_t)range * per + per : n);
   const uint64_t lo0 = (uint64_t)range * per + part * sub;  // 16-byte aligned
   const uint64_t lo = lo0 < rhi ? lo0 : rhi;
   const uint64_t hi = (part + 1 == kRsUpSplit) ? rhi : (lo0 + sub < rhi ? lo0 + sub : rhi);
@@ -467,13 +470,24 @@ __global__ void __launch_bounds__(256) k_rs_up(K* keys, uint64_t n, uint64_t per
     Vec x[U];
 #pragma unroll
     for (int u = 0; u < U; ++u) x[u] = vp[v0 + u * 256];
+    // all U * V map gathers are issued before any histogram update (the gathers are L2-latency
+    // bound; interleaving them with shared atomics serialised them)
+    if (map) {
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        K* kk = (K*)&x[u];
+#pragma unroll
+        for (int j = 0; j < V; ++j)
+          if (!rs_hole<K, HOLES>(kk[j], kmask)) kk[j] = (K)__ldg(&map[(uint32_t)(kk[j] & kmask)]) | (kk[j] & ~kmask);
+      }
+    }
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       K* kk = (K*)&x[u];
 #pragma unroll
       for (int j = 0; j < V; ++j) {
+        // a mapped hole stays a hole: map values keep the bits above kmask of a non-hole
         const bool hole = rs_hole<K, HOLES>(kk[j], kmask);
-        if (map && !hole) kk[j] = (K)__ldg(&map[(uint32_t)(kk[j] & kmask)]) | (kk[j] & ~kmask);
         if (!hole) atomicAdd(&h[w][(uint32_t)(rs_dkey<K, MASK>(kk[j], kmask) >> shift) & 255u], 1u);
       }
       if (map) vp[v0 + u * 256] = x[u];
@@ -639,7 +653,7 @@ template <typename K, bool HOLES, bool MASK>
 __global__ void __launch_bounds__(kDsThreads, 2) k_rs_down2(const K* __restrict__ kin, const uint32_t* __restrict__ vin,
                                                          K* __restrict__ kout, uint32_t* __restrict__ vout, uint64_t n,
                                                          uint64_t per, int shift, const uint32_t* __restrict__ offs,
-                                                         K kmask) {
+                                                         K kmask, const uint32_t* __restrict__ rlen) {
   extern __shared__ __align__(128) unsigned char os_smem[];
   __shared__ __align__(8) uint64_t bar[2];
   __shared__ uint32_t wcnt[kDsWarps][256];
@@ -657,7 +671,7 @@ __global__ void __launch_bounds__(kDsThreads, 2) k_rs_down2(const K* __restrict_
   const int w = threadIdx.x >> 5;
   const uint32_t lt = (1u << lane) - 1u;
   const uint64_t lo = (uint64_t)blockIdx.x * per;
-  const uint64_t hi = lo + per < n ? lo + per : n;
+  const uint64_t hi = rlen ? lo + rlen[blockIdx.x] : (lo + per < n ? lo + per : n);
   if (lo >= hi) return;
 
   auto issue = [&](int s, uint64_t base) {  // thread 0

@@ -52,7 +52,7 @@ struct EmitOut {
   uint32_t* hot_tf;        // hot term x document token counts
   Slot* table;             // chunk hash table
   uint32_t* slot_ref;      // per slot: first-occurrence offset (written by the inserter)
-  uint32_t mask;           // capacity - 1 (power of two)
+  uint32_t cap;            // capacity (slots; any value >= 1)
   uint32_t doc_base;       // global DocID of local document 0
   uint32_t* slot;          // per kept token: table slot
   uint32_t* doc;           // per kept token: global DocID
@@ -308,7 +308,8 @@ __device__ __forceinline__ uint32_t win_word(const uint32_t* win32, uint32_t s, 
 }
 
 // 32-bit term hash over the folded, zero-padded little-endian words (cheap integer ops: the emit
-// kernel is instruction-bound).  Slot index = h & mask; the slot tag is a second mix of h.
+// kernel is instruction-bound).  First slot = mulhi(h, capacity) (any capacity, so the table can be
+// sized to the expected unique terms instead of the next power of two); the slot tag is a second mix.
 __device__ __forceinline__ uint32_t hash_init(uint32_t len) { return len * 0x9E3779B1u + 0x7F4A7C15u; }
 __device__ __forceinline__ uint32_t hash_mix(uint32_t h, uint32_t w) {
   h = (h ^ w) * 0x85EBCA77u;
@@ -321,10 +322,10 @@ __device__ __forceinline__ uint32_t hash_fin(uint32_t h) {
 }
 __device__ __forceinline__ uint32_t hash_tag(uint32_t h) { return (h * 0x9E3779B1u) >> 8; }
 
-__device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* table, uint32_t* slot_ref, uint32_t mask,
+__device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* table, uint32_t* slot_ref, uint32_t cap,
                                                  uint64_t h, uint64_t k0, uint64_t k1, uint32_t s_abs, uint32_t len,
                                                  const uint32_t* win32, uint32_t s_win, uint32_t* overflow) {
-  uint32_t i = (uint32_t)h & mask;
+  uint32_t i = __umulhi((uint32_t)h, cap);
   for (int probe = 0; probe < 4096; ++probe) {
     // Slots are claimed once (CAS on k0) and published once (k1), so a cached read can only be
     // stale-empty: the CAS or the volatile re-read below resolves it.
@@ -352,7 +353,7 @@ __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* tabl
         if (eq) return i;
       }
     }
-    i = (i + 1) & mask;
+    i = i + 1 == cap ? 0u : i + 1;
   }
   atomicExch(overflow, 1u);
   return kMiss;
@@ -448,7 +449,7 @@ __global__ void __launch_bounds__(kTokThreads, 5) k_tok_emit(ChunkView cv, uint3
           __stcs(eo.slot + out, 0u);
         } else {
           const uint32_t slot =
-              table_insert(cv.text, eo.table, eo.slot_ref, eo.mask, h, k0, k1, s_abs, len, w32, s_win, eo.overflow);
+              table_insert(cv.text, eo.table, eo.slot_ref, eo.cap, h, k0, k1, s_abs, len, w32, s_win, eo.overflow);
           __stcs(eo.slot + out, slot | (1u << 25));  // stream element: slot | count 1 << 25
           __stcs(eo.doc + out, doc);
         }

@@ -30,23 +30,37 @@ int main(int argc, char** argv) {
   cudaMalloc(&k0, n * 4); cudaMalloc(&v0, n * 4); cudaMalloc(&k, n * 4 + 64); cudaMalloc(&v, n * 4 + 64);
   cudaMemcpy(k0, hk.data(), n * 4, cudaMemcpyHostToDevice);
   cudaMemcpy(v0, hv.data(), n * 4, cudaMemcpyHostToDevice);
-  const uint32_t ntiles = (uint32_t)((n + kDcTile - 1) / kDcTile);
-  uint64_t* lk; cudaMalloc(&lk, (ntiles + 2) * 8);
-  uint32_t* nout; cudaMalloc(&nout, 4);
+  uint64_t per = (n + 296 - 1) / 296;
+  per = (per + kDcTile - 1) / kDcTile * kDcTile;
+  const uint32_t G = (uint32_t)((n + per - 1) / per);
+  uint32_t* rl; cudaMalloc(&rl, G * 4);
   cudaFuncSetAttribute(k_doc_combine, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dc_smem_bytes());
+  int occ = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_doc_combine, kDcThreads, dc_smem_bytes());
   cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
-  float best = 1e9; uint32_t m = 0;
+  float best = 1e9;
   for (int it = 0; it < 5; ++it) {
     cudaMemcpy(k, k0, n * 4, cudaMemcpyDeviceToDevice);
     cudaMemcpy(v, v0, n * 4, cudaMemcpyDeviceToDevice);
-    cudaMemset(lk, 0, (ntiles + 2) * 8);
     cudaEventRecord(a);
-    k_doc_combine<<<ntiles, kDcThreads, dc_smem_bytes()>>>(k, v, n, ntiles, lk, (uint32_t*)(lk + ntiles), nout);
+    k_doc_combine<<<G, kDcThreads, dc_smem_bytes()>>>(k, v, n, per, rl);
     cudaEventRecord(b); cudaEventSynchronize(b);
     float ms; cudaEventElapsedTime(&ms, a, b); if (it) best = std::min(best, ms);
   }
-  cudaMemcpy(&m, nout, 4, cudaMemcpyDeviceToHost);
-  printf("doc_combine n=%llu -> %u elements (%.3f): %.3f ms  err=%s\n", (unsigned long long)n, m, (double)m / n, best,
+  std::vector<uint32_t> hl(G);
+  cudaMemcpy(hl.data(), rl, G * 4, cudaMemcpyDeviceToHost);
+  uint64_t m = 0; for (auto x : hl) m += x;
+  // check: per range, sum of counts == range tokens, and elements are (id, doc) with ascending doc
+  std::vector<uint32_t> ok(n), ov(n);
+  cudaMemcpy(ok.data(), k, n * 4, cudaMemcpyDeviceToHost);
+  cudaMemcpy(ov.data(), v, n * 4, cudaMemcpyDeviceToHost);
+  uint64_t bad = 0;
+  for (uint32_t c = 0; c < G; ++c) {
+    uint64_t lo = (uint64_t)c * per, hi = std::min<uint64_t>(n, lo + per), tok = 0;
+    for (uint64_t i = lo; i < lo + hl[c]; ++i) { tok += ok[i] >> 25; if (i > lo && ov[i] < ov[i - 1]) ++bad; }
+    if (tok != hi - lo) ++bad;
+  }
+  printf("doc_combine n=%llu -> %llu elements (%.3f): %.3f ms  occ=%d/SM bad=%llu err=%s\n", (unsigned long long)n, (unsigned long long)m, (double)m / n, best, occ, (unsigned long long)bad,
          cudaGetErrorString(cudaGetLastError()));
   return 0;
 }
