@@ -48,6 +48,7 @@ KERNEL_BYTES = {
     "sort_hist": lambda T, N, P, E: 4 * E,                  # read u32 keys
     "sort_scatter": lambda T, N, P, E: 16 * E,              # read + write (u32 key, u32 doc) per element
     "rle_emit": lambda T, N, P, E: 8 * E + 8 * P,           # read (key, doc), write (docid, tf)
+    "copy_partials": lambda T, N, P, E: 16 * P,             # read + write (docid, tf) per posting
 }
 
 

@@ -113,8 +113,9 @@ enum {
   WJ_KERNEL_SORT_HIST,          /* finalize: radix digit histogram (token stream)                  */
   WJ_KERNEL_SORT_SCATTER,       /* finalize: stable radix scatter (token stream)                   */
   WJ_KERNEL_RLE_EMIT,           /* finalize: run-length (docID, tf) emit                           */
-  WJ_KERNEL_DOC_COMBINE,        /* per-document pre-aggregation of a chunk's stream (combine.cuh)   */
-  WJ_KERNEL_COUNT = 9
+  WJ_KERNEL_DOC_COMBINE,        /* per-document pre-aggregation of the stream (combine.cuh, opt-in) */
+  WJ_KERNEL_COPY_PARTIALS,      /* finalize: copy each chunk's partial postings lists into place    */
+  WJ_KERNEL_COUNT = 10
 };
 
 typedef struct {

@@ -247,7 +247,7 @@ __global__ void k_probe(DictView dv, UniqueView uv, uint32_t U, uint32_t* tid_ou
 // 11 folded bytes come from the slot itself, longer terms read their first occurrence
 __global__ void k_unique_gather(const Slot* table, const uint32_t* slot_ref, uint32_t C, const uint32_t* uid,
                                 const uint8_t* text, uint4* u_w, uint32_t* u_ref, uint32_t* u_len, uint32_t* u_bucket,
-                                uint32_t* u_cache, uint64_t* u_key) {
+                                uint32_t* u_cache, uint64_t* u_key, uint32_t* u_slot) {
   const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= C) return;
   const ulonglong2 e = *(const ulonglong2*)(table + i);
@@ -264,6 +264,7 @@ __global__ void k_unique_gather(const Slot* table, const uint32_t* slot_ref, uin
   }
   const TermInfo ti = term_info_w(w, text, ref, len);
   u_w[u] = w; u_ref[u] = ref; u_len[u] = len; u_bucket[u] = ti.bucket; u_cache[u] = ti.cache; u_key[u] = ti.key;
+  u_slot[u] = i;
 }
 
 // compact the misses: nk_key/nk_val in unique order (radix-sorted next)

@@ -12,6 +12,7 @@
 #include "dict.cuh"
 #include "dist.cuh"
 #include "hot.cuh"
+#include "partials.cuh"
 #include "exchange.h"
 #include "postings.cuh"
 #include "radix.cuh"
@@ -183,6 +184,23 @@ struct wj_index {
   // (profiles/r01_README.md)
   bool combine_on = false;
   DevBuf dc_len;
+  // Partial postings per chunk (partials.cuh; single GPU, no stemming / stop words / hot terms): the
+  // chunk's stream is sorted by slot and run-length encoded on side_st while the dictionary update
+  // runs on st; finalize combines the partial lists.  WJ_PARTIALS=0: global stream
+  // sorted at finalize instead.
+  bool pm = false;
+  cudaStream_t side_st = nullptr, hp_st = nullptr;  // side: lowest priority; hp: dictionary, highest
+  cudaEvent_t ev_fork = nullptr, ev_side = nullptr, ev_dict = nullptr;
+  DevBuf side_scan, side_hist, side_hist_scan;
+  DevBuf pc_key, pc_doc, pc_po, pc_cs, u_slot, pp_doc, pp_tf, rec_tid, rec_start, rec_df, rec_cf, rec_before, df_totb,
+      cf_totb;
+  uint64_t pbase = 0, nrec = 0;      // partial postings / records of the chunks so far
+  uint32_t rs_ctas = kRsCtas;        // radix downsweep CTAs (ranges) of sort_pairs
+  uint32_t side_ctas = kRsCtas;      // ... for the side stream's sort (WJ_SIDE_CTAS): fewer leave SMs to st
+  bool pc_pending = false;           // the last chunk's posting count is still on the device (dscal[13])
+  bool pc_join = false;              // the last chunk's side-stream work is not joined yet
+  uint64_t pc_U = 0, pc_Nc = 0;
+  std::vector<uint64_t> rec_end;     // end of each chunk's records
   uint64_t sorted_elems = 0;    // stream elements the last finalize sorted (after the combine)
   // Sampled hot-term path (hot.cuh) is opt-in: on config 2 it removes ~30% of the
   // stream elements but its per-document counters cost more global atomics in the emit kernel than
@@ -269,7 +287,9 @@ struct wj_index {
                      &dbg_doc, &lexg, &qbuf, &qres, &rank_of, &term_at, &sk1, &sv1, &pidx, &out_doc, &out_tf,
                      &post_off, &df, &cf, &term_off, &term_bytes, &vb_first, &vb_tiles, &vb_code, &vb_boff, &samp_hist, &owner_tab,
                      &table_s, &uid_s, &st_off, &st_text, &st_keep, &st_tidx, &st_m1, &st_slot, &st_doc, &st_tiles,
-                     &st_doff, &stop_keys};
+                     &st_doff, &stop_keys, &dc_len, &side_scan, &side_hist, &side_hist_scan, &pc_key, &pc_doc, &pc_po,
+                     &pc_cs, &u_slot, &pp_doc, &pp_tf, &rec_tid, &rec_start, &rec_df, &rec_cf, &rec_before, &df_totb,
+                     &cf_totb};
     for (DevBuf* b : all) {
       if (b->p) cudaFree(b->p);
       b->p = nullptr;
@@ -345,6 +365,7 @@ struct wj_index {
     if (recs.empty() && krecs.empty()) return;
     if (cur_phase >= 0) phase(-1);
     sync();
+    if (side_st) WJ_CUDA_CHECK(cudaStreamSynchronize(side_st));  // side-stream events (partials)
     for (auto& r : recs) {
       float ms = 0;
       WJ_CUDA_CHECK(cudaEventElapsedTime(&ms, r.a, r.b));
@@ -378,6 +399,7 @@ struct wj_index {
   // ---------------------------------------------------------------- init / reset
   void reset_state() {
     if (cs) WJ_CUDA_CHECK(cudaStreamSynchronize(cs));
+    if (side_st) WJ_CUDA_CHECK(cudaStreamSynchronize(side_st));  // an unjoined chunk (partials)
     pend = false;  // a pending (copied, not yet indexed) host chunk is dropped
     collect_phases();
     chunk_tok.clear();
@@ -385,6 +407,9 @@ struct wj_index {
     n_docs = n_tokens = n_dropped = n_chunks = n_elems = 0;
     stream_has_hot = false;
     sorted_elems = 0;
+    pbase = nrec = 0;
+    pc_pending = pc_join = false;
+    rec_end.clear();
     unique_last = new_last = n_nodes = height_max = 0;
     exchange_bytes = 0;
     V = 0;
@@ -702,8 +727,9 @@ struct wj_index {
     uint32_t* ub = buf<uint32_t>(u_bucket, U);
     uint32_t* uc = buf<uint32_t>(u_cache, U);
     uint64_t* uk = buf<uint64_t>(u_key, U);
+    uint32_t* us = buf<uint32_t>(u_slot, U);
     k_unique_gather<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, (const uint32_t*)slotref.p, (uint32_t)C,
-                                                      slot_uid, cv.text, uw, ur, ul, ub, uc, uk);
+                                                      slot_uid, cv.text, uw, ur, ul, ub, uc, uk, us);
     launched();
     return Nc;
   }
@@ -858,6 +884,125 @@ struct wj_index {
     }
   }
 
+  // run the following launches on side_st with its own scan / histogram scratch (no host syncs there)
+  void swap_side() {
+    std::swap(st, side_st);
+    std::swap(scan_scr, side_scan);
+    std::swap(hist, side_hist);
+    std::swap(hist_scan, side_hist_scan);
+    std::swap(rs_ctas, side_ctas);
+  }
+
+  // run-length pass over a sorted stream (postings.cuh): docid/tf into od/of, post_off / cstart at each
+  // term's key (key & kRankMask); the posting count is left in dscal[8] (u32, no host round trip)
+  void rle(const uint32_t* key, const uint32_t* docs, uint64_t N, bool counts, uint32_t* od, uint32_t* of, uint64_t* po,
+           uint64_t* csp) {
+    uint64_t per = (N + 148 * 2 - 1) / (148 * 2);
+    per = (per + kRleTile - 1) / kRleTile * kRleTile;
+    const uint32_t G = (uint32_t)((N + per - 1) / per);
+    uint32_t* rc = buf<uint32_t>(rle_p0, (uint64_t)G + 1);
+    uint32_t* rl = buf<uint32_t>(rle_lead, (uint64_t)G + 1);
+    uint64_t* rt = buf<uint64_t>(rle_tok, (uint64_t)G + 1);
+    ktime(WJ_KERNEL_RLE_EMIT, [&] {
+      if (counts) k_rle_count<true><<<G, kRleThreads, 0, st>>>(key, docs, N, per, rc, rt);
+      else k_rle_count<false><<<G, kRleThreads, 0, st>>>(key, docs, N, per, rc, rt);
+      launched();
+      scan<uint32_t>(ArrayIn<uint32_t>{rc}, G, rc, (uint32_t*)(dscal() + 8));
+      scan<uint64_t>(ArrayIn<uint64_t>{rt}, G, rt, (uint64_t*)(dscal() + 11));
+      if (counts)
+        k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(key, docs, N, per, rc, rt, od, of, po, csp, rl);
+      else
+        k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(), st>>>(key, docs, N, per, rc, rt, od, of, po, csp, rl);
+      launched();
+    });
+    k_rle_fixup<<<grid_for(G, 256), 256, 0, st>>>(rc, rl, G, of);
+    launched();
+    WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 8) + 1, 0, 4, st));
+  }
+
+  // the previous chunk's posting count (partials mode): read once its side-stream work is joined
+  void settle_partials() {
+    if (!pc_pending) return;
+    sync();
+    pbase += (uint32_t)h_scal[13];
+    pc_pending = false;
+  }
+
+  // Partials mode, one chunk: the stream (pc_key, pc_doc)[Nc] of C slots, U unique terms.  Sort by slot
+  // + run-length on side_st (the partial lists of the run) while the dictionary update runs on
+  // st; then one record per unique term.
+  void chunk_partials(const uint8_t* text, uint64_t Nc, uint64_t C, uint64_t U) {
+    settle_partials();  // the previous chunk is joined (add_chunk), its posting count read here
+    uint32_t* kt = (uint32_t*)pc_key.p;
+    uint32_t* dt = (uint32_t*)pc_doc.p;
+    uint32_t* k1 = buf<uint32_t>(sk1, Nc + 16);
+    uint32_t* v1 = buf<uint32_t>(sv1, Nc + 16);
+    uint32_t* od = buf_keep<uint32_t>(pp_doc, pbase + Nc + 16, pbase);  // P_c <= N_c
+    uint32_t* of = buf_keep<uint32_t>(pp_tf, pbase + Nc + 16, pbase);
+    uint64_t* po = buf<uint64_t>(pc_po, C + 1);
+    uint64_t* cs = buf<uint64_t>(pc_cs, C + 1);
+    int bits = 0;
+    while (bits < 32 && ((uint64_t)1 << bits) < C) ++bits;
+    phase(-1);
+    WJ_CUDA_CHECK(cudaEventRecord(ev_fork, st));
+    WJ_CUDA_CHECK(cudaStreamWaitEvent(side_st, ev_fork, 0));
+    swap_side();
+    try {
+      phase(WJ_PHASE_SORT);
+      const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, bits, nullptr, true);
+      phase(WJ_PHASE_POSTINGS);
+      rle(in1 ? k1 : kt, in1 ? v1 : dt, Nc, false, od + pbase, of + pbase, po, cs);
+      phase(-1);
+      WJ_CUDA_CHECK(cudaEventRecord(ev_side, st));
+    } catch (...) {
+      swap_side();
+      throw;
+    }
+    swap_side();
+    // the dictionary update (latency-bound small kernels with host round trips) on a high-priority
+    // stream, so its CTAs are scheduled ahead of the side stream's whenever SMs free up
+    WJ_CUDA_CHECK(cudaStreamWaitEvent(hp_st, ev_fork, 0));
+    std::swap(st, hp_st);
+    try {
+      dictionary_update(text, U);
+      phase(-1);
+      WJ_CUDA_CHECK(cudaEventRecord(ev_dict, st));
+    } catch (...) {
+      std::swap(st, hp_st);
+      throw;
+    }
+    std::swap(st, hp_st);
+    WJ_CUDA_CHECK(cudaStreamWaitEvent(st, ev_dict, 0));
+    pc_join = true;
+    pc_U = U;
+    pc_Nc = Nc;
+  }
+
+  // Join the last chunk's side-stream work and write its records; runs before the next chunk's
+  // tokenizer reuses the chunk buffers, or in finalize after the work that does not need postings.
+  void join_partials() {
+    if (!pc_join) return;
+    pc_join = false;
+    const uint64_t U = pc_U, Nc = pc_Nc;
+    phase(WJ_PHASE_STREAM);
+    WJ_CUDA_CHECK(cudaStreamWaitEvent(st, ev_side, 0));
+    const uint64_t* po = (const uint64_t*)pc_po.p;
+    const uint64_t* cs = (const uint64_t*)pc_cs.p;
+    uint32_t* rt = buf_keep<uint32_t>(rec_tid, nrec + U, nrec);
+    uint64_t* rs = buf_keep<uint64_t>(rec_start, nrec + U, nrec);
+    uint32_t* rd = buf_keep<uint32_t>(rec_df, nrec + U, nrec);
+    uint32_t* rc = buf_keep<uint32_t>(rec_cf, nrec + U, nrec);
+    k_chunk_records<<<grid_for(U, 256), 256, 0, st>>>((const uint32_t*)u_slot.p, (uint32_t)U, po, cs,
+                                                      (const uint32_t*)(dscal() + 8), Nc, (const uint32_t*)u_tid.p, pbase,
+                                                      rt + nrec, rs + nrec, rd + nrec, rc + nrec);
+    launched();
+    WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 13, dscal() + 8, 8, cudaMemcpyDeviceToHost, st));
+    pc_pending = true;
+    nrec += U;
+    rec_end.push_back(nrec);
+    phase(-1);
+  }
+
   // the chunk's (slot, docID) stream is the postings input; keep its slot -> termID map
   void register_chunk_map(uint64_t C, uint64_t tok_start) {
     phase(WJ_PHASE_STREAM);
@@ -918,6 +1063,7 @@ struct wj_index {
   void add_chunk(const void* bytes, uint64_t n_bytes, const uint64_t* doc_off_in, uint64_t nd) {
     const uint8_t* text = nullptr;
     const uint64_t* off = nullptr;
+    if (pm) join_partials();  // the previous chunk's side work, before its buffers are reused
     stage(bytes, n_bytes, doc_off_in, nd, &text, &off);
     ++n_chunks;
     if (xport) {
@@ -937,6 +1083,12 @@ struct wj_index {
     uint32_t *so = nullptr, *dout = nullptr;
     const bool norm = stem_on || stop_on;
     const uint64_t Nc = tokenize_dedup(cv, doc_base, [&](uint64_t nc, uint32_t*& sp, uint32_t*& dp) {
+      if (pm) {  // the chunk's own stream; the previous chunk's side work is joined on st already
+        if (nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 tokens in one chunk"};
+        sp = buf<uint32_t>(pc_key, nc + 16);  // +16: TMA round-up reads
+        dp = buf<uint32_t>(pc_doc, nc + 16);
+        return;
+      }
       if (n_elems + nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 stream elements"};
       sp = buf_keep<uint32_t>(g_tid, n_elems + nc + 16, n_elems) + n_elems;  // +16: TMA round-up reads
       dp = buf_keep<uint32_t>(g_doc, n_elems + nc + 16, n_elems) + n_elems;
@@ -959,6 +1111,10 @@ struct wj_index {
         n_elems += kept;
         n_tokens += kept;
       }
+    } else if (Nc > 0 && pm) {
+      chunk_partials(text, Nc, C, U);
+      n_elems += Nc;
+      n_tokens += Nc;
     } else if (Nc > 0) {
       uint64_t NH = 0;
       if (hot_H) {  // hot (term, document) counters -> stream elements after the chunk's tokens
@@ -1353,7 +1509,7 @@ struct wj_index {
       rlen = rl;
     }
     for (int p = 0; p < passes; ++p) {
-      uint64_t per = (cur_n + kRsCtas - 1) / kRsCtas;
+      uint64_t per = (cur_n + rs_ctas - 1) / rs_ctas;
       per = (per + kOsTile - 1) / kOsTile * kOsTile;
       const uint32_t G = (uint32_t)((cur_n + per - 1) / per);
       uint32_t* h1 = buf<uint32_t>(hist, (uint64_t)256 * G);
@@ -1407,6 +1563,26 @@ struct wj_index {
     return in1;
   }
 
+  // final dictionary bytes: term_off by scan, restored trie prefix + stored suffix (needs ranks only)
+  void dict_bytes() {
+    const uint2* ta = (const uint2*)term_at.p;  // rank_info (k_lexrank)
+    phase(WJ_PHASE_DICT);
+    uint64_t* to = buf<uint64_t>(term_off, (uint64_t)V + 1);
+    TB = 0;
+    if (V > 0) {
+      scan<uint64_t>(TermFullLen{ta},
+                     V, to, to + V);
+      WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 9, to + V, 8, cudaMemcpyDeviceToHost, st));
+      sync();
+      TB = h_scal[9];
+      uint8_t* tbp = buf<uint8_t>(term_bytes, TB);
+      k_term_bytes<<<grid_for(V, 256), 256, 0, st>>>(ta, V, (const uint8_t*)arena.p, to, tbp);
+      launched();
+    } else {
+      WJ_CUDA_CHECK(cudaMemsetAsync(to, 0, 8, st));
+    }
+  }
+
   // ---------------------------------------------------------------- finalize
   void finalize() {
     drain();
@@ -1432,7 +1608,56 @@ struct wj_index {
     uint64_t* cfp = buf<uint64_t>(cf, V);
     uint64_t* csp = buf<uint64_t>(cstart_b, (uint64_t)V + 1);
     P = 0;
-    if (NE > 0 && V > 0) {
+    if (pm) {
+      // the dictionary bytes need no postings: they overlap the last chunk's side-stream work; then
+      // combine the chunks' partial lists (partials.cuh): totals per term in chunk order, post_off in
+      // rank order, one copy of every partial list to its place
+      dict_bytes();
+      join_partials();
+      settle_partials();
+      sorted_elems = n_elems;
+      if (nrec > 0 && V > 0) {
+        phase(WJ_PHASE_POSTINGS);
+        uint32_t* dft = buf<uint32_t>(df_totb, V);
+        uint64_t* cft = buf<uint64_t>(cf_totb, V);
+        uint32_t* bef = buf<uint32_t>(rec_before, nrec);
+        const uint32_t* rt = (const uint32_t*)rec_tid.p;
+        const uint32_t* rd = (const uint32_t*)rec_df.p;
+        if (rec_end.size() == 1) {  // one run: every partial list is its term's whole list
+          WJ_CUDA_CHECK(cudaMemsetAsync(bef, 0, nrec * 4, st));
+          k_rank_scatter_rec<<<grid_for(nrec, 256), 256, 0, st>>>(rt, rd, (const uint32_t*)rec_cf.p, nrec, ro, dfp, cfp);
+          launched();
+        } else {
+          WJ_CUDA_CHECK(cudaMemsetAsync(dft, 0, (size_t)V * 4, st));
+          WJ_CUDA_CHECK(cudaMemsetAsync(cft, 0, (size_t)V * 8, st));
+          uint64_t lo = 0;
+          for (const uint64_t hi : rec_end) {
+            if (hi > lo) {
+              k_rec_accum<<<grid_for(hi - lo, 256), 256, 0, st>>>(rt, rd, (const uint32_t*)rec_cf.p, lo, hi, dft, cft, bef);
+              launched();
+            }
+            lo = hi;
+          }
+          k_rank_scatter<<<grid_for(V, 256), 256, 0, st>>>(ro, V, dft, cft, dfp, cfp);
+          launched();
+        }
+        scan<uint64_t>(U32AsU64{dfp}, V, po, po + V);
+        WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 8, po + V, 8, cudaMemcpyDeviceToHost, st));
+        sync();
+        P = h_scal[8];
+        uint32_t* od = buf<uint32_t>(out_doc, P + 1);
+        uint32_t* of = buf<uint32_t>(out_tf, P + 1);
+        ktime(WJ_KERNEL_COPY_PARTIALS, [&] {
+          k_copy_partials<<<grid_for((P + kCopyChunk - 1) / kCopyChunk * 32, 256), 256, 0, st>>>(
+              rt, (const uint64_t*)rec_start.p, rd, bef, nrec, P, ro, po,
+                                                                   (const uint32_t*)pp_doc.p, (const uint32_t*)pp_tf.p,
+                                                                   od, of);
+          launched();
+        });
+      } else {
+        WJ_CUDA_CHECK(cudaMemsetAsync(po, 0, 8, st));
+      }
+    } else if (NE > 0 && V > 0) {
       phase(WJ_PHASE_SORT);
       uint32_t* kt = (uint32_t*)g_tid.p;
       uint32_t* dt = (uint32_t*)g_doc.p;
@@ -1495,21 +1720,7 @@ struct wj_index {
     }
     PB = 0;
     if (vbyte) encode_vbyte();
-    phase(WJ_PHASE_DICT);
-    uint64_t* to = buf<uint64_t>(term_off, (uint64_t)V + 1);
-    TB = 0;
-    if (V > 0) {
-      scan<uint64_t>(TermFullLen{ta},
-                     V, to, to + V);
-      WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 9, to + V, 8, cudaMemcpyDeviceToHost, st));
-      sync();
-      TB = h_scal[9];
-      uint8_t* tbp = buf<uint8_t>(term_bytes, TB);
-      k_term_bytes<<<grid_for(V, 256), 256, 0, st>>>(ta, V, (const uint8_t*)arena.p, to, tbp);
-      launched();
-    } else {
-      WJ_CUDA_CHECK(cudaMemsetAsync(to, 0, 8, st));
-    }
+    if (!pm) dict_bytes();
     phase(-1);
     sync();
     finalized = true;
@@ -1659,8 +1870,22 @@ int index_init(wj_index** out, const wj_config* cfg) {
         WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->pipe_done[i], cudaEventDisableTiming));
       }
     }
+    // a transport (world > 1, or a communicator at world 1) runs the distributed path: global stream
+    ix->pm = ix->world == 1 && !cfg->nccl_unique_id && !ix->stem_on && !ix->stop_on;
+    if (const char* e = getenv("WJ_PARTIALS")) ix->pm = ix->pm && strtoull(e, nullptr, 10) != 0;
     if (const char* e = getenv("WJ_DOC_COMBINE")) ix->combine_on = strtoull(e, nullptr, 10) != 0;
     if (const char* e = getenv("WJ_HOT_MIN_BYTES")) ix->hot_min_bytes = strtoull(e, nullptr, 10);
+    if (ix->hot_min_bytes != ~0ull) ix->pm = false;  // hot-term elements need the global stream
+    if (const char* e = getenv("WJ_SIDE_CTAS")) ix->side_ctas = std::max<uint32_t>((uint32_t)strtoul(e, nullptr, 10), 1);
+    if (ix->pm) {
+      int least = 0, greatest = 0;
+      WJ_CUDA_CHECK(cudaDeviceGetStreamPriorityRange(&least, &greatest));
+      WJ_CUDA_CHECK(cudaStreamCreateWithPriority(&ix->side_st, cudaStreamNonBlocking, least));
+      WJ_CUDA_CHECK(cudaStreamCreateWithPriority(&ix->hp_st, cudaStreamNonBlocking, greatest));
+      WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->ev_fork, cudaEventDisableTiming));
+      WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->ev_side, cudaEventDisableTiming));
+      WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->ev_dict, cudaEventDisableTiming));
+    }
     if (const char* e = getenv("WJ_TABLE_POW2")) ix->table_pow2 = strtoull(e, nullptr, 10) != 0;
     if (const char* e = getenv("WJ_TABLE_PCT")) ix->table_pct = std::max<uint64_t>(strtoull(e, nullptr, 10), 110);
     if (cfg->world > 1 || cfg->nccl_unique_id) {  // a transport at world 1 runs the same distributed path
@@ -2064,6 +2289,17 @@ void index_destroy(wj_index* ix) {
     if (ix->pipe_done[i]) cudaEventDestroy(ix->pipe_done[i]);
   }
   if (ix->cs) cudaStreamDestroy(ix->cs);
+  if (ix->side_st) {
+    cudaStreamSynchronize(ix->side_st);
+    cudaStreamDestroy(ix->side_st);
+  }
+  if (ix->hp_st) {
+    cudaStreamSynchronize(ix->hp_st);
+    cudaStreamDestroy(ix->hp_st);
+  }
+  if (ix->ev_dict) cudaEventDestroy(ix->ev_dict);
+  if (ix->ev_fork) cudaEventDestroy(ix->ev_fork);
+  if (ix->ev_side) cudaEventDestroy(ix->ev_side);
   delete ix->xport;
   for (auto e : ix->ev_pool) cudaEventDestroy(e);
   if (ix->h_scal) cudaFreeHost(ix->h_scal);

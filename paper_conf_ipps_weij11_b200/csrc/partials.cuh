@@ -1,0 +1,159 @@
+// Partial postings lists per run, combined at finalize.
+//
+// The paper's indexer appends each run's postings to partial lists and post-processing combines the
+// partial lists of a term in run order (docIDs ascend across runs).  Here a run is one
+// index_add_stream chunk: its (slot, docID) stream is sorted by chunk slot and run-length encoded on
+// a side stream while the dictionary update of the same chunk runs on the main stream, giving per
+// chunk a CSR by slot.  Once the chunk's slots are mapped to termIDs, one record per unique term
+// (termID, start, df, cf) describes the term's partial list.  Finalize accumulates df / cf per term
+// over the chunks (in chunk order, which also gives each partial its offset inside the term's final
+// list), scans df in lexicographic rank order into post_off, and copies every partial list to its
+// final place.
+#pragma once
+#include "common.cuh"
+
+namespace wj {
+
+// Per unique term u of a chunk (u ascending = slot ascending = the order of the sorted runs):
+// start / df / cf of its partial list from the run-length output (post_off / cstart indexed by slot).
+__global__ void k_chunk_records(const uint32_t* __restrict__ u_slot, uint32_t U, const uint64_t* __restrict__ post_off,
+                                const uint64_t* __restrict__ cstart, const uint32_t* __restrict__ P_dev, uint64_t Nc,
+                                const uint32_t* __restrict__ u_tid, uint64_t pbase, uint32_t* rec_tid,
+                                uint64_t* rec_start, uint32_t* rec_df, uint32_t* rec_cf) {
+  const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
+  if (u >= U) return;
+  const uint32_t s = u_slot[u];
+  const uint64_t a = post_off[s], ta = cstart[s];
+  uint64_t b, tb;
+  if (u + 1 < U) {
+    const uint32_t s2 = u_slot[u + 1];
+    b = post_off[s2];
+    tb = cstart[s2];
+  } else {
+    b = *P_dev;
+    tb = Nc;
+  }
+  rec_tid[u] = u_tid[u];
+  rec_start[u] = pbase + a;
+  rec_df[u] = (uint32_t)(b - a);
+  rec_cf[u] = (uint32_t)(tb - ta);
+}
+
+// One chunk's records, in chunk order: offset of the partial inside its term's list = postings of
+// the term in earlier chunks; termIDs are distinct within a chunk, so there is no conflict.
+__global__ void k_rec_accum(const uint32_t* __restrict__ rec_tid, const uint32_t* __restrict__ rec_df,
+                            const uint32_t* __restrict__ rec_cf, uint64_t lo, uint64_t hi, uint32_t* df_tot,
+                            uint64_t* cf_tot, uint32_t* before) {
+  const uint64_t i = lo + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= hi) return;
+  const uint32_t t = rec_tid[i];
+  before[i] = df_tot[t];
+  df_tot[t] += rec_df[i];
+  cf_tot[t] += rec_cf[i];
+}
+
+// termID-indexed totals -> rank order (df, cf of the final dictionary)
+__global__ void k_rank_scatter(const uint32_t* __restrict__ rank_of, uint32_t V, const uint32_t* __restrict__ df_tot,
+                               const uint64_t* __restrict__ cf_tot, uint32_t* df, uint64_t* cf) {
+  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= V) return;
+  const uint32_t r = rank_of[t];
+  df[r] = df_tot[t];
+  cf[r] = cf_tot[t];
+}
+
+// a single run: the records are the terms, df / cf straight to rank order
+__global__ void k_rank_scatter_rec(const uint32_t* __restrict__ rec_tid, const uint32_t* __restrict__ rec_df,
+                                   const uint32_t* __restrict__ rec_cf, uint64_t R, const uint32_t* __restrict__ rank_of,
+                                   uint32_t* df, uint64_t* cf) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= R) return;
+  const uint32_t r = rank_of[rec_tid[i]];
+  df[r] = rec_df[i];
+  cf[r] = rec_cf[i];
+}
+
+struct U32AsU64 {
+  const uint32_t* p;
+  __device__ __forceinline__ uint64_t operator()(uint64_t i) const { return p[i]; }
+};
+
+// Copy every partial list to post_off[rank(term)] + before.  The partial lists lie back to back in
+// record order, so warp w copies the source postings [w * kCopyChunk, (w + 1) * kCopyChunk): it finds
+// the record holding its first posting (binary search on rec_start), then walks windows of 32
+// records, 32 postings at a time (coalesced reads; each lane finds its record in the window with a
+// 5-step shuffle search); writes are contiguous within each record's list.  Long lists (the Zipf
+// head) are spread over many warps.
+constexpr uint32_t kCopyChunk = 1024;
+
+__global__ void __launch_bounds__(256) k_copy_partials(const uint32_t* __restrict__ rec_tid,
+                                                       const uint64_t* __restrict__ rec_start,
+                                                       const uint32_t* __restrict__ rec_df,
+                                                       const uint32_t* __restrict__ before, uint64_t R, uint64_t P,
+                                                       const uint32_t* __restrict__ rank_of,
+                                                       const uint64_t* __restrict__ post_off,
+                                                       const uint32_t* __restrict__ pdoc, const uint32_t* __restrict__ ptf,
+                                                       uint32_t* __restrict__ out_doc, uint32_t* __restrict__ out_tf) {
+  const uint64_t w = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t lane = threadIdx.x & 31;
+  uint64_t lo = w * kCopyChunk;
+  if (lo >= P) return;
+  const uint64_t hi = lo + kCopyChunk < P ? lo + kCopyChunk : P;
+  // first record: the last one with rec_start <= lo (rec_start is increasing; record 0 starts at 0)
+  uint64_t r = 0;
+  if (lane == 0) {
+    uint64_t a = 0, b = R;  // invariant: rec_start[a] <= lo, answer in [a, b)
+    while (b - a > 1) {
+      const uint64_t m = (a + b) >> 1;
+      if (rec_start[m] <= lo) a = m; else b = m;
+    }
+    r = a;
+  }
+  r = __shfl_sync(0xffffffffu, r, 0);
+  for (;;) {
+    const uint64_t i = r + lane;
+    const bool v = i < R;
+    const uint64_t st = v ? rec_start[i] : ~0ull;
+    const uint32_t n = v ? rec_df[i] : 0u;
+    const uint64_t dst = v ? post_off[rank_of[rec_tid[i]]] + before[i] : 0ull;
+    const uint64_t wend = __shfl_sync(0xffffffffu, v ? st + n : 0ull, 31);  // end of the window
+    const uint64_t last = (r + 31 < R) ? wend : P;
+    const uint64_t e = last < hi ? last : hi;
+    // window-relative starts (u32) for cheaper shuffles; 4 x 32 postings per step, loads before stores
+    const uint64_t ws = __shfl_sync(0xffffffffu, st, 0);
+    const uint32_t srel = v ? (uint32_t)(st - ws) : 0xFFFFFFFFu;
+    for (uint64_t base = lo; base < e; base += 128) {  // warp-uniform trip count
+      uint32_t dv[4], tv[4];
+      uint64_t dd[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint64_t p = base + 32 * q + lane;
+        const uint32_t pr = (uint32_t)(p - ws);
+        uint32_t j = 0;  // last lane of the window with start <= p
+#pragma unroll
+        for (int b = 16; b > 0; b >>= 1) {
+          const uint32_t sj = __shfl_sync(0xffffffffu, srel, j + b);
+          if (sj <= pr) j += b;
+        }
+        const uint32_t sj = __shfl_sync(0xffffffffu, srel, j);
+        dd[q] = __shfl_sync(0xffffffffu, dst, j) + (pr - sj);
+        if (p < e) {
+          dv[q] = __ldcs(pdoc + p);
+          tv[q] = __ldcs(ptf + p);
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        if (base + 32 * q + lane < e) {
+          __stcs(out_doc + dd[q], dv[q]);
+          __stcs(out_tf + dd[q], tv[q]);
+        }
+      }
+    }
+    if (e >= hi) break;
+    lo = e;
+    r += 32;
+  }
+}
+
+}  // namespace wj

@@ -490,6 +490,7 @@ def combine_off(monkeypatch):
 @pytest.fixture
 def combine_on(monkeypatch):
     monkeypatch.setenv("WJ_DOC_COMBINE", "1")
+    monkeypatch.setenv("WJ_PARTIALS", "0")  # the combine runs on the global stream's finalize sort
     yield
 
 
@@ -530,3 +531,39 @@ def test_combine_off_same_bytes(combine_off):
         got = ix.serialize()
         assert ix.stats()["stream_elems"] == ix.stats()["n_tokens"]
     assert_same_index(got, oracle.index_bytes(text, off))
+
+
+# ------------------------------------------------------------------ partial lists per run (partials.cuh)
+@pytest.mark.parametrize("partials", ["1", "0"])
+def test_partials_and_global_stream_paths(monkeypatch, partials):
+    # default single-GPU path: per-chunk partial postings combined at finalize;
+    # WJ_PARTIALS=0: the global stream sorted at finalize.  Both must give the oracle's bytes, with
+    # chunks of very different sizes, empty chunks and a single-document chunk.
+    monkeypatch.setenv("WJ_PARTIALS", partials)
+    cfg = gen.CONFIGS[3].scaled(chunk_bytes=3 << 20, vocab=50_000)
+    text, off = gen.generate(cfg)
+    n = len(off) - 1
+    want = oracle.index_bytes(text, off)
+    for cuts in ([0, n], [0, 1, 1, n // 7, n // 2, n - 1, n], [0, n // 3, 2 * n // 3, n]):
+        assert_same_index(gpu_index(text, off, cuts=cuts), want)
+    assert_same_index(gpu_index(text, off, cuts=[0, n // 2, n], vbyte=True), oracle.index_bytes(text, off, vbyte=True))
+
+
+def test_partials_repeated_reset_and_read_postings():
+    cfg = gen.CONFIGS[2].scaled(chunk_bytes=2 << 20, vocab=20_000)
+    text, off = gen.generate(cfg)
+    want = oracle.index_bytes(text, off)
+    w = wjformat.parse(want)
+    with wj.Index(device=0) as ix:
+        for _ in range(3):
+            ix.reset()
+            n = len(off) - 1
+            for a, b in ((0, n // 2), (n // 2, n)):
+                ix.add_stream(text[int(off[a]):int(off[b])], (off[a:b + 1] - off[a]).astype(np.uint64))
+            ix.finalize()
+            assert_same_index(ix.serialize(), want)
+        terms = w.terms()
+        for i in (0, len(terms) // 2, len(terms) - 1):
+            d, t = ix.read_postings(terms[i])
+            lo, hi = int(w.post_off[i]), int(w.post_off[i + 1])
+            assert np.array_equal(d, w.docid[lo:hi]) and np.array_equal(t, w.tf[lo:hi])
