@@ -1624,8 +1624,8 @@ struct wj_index {
         const uint32_t* rt = (const uint32_t*)rec_tid.p;
         const uint32_t* rd = (const uint32_t*)rec_df.p;
         if (rec_end.size() == 1) {  // one run: every partial list is its term's whole list
-          WJ_CUDA_CHECK(cudaMemsetAsync(bef, 0, nrec * 4, st));
-          k_rank_scatter_rec<<<grid_for(nrec, 256), 256, 0, st>>>(rt, rd, (const uint32_t*)rec_cf.p, nrec, ro, dfp, cfp);
+          k_rank_scatter_rec<<<grid_for(nrec, 256), 256, 0, st>>>(rt, rd, (const uint32_t*)rec_cf.p, nrec, ro, dfp, cfp,
+                                                                  bef);
           launched();
         } else {
           WJ_CUDA_CHECK(cudaMemsetAsync(dft, 0, (size_t)V * 4, st));
@@ -1648,6 +1648,12 @@ struct wj_index {
         uint32_t* od = buf<uint32_t>(out_doc, P + 1);
         uint32_t* of = buf<uint32_t>(out_tf, P + 1);
         ktime(WJ_KERNEL_COPY_PARTIALS, [&] {
+          if (rec_end.size() == 1) {  // one run: bef holds the record of each rank
+            k_copy_by_rank<<<grid_for((P + kCopyChunk - 1) / kCopyChunk * 32, 256), 256, 0, st>>>(
+                bef, (const uint64_t*)rec_start.p, V, P, po, (const uint32_t*)pp_doc.p, (const uint32_t*)pp_tf.p, od, of);
+            launched();
+            return;
+          }
           k_copy_partials<<<grid_for((P + kCopyChunk - 1) / kCopyChunk * 32, 256), 256, 0, st>>>(
               rt, (const uint64_t*)rec_start.p, rd, bef, nrec, P, ro, po,
                                                                    (const uint32_t*)pp_doc.p, (const uint32_t*)pp_tf.p,

@@ -62,16 +62,26 @@ __global__ void k_rank_scatter(const uint32_t* __restrict__ rank_of, uint32_t V,
   cf[r] = cf_tot[t];
 }
 
-// a single run: the records are the terms, df / cf straight to rank order
+// a single run: the records are the terms, df / cf straight to rank order, and the record of each rank
 __global__ void k_rank_scatter_rec(const uint32_t* __restrict__ rec_tid, const uint32_t* __restrict__ rec_df,
                                    const uint32_t* __restrict__ rec_cf, uint64_t R, const uint32_t* __restrict__ rank_of,
-                                   uint32_t* df, uint64_t* cf) {
+                                   uint32_t* df, uint64_t* cf, uint32_t* rec_of_rank) {
   const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= R) return;
   const uint32_t r = rank_of[rec_tid[i]];
   df[r] = rec_df[i];
   cf[r] = rec_cf[i];
+  rec_of_rank[r] = (uint32_t)i;
 }
+
+// Single run: the same copy walked in destination (rank) order -- warp w writes the final postings
+// [w * kCopyChunk, (w + 1) * kCopyChunk) coalesced and gathers them from the partial lists (each
+// term's list is contiguous in both).
+__global__ void __launch_bounds__(256) k_copy_by_rank(const uint32_t* __restrict__ rec_of_rank,
+                                                      const uint64_t* __restrict__ rec_start, uint32_t V, uint64_t P,
+                                                      const uint64_t* __restrict__ post_off,
+                                                      const uint32_t* __restrict__ pdoc, const uint32_t* __restrict__ ptf,
+                                                      uint32_t* __restrict__ out_doc, uint32_t* __restrict__ out_tf);
 
 struct U32AsU64 {
   const uint32_t* p;
@@ -147,6 +157,69 @@ __global__ void __launch_bounds__(256) k_copy_partials(const uint32_t* __restric
         if (base + 32 * q + lane < e) {
           __stcs(out_doc + dd[q], dv[q]);
           __stcs(out_tf + dd[q], tv[q]);
+        }
+      }
+    }
+    if (e >= hi) break;
+    lo = e;
+    r += 32;
+  }
+}
+
+__global__ void __launch_bounds__(256) k_copy_by_rank(const uint32_t* __restrict__ rec_of_rank,
+                                                      const uint64_t* __restrict__ rec_start, uint32_t V, uint64_t P,
+                                                      const uint64_t* __restrict__ post_off,
+                                                      const uint32_t* __restrict__ pdoc, const uint32_t* __restrict__ ptf,
+                                                      uint32_t* __restrict__ out_doc, uint32_t* __restrict__ out_tf) {
+  const uint64_t w = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t lane = threadIdx.x & 31;
+  uint64_t lo = w * kCopyChunk;
+  if (lo >= P) return;
+  const uint64_t hi = lo + kCopyChunk < P ? lo + kCopyChunk : P;
+  uint64_t r = 0;  // last rank with post_off <= lo
+  if (lane == 0) {
+    uint64_t a = 0, b = V;
+    while (b - a > 1) {
+      const uint64_t m = (a + b) >> 1;
+      if (post_off[m] <= lo) a = m; else b = m;
+    }
+    r = a;
+  }
+  r = __shfl_sync(0xffffffffu, r, 0);
+  for (;;) {
+    const uint64_t i = r + lane;
+    const bool v = i < V;
+    const uint64_t d0 = v ? post_off[i] : ~0ull;
+    const uint64_t src = v ? rec_start[rec_of_rank[i]] : 0ull;
+    const uint64_t wend = (r + 32 < V) ? post_off[r + 32] : P;  // first posting after the window
+    const uint64_t e = wend < hi ? wend : hi;
+    const uint64_t ws = __shfl_sync(0xffffffffu, d0, 0);
+    const uint32_t drel = v ? (uint32_t)(d0 - ws) : 0xFFFFFFFFu;
+    for (uint64_t base = lo; base < e; base += 128) {  // warp-uniform trip count
+      uint32_t dv[4], tv[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint64_t p = base + 32 * q + lane;
+        const uint32_t pr = (uint32_t)(p - ws);
+        uint32_t j = 0;  // last lane of the window whose list starts at or before p
+#pragma unroll
+        for (int b = 16; b > 0; b >>= 1) {
+          const uint32_t dj = __shfl_sync(0xffffffffu, drel, j + b);
+          if (dj <= pr) j += b;
+        }
+        const uint32_t dj = __shfl_sync(0xffffffffu, drel, j);
+        const uint64_t sp = __shfl_sync(0xffffffffu, src, j) + (pr - dj);
+        if (p < e) {
+          dv[q] = __ldg(pdoc + sp);
+          tv[q] = __ldg(ptf + sp);
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint64_t p = base + 32 * q + lane;
+        if (p < e) {
+          __stcs(out_doc + p, dv[q]);
+          __stcs(out_tf + p, tv[q]);
         }
       }
     }
