@@ -29,7 +29,10 @@ constexpr int kTokThreads = 256;
 constexpr int kTokWarps = kTokThreads / 32;
 constexpr int kSegsPerWarp = 4;
 constexpr int kWinBytes = (kSegsPerWarp + 1) * kSegBytes + 16;  // staged range + 1 segment + pad
-constexpr int kQueueCap = kSegBytes;                            // >= tokens of one segment
+#ifndef WJ_QUEUE_CAP
+#define WJ_QUEUE_CAP 320
+#endif
+constexpr int kQueueCap = WJ_QUEUE_CAP;  // >= tokens of one segment (<= 257) + 1
 
 struct ChunkView {
   const uint8_t* text;     // 16-byte aligned device pointer
@@ -359,8 +362,12 @@ __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* tabl
   return kMiss;
 }
 
-// 5 CTAs/SM (48 registers): 0.3 ms/step faster than 4 CTAs (64 registers) on config 2
-__global__ void __launch_bounds__(kTokThreads, 5) k_tok_emit(ChunkView cv, uint32_t n_segs, const uint64_t* kstart,
+// 6 CTAs/SM (40 registers, 320-entry token queues, 31 KB of shared memory per CTA): emit 2.43 -> 2.34 ms
+// on config 2 vs 5 CTAs/SM (48 registers, 512-entry queues); 4 CTAs/SM (64 registers) was 0.3 ms slower still
+#ifndef WJ_EMIT_MINB
+#define WJ_EMIT_MINB 6
+#endif
+__global__ void __launch_bounds__(kTokThreads, WJ_EMIT_MINB) k_tok_emit(ChunkView cv, uint32_t n_segs, const uint64_t* kstart,
                                                           const uint32_t* range_off, EmitOut eo) {
   __shared__ __align__(16) uint32_t win[kTokWarps][kWinBytes / 4];
   __shared__ uint32_t queue[kTokWarps][kQueueCap + 1];
