@@ -388,6 +388,7 @@ def main():
             "e2e": e2e,
             "gpu_launches": int(round(launches * args.steps)),
             "gpu_launches_per_step": launches,
+            "host_syncs_per_step": (s1["host_syncs"] - s0["host_syncs"]) / args.steps,
             "clocks": clk,
             "phases_ms_per_step": phases,
             "kernels": kernels,
