@@ -912,7 +912,7 @@ struct wj_index {
       if (counts)
         k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(key, docs, N, per, rc, rt, od, of, po, csp, rl);
       else
-        k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(), st>>>(key, docs, N, per, rc, rt, od, of, po, csp, rl);
+        k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(false), st>>>(key, docs, N, per, rc, rt, od, of, po, csp, rl);
       launched();
     });
     k_rle_fixup<<<grid_for(G, 256), 256, 0, st>>>(rc, rl, G, of);
@@ -1711,7 +1711,7 @@ struct wj_index {
         if (stream_has_hot || combine)
           k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl);
         else
-          k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl);
+          k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(false), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl);
         launched();
       });
       k_rle_fixup<<<grid_for(G, 256), 256, 0, st>>>(rc, rl, G, of);

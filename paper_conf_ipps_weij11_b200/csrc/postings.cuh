@@ -153,15 +153,23 @@ __global__ void __launch_bounds__(kRleThreads) k_rle_count(const uint32_t* __res
   }
 }
 
-inline size_t rle_smem_bytes() {
+inline size_t rle_smem_bytes(bool counts = true) {
   return (size_t)4 * kRleTile * 4 /*2 stages x (key, doc)*/ + 2 * kRleTile * 4 /*staged docid, tf*/ +
-         (kRleTile + 4) * 4 /*item token-count prefix*/;
+         (counts ? (kRleTile + 4) * 4 : 0) /*item token-count prefix (COUNTS only)*/;
 }
 
 // COUNTS = false: every element is one token (no hot-term elements in the stream), so token prefixes
 // are element positions and the second block scan and the prefix array are skipped.
 template <bool COUNTS>
-__global__ void __launch_bounds__(kRleThreads, WJ_RLE_MINB) k_rle_write_tma(const uint32_t* __restrict__ key,
+#ifndef WJ_RLE_MAXREG
+#define WJ_RLE_MAXREG 0
+#endif
+#if WJ_RLE_MAXREG > 0
+#define WJ_RLE_BOUNDS __maxnreg__(WJ_RLE_MAXREG)
+#else
+#define WJ_RLE_BOUNDS __launch_bounds__(kRleThreads, WJ_RLE_MINB)
+#endif
+__global__ void WJ_RLE_BOUNDS k_rle_write_tma(const uint32_t* __restrict__ key,
                                                                const uint32_t* __restrict__ doc, uint64_t N,
                                                                uint64_t per, const uint32_t* __restrict__ range_off,
                                                                const uint64_t* __restrict__ range_tok_off,
