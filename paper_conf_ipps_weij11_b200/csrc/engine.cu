@@ -1609,13 +1609,33 @@ struct wj_index {
     uint64_t* csp = buf<uint64_t>(cstart_b, (uint64_t)V + 1);
     P = 0;
     if (pm) {
-      // the dictionary bytes need no postings: they overlap the last chunk's side-stream work; then
       // combine the chunks' partial lists (partials.cuh): totals per term in chunk order, post_off in
-      // rank order, one copy of every partial list to its place
-      dict_bytes();
+      // rank order, one copy of every partial list to its place.  The dictionary bytes need no
+      // postings: they run on the side stream (idle once the last chunk is joined) meanwhile.
       join_partials();
       settle_partials();
       sorted_elems = n_elems;
+      phase(-1);
+      WJ_CUDA_CHECK(cudaEventRecord(ev_fork, st));  // ranks (k_lexrank) are ready in st order
+      bool dict_started = false;
+      auto side_dict = [&] {  // enqueue dict_bytes on side_st (its size readback waits for side_st only)
+        if (dict_started) return;
+        dict_started = true;
+        const int open = cur_phase;
+        phase(-1);
+        WJ_CUDA_CHECK(cudaStreamWaitEvent(side_st, ev_fork, 0));
+        swap_side();
+        try {
+          dict_bytes();
+          phase(-1);
+          WJ_CUDA_CHECK(cudaEventRecord(ev_side, st));
+        } catch (...) {
+          swap_side();
+          throw;
+        }
+        swap_side();
+        if (open >= 0) phase(open);
+      };
       if (nrec > 0 && V > 0) {
         phase(WJ_PHASE_POSTINGS);
         uint32_t* dft = buf<uint32_t>(df_totb, V);
@@ -1643,6 +1663,7 @@ struct wj_index {
         }
         scan<uint64_t>(U32AsU64{dfp}, V, po, po + V);
         WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 8, po + V, 8, cudaMemcpyDeviceToHost, st));
+        side_dict();
         sync();
         P = h_scal[8];
         uint32_t* od = buf<uint32_t>(out_doc, P + 1);
@@ -1663,6 +1684,8 @@ struct wj_index {
       } else {
         WJ_CUDA_CHECK(cudaMemsetAsync(po, 0, 8, st));
       }
+      side_dict();
+      WJ_CUDA_CHECK(cudaStreamWaitEvent(st, ev_side, 0));
     } else if (NE > 0 && V > 0) {
       phase(WJ_PHASE_SORT);
       uint32_t* kt = (uint32_t*)g_tid.p;
