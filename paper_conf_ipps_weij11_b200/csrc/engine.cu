@@ -1497,7 +1497,7 @@ struct wj_index {
     // per-document combine (combine.cuh) on the first pass's ranges: range c keeps rlen[c] elements
     const uint32_t* rlen = nullptr;
     if (combine) {
-      uint64_t per = (n + kRsCtas - 1) / kRsCtas;
+      uint64_t per = (n + rs_ctas - 1) / rs_ctas;  // the first pass's ranges
       per = (per + kOsTile - 1) / kOsTile * kOsTile;
       const uint32_t G = (uint32_t)((n + per - 1) / per);
       uint32_t* rl = buf<uint32_t>(dc_len, G);

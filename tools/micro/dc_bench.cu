@@ -1,5 +1,5 @@
 // Microbenchmark (not product code): k_doc_combine on a synthetic Zipf (slot, doc) stream of
-// config-2 size; variants selected by -DDC_VARIANT in combine.cuh experiments.
+// config-2 size, checking per-range token counts and docID order of the merged elements.
 #include <cstdio>
 #include <cstdint>
 #include <vector>
