@@ -567,3 +567,24 @@ def test_partials_repeated_reset_and_read_postings():
             d, t = ix.read_postings(terms[i])
             lo, hi = int(w.post_off[i]), int(w.post_off[i + 1])
             assert np.array_equal(d, w.docid[lo:hi]) and np.array_equal(t, w.tf[lo:hi])
+
+
+def test_partials_profiled_stats_between_chunks():
+    # WJ_FLAG_PROFILE with the side / dictionary streams: stats between add_stream calls (an unjoined
+    # chunk, events on three streams), reset with a pending chunk, then a full pass
+    cfg = gen.CONFIGS[2].scaled(chunk_bytes=3 << 20, vocab=40_000)
+    text, off = gen.generate(cfg)
+    n = len(off) - 1
+    want = oracle.index_bytes(text, off)
+    with wj.Index(device=0, profile=True) as ix:
+        ix.add_stream(text[:int(off[n // 2])], off[:n // 2 + 1].astype(np.uint64))
+        s = ix.stats()
+        assert s["n_tokens"] > 0 and s["phase_ms"]["sort"] > 0 and s["kernel_count"]["sort_scatter"] > 0
+        ix.reset()
+        for a, b in ((0, n // 2), (n // 2, n)):
+            ix.add_stream(text[int(off[a]):int(off[b])], (off[a:b + 1] - off[a]).astype(np.uint64))
+            ix.stats()
+        ix.finalize()
+        assert_same_index(ix.serialize(), want)
+        s = ix.stats()
+        assert s["kernel_count"]["copy_partials"] >= 1 and s["stream_elems"] == s["n_tokens"]
