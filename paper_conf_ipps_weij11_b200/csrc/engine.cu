@@ -1948,6 +1948,9 @@ int index_init(wj_index** out, const wj_config* cfg) {
 #undef WJ_DS_ATTR
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_doc_combine, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)dc_smem_bytes()));
+    if (const char* e = getenv("WJ_EMIT_CARVEOUT"))
+      WJ_CUDA_CHECK(cudaFuncSetAttribute(k_tok_emit, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                         (int)strtol(e, nullptr, 10)));
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rle_write_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)rle_smem_bytes()));
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rle_write_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,

@@ -362,8 +362,11 @@ __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* tabl
   return kMiss;
 }
 
-// 6 CTAs/SM (40 registers, 320-entry token queues, 31 KB of shared memory per CTA): emit 2.43 -> 2.34 ms
-// on config 2 vs 5 CTAs/SM (48 registers, 512-entry queues); 4 CTAs/SM (64 registers) was 0.3 ms slower still
+// Launch bounds for 6 CTAs/SM (40 registers) with 320-entry token queues (31 KB of shared memory per
+// CTA): emit 2.43 -> 2.34 ms on config 2 vs 48 registers and 512-entry queues.  The L1 share matters as
+// much as the warps: with the driver's default carveout the kernel runs at ~66% occupancy; forcing a
+// 86-100% shared-memory carveout (more CTAs, less L1 for the table probes) costs ~1 ms, 58-64% costs
+// 0.18 ms (profiles/r01_README.md)
 #ifndef WJ_EMIT_MINB
 #define WJ_EMIT_MINB 6
 #endif
