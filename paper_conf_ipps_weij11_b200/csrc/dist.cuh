@@ -118,4 +118,14 @@ __global__ void k_xid_map(const uint32_t* syn_slot, uint32_t n, const Slot* tabl
   map[x] = table[sl].k0 ? u_tid[slot_uid[sl]] : 0u;
 }
 
+// Owner side on the per-run partials path: a record of source s carries
+// xid = index of its term in the text s sent; replace it by that term's stream element in the owner's
+// chunk table (slot | count 1 << 25, as k_tok_emit writes it), so the received records are a chunk
+// stream like a single-GPU chunk's and are sorted by slot on the side stream (partials.cuh).
+__global__ void k_xid_to_slot(uint32_t* key, uint64_t n, const uint32_t* syn_slot) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  key[i] = syn_slot[key[i] & kXidMask];
+}
+
 }  // namespace wj

@@ -1293,8 +1293,9 @@ struct wj_index {
     // registered below, so no per-record translation pass is needed
     const uint64_t R = rr_off[K];
     if (n_elems + R > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 stream elements"};
-    uint32_t* recv_key = buf_keep<uint32_t>(g_tid, n_elems + R + 16, n_elems) + n_elems;
-    uint32_t* recv_doc = buf_keep<uint32_t>(g_doc, n_elems + R + 16, n_elems) + n_elems;
+    // partials path (pm): the records land in the chunk stream buffers of the per-run partial lists
+    uint32_t* recv_key = pm ? buf<uint32_t>(pc_key, R + 16) : buf_keep<uint32_t>(g_tid, n_elems + R + 16, n_elems) + n_elems;
+    uint32_t* recv_doc = pm ? buf<uint32_t>(pc_doc, R + 16) : buf_keep<uint32_t>(g_doc, n_elems + R + 16, n_elems) + n_elems;
     std::vector<uint64_t> rec_soff(K + 1), rec_roff(K + 1);
     for (int o = 0; o <= K; ++o) { rec_soff[o] = r_off[o] * 4; rec_roff[o] = rr_off[o] * 4; }
     const uint64_t t0 = xport->sent;
@@ -1321,6 +1322,22 @@ struct wj_index {
       }, C2, U2, sslot, sdoc);
       n_dropped = dropped0;
       if (Ns != rt_off[K]) throw StatusError{WJ_ERR_CUDA, "received term text: token count mismatch (internal)"};
+      if (pm) {  // records -> owner chunk-table stream elements; sort by slot beside the dictionary update
+        phase(WJ_PHASE_STREAM);
+        for (int src = 0; src < K; ++src) {
+          const uint64_t nr = rr_off[src + 1] - rr_off[src];
+          if (nr == 0) continue;
+          k_xid_to_slot<<<grid_for(nr, 256), 256, 0, st>>>(recv_key + rr_off[src], nr, sslot + rt_off[src]);
+          launched();
+        }
+        phase(-1);
+        if (R > 0) chunk_partials(recv_terms, R, C2, U2);
+        n_elems += R;
+        n_tokens += R;
+        n_docs += tot_docs;
+        sync();  // exchange buffers are reused by the next chunk
+        return;
+      }
       dictionary_update(recv_terms, U2);
       phase(WJ_PHASE_STREAM);
       // source s's records: key & kRankMask = xid = index into the terms s sent; map xid -> termID
@@ -1899,8 +1916,15 @@ int index_init(wj_index** out, const wj_config* cfg) {
         WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->pipe_done[i], cudaEventDisableTiming));
       }
     }
-    // a transport (world > 1, or a communicator at world 1) runs the distributed path: global stream
-    ix->pm = ix->world == 1 && !cfg->nccl_unique_id && !ix->stem_on && !ix->stop_on;
+    // per-run partial lists on one GPU; the distributed path (a transport: world > 1, or a
+    // communicator at world 1) keeps the global stream unless WJ_DIST_PARTIALS=1 (owner-side partial
+    // lists, parity-green but 11.53 -> 11.86-11.92 ms/step at K = 1 on config 2: the dictionary
+    // update it overlaps is ~1.2 ms there, less than the partial-list combine costs; profiles/r01_README.md)
+    ix->pm = !ix->stem_on && !ix->stop_on;
+    if (ix->world > 1 || cfg->nccl_unique_id) {
+      const char* e = getenv("WJ_DIST_PARTIALS");
+      ix->pm = ix->pm && e && strtoull(e, nullptr, 10) != 0;
+    }
     if (const char* e = getenv("WJ_PARTIALS")) ix->pm = ix->pm && strtoull(e, nullptr, 10) != 0;
     if (const char* e = getenv("WJ_DOC_COMBINE")) ix->combine_on = strtoull(e, nullptr, 10) != 0;
     if (const char* e = getenv("WJ_HOT_MIN_BYTES")) ix->hot_min_bytes = strtoull(e, nullptr, 10);

@@ -77,6 +77,19 @@ def test_loopback_config1(K):
     assert wj.merge_serialized(slices) == want
 
 
+@pytest.mark.parametrize("K", [1, 2, 3])
+@pytest.mark.parametrize("dist_partials", ["0", "1"])
+def test_loopback_owner_partials(K, dist_partials, monkeypatch):
+    """Owner side on per-run partial lists (WJ_DIST_PARTIALS=1: received records sorted by the owner's
+    chunk-table slot on the side stream) and on the global stream (default): both
+    byte-identical to the oracle over three chunks."""
+    monkeypatch.setenv("WJ_DIST_PARTIALS", dist_partials)
+    text, off = gen.generate(gen.CONFIGS[1])
+    want = oracle.index_bytes(text, off)
+    slices, _ = dist_index(text, off, K, cuts=[0, 300, 301, 1000])
+    assert wj.merge_serialized(slices) == want
+
+
 def test_loopback_edges_and_queries():
     docs = [b"", b"a", b"b", b"Apple apple APPLE", b"x" * 300 + b" zoo 01 0195 954", b"", b"aaat aabomycin zzzy",
             b"application lication"] * 5
