@@ -42,7 +42,9 @@ typedef enum {
   WJ_ERR_CUDA = -3,            /* CUDA runtime / kernel error, or no CUDA device                  */
   WJ_ERR_NCCL = -4,            /* NCCL error (world > 1)                                          */
   WJ_ERR_OOM = -5,             /* device allocation failed (or caller workspace exhausted)        */
-  WJ_ERR_CAPACITY = -6,        /* > 2^32-1 documents, tokens or terms; arena > 4 GiB              */
+  WJ_ERR_CAPACITY = -6,        /* > 2^32-1 documents or tokens; > 2^32-2 terms (one GPU) or 2^25 */
+                               /* terms per slice (world > 1, stemming); > 2^25 distinct terms in  */
+                               /* one index_add_stream call; string arena > 4 GiB                  */
   WJ_ERR_BUFFER_TOO_SMALL = -7 /* output buffer smaller than needed; *n_out holds the size needed */
 } wj_status;
 
@@ -131,6 +133,8 @@ typedef struct {
   uint64_t device_bytes;           /* device memory held by the context                              */
   uint64_t stream_elems;           /* (term, docID) stream elements of the index so far: tokens after */
                                    /* the per-document combine (elements the finalize sort moves)    */
+  uint64_t table_retries;          /* chunk hash-table probe overflows retried with a doubled table   */
+                                   /* (cumulative since index_init)                                   */
   /* The fields below are cumulative since index_init (index_reset does not clear them).          */
   double phase_ms[WJ_PHASE_COUNT]; /* WJ_FLAG_PROFILE: accumulated CUDA-event time per phase        */
   uint64_t phase_launches[WJ_PHASE_COUNT];

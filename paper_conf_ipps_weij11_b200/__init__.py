@@ -56,7 +56,7 @@ class Stats(ctypes.Structure):
     _fields_ = [(n, ctypes.c_uint64) for n in
                 ("n_docs", "n_tokens", "n_dropped", "n_terms", "n_postings", "n_term_bytes", "n_chunks",
                  "kernel_launches", "host_syncs", "unique_terms_last", "new_terms_last", "btree_nodes",
-                 "btree_height_max", "exchange_bytes", "device_bytes", "stream_elems")] + [
+                 "btree_height_max", "exchange_bytes", "device_bytes", "stream_elems", "table_retries")] + [
         ("phase_ms", ctypes.c_double * 16), ("phase_launches", ctypes.c_uint64 * 16),
         ("kernel_ms", ctypes.c_double * len(KERNELS)), ("kernel_count", ctypes.c_uint64 * len(KERNELS))]
 
@@ -256,7 +256,7 @@ class Index:
     def stats(self) -> dict:
         s = Stats()
         self._check(self._lib.index_stats(self._h, ctypes.byref(s)))
-        out = {name: getattr(s, name) for name, _ in Stats._fields_[:16]}
+        out = {name: getattr(s, name) for name, _ in Stats._fields_[:17]}
         out["phase_ms"] = {PHASES[i]: s.phase_ms[i] for i in range(len(PHASES))}
         out["phase_launches"] = {PHASES[i]: s.phase_launches[i] for i in range(len(PHASES))}
         out["kernel_ms"] = {KERNELS[i]: s.kernel_ms[i] for i in range(len(KERNELS))}

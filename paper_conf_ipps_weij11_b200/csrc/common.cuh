@@ -45,6 +45,14 @@ __host__ __device__ inline uint32_t ceil_div32(uint64_t a, uint32_t b) { return 
 
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
 
+// ld.acquire.gpu of a 64-bit word: later loads of this thread observe what the releasing writer
+// stored before its release (PTX memory model)
+__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+
 // ---- SWAR byte classification (4 bytes per u32, little-endian byte order) -------------------
 // Token bytes (reading S1): [0-9] U [A-Z] U [a-z] U [0x80-0xFF].  Returns bit i = byte i.
 __device__ __forceinline__ uint32_t tokmask4(uint32_t x) {

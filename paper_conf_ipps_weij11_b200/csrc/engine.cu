@@ -159,6 +159,7 @@ struct wj_index {
   uint32_t V = 0;
   uint64_t arena_used = 0;
   uint64_t table_est = 0;
+  uint64_t table_retries = 0;  // chunk-table probe overflows retried with a larger table (cumulative)
   // chunk table capacity = table_pct% of the expected unique terms (WJ_TABLE_PCT), any multiple of
   // 4096 slots (mulhi indexing).  On config 2 the emit kernel gets faster with capacity (2.82 / 2.45 /
   // 2.36 ms at 125 / 190 / 320%: shorter probe runs) while the slot -> rank gather of the first sort
@@ -692,7 +693,9 @@ struct wj_index {
     // the last U); a probe-sequence overflow retries with a doubled table
     uint64_t est = std::max<uint64_t>({table_est, Nc / 32, 4096});
     est = std::min<uint64_t>(est, Nc + 16);
-    C = table_cap(est * table_pct / 100);
+    // stream elements carry the slot below the count bits (slot | count << kCountShift): C <= 2^25
+    constexpr uint64_t kMaxC = (uint64_t)kRankMask + 1;
+    C = std::min<uint64_t>(table_cap(est * table_pct / 100), kMaxC);
     uint32_t* slot_uid = nullptr;
     for (;;) {
       Slot* tab = buf<Slot>(table, C);
@@ -715,7 +718,11 @@ struct wj_index {
       readback(2, 4);
       U = (uint32_t)h_scal[2];
       if (((uint32_t)h_scal[5]) == 0) break;
-      C *= 2;  // probe sequence overflow: retry with a larger table
+      // probe sequence overflow: retry with a larger table
+      if (C >= kMaxC)
+        throw StatusError{WJ_ERR_CAPACITY, "more than ~2^25 distinct terms in one index_add_stream call: pass smaller chunks"};
+      C = std::min<uint64_t>(C * 2, kMaxC);
+      ++table_retries;
       phase(WJ_PHASE_TOKENIZE);
     }
     unique_last = U;
@@ -877,7 +884,11 @@ struct wj_index {
     const uint64_t Nn = (uint32_t)h_scal[3];
     new_last = Nn;
     if (Nn > 0) {
-      if ((uint64_t)V + Nn > 0xFFFFFFFEull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-2 terms"};
+      // the per-run partial lists carry u32 termIDs; the global-stream path (multi-rank, stemming)
+      // sorts rank | count << kCountShift keys, so its dictionary slice is limited to 2^25 terms
+      const uint64_t vmax = pm ? 0xFFFFFFFEull : (uint64_t)kRankMask + 1;
+      if ((uint64_t)V + Nn > vmax)
+        throw StatusError{WJ_ERR_CAPACITY, pm ? "more than 2^32-2 terms" : "more than 2^25 terms in one dictionary slice"};
       insert_new(text, U, Nn);
       phase(WJ_PHASE_REBUILD);
       rebuild();
@@ -1606,7 +1617,7 @@ struct wj_index {
     const uint64_t NE = n_elems;  // stream elements (tokens, aggregated hot entries, holes)
     uint32_t* ro = buf<uint32_t>(rank_of, V);
     uint2* ta = buf<uint2>(term_at, V);  // rank_info
-    if ((uint64_t)V > (uint64_t)kRankMask + 1)
+    if (!pm && (uint64_t)V > (uint64_t)kRankMask + 1)  // enforced at insert already (dictionary_update)
       throw StatusError{WJ_ERR_CAPACITY, "more than 2^25 terms in one dictionary slice"};
     if (V > 0) {
       phase(WJ_PHASE_LEXRANK);
@@ -2084,6 +2095,7 @@ int index_stats(wj_index* ix, wj_stats* out) {
     out->exchange_bytes = ix->exchange_bytes;
     out->device_bytes = ix->device_bytes;
     out->stream_elems = ix->finalized ? ix->sorted_elems : ix->n_elems;
+    out->table_retries = ix->table_retries;
     for (int i = 0; i < WJ_PHASE_COUNT; ++i) {
       out->phase_ms[i] = ix->phase_ms[i];
       out->phase_launches[i] = ix->phase_launches[i];

@@ -32,7 +32,7 @@ constexpr int kWinBytes = (kSegsPerWarp + 1) * kSegBytes + 16;  // staged range 
 #ifndef WJ_QUEUE_CAP
 #define WJ_QUEUE_CAP 320
 #endif
-constexpr int kQueueCap = WJ_QUEUE_CAP;  // >= tokens of one segment (<= 257) + 1
+constexpr int kQueueCap = WJ_QUEUE_CAP;  // a segment with more kept starts is queued in rounds (emit)
 
 struct ChunkView {
   const uint8_t* text;     // 16-byte aligned device pointer
@@ -359,6 +359,8 @@ __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* tabl
       while (e.y == 0) e.y = *(volatile unsigned long long*)&table[i].k1;
       if (e.y == k1) {
         if (len <= kSlotBytes) return i;
+        // acquire: the inserter wrote slot_ref[i] before its release of k1 (__threadfence + store)
+        (void)ld_acquire_u64(&table[i].k1);
         const uint32_t r = *(volatile uint32_t*)&slot_ref[i];
         const TermWords other(text, r, len);
         bool eq = true;
@@ -523,15 +525,36 @@ __global__ void __launch_bounds__(kTokThreads, WJ_EMIT_MINB) k_tok_emit(ChunkVie
     }
     const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
     if (qn + tot > (uint32_t)kQueueCap) flush();
-    uint32_t pos_q = qn + inc - c;
-    for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
-      const int jb = __ffs(sm) - 1;
-      const uint32_t pos = 16 * lane + jb;
-      if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
-      const uint32_t len = tok_end_rel(sb, tk, jb) - pos;
-      if (len <= kMaxTermLen) q[pos_q++] = ((s0 + pos - B0) << 8) | len;
+    if (tot <= (uint32_t)kQueueCap) {
+      uint32_t pos_q = qn + inc - c;
+      for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
+        const int jb = __ffs(sm) - 1;
+        const uint32_t pos = 16 * lane + jb;
+        if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
+        const uint32_t len = tok_end_rel(sb, tk, jb) - pos;
+        if (len <= kMaxTermLen) q[pos_q++] = ((s0 + pos - B0) << 8) | len;
+      }
+      qn += tot;
+    } else {
+      // Rare: more kept tokens start in this segment than the queue holds (up to 512: dense
+      // document starts, e.g. consecutive 1-byte documents).  Queue them in rounds of kQueueCap,
+      // flushing between rounds (the queue is empty here: tot > kQueueCap forced the flush above).
+      for (uint32_t r0 = 0; r0 < tot; r0 += (uint32_t)kQueueCap) {
+        uint32_t pos_q = inc - c;  // segment-relative index of the lane's first kept token
+        for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
+          const int jb = __ffs(sm) - 1;
+          const uint32_t pos = 16 * lane + jb;
+          if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
+          const uint32_t len = tok_end_rel(sb, tk, jb) - pos;
+          if (len > kMaxTermLen) continue;
+          if (pos_q >= r0 && pos_q < r0 + (uint32_t)kQueueCap) q[pos_q - r0] = ((s0 + pos - B0) << 8) | len;
+          ++pos_q;
+        }
+        qn = min(tot - r0, (uint32_t)kQueueCap);
+        __syncwarp();
+        flush();
+      }
     }
-    qn += tot;
     if (tk.open_lane >= 0) { open = true; open_start = s0 + tk.open_pos; }
     __syncwarp();
   }

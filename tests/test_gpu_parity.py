@@ -588,3 +588,36 @@ def test_partials_profiled_stats_between_chunks():
         assert_same_index(ix.serialize(), want)
         s = ix.stats()
         assert s["kernel_count"]["copy_partials"] >= 1 and s["stream_elems"] == s["n_tokens"]
+
+
+# ------------------------------------------------------------------ robustness (round 2)
+@pytest.mark.parametrize("doc", [b"a", b"ab", b"a b", b"a,", b"Zz9"])
+def test_dense_tiny_documents(doc):
+    """Thousands of consecutive 1-3 byte documents: up to 512 token starts in one 512-byte segment
+    (every byte a document start), more than the emit kernel's per-warp token queue holds; the
+    segment is queued in rounds (tokenize.cuh)."""
+    docs = [doc] * 5000 + [b"tail word"] + [doc] * 3001
+    text, off = docs_to_corpus(docs)
+    want = oracle.index_bytes(text, off)
+    assert_same_index(gpu_index(text, off), want)
+    assert_same_index(gpu_index(text, off, cuts=[0, 777, 778, len(docs)]), want)
+    with wj.Index() as ix:
+        assert ix.debug_tokens(text, off) == oracle.dump_tokens(text, off)
+
+
+def test_table_overflow_retry_forced():
+    """A first chunk whose distinct-term count is far above the table's estimate (N/32): the
+    probe sequences overflow and the chunk is retokenised with a doubled table (engine.cu
+    tokenize_dedup); table_retries counts it and the index stays bit-exact."""
+    rng = np.random.default_rng(11)
+    words = [bytes(rng.choice(list(b"abcdefghijklmnopqrstuvwxyz"), size=int(rng.integers(4, 14))))
+             for _ in range(60_000)]
+    docs = [b" ".join(words[i:i + 40]) for i in range(0, len(words), 40)]
+    text, off = docs_to_corpus(docs)
+    want = oracle.index_bytes(text, off)
+    with wj.Index(device=0) as ix:
+        ix.add_stream(text, off)
+        ix.finalize()
+        got = ix.serialize()
+        assert ix.stats()["table_retries"] >= 1
+    assert_same_index(got, want)
