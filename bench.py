@@ -44,7 +44,6 @@ KERNEL_BYTES = {
     "tokenize_emit": lambda T, N, P, E: T + 8 * N,          # read text, write (slot u32, doc u32) per token
     "slot_to_tid": lambda T, N, P, E: 8 * N,                # read + write u32 per token
     "map_rank": lambda T, N, P, E: 8 * E,                   # read + write u32 per element
-    "doc_combine": lambda T, N, P, E: 8 * N + 8 * E,        # read (slot, doc) per token, write per element
     "sort_hist": lambda T, N, P, E: 4 * E,                  # read u32 keys
     "sort_scatter": lambda T, N, P, E: 16 * E,              # read + write (u32 key, u32 doc) per element
     "rle_emit": lambda T, N, P, E: 8 * E + 8 * P,           # read (key, doc), write (docid, tf)

@@ -112,12 +112,11 @@ enum {
   WJ_KERNEL_PROBE,              /* K3 warp-per-key B-tree descent                                   */
   WJ_KERNEL_SLOT_TO_TID,        /* stream slot -> termID                                           */
   WJ_KERNEL_MAP_RANK,           /* finalize: termID -> lexicographic rank                          */
-  WJ_KERNEL_SORT_HIST,          /* finalize: radix digit histogram (token stream)                  */
-  WJ_KERNEL_SORT_SCATTER,       /* finalize: stable radix scatter (token stream)                   */
-  WJ_KERNEL_RLE_EMIT,           /* finalize: run-length (docID, tf) emit                           */
-  WJ_KERNEL_DOC_COMBINE,        /* per-document pre-aggregation of the stream (combine.cuh, opt-in) */
+  WJ_KERNEL_SORT_HIST,          /* radix digit histogram of the (term, docID) stream                */
+  WJ_KERNEL_SORT_SCATTER,       /* stable radix scatter of the (term, docID) stream                 */
+  WJ_KERNEL_RLE_EMIT,           /* run-length (docID, tf) emit of the sorted stream                 */
   WJ_KERNEL_COPY_PARTIALS,      /* finalize: copy each chunk's partial postings lists into place    */
-  WJ_KERNEL_COUNT = 10
+  WJ_KERNEL_COUNT = 9
 };
 
 typedef struct {
@@ -131,8 +130,8 @@ typedef struct {
   uint64_t btree_height_max;       /* tallest trie-collection B-tree                                 */
   uint64_t exchange_bytes;         /* world > 1: bytes this rank sent                                */
   uint64_t device_bytes;           /* device memory held by the context                              */
-  uint64_t stream_elems;           /* (term, docID) stream elements of the index so far: tokens after */
-                                   /* the per-document combine (elements the finalize sort moves)    */
+  uint64_t stream_elems;           /* (term, docID) stream elements of the index so far (tokens, and  */
+                                   /* aggregated hot-term elements with WJ_FLAG_HOT_TERMS)            */
   uint64_t table_retries;          /* chunk hash-table probe overflows retried with a doubled table   */
                                    /* (cumulative since index_init)                                   */
   /* The fields below are cumulative since index_init (index_reset does not clear them).          */

@@ -24,7 +24,7 @@ WJ_FLAG_PROFILE = 1
 PHASES = ["h2d", "tokenize", "unique", "probe", "insert", "rebuild", "stream", "lexrank", "sort", "postings",
           "dict", "exchange", "vbyte", "stem"]
 KERNELS = ["tokenize_count", "tokenize_emit", "probe", "slot_to_tid", "map_rank", "sort_hist", "sort_scatter",
-           "rle_emit", "doc_combine", "copy_partials"]
+           "rle_emit", "copy_partials"]
 N_COLLECTIONS = 17613
 
 EXPORTS = ["index_init", "index_add_stream", "index_finalize", "index_read_postings", "index_serialize",

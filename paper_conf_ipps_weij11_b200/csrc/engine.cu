@@ -7,7 +7,6 @@
 #include <vector>
 
 #include "../../include/wjindex.h"
-#include "combine.cuh"
 #include "common.cuh"
 #include "dict.cuh"
 #include "dist.cuh"
@@ -178,13 +177,6 @@ struct wj_index {
       samp_ck2, samp_cv2, samp_n;
   uint32_t hot_H = 0, hot_D = 0;
   bool stream_has_hot = false;  // some chunk appended hot-term elements (holes + counts > 1)
-  // Per-document pre-aggregation of the stream before the finalize sort (combine.cuh) is opt-in
-  // (WJ_DOC_COMBINE=1): it shrinks the sorted stream to 0.68 N on config 2 (sort 3.76 -> 2.66 ms), but
-  // merging needs a shared hash table per tile and neither a CAS insert (returning shared atomics run
-  // at ~2 cycles/lane: 3.6 ms) nor a CAS-free round-based insert (5.8 ms) costs less than it saves
-  // (profiles/r01_README.md)
-  bool combine_on = false;
-  DevBuf dc_len;
   // Partial postings per chunk (partials.cuh; single GPU, no stemming / stop words / hot terms): the
   // chunk's stream is sorted by slot and run-length encoded on side_st while the dictionary update
   // runs on st; finalize combines the partial lists.  WJ_PARTIALS=0: global stream
@@ -202,7 +194,7 @@ struct wj_index {
   bool pc_join = false;              // the last chunk's side-stream work is not joined yet
   uint64_t pc_U = 0, pc_Nc = 0;
   std::vector<uint64_t> rec_end;     // end of each chunk's records
-  uint64_t sorted_elems = 0;    // stream elements the last finalize sorted (after the combine)
+  uint64_t sorted_elems = 0;    // stream elements the last finalize sorted (after hole compaction)
   // Sampled hot-term path (hot.cuh) is opt-in: on config 2 it removes ~30% of the
   // stream elements but its per-document counters cost more global atomics in the emit kernel than
   // the sort saves (profiles/r01_README.md).  WJ_HOT_MIN_BYTES=<bytes> enables it for larger chunks.
@@ -214,7 +206,6 @@ struct wj_index {
       t_bucket;
   // device scalars: [0] tokens, [1] dropped, [2] U, [3] Nnew, [4] arena total, [5] overflow|bad,
   // [6] tid counter (u32 view), [7] level count, [8] P, [9] TB, [10] bad doc_off, [11] rle tokens,
-  // [12] doc-combine output length
   DevBuf scal;
   uint64_t* h_scal = nullptr;  // pinned
   // token stream (termID, docID) of all chunks
@@ -288,7 +279,7 @@ struct wj_index {
                      &dbg_doc, &lexg, &qbuf, &qres, &rank_of, &term_at, &sk1, &sv1, &pidx, &out_doc, &out_tf,
                      &post_off, &df, &cf, &term_off, &term_bytes, &vb_first, &vb_tiles, &vb_code, &vb_boff, &samp_hist, &owner_tab,
                      &table_s, &uid_s, &st_off, &st_text, &st_keep, &st_tidx, &st_m1, &st_slot, &st_doc, &st_tiles,
-                     &st_doff, &stop_keys, &dc_len, &side_scan, &side_hist, &side_hist_scan, &pc_key, &pc_doc, &pc_po,
+                     &st_doff, &stop_keys, &side_scan, &side_hist, &side_hist_scan, &pc_key, &pc_doc, &pc_po,
                      &pc_cs, &u_slot, &pp_doc, &pp_tf, &rec_tid, &rec_start, &rec_df, &rec_cf, &rec_before, &df_totb,
                      &cf_totb};
     for (DevBuf* b : all) {
@@ -1493,7 +1484,7 @@ struct wj_index {
                   const uint32_t* rank_of, bool timed,
                   const std::vector<std::pair<uint64_t, const uint32_t*>>* segs = nullptr, K kmask = ~K(0),
                   bool skip0 = false, uint64_t* n_out = nullptr, bool mask_digits = true,
-                  std::vector<uint64_t>* digit_start = nullptr, bool combine = false) {
+                  std::vector<uint64_t>* digit_start = nullptr) {
     if (n_out) *n_out = n;
     if (n == 0) return false;
     int passes = end_bit > begin_bit ? (end_bit - begin_bit + 7) / 8 : 0;
@@ -1522,20 +1513,6 @@ struct wj_index {
     const uint32_t* first_map = (segs && !multi_map) ? (*segs)[0].second : rank_of;
     bool in1 = false;
     uint64_t cur_n = n;
-    // per-document combine (combine.cuh) on the first pass's ranges: range c keeps rlen[c] elements
-    const uint32_t* rlen = nullptr;
-    if (combine) {
-      uint64_t per = (n + rs_ctas - 1) / rs_ctas;  // the first pass's ranges
-      per = (per + kOsTile - 1) / kOsTile * kOsTile;
-      const uint32_t G = (uint32_t)((n + per - 1) / per);
-      uint32_t* rl = buf<uint32_t>(dc_len, G);
-      auto c = [&] {
-        k_doc_combine<<<G, kDcThreads, dc_smem_bytes(), st>>>((uint32_t*)k0, v0, n, per, rl);
-        launched();
-      };
-      if (timed) ktime(WJ_KERNEL_DOC_COMBINE, c); else c();
-      rlen = rl;
-    }
     for (int p = 0; p < passes; ++p) {
       uint64_t per = (cur_n + rs_ctas - 1) / rs_ctas;
       per = (per + kOsTile - 1) / kOsTile * kOsTile;
@@ -1549,26 +1526,25 @@ struct wj_index {
       const int shift = begin_bit + 8 * p;
       const uint32_t* mp = p == 0 ? first_map : nullptr;
       const bool holes = skip0 && p == 0;
-      const uint32_t* rl = p == 0 ? rlen : nullptr;
       // the count bits of stream elements only reach a digit when passes cover bits >= 25
       const bool masked = mask_digits && kmask != ~K(0) && begin_bit + 8 * passes > kCountShift;
       auto up = [&] {
         WJ_CUDA_CHECK(cudaMemsetAsync(h1, 0, (size_t)256 * G * 4, st));
         const uint32_t GU = G * kRsUpSplit;
-        if (holes && masked) k_rs_up<K, true, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, rl);
-        else if (holes) k_rs_up<K, true, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, rl);
-        else if (masked) k_rs_up<K, false, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, rl);
-        else k_rs_up<K, false, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, rl);
+        if (holes && masked) k_rs_up<K, true, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
+        else if (holes) k_rs_up<K, true, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
+        else if (masked) k_rs_up<K, false, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
+        else k_rs_up<K, false, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
         launched();
       };
       if (timed) ktime(WJ_KERNEL_SORT_HIST, up); else up();
       scan<uint32_t>(ArrayIn<uint32_t>{h1}, (uint64_t)256 * G, h2, h2 + (uint64_t)256 * G);
       auto down = [&] {
         const size_t sm = ds_smem_bytes<K>();
-        if (holes && masked) k_rs_down2<K, true, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, rl);
-        else if (holes) k_rs_down2<K, true, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, rl);
-        else if (masked) k_rs_down2<K, false, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, rl);
-        else k_rs_down2<K, false, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, rl);
+        if (holes && masked) k_rs_down2<K, true, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
+        else if (holes) k_rs_down2<K, true, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
+        else if (masked) k_rs_down2<K, false, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
+        else k_rs_down2<K, false, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
         launched();
       };
       if (timed) ktime(WJ_KERNEL_SORT_SCATTER, down); else down();
@@ -1579,7 +1555,7 @@ struct wj_index {
         sync();
         digit_start->assign(ds.begin(), ds.end());
       }
-      if (holes || rl) {  // elements that survive the compaction / the combine
+      if (holes) {  // elements that survive the compaction
         uint32_t tot = 0;
         WJ_CUDA_CHECK(cudaMemcpyAsync(&tot, h2 + (uint64_t)256 * G, 4, cudaMemcpyDeviceToHost, st));
         sync();
@@ -1732,11 +1708,9 @@ struct wj_index {
         segs.emplace_back(chunk_tok[c], m);
       }
       uint64_t N = NE;
-      // the combine needs single-token input elements (no hot-term count elements or holes)
-      const bool combine = combine_on && !stream_has_hot;
       const bool in1 =
           sort_pairs<uint32_t>(kt, dt, k1, v1, NE, 0, bits, nullptr, true, &segs, kRankMask, stream_has_hot, &N, true,
-                               nullptr, combine);
+                               nullptr);
       sorted_elems = N;
       f_key = in1 ? k1 : kt;
       f_doc = in1 ? v1 : dt;
@@ -1752,14 +1726,14 @@ struct wj_index {
       uint32_t* od = buf<uint32_t>(out_doc, N);
       uint32_t* of = buf<uint32_t>(out_tf, N);
       ktime(WJ_KERNEL_RLE_EMIT, [&] {
-        if (stream_has_hot || combine)
+        if (stream_has_hot)
           k_rle_count<true><<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc, rt);
         else
           k_rle_count<false><<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc, rt);
         launched();
         scan<uint32_t>(ArrayIn<uint32_t>{rc}, G, rc, (uint32_t*)(dscal() + 8));
         scan<uint64_t>(ArrayIn<uint64_t>{rt}, G, rt, (uint64_t*)(dscal() + 11));
-        if (stream_has_hot || combine)
+        if (stream_has_hot)
           k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl);
         else
           k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(false), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl);
@@ -1937,7 +1911,6 @@ int index_init(wj_index** out, const wj_config* cfg) {
       ix->pm = ix->pm && e && strtoull(e, nullptr, 10) != 0;
     }
     if (const char* e = getenv("WJ_PARTIALS")) ix->pm = ix->pm && strtoull(e, nullptr, 10) != 0;
-    if (const char* e = getenv("WJ_DOC_COMBINE")) ix->combine_on = strtoull(e, nullptr, 10) != 0;
     if (const char* e = getenv("WJ_HOT_MIN_BYTES")) ix->hot_min_bytes = strtoull(e, nullptr, 10);
     if (ix->hot_min_bytes != ~0ull) ix->pm = false;  // hot-term elements need the global stream
     if (const char* e = getenv("WJ_SIDE_CTAS")) ix->side_ctas = std::max<uint32_t>((uint32_t)strtoul(e, nullptr, 10), 1);
@@ -1962,18 +1935,6 @@ int index_init(wj_index** out, const wj_config* cfg) {
         throw StatusError{WJ_ERR_NCCL, e.msg};
       }
     }
-    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_os_pass<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)os_smem_bytes<uint64_t>()));
-    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_os_pass<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)os_smem_bytes<uint32_t>()));
-    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_os_pass_tma<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)os_tma_smem_bytes<uint64_t>()));
-    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_os_pass_tma<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)os_tma_smem_bytes<uint32_t>()));
-    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rs_down<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)os_tma_smem_bytes<uint64_t>()));
-    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rs_down<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)os_tma_smem_bytes<uint32_t>()));
 #define WJ_DS_ATTR(K, H, M)                                                                           \
   WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rs_down2<K, H, M>, cudaFuncAttributeMaxDynamicSharedMemorySize, \
                                      (int)ds_smem_bytes<K>()))
@@ -1981,8 +1942,6 @@ int index_init(wj_index** out, const wj_config* cfg) {
     WJ_DS_ATTR(uint64_t, true, true); WJ_DS_ATTR(uint32_t, false, false); WJ_DS_ATTR(uint32_t, true, false);
     WJ_DS_ATTR(uint32_t, false, true); WJ_DS_ATTR(uint32_t, true, true);
 #undef WJ_DS_ATTR
-    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_doc_combine, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)dc_smem_bytes()));
     if (const char* e = getenv("WJ_EMIT_CARVEOUT"))
       WJ_CUDA_CHECK(cudaFuncSetAttribute(k_tok_emit, cudaFuncAttributePreferredSharedMemoryCarveout,
                                          (int)strtol(e, nullptr, 10)));

@@ -480,59 +480,6 @@ def test_new_terms_sharing_long_prefixes(seed):
     assert_same_index(gpu_index(text, off, cuts=[0, 3, 5, 8]), want)
 
 
-# ------------------------------------------------------------------ per-document combine (combine.cuh)
-@pytest.fixture
-def combine_off(monkeypatch):
-    monkeypatch.setenv("WJ_DOC_COMBINE", "0")
-    yield
-
-
-@pytest.fixture
-def combine_on(monkeypatch):
-    monkeypatch.setenv("WJ_DOC_COMBINE", "1")
-    monkeypatch.setenv("WJ_PARTIALS", "0")  # the combine runs on the global stream's finalize sort
-    yield
-
-
-def test_combine_repetitive_docs(combine_on):
-    # per-(term, doc) counts above 127 (split elements), documents spanning several 4096-element
-    # tiles (one pair split across tiles), one-token documents, empty documents
-    docs = ([b"the " * 600 + b"cat", b"the", b"", b"The the THE"] * 300 + [b"x y z " * 5000]
-            + [b"w%d" % (i % 7) for i in range(9000)] + [b"the " * 20000])
-    text, off = gen.from_docs(docs)
-    want = oracle.index_bytes(text, off)
-    assert_same_index(gpu_index(text, off), want)
-    n = len(off) - 1
-    assert_same_index(gpu_index(text, off, cuts=[0, 1, n // 2, n - 1, n]), want)
-
-
-@pytest.mark.parametrize("cfg_id", [2, 3, 4])
-def test_combine_shrinks_stream_and_matches(combine_on, cfg_id):
-    cfg = gen.CONFIGS[cfg_id].scaled(chunk_bytes=8 << 20, vocab=300_000)
-    text, off = gen.generate(cfg)
-    want = oracle.index_bytes(text, off)
-    with wj.Index(device=0) as ix:
-        ix.add_stream(text, np.asarray(off, dtype=np.uint64))
-        ix.finalize()
-        got = ix.serialize()
-        s = ix.stats()
-    assert_same_index(got, want)
-    hdr = wjformat.parse(want)
-    # at least one element per posting, at most one per token
-    assert hdr.n_postings <= s["stream_elems"] < s["n_tokens"]
-
-
-def test_combine_off_same_bytes(combine_off):
-    cfg = gen.CONFIGS[2].scaled(chunk_bytes=4 << 20, vocab=100_000)
-    text, off = gen.generate(cfg)
-    with wj.Index(device=0) as ix:
-        ix.add_stream(text, np.asarray(off, dtype=np.uint64))
-        ix.finalize()
-        got = ix.serialize()
-        assert ix.stats()["stream_elems"] == ix.stats()["n_tokens"]
-    assert_same_index(got, oracle.index_bytes(text, off))
-
-
 # ------------------------------------------------------------------ partial lists per run (partials.cuh)
 @pytest.mark.parametrize("partials", ["1", "0"])
 def test_partials_and_global_stream_paths(monkeypatch, partials):
@@ -610,8 +557,8 @@ def test_table_overflow_retry_forced():
     probe sequences overflow and the chunk is retokenised with a doubled table (engine.cu
     tokenize_dedup); table_retries counts it and the index stays bit-exact."""
     rng = np.random.default_rng(11)
-    words = [bytes(rng.choice(list(b"abcdefghijklmnopqrstuvwxyz"), size=int(rng.integers(4, 14))))
-             for _ in range(60_000)]
+    letters = np.frombuffer(b"abcdefghijklmnopqrstuvwxyz", dtype=np.uint8)
+    words = [rng.choice(letters, size=int(rng.integers(4, 14))).tobytes() for _ in range(60_000)]
     docs = [b" ".join(words[i:i + 40]) for i in range(0, len(words), 40)]
     text, off = docs_to_corpus(docs)
     want = oracle.index_bytes(text, off)
