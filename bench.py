@@ -225,6 +225,56 @@ def run_reference(args, rank, world):
     print_json(line)
 
 
+def steady_state(wj, ix, args, device):
+    """Multi-chunk leg (N = 1): S device-resident 1 GiB chunks of config 5 per step (reset + S x
+    add_stream + finalize), so every chunk after the first probes and extends a non-empty dictionary
+    ("Fig. 11").  Reports MB/s, ms per chunk and the per-kernel / per-phase ms per chunk."""
+    import torch
+
+    S = args.steady_chunks
+    parts = []
+    for c in range(S):
+        t, o = corpus(5, c)
+        parts.append((torch.from_numpy(t).cuda(), torch.from_numpy(o.astype(np.int64)).cuda(), len(t)))
+    T = sum(p[2] for p in parts)
+
+    def step():
+        ix.reset()
+        for t, o, _ in parts:
+            ix.add_stream(t, o)
+        ix.finalize()
+
+    step()
+    torch.cuda.synchronize()
+    s0 = ix.stats()
+    steps = 3
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(steps):
+        step()
+    e1.record()
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / steps
+    s1 = ix.stats()
+    kms = {k: round((s1["kernel_ms"][k] - s0["kernel_ms"][k]) / steps / S, 4) for k in wj.KERNELS
+           if s1["kernel_count"][k] > s0["kernel_count"][k]}
+    pms = {k: round((s1["phase_ms"][k] - s0["phase_ms"][k]) / steps / S, 4) for k in wj.PHASES
+           if s1["phase_ms"][k] > s0["phase_ms"][k]}
+    b_min = T + 8 * s1["n_postings"] + s1["n_term_bytes"] + 28 * s1["n_terms"]
+    peak, _ = measured_peak()
+    del parts
+    torch.cuda.empty_cache()
+    return {"workload": f"config 5 (ClueWeb09-shaped) prefix: {S} x 1 GiB chunks, device-resident", "chunks": S,
+            "bytes": T, "ms_per_step": ms, "ms_per_chunk": ms / S, "value": T / (ms / 1e3) / 1e6, "unit": "MB/s",
+            "n_terms": s1["n_terms"], "n_postings": s1["n_postings"], "n_tokens": s1["n_tokens"],
+            "btree_height_max": s1["btree_height_max"], "new_terms_last_chunk": s1["new_terms_last"],
+            "roofline_frac": b_min / (ms / 1e3) / 1e9 / peak, "steps": steps,
+            "kernels_ms_per_chunk": kms, "phases_ms_per_chunk": pms,
+            "host_syncs_per_chunk": (s1["host_syncs"] - s0["host_syncs"]) / steps / S,
+            "launches_per_chunk": (s1["kernel_launches"] - s0["kernel_launches"]) / steps / S}
+
+
 def print_json(obj):  # replaced in main() by a writer bound to the real stdout
     print(json.dumps(obj), flush=True)
 
@@ -248,6 +298,10 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--e2e-chunks", type=int, default=4,
                     help="e2e: feed the step as this many pinned host chunks through the host pipeline")
+    ap.add_argument("--steady-chunks", type=int, default=4,
+                    help="multi-chunk leg: this many 1 GiB chunks of config 5 (ClueWeb scale, SURVEY 8(d)) per step, "
+                         "device-resident, so the B-tree probe, merge and rebuild run on a non-empty dictionary (0: off)")
+    ap.add_argument("--hot", action="store_true", help="sampled hot-term aggregation (SURVEY 8(f2)(ii), opt-in)")
     ap.add_argument("--vbyte", action="store_true",
                     help="also encode the postings as d-gaps + variable-byte code (SURVEY 8(f1), WJINV002)")
     args = ap.parse_args()
@@ -276,6 +330,7 @@ def main():
     off_d = off_h.cuda()
     torch.cuda.synchronize()
 
+    hot = args.hot
     force_dist = os.environ.get("WJ_BENCH_FORCE_DIST") == "1"  # exercise the NCCL path at N=1
     if world > 1 or force_dist:
         nid = [wj.nccl_unique_id() if rank == 0 else None]
@@ -284,7 +339,7 @@ def main():
         ix = wj.Index(device=local, profile=True, rank=rank, world=world, nccl_id=nid[0], vbyte=args.vbyte,
                       balanced=world > 1)
     else:
-        ix = wj.Index(device=local, profile=True, vbyte=args.vbyte)
+        ix = wj.Index(device=local, profile=True, vbyte=args.vbyte, hot=hot)
 
     def step(t, o):
         ix.reset()
@@ -408,6 +463,10 @@ def main():
         if ixe is not ix:
             ixe.close()
 
+    steady = None
+    if args.steady_chunks > 0 and world == 1 and not force_dist:
+        steady = steady_state(wj, ix, args, local)
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(text, doc_off)
@@ -440,6 +499,7 @@ def main():
                                   "def": "implementation bytes of DESIGN.md section 7 (design evidence, not the headline)"},
             "cpu_baseline": cpu,
             "e2e": e2e,
+            "steady_state": steady,
             "gpu_launches": int(round(launches * args.steps)),
             "gpu_launches_per_step": launches,
             "host_syncs_per_step": (s1["host_syncs"] - s0["host_syncs"]) / args.steps,

@@ -68,6 +68,14 @@ typedef enum {
 #define WJ_FLAG_STEM 0x20u     /* parser Step 3 (reading S20): every term of   */
                                /* >= 3 bytes made only of a-z is replaced by its Porter (1980) stem */
                                /* before indexing; the dictionary holds stems (query by the stem)  */
+#define WJ_FLAG_HOT_TERMS 0x80u /* opt-in: per chunk of >= 64 KiB the <= 127 most frequent terms of */
+                               /* a 1 MiB sample are merged per       */
+                               /* document in the tokenizer (one stream element with a count).      */
+                               /* Same bytes; measured slower on config 2            */
+#define WJ_FLAG_GLOBAL_STREAM 0x200u /* one GPU: instead of per-run partial postings lists (sorted  */
+                               /* and run-length encoded per add_stream call beside the dictionary */
+                               /* update, combined at finalize), keep one global      */
+                               /* (term, docID) stream and sort it once at finalize.  Same bytes.   */
 #define WJ_FLAG_STOPWORDS 0x40u /* parser Step 4 (reading S20): tokens whose (stemmed, with */
                                /* WJ_FLAG_STEM) term equals the (stemmed) form of a word of the     */
                                /* built-in 318-word English stop list are dropped; they count in    */
@@ -84,6 +92,12 @@ typedef struct {
   uint64_t max_chunk_bytes;  /* hint: largest n_bytes of one index_add_stream call (0 = no hint)   */
   uint32_t flags;            /* WJ_FLAG_* ; other bits must be 0                                   */
   uint32_t reserved;         /* must be 0                                                          */
+  void* workspace;           /* optional caller-owned device arena (e.g. a torch tensor's memory): */
+  uint64_t workspace_bytes;  /* when non-NULL the library sub-allocates ALL its device buffers from */
+                             /* it (first fit, 256-byte granules) and never calls cudaMalloc for    */
+                             /* index state; the caller keeps it alive and unused until             */
+                             /* index_destroy.  Exhausting it returns WJ_ERR_OOM.  NULL = the       */
+                             /* library allocates with cudaMalloc.                                  */
 } wj_config;
 
 enum {
@@ -134,6 +148,10 @@ typedef struct {
                                    /* aggregated hot-term elements with WJ_FLAG_HOT_TERMS)            */
   uint64_t table_retries;          /* chunk hash-table probe overflows retried with a doubled table   */
                                    /* (cumulative since index_init)                                   */
+  uint64_t hot_elems_saved;        /* stream elements merged away by the hot-term aggregation         */
+                                   /* (cumulative since index_init)                                   */
+  double exchange_ms;              /* world > 1: host wall time of the all-to-all-v rounds, device-    */
+                                   /* synchronised (cumulative since index_init)                      */
   /* The fields below are cumulative since index_init (index_reset does not clear them).          */
   double phase_ms[WJ_PHASE_COUNT]; /* WJ_FLAG_PROFILE: accumulated CUDA-event time per phase        */
   uint64_t phase_launches[WJ_PHASE_COUNT];

@@ -38,6 +38,8 @@ WJ_FLAG_HOST_PIPELINE = 8
 WJ_FLAG_BALANCED_OWNERS = 16
 WJ_FLAG_STEM = 32
 WJ_FLAG_STOPWORDS = 64
+WJ_FLAG_HOT_TERMS = 128
+WJ_FLAG_GLOBAL_STREAM = 512
 
 
 class WJError(RuntimeError):
@@ -49,14 +51,16 @@ class WJError(RuntimeError):
 class Config(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("nccl_unique_id", ctypes.c_void_p), ("stream", ctypes.c_void_p),
-                ("max_chunk_bytes", ctypes.c_uint64), ("flags", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
+                ("max_chunk_bytes", ctypes.c_uint64), ("flags", ctypes.c_uint32), ("reserved", ctypes.c_uint32),
+                ("workspace", ctypes.c_void_p), ("workspace_bytes", ctypes.c_uint64)]
 
 
 class Stats(ctypes.Structure):
     _fields_ = [(n, ctypes.c_uint64) for n in
                 ("n_docs", "n_tokens", "n_dropped", "n_terms", "n_postings", "n_term_bytes", "n_chunks",
                  "kernel_launches", "host_syncs", "unique_terms_last", "new_terms_last", "btree_nodes",
-                 "btree_height_max", "exchange_bytes", "device_bytes", "stream_elems", "table_retries")] + [
+                 "btree_height_max", "exchange_bytes", "device_bytes", "stream_elems", "table_retries",
+                 "hot_elems_saved")] + [("exchange_ms", ctypes.c_double)] + [
         ("phase_ms", ctypes.c_double * 16), ("phase_launches", ctypes.c_uint64 * 16),
         ("kernel_ms", ctypes.c_double * len(KERNELS)), ("kernel_count", ctypes.c_uint64 * len(KERNELS))]
 
@@ -153,7 +157,7 @@ class Index:
     def __init__(self, device: int = 0, stream=None, profile: bool = False, rank: int = 0, world: int = 1,
                  nccl_id: bytes | None = None, hub: "LoopbackHub | None" = None, own_stream: bool = False,
                  vbyte: bool = False, pipeline: bool = False, balanced: bool = False, stem: bool = False,
-                 stop: bool = False):
+                 stop: bool = False, hot: bool = False, workspace=None, global_stream: bool = False):
         """world > 1: pass nccl_id (128 bytes from nccl_unique_id(), broadcast by the caller) or a
         LoopbackHub shared by `world` contexts of this process (one host thread each).
         vbyte: finalize also builds the d-gap + variable-byte postings code; serialize() then
@@ -162,20 +166,31 @@ class Index:
         (Fig. 9); keep each host buffer unchanged until the next call returns.
         balanced: world > 1, owners of the trie collections from a sampled bin-packing.
         stem / stop: the parser's Steps 3-4 (reading S20): Porter (1980)
-        stems and removal of the built-in stop words (stop_words())."""
+        stems and removal of the built-in stop words (stop_words()).
+        hot: sampled hot terms merged per document in the tokenizer for every chunk of >= 64 KiB
+        (opt-in).
+        workspace: a CUDA torch tensor (any dtype) whose memory the library sub-allocates for all of
+        its device state instead of calling cudaMalloc; keep it alive until close().
+        global_stream: one GPU, sort one global (term, docID) stream at finalize instead of building
+        per-run partial postings lists (same bytes)."""
         self._lib = load_library()
         flags = (WJ_FLAG_PROFILE if profile else 0) | (WJ_FLAG_LOOPBACK if hub is not None else 0) | (
             WJ_FLAG_VBYTE if vbyte else 0) | (WJ_FLAG_HOST_PIPELINE if pipeline else 0) | (
             WJ_FLAG_BALANCED_OWNERS if balanced else 0) | (WJ_FLAG_STEM if stem else 0) | (
-            WJ_FLAG_STOPWORDS if stop else 0)
+            WJ_FLAG_STOPWORDS if stop else 0) | (WJ_FLAG_HOT_TERMS if hot else 0) | (
+            WJ_FLAG_GLOBAL_STREAM if global_stream else 0)
         self._nid = ctypes.create_string_buffer(bytes(nccl_id), 128) if nccl_id is not None else None
         uid = hub._h if hub is not None else (ctypes.cast(self._nid, ctypes.c_void_p) if self._nid is not None else None)
         if own_stream:
             strm = ctypes.c_void_p(0)
         else:
             strm = stream if stream is not None else _current_stream(device)
+        ws_ptr, ws_bytes = None, 0
+        self._ws = workspace
+        if workspace is not None:
+            ws_ptr, ws_bytes = workspace.data_ptr(), workspace.numel() * workspace.element_size()
         cfg = Config(device=device, rank=rank, world=world, nccl_unique_id=uid, stream=strm,
-                     max_chunk_bytes=0, flags=flags, reserved=0)
+                     max_chunk_bytes=0, flags=flags, reserved=0, workspace=ws_ptr, workspace_bytes=ws_bytes)
         h = ctypes.c_void_p()
         rc = self._lib.index_init(ctypes.byref(h), ctypes.byref(cfg))
         if rc != WJ_OK:
@@ -256,7 +271,7 @@ class Index:
     def stats(self) -> dict:
         s = Stats()
         self._check(self._lib.index_stats(self._h, ctypes.byref(s)))
-        out = {name: getattr(s, name) for name, _ in Stats._fields_[:17]}
+        out = {name: getattr(s, name) for name, _ in Stats._fields_[:19]}
         out["phase_ms"] = {PHASES[i]: s.phase_ms[i] for i in range(len(PHASES))}
         out["phase_launches"] = {PHASES[i]: s.phase_launches[i] for i in range(len(PHASES))}
         out["kernel_ms"] = {KERNELS[i]: s.kernel_ms[i] for i in range(len(KERNELS))}

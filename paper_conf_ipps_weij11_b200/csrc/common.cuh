@@ -40,6 +40,9 @@ struct __align__(16) Slot {
   unsigned long long k1;
 };
 constexpr uint32_t kSlotBytes = 11;
+// k1 bits 57..63 of a slot seeded with a sampled hot term (k_hot_seed) hold its hot id (1..127)
+constexpr int kHotShift = 57;
+constexpr unsigned long long kSlotK1Mask = (1ull << kHotShift) - 1ull;
 
 __host__ __device__ inline uint32_t ceil_div32(uint64_t a, uint32_t b) { return (uint32_t)((a + b - 1) / b); }
 

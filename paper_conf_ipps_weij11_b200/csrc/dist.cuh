@@ -118,14 +118,56 @@ __global__ void k_xid_map(const uint32_t* syn_slot, uint32_t n, const Slot* tabl
   map[x] = table[sl].k0 ? u_tid[slot_uid[sl]] : 0u;
 }
 
-// Owner side on the per-run partials path: a record of source s carries
-// xid = index of its term in the text s sent; replace it by that term's stream element in the owner's
-// chunk table (slot | count 1 << 25, as k_tok_emit writes it), so the received records are a chunk
-// stream like a single-GPU chunk's and are sorted by slot on the side stream (partials.cuh).
-__global__ void k_xid_to_slot(uint32_t* key, uint64_t n, const uint32_t* syn_slot) {
-  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= n) return;
-  key[i] = syn_slot[key[i] & kXidMask];
+// ------------------------------------------------------------------ sender-side partial lists
+// (SURVEY 8(e)): every rank sorts and run-length encodes its own documents' stream by
+// gpos = (owner's first term index + xid), so the postings it sends to owner o are one contiguous range
+// of (docID, tf) pairs, grouped per term (P:160-162's per-term grouping, aggregated to one posting per
+// (term, document)); a header (df, cf) per term and the folded term bytes go with them.
+
+// slot -> gpos of its unique term (the stream sort key)
+__global__ void k_slot_gpos(const Slot* table, uint32_t C, const uint32_t* slot_uid, const uint32_t* u_owner,
+                            const uint32_t* xid, const uint64_t* t_off, uint32_t* km) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= C || table[i].k0 == 0) return;
+  const uint32_t u = slot_uid[i];
+  km[i] = (uint32_t)t_off[u_owner[u]] + xid[u];
+}
+
+// per term (gpos g): df, cf of its local partial list from the run-length output (post_off / cstart
+// indexed by gpos; every gpos occurs); P_dev = postings of the chunk, NT = its tokens
+__global__ void k_term_hdr(const uint64_t* post_off, const uint64_t* cstart, uint32_t U, const uint32_t* P_dev, uint64_t NT,
+                           uint32_t* df, uint32_t* cf) {
+  const uint32_t g = blockIdx.x * blockDim.x + threadIdx.x;
+  if (g >= U) return;
+  const uint64_t b = g + 1 < U ? post_off[g + 1] : (uint64_t)*P_dev;
+  const uint64_t tb = g + 1 < U ? cstart[g + 1] : NT;
+  df[g] = (uint32_t)(b - post_off[g]);
+  cf[g] = (uint32_t)(tb - cstart[g]);
+}
+
+// per owner o (o <= K): postings / tokens before its first term; bounds[o] = t_off[o] (U: the end)
+__global__ void k_owner_bounds(const uint64_t* post_off, const uint64_t* cstart, const uint64_t* t_off, uint32_t K,
+                               uint32_t U, const uint32_t* P_dev, uint64_t NT, uint64_t* p_off, uint64_t* c_off) {
+  const uint32_t o = blockIdx.x * blockDim.x + threadIdx.x;
+  if (o > K) return;
+  const uint64_t g = t_off[o];
+  p_off[o] = g < U ? post_off[g] : (uint64_t)*P_dev;
+  c_off[o] = g < U ? cstart[g] : NT;
+}
+
+// owner side: the records of source s's terms (xid order = the order s sent them): termID from the
+// owner's dictionary, start = base + exclusive prefix of df, df, cf
+__global__ void k_recv_records(const uint32_t* syn_slot, uint32_t n, const Slot* table, const uint32_t* slot_uid,
+                               const uint32_t* u_tid, const uint32_t* hdf, const uint32_t* hcf, const uint64_t* dprefix,
+                               uint64_t base, uint32_t* rec_tid, uint64_t* rec_start, uint32_t* rec_df,
+                               uint32_t* rec_cf) {
+  const uint32_t x = blockIdx.x * blockDim.x + threadIdx.x;
+  if (x >= n) return;
+  const uint32_t sl = syn_slot[x] & kXidMask;
+  rec_tid[x] = u_tid[slot_uid[sl]];
+  rec_start[x] = base + dprefix[x];
+  rec_df[x] = hdf[x];
+  rec_cf[x] = hcf[x];
 }
 
 }  // namespace wj

@@ -1,6 +1,8 @@
 // Engine + C ABI (include/wjindex.h): owns device state, orders the kernels of one chunk and of
 // finalize on the context stream, and turns CUDA errors into wj_status codes.
 #include <algorithm>
+#include <chrono>
+#include <map>
 #include <cstring>
 #include <new>
 #include <string>
@@ -32,6 +34,56 @@ struct StatusError {
 struct DevBuf {
   void* p = nullptr;
   size_t cap = 0;  // bytes
+};
+
+// Caller-owned device workspace (wj_config.workspace, e.g. a torch tensor): the library sub-allocates
+// every device buffer from it, first fit with coalescing of freed neighbours, 256-byte granules.
+struct Arena {
+  uintptr_t base = 0;
+  uint64_t bytes = 0;
+  std::map<uint64_t, uint64_t> free_;  // offset -> size
+  std::map<uint64_t, uint64_t> used_;  // offset -> size
+  void init(void* p, uint64_t n) {
+    const uintptr_t a = ((uintptr_t)p + 255) & ~(uintptr_t)255;
+    base = a;
+    bytes = n > (a - (uintptr_t)p) ? (n - (a - (uintptr_t)p)) & ~(uint64_t)255 : 0;
+    free_.clear();
+    used_.clear();
+    if (bytes) free_[0] = bytes;
+  }
+  void* alloc(uint64_t n) {
+    n = (n + 255) & ~(uint64_t)255;
+    for (auto it = free_.begin(); it != free_.end(); ++it) {
+      if (it->second < n) continue;
+      const uint64_t off = it->first, sz = it->second;
+      free_.erase(it);
+      if (sz > n) free_[off + n] = sz - n;
+      used_[off] = n;
+      return (void*)(base + off);
+    }
+    return nullptr;
+  }
+  void release(void* p) {
+    const uint64_t off = (uint64_t)((uintptr_t)p - base);
+    auto u = used_.find(off);
+    if (u == used_.end()) return;
+    uint64_t o = off, n = u->second;
+    used_.erase(u);
+    auto nx = free_.lower_bound(o);
+    if (nx != free_.end() && nx->first == o + n) {
+      n += nx->second;
+      nx = free_.erase(nx);
+    }
+    if (nx != free_.begin()) {
+      auto pv = std::prev(nx);
+      if (pv->first + pv->second == o) {
+        o = pv->first;
+        n += pv->second;
+        free_.erase(pv);
+      }
+    }
+    free_[o] = n;
+  }
 };
 
 struct PhaseRec {
@@ -159,8 +211,8 @@ struct wj_index {
   uint64_t arena_used = 0;
   uint64_t table_est = 0;
   uint64_t table_retries = 0;  // chunk-table probe overflows retried with a larger table (cumulative)
-  // chunk table capacity = table_pct% of the expected unique terms (WJ_TABLE_PCT), any multiple of
-  // 4096 slots (mulhi indexing).  On config 2 the emit kernel gets faster with capacity (2.82 / 2.45 /
+  // chunk table capacity = table_pct% of the expected unique terms, any multiple of 4096 slots
+  // (mulhi indexing).  On config 2 the emit kernel gets faster with capacity (2.82 / 2.45 /
   // 2.36 ms at 125 / 190 / 320%: shorter probe runs) while the slot -> rank gather of the first sort
   // pass and the slot scans get slower; 190-230% was the best step time (profiles/r01_README.md)
   uint64_t table_pct = 200;
@@ -172,10 +224,10 @@ struct wj_index {
   uint64_t exchange_bytes = 0;
 
   Transport* xport = nullptr;  // world > 1
-  // sampled hot terms of the current chunk (hot.cuh)
-  DevBuf hot_tab, hot_tfb, hot_slotb, hot_kb, hot_offb, samp_off, samp_slot, samp_doc, samp_cnt, samp_ck, samp_cv,
+  // sampled hot terms of the current chunk (hot.cuh): hot_slotb = hot id -> chunk-table slot
+  DevBuf hot_samp, hot_slotb, hot_kb, samp_off, samp_slot, samp_doc, samp_cnt, samp_ck, samp_cv,
       samp_ck2, samp_cv2, samp_n;
-  uint32_t hot_H = 0, hot_D = 0;
+  uint32_t hot_H = 0;
   bool stream_has_hot = false;  // some chunk appended hot-term elements (holes + counts > 1)
   // Partial postings per chunk (partials.cuh; single GPU, no stemming / stop words / hot terms): the
   // chunk's stream is sorted by slot and run-length encoded on side_st while the dictionary update
@@ -189,18 +241,21 @@ struct wj_index {
       cf_totb;
   uint64_t pbase = 0, nrec = 0;      // partial postings / records of the chunks so far
   uint32_t rs_ctas = kRsCtas;        // radix downsweep CTAs (ranges) of sort_pairs
-  uint32_t side_ctas = kRsCtas;      // ... for the side stream's sort (WJ_SIDE_CTAS): fewer leave SMs to st
+  uint32_t side_ctas = kRsCtas;      // ... for the side stream's sort (148 / 222 measured slower)
   bool pc_pending = false;           // the last chunk's posting count is still on the device (dscal[13])
   bool pc_join = false;              // the last chunk's side-stream work is not joined yet
   uint64_t pc_U = 0, pc_Nc = 0;
   std::vector<uint64_t> rec_end;     // end of each chunk's records
   uint64_t sorted_elems = 0;    // stream elements the last finalize sorted (after hole compaction)
-  // Sampled hot-term path (hot.cuh) is opt-in: on config 2 it removes ~30% of the
-  // stream elements but its per-document counters cost more global atomics in the emit kernel than
-  // the sort saves (profiles/r01_README.md).  WJ_HOT_MIN_BYTES=<bytes> enables it for larger chunks.
+  // Sampled hot terms (hot.cuh) merged per document in the emit kernel: opt-in
+  // (WJ_FLAG_HOT_TERMS, every chunk of >= 64 KiB); measured slower on config 2 (profiles/r02_README.md)
   uint64_t hot_min_bytes = ~0ull;
+  uint64_t hot_elems_saved = 0;  // stream elements merged away by the hot-term aggregation (cumulative)
+  uint64_t pm_merged = 0;        // ... of this index on the partials path (its stream_elems exclude them)
   DevBuf x_owner, x_iota, x_sorted, x_sorted2, x_owner2, x_xid, x_cnt, x_toff, x_boff, x_send, x_tkey, x_tidx, x_tkey2,
-      x_tidx2, x_rkey, x_rdoc, x_keymap, x_recv_terms, x_recv_key, x_recv_doc, x_loc_slot, x_loc_doc, x_syn_slot, x_syn_doc, x_syn_off, x_roff, x_tbase;
+      x_tidx2, x_rkey, x_rdoc, x_keymap, x_recv_terms, x_recv_key, x_recv_doc, x_loc_slot, x_loc_doc, x_syn_slot, x_syn_doc, x_syn_off, x_roff, x_tbase,
+      x_hdf, x_hcf, x_rhdf, x_rhcf, x_rpre, x_bnd;
+  double exchange_ms = 0;  // host wall time inside the all-to-all-v calls (cumulative)
   // persistent dictionary
   DevBuf nodes, coll_root, coll_n, coll_base, coll_base2, e_tid, e_bkt, e_tid2, e_bkt2, arena, t_arena, t_cache,
       t_bucket;
@@ -243,20 +298,39 @@ struct wj_index {
   size_t device_bytes = 0;
 
   // ---------------------------------------------------------------- memory
+  bool use_arena = false;  // wj_config.workspace given: every device buffer comes from it
+  Arena arena_ws;
+  void* dev_alloc(size_t n) {
+    if (use_arena) {
+      void* p = arena_ws.alloc(n);
+      if (!p) throw StatusError{WJ_ERR_OOM, "workspace exhausted (" + std::to_string(n) + " more bytes needed)"};
+      return p;
+    }
+    void* p = nullptr;
+    cudaError_t e = cudaMalloc(&p, n);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      throw StatusError{WJ_ERR_OOM, "cudaMalloc(" + std::to_string(n) + ") failed: " + cudaGetErrorString(e)};
+    }
+    return p;
+  }
+  void dev_free(void* p) {
+    if (!p) return;
+    if (use_arena) arena_ws.release(p);
+    else cudaFree(p);
+  }
   void* grow(DevBuf& b, size_t bytes, bool keep = false, size_t keep_bytes = 0) {
     if (bytes <= b.cap && b.p) return b.p;
     size_t nc = std::max(bytes, b.cap + b.cap / 2);
     nc = (nc + 255) & ~(size_t)255;
-    void* np = nullptr;
-    cudaError_t e = cudaMalloc(&np, nc);
-    if (e != cudaSuccess) {
-      cudaGetLastError();
-      throw StatusError{WJ_ERR_OOM, "cudaMalloc(" + std::to_string(nc) + ") failed: " + cudaGetErrorString(e)};
-    }
+    void* np = dev_alloc(nc);
     if (keep && b.p && keep_bytes) WJ_CUDA_CHECK(cudaMemcpyAsync(np, b.p, keep_bytes, cudaMemcpyDeviceToDevice, st));
     if (b.p) {
+      // other streams (side / dictionary) may still read the old buffer: wait for the device
       WJ_CUDA_CHECK(cudaStreamSynchronize(st));
-      WJ_CUDA_CHECK(cudaFree(b.p));
+      if (side_st) WJ_CUDA_CHECK(cudaStreamSynchronize(side_st));
+      if (hp_st) WJ_CUDA_CHECK(cudaStreamSynchronize(hp_st));
+      dev_free(b.p);
       device_bytes -= b.cap;
     }
     b.p = np;
@@ -283,23 +357,24 @@ struct wj_index {
                      &pc_cs, &u_slot, &pp_doc, &pp_tf, &rec_tid, &rec_start, &rec_df, &rec_cf, &rec_before, &df_totb,
                      &cf_totb};
     for (DevBuf* b : all) {
-      if (b->p) cudaFree(b->p);
+      dev_free(b->p);
       b->p = nullptr;
       b->cap = 0;
     }
-    DevBuf* hs[] = {&hot_tab, &hot_tfb, &hot_slotb, &hot_kb, &hot_offb, &samp_off, &samp_slot, &samp_doc, &samp_cnt,
+    DevBuf* hs[] = {&hot_samp, &hot_slotb, &hot_kb, &samp_off, &samp_slot, &samp_doc, &samp_cnt,
                     &samp_ck, &samp_cv, &samp_ck2, &samp_cv2, &samp_n};
-    for (DevBuf* b : hs) { if (b->p) cudaFree(b->p); *b = DevBuf{}; }
+    for (DevBuf* b : hs) { dev_free(b->p); *b = DevBuf{}; }
     DevBuf* xs[] = {&x_owner, &x_iota, &x_sorted, &x_sorted2, &x_owner2, &x_xid, &x_cnt, &x_toff, &x_boff, &x_send,
                     &x_tkey, &x_tidx, &x_tkey2, &x_tidx2, &x_rkey, &x_rdoc, &x_keymap, &x_recv_terms, &x_recv_key, &x_recv_doc, &x_loc_slot,
-                    &x_loc_doc, &x_syn_slot, &x_syn_doc, &x_syn_off, &x_roff, &x_tbase};
-    for (DevBuf* b : xs) { if (b->p) cudaFree(b->p); *b = DevBuf{}; }
-    for (auto& b : chunk_map) if (b.p) cudaFree(b.p);
+                    &x_loc_doc, &x_syn_slot, &x_syn_doc, &x_syn_off, &x_roff, &x_tbase, &x_hdf, &x_hcf, &x_rhdf,
+                    &x_rhcf, &x_rpre, &x_bnd};
+    for (DevBuf* b : xs) { dev_free(b->p); *b = DevBuf{}; }
+    for (auto& b : chunk_map) dev_free(b.p);
     chunk_map.clear();
-    for (DevBuf* b : {&rle_look, &rle_p0, &rle_lead, &rle_tok, &cstart_b}) { if (b->p) cudaFree(b->p); *b = DevBuf{}; }
+    for (DevBuf* b : {&rle_look, &rle_p0, &rle_lead, &rle_tok, &cstart_b}) { dev_free(b->p); *b = DevBuf{}; }
     for (int i = 0; i < 4; ++i) {
-      if (lvA[i].p) cudaFree(lvA[i].p);
-      if (lvB[i].p) cudaFree(lvB[i].p);
+      dev_free(lvA[i].p);
+      dev_free(lvB[i].p);
       lvA[i] = DevBuf{};
       lvB[i] = DevBuf{};
     }
@@ -400,6 +475,7 @@ struct wj_index {
     stream_has_hot = false;
     sorted_elems = 0;
     pbase = nrec = 0;
+    pm_merged = 0;
     pc_pending = pc_join = false;
     rec_end.clear();
     unique_last = new_last = n_nodes = height_max = 0;
@@ -492,10 +568,7 @@ struct wj_index {
     if (clear_table) WJ_CUDA_CHECK(cudaMemsetAsync(tab, 0, C * sizeof(Slot), st));
     WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 5, 0, 8, st));
     EmitOut eo;
-    eo.hot = (use_hot && hot_H) ? (const HotEntry*)hot_tab.p : nullptr;
-    eo.hot_mask = kHotTable - 1;
-    eo.hot_docs = hot_D;
-    eo.hot_tf = (uint32_t*)hot_tfb.p;
+    eo.hot_slot = (use_hot && hot_H) ? (const uint32_t*)hot_slotb.p : nullptr;
     eo.table = tab;
     eo.slot_ref = sref;
     eo.cap = (uint32_t)C;
@@ -506,10 +579,16 @@ struct wj_index {
     eo.dbg_len = dlen;
     eo.overflow = (uint32_t*)(dscal() + 5);
     const uint64_t ranges = (n_segs + kSegsPerWarp - 1) / kSegsPerWarp;
-    const unsigned grid = (unsigned)((ranges + kTokWarps - 1) / kTokWarps);
+    const uint32_t sub = eo.hot_slot ? emit_sub<true>() : emit_sub<false>();
+    const uint64_t warps = (ranges + sub - 1) / sub;  // a warp walks `sub` ranges
+    const unsigned grid = (unsigned)((warps + kTokWarps - 1) / kTokWarps);
     ktime(WJ_KERNEL_TOKENIZE_EMIT, [&] {
-      k_tok_emit<<<grid, kTokThreads, 0, st>>>(cv, (uint32_t)n_segs, (const uint64_t*)kstart.p,
-                                               (const uint32_t*)seg_cnt.p, eo);
+      if (eo.hot_slot)
+        k_tok_emit<true><<<grid, kTokThreads, 0, st>>>(cv, (uint32_t)n_segs, (const uint64_t*)kstart.p,
+                                                       (const uint32_t*)seg_cnt.p, eo);
+      else
+        k_tok_emit<false><<<grid, kTokThreads, 0, st>>>(cv, (uint32_t)n_segs, (const uint64_t*)kstart.p,
+                                                        (const uint32_t*)seg_cnt.p, eo);
       launched();
     });
   }
@@ -608,12 +687,13 @@ struct wj_index {
       if (tk[i] >= kHotMinCount) hot_slots.push_back(tv[i]);
     const uint32_t H = (uint32_t)hot_slots.size();
     if (H == 0) return 0;
-    uint32_t* hs = buf<uint32_t>(hot_slotb, kHotMax);
+    uint32_t* hs = buf<uint32_t>(hot_samp, kHotMax);
     WJ_CUDA_CHECK(cudaMemcpyAsync(hs, hot_slots.data(), H * 4, cudaMemcpyHostToDevice, st));
     ulonglong2* hk = (ulonglong2*)grow(hot_kb, kHotMax * sizeof(ulonglong2));
     k_hot_extract<<<1, kHotMax, 0, st>>>((const Slot*)table.p, hs, H, hk);
     launched();
-    sync();  // hot_slot_b is rewritten with main-table slots by k_hot_build
+    buf<uint32_t>(hot_slotb, kHotMax + 1);  // written by k_hot_seed
+    sync();  // hot_slots (host) is read by the copy above
     return H;
   }
 
@@ -643,13 +723,8 @@ struct wj_index {
     if (!bytes && cudaCtxResetPersistingL2Cache() != cudaSuccess) cudaGetLastError();
   }
 
-  // chunk table capacity: WJ_TABLE_POW2=1 rounds to a power of two (the layout before mulhi indexing),
-  // else to a multiple of 4096 slots
-  bool table_pow2 = false;
-  uint64_t table_cap(uint64_t x) const {
-    if (table_pow2) return pow2_at_least(x);
-    return std::max<uint64_t>((x + 4095) / 4096 * 4096, 4096);
-  }
+  // chunk table capacity: a multiple of 4096 slots (mulhi indexing takes any capacity)
+  uint64_t table_cap(uint64_t x) const { return std::max<uint64_t>((x + 4095) / 4096 * 4096, 4096); }
   static uint64_t pow2_at_least(uint64_t x) {
     uint64_t c = 1;
     while (c < x) c <<= 1;
@@ -667,15 +742,7 @@ struct wj_index {
     U = 0;
     phase(WJ_PHASE_TOKENIZE);
     hot_H = 0;
-    hot_D = 0;
-    if (allow_hot && cv.n_bytes >= hot_min_bytes && cv.n_docs > 0) {
-      const uint64_t cap = 64ull << 20;  // hot x documents counters
-      if (cv.n_docs <= cap / 16) {
-        hot_H = select_hot(cv);
-        hot_H = (uint32_t)std::min<uint64_t>(hot_H, cap / cv.n_docs);
-        hot_D = (uint32_t)cv.n_docs;
-      }
-    }
+    if (allow_hot && cv.n_bytes >= hot_min_bytes && cv.n_docs > 0) hot_H = select_hot(cv);
     const uint64_t Nc = count_tokens(cv, n_segs);
     n_dropped += h_scal[1];
     out_alloc(Nc, slot_out, doc_out);
@@ -692,14 +759,11 @@ struct wj_index {
       Slot* tab = buf<Slot>(table, C);
       uint32_t* sref = buf<uint32_t>(slotref, C);
       WJ_CUDA_CHECK(cudaMemsetAsync(tab, 0, C * sizeof(Slot), st));
-      if (hot_H) {  // hot terms first: their slots in this table, and the lookup table for the emit
+      if (hot_H) {  // hot terms first: their slots in this table carry their hot ids
         WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 5, 0, 8, st));
-        HotEntry* ht = (HotEntry*)grow(hot_tab, kHotTable * sizeof(HotEntry));
-        k_hot_build<<<1, 1, 0, st>>>((const ulonglong2*)hot_kb.p, hot_H, tab, sref, (uint32_t)C, ht,
-                                     (uint32_t*)hot_slotb.p, (uint32_t*)(dscal() + 5));
+        k_hot_seed<<<1, 128, 0, st>>>((const ulonglong2*)hot_kb.p, hot_H, tab, sref, (uint32_t)C,
+                                      (uint32_t*)hot_slotb.p, (uint32_t*)(dscal() + 5));
         launched();
-        uint32_t* tf = buf<uint32_t>(hot_tfb, (uint64_t)hot_H * hot_D);
-        WJ_CUDA_CHECK(cudaMemsetAsync(tf, 0, (uint64_t)hot_H * hot_D * 4, st));
       }
       emit_tokens(cv, n_segs, slot_out, doc_out, doc_base, C, nullptr, nullptr, hot_H > 0, false);
       phase(WJ_PHASE_UNIQUE);
@@ -933,7 +997,8 @@ struct wj_index {
   // Partials mode, one chunk: the stream (pc_key, pc_doc)[Nc] of C slots, U unique terms.  Sort by slot
   // + run-length on side_st (the partial lists of the run) while the dictionary update runs on
   // st; then one record per unique term.
-  void chunk_partials(const uint8_t* text, uint64_t Nc, uint64_t C, uint64_t U) {
+  // hot: the stream holds merged hot-term elements (counts) and holes (hot.cuh)
+  void chunk_partials(const uint8_t* text, uint64_t Nc, uint64_t C, uint64_t U, bool hot) {
     settle_partials();  // the previous chunk is joined (add_chunk), its posting count read here
     uint32_t* kt = (uint32_t*)pc_key.p;
     uint32_t* dt = (uint32_t*)pc_doc.p;
@@ -951,9 +1016,13 @@ struct wj_index {
     swap_side();
     try {
       phase(WJ_PHASE_SORT);
-      const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, bits, nullptr, true);
+      // holes (merged hot tokens, key 0) are dropped by the first pass: Ns elements remain
+      uint64_t Ns = Nc;
+      const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, bits, nullptr, true, nullptr, kRankMask, hot, &Ns);
+      hot_elems_saved += Nc - Ns;
+      pm_merged += Nc - Ns;
       phase(WJ_PHASE_POSTINGS);
-      rle(in1 ? k1 : kt, in1 ? v1 : dt, Nc, false, od + pbase, of + pbase, po, cs);
+      rle(in1 ? k1 : kt, in1 ? v1 : dt, Ns, hot, od + pbase, of + pbase, po, cs);
       phase(-1);
       WJ_CUDA_CHECK(cudaEventRecord(ev_side, st));
     } catch (...) {
@@ -1068,6 +1137,11 @@ struct wj_index {
     if (pm) join_partials();  // the previous chunk's side work, before its buffers are reused
     stage(bytes, n_bytes, doc_off_in, nd, &text, &off);
     ++n_chunks;
+    if (xport && pm) {
+      add_chunk_dist_pl(text, nd ? n_bytes : 0, off, nd);
+      phase(-1);
+      return;
+    }
     if (xport) {
       add_chunk_dist(text, nd ? n_bytes : 0, off, nd);
       phase(-1);
@@ -1114,35 +1188,245 @@ struct wj_index {
         n_tokens += kept;
       }
     } else if (Nc > 0 && pm) {
-      chunk_partials(text, Nc, C, U);
+      chunk_partials(text, Nc, C, U, hot_H > 0);
       n_elems += Nc;
       n_tokens += Nc;
     } else if (Nc > 0) {
-      uint64_t NH = 0;
-      if (hot_H) {  // hot (term, document) counters -> stream elements after the chunk's tokens
-        const uint64_t HD = (uint64_t)hot_H * hot_D;
-        uint32_t* ho = buf<uint32_t>(hot_offb, HD + 1);
-        scan<uint32_t>(HotElemCount{(const uint32_t*)hot_tfb.p}, HD, ho, ho + HD);
-        uint32_t nh = 0;
-        WJ_CUDA_CHECK(cudaMemcpyAsync(&nh, ho + HD, 4, cudaMemcpyDeviceToHost, st));
-        sync();
-        NH = nh;
-        const uint64_t base = n_elems + Nc;
-        if (base + NH > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 stream elements"};
-        uint32_t* gt = buf_keep<uint32_t>(g_tid, base + NH + 16, base);
-        uint32_t* gd = buf_keep<uint32_t>(g_doc, base + NH + 16, base);
-        k_hot_elems<<<grid_for(HD, 256), 256, 0, st>>>((const uint32_t*)hot_tfb.p, HD, hot_D, ho,
-                                                       (const uint32_t*)hot_slotb.p, doc_base, gt + base, gd + base);
-        launched();
-      }
       dictionary_update(text, U);
       register_chunk_map(C, n_elems);
       if (hot_H) stream_has_hot = true;
-      n_elems += Nc + NH;
+      n_elems += Nc;
       n_tokens += Nc;
     }
     n_docs += nd;
     phase(-1);
+  }
+
+  // ---------------------------------------------------------------- one chunk, world > 1
+  // Sender-side partial lists: every rank tokenises its own documents,
+  // groups its unique terms by owner (collection b -> b mod K, or the balanced map),
+  // sorts + run-length encodes its stream by (owner, term) into (docID, tf) postings written straight
+  // into its partial-list buffer, and sends each owner its terms (folded bytes), a (df, cf) header per
+  // term and that term's postings in one all-to-all-v round.  The owner deduplicates the received
+  // terms, updates its exclusive dictionary slice and appends one partial-list record per
+  // (source, term), in source-rank order = docID order; its own postings never move.  Finalize
+  // is the single-GPU partial-list combine.
+  void add_chunk_dist_pl(const uint8_t* text, uint64_t n_bytes, const uint64_t* off, uint64_t nd) {
+    const int K = world;
+    phase(WJ_PHASE_EXCHANGE);
+    std::vector<uint64_t> ndall(K);
+    const uint64_t mine = nd;
+    xport->allgather(&mine, 1, ndall.data(), st);
+    uint64_t base = n_docs, tot_docs = 0;
+    for (int r = 0; r < K; ++r) {
+      if (r < rank) base += ndall[r];
+      tot_docs += ndall[r];
+    }
+    if (n_docs + tot_docs > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 documents"};
+    if (balanced && !owner_ready) {
+      ChunkView cv0{text, n_bytes, off, nd};
+      build_owner_map(nd > 0 && n_bytes > 0 ? &cv0 : nullptr);
+      phase(WJ_PHASE_EXCHANGE);
+    }
+    // 1. local tokenize + dedup of this rank's documents (stream into pc_key / pc_doc)
+    uint64_t C = 0, U = 0, Nc = 0;
+    uint32_t *lslot = nullptr, *ldoc = nullptr;
+    if (nd > 0 && n_bytes > 0) {
+      ChunkView cv{text, n_bytes, off, nd};
+      Nc = tokenize_dedup(cv, (uint32_t)base, [&](uint64_t nc, uint32_t*& sp, uint32_t*& dp) {
+        if (nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 tokens in one chunk"};
+        sp = buf<uint32_t>(pc_key, nc + 16);
+        dp = buf<uint32_t>(pc_doc, nc + 16);
+      }, C, U, lslot, ldoc, true);
+    }
+    const bool hot = hot_H > 0;
+    std::vector<uint64_t> t_off(K + 1, 0), b_off(K + 1, 0), p_off(K + 1, 0), c_off(K + 1, 0);
+    uint8_t* send_terms = (uint8_t*)grow(x_send, 16);
+    uint64_t P_local = 0;
+    // the chunk's postings: K == 1 straight into the partial-list buffer; K > 1 into scratch, from where
+    // every owner's range (the own one by a device copy) lands in the owners' partial-list buffers in
+    // source-rank order, so each chunk's partial lists are back to back in record order
+    uint32_t *od = nullptr, *of = nullptr;
+    if (K == 1) {
+      od = buf_keep<uint32_t>(pp_doc, pbase + Nc + 16, pbase) + pbase;
+      of = buf_keep<uint32_t>(pp_tf, pbase + Nc + 16, pbase) + pbase;
+    } else {
+      od = buf<uint32_t>(x_rkey, Nc + 16);
+      of = buf<uint32_t>(x_rdoc, Nc + 16);
+    }
+    if (U > 0) {
+      // 2. unique terms grouped by owner (stable): t_off, xid, gpos map, packed term bytes
+      uint32_t* own = buf<uint32_t>(x_owner, U + 16);
+      uint32_t* iota = buf<uint32_t>(x_iota, U + 16);
+      uint32_t* own2 = buf<uint32_t>(x_owner2, U + 16);
+      uint32_t* srt2 = buf<uint32_t>(x_sorted2, U + 16);
+      uint32_t* oc = buf<uint32_t>(x_cnt, 2 * K);
+      WJ_CUDA_CHECK(cudaMemsetAsync(oc, 0, 2 * K * 4, st));
+      k_owner<<<grid_for(U, 256), 256, 0, st>>>((const uint32_t*)u_bucket.p, (uint32_t)U, (uint32_t)K,
+                                                owner_ready ? (const uint32_t*)owner_tab.p : nullptr, own, iota, oc);
+      launched();
+      const uint32_t* sorted_u = iota;
+      if (K > 1) {
+        WJ_CUDA_CHECK(cudaMemcpyAsync(own2, own, U * 4, cudaMemcpyDeviceToDevice, st));
+        int obits = 0;
+        while ((1 << obits) < K) ++obits;
+        uint32_t* srt1 = (uint32_t*)grow(x_sorted, (U + 16) * 4);
+        sorted_u = sort_pairs<uint32_t>(own2, iota, srt1, srt2, U, 0, obits, nullptr, false) ? srt2 : iota;
+      }
+      std::vector<uint32_t> oc_h(K);
+      WJ_CUDA_CHECK(cudaMemcpyAsync(oc_h.data(), oc, K * 4, cudaMemcpyDeviceToHost, st));
+      sync();
+      for (int o = 0; o < K; ++o) t_off[o + 1] = t_off[o] + oc_h[o];
+      uint64_t* toff_d = buf<uint64_t>(x_toff, K + 1);
+      WJ_CUDA_CHECK(cudaMemcpyAsync(toff_d, t_off.data(), (K + 1) * 8, cudaMemcpyHostToDevice, st));
+      uint32_t* xid = buf<uint32_t>(x_xid, U);
+      k_xid<<<grid_for(U, 256), 256, 0, st>>>(sorted_u, (uint32_t)U, own, toff_d, xid);
+      launched();
+      uint32_t* km = buf<uint32_t>(x_keymap, C);
+      k_slot_gpos<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, (uint32_t)C, (const uint32_t*)uid.p, own, xid,
+                                                    toff_d, km);
+      launched();
+      uint64_t* boff = buf<uint64_t>(x_boff, U + 1);
+      scan<uint64_t>(PackTermSize{sorted_u, (const uint32_t*)u_len.p}, U, boff, boff + U);
+      // 3. the stream sorted by gpos (map applied by the first pass; holes of merged hot tokens dropped),
+      //    run-length encoded into this rank's partial-list buffer
+      int bits = 0;
+      while (bits < 32 && ((uint64_t)1 << bits) < U) ++bits;
+      uint32_t* kt = (uint32_t*)pc_key.p;
+      uint32_t* dt = (uint32_t*)pc_doc.p;
+      uint32_t* k1 = buf<uint32_t>(sk1, Nc + 16);
+      uint32_t* v1 = buf<uint32_t>(sv1, Nc + 16);
+      uint64_t* po = buf<uint64_t>(pc_po, U + 1);
+      uint64_t* cs = buf<uint64_t>(pc_cs, U + 1);
+      phase(WJ_PHASE_SORT);
+      std::vector<std::pair<uint64_t, const uint32_t*>> segs{{0, km}};
+      uint64_t Ns = Nc;
+      bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, std::max(bits, 1), nullptr, true, &segs, kRankMask, hot,
+                                      &Ns);
+      hot_elems_saved += Nc - Ns;
+      phase(WJ_PHASE_POSTINGS);
+      rle(in1 ? k1 : kt, in1 ? v1 : dt, Ns, hot, od, of, po, cs);
+      phase(WJ_PHASE_EXCHANGE);
+      uint32_t* hdf = buf<uint32_t>(x_hdf, U);
+      uint32_t* hcf = buf<uint32_t>(x_hcf, U);
+      k_term_hdr<<<grid_for(U, 256), 256, 0, st>>>(po, cs, (uint32_t)U, (const uint32_t*)(dscal() + 8), Nc, hdf, hcf);
+      launched();
+      uint64_t* bnd = buf<uint64_t>(x_bnd, 2 * (K + 1));
+      k_owner_bounds<<<grid_for(K + 1, 256), 256, 0, st>>>(po, cs, toff_d, (uint32_t)K, (uint32_t)U,
+                                                          (const uint32_t*)(dscal() + 8), Nc, bnd, bnd + K + 1);
+      launched();
+      std::vector<uint64_t> hb(2 * (K + 1));
+      WJ_CUDA_CHECK(cudaMemcpyAsync(hb.data(), bnd, hb.size() * 8, cudaMemcpyDeviceToHost, st));
+      for (int o = 0; o <= K; ++o)
+        WJ_CUDA_CHECK(cudaMemcpyAsync(&b_off[o], boff + t_off[o], 8, cudaMemcpyDeviceToHost, st));
+      sync();
+      for (int o = 0; o <= K; ++o) {
+        p_off[o] = hb[o];
+        c_off[o] = hb[K + 1 + o];
+      }
+      P_local = p_off[K];
+      send_terms = (uint8_t*)grow(x_send, b_off[K] + 16);
+      k_pack_terms<<<grid_for(U, 256), 256, 0, st>>>(sorted_u, (uint32_t)U, boff, (const uint4*)u_w.p, text,
+                                                    (const uint32_t*)u_ref.p, (const uint32_t*)u_len.p, send_terms);
+      launched();
+    }
+    // 4. exchange: per owner [terms, term bytes, postings, tokens]; then the term bytes, the headers and
+    //    the postings (own postings stay in place: zero-size self segment)
+    std::vector<uint64_t> cnt(4 * K, 0), all(4 * K * K);
+    for (int o = 0; o < K; ++o) {
+      cnt[o] = t_off[o + 1] - t_off[o];
+      cnt[K + o] = b_off[o + 1] - b_off[o];
+      cnt[2 * K + o] = p_off[o + 1] - p_off[o];
+      cnt[3 * K + o] = c_off[o + 1] - c_off[o];
+    }
+    xport->allgather(cnt.data(), 4 * K, all.data(), st);
+    std::vector<uint64_t> rt(K + 1, 0), rb(K + 1, 0), rp(K + 1, 0);
+    uint64_t my_tokens = 0;
+    for (int s = 0; s < K; ++s) {
+      const uint64_t* c = all.data() + (size_t)s * 4 * K;
+      rt[s + 1] = rt[s] + c[rank];
+      rb[s + 1] = rb[s] + c[K + rank];
+      rp[s + 1] = rp[s] + c[2 * K + rank];
+      my_tokens += c[3 * K + rank];
+    }
+    const uint64_t RT = rt[K], RP = rp[K];  // RP: postings of this owner's terms over all sources
+    uint8_t* recv_terms = (uint8_t*)grow(x_recv_terms, rb[K] + 32);
+    uint32_t* rhdf = buf<uint32_t>(x_rhdf, RT + 1);
+    uint32_t* rhcf = buf<uint32_t>(x_rhcf, RT + 1);
+    uint32_t* hdf = buf<uint32_t>(x_hdf, std::max<uint64_t>(U, 1));
+    uint32_t* hcf = buf<uint32_t>(x_hcf, std::max<uint64_t>(U, 1));
+    std::vector<uint64_t> s4(K + 1), r4(K + 1), rpb(K + 1);
+    for (int o = 0; o <= K; ++o) {
+      s4[o] = t_off[o] * 4;
+      r4[o] = rt[o] * 4;
+    }
+    const uint64_t t0 = xport->sent;
+    {
+      const auto tx = std::chrono::steady_clock::now();
+      try {
+        xport->alltoallv(send_terms, b_off.data(), recv_terms, rb.data(), st);
+        xport->alltoallv(hdf, s4.data(), rhdf, r4.data(), st);
+        xport->alltoallv(hcf, s4.data(), rhcf, r4.data(), st);
+        if (K > 1) {  // postings: owner o's range of the scratch -> o's partial-list buffer
+          uint32_t* pd = buf_keep<uint32_t>(pp_doc, pbase + RP + 16, pbase) + pbase;
+          uint32_t* pt = buf_keep<uint32_t>(pp_tf, pbase + RP + 16, pbase) + pbase;
+          std::vector<uint64_t> spb(K + 1);
+          for (int o = 0; o <= K; ++o) {
+            spb[o] = p_off[o] * 4;
+            rpb[o] = rp[o] * 4;
+          }
+          xport->alltoallv(od, spb.data(), pd, rpb.data(), st);
+          xport->alltoallv(of, spb.data(), pt, rpb.data(), st);
+        }
+      } catch (const ExchangeError& e) {
+        throw StatusError{WJ_ERR_NCCL, e.msg};
+      }
+      WJ_CUDA_CHECK(cudaStreamSynchronize(st));
+      exchange_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - tx).count();
+    }
+    exchange_bytes += xport->sent - t0;
+    // 5. owner side: the received terms through the tokenizer / dedup / dictionary, then one record
+    //    per (source, term) in source-rank order
+    if (RT > 0) {
+      uint64_t* so = buf<uint64_t>(x_syn_off, 2);
+      const uint64_t h2[2] = {0, rb[K]};
+      WJ_CUDA_CHECK(cudaMemcpyAsync(so, h2, 16, cudaMemcpyHostToDevice, st));
+      ChunkView sv{recv_terms, rb[K], so, 1};
+      uint64_t C2 = 0, U2 = 0;
+      uint32_t *sslot = nullptr, *sdoc = nullptr;
+      const uint64_t dropped0 = n_dropped;
+      const uint64_t Ns2 = tokenize_dedup(sv, 0, [&](uint64_t nc, uint32_t*& sp2, uint32_t*& dp2) {
+        sp2 = buf<uint32_t>(x_syn_slot, nc + 16);
+        dp2 = buf<uint32_t>(x_syn_doc, nc + 16);
+      }, C2, U2, sslot, sdoc);
+      n_dropped = dropped0;
+      if (Ns2 != RT) throw StatusError{WJ_ERR_CUDA, "received term text: token count mismatch (internal)"};
+      dictionary_update(recv_terms, U2);
+      phase(WJ_PHASE_STREAM);
+      uint64_t* pre = buf<uint64_t>(x_rpre, RT + 1);
+      uint32_t* rtid = buf_keep<uint32_t>(rec_tid, nrec + RT, nrec);
+      uint64_t* rst = buf_keep<uint64_t>(rec_start, nrec + RT, nrec);
+      uint32_t* rdf = buf_keep<uint32_t>(rec_df, nrec + RT, nrec);
+      uint32_t* rcf = buf_keep<uint32_t>(rec_cf, nrec + RT, nrec);
+      for (int s = 0; s < K; ++s) {
+        const uint64_t nt = rt[s + 1] - rt[s];
+        if (nt == 0) continue;
+        scan<uint64_t>(U32AsU64{rhdf + rt[s]}, nt, pre + rt[s], (uint64_t*)nullptr);
+        const uint64_t pb = pbase + rp[s];
+        k_recv_records<<<grid_for(nt, 256), 256, 0, st>>>(sslot + rt[s], (uint32_t)nt, (const Slot*)table.p,
+                                                          (const uint32_t*)uid.p, (const uint32_t*)u_tid.p, rhdf + rt[s],
+                                                          rhcf + rt[s], pre + rt[s], pb, rtid + nrec + rt[s],
+                                                          rst + nrec + rt[s], rdf + nrec + rt[s], rcf + nrec + rt[s]);
+        launched();
+        rec_end.push_back(nrec + rt[s + 1]);
+      }
+      nrec += RT;
+    }
+    pbase += RP;
+    n_tokens += my_tokens;
+    n_elems += Nc;
+    n_docs += tot_docs;
+    sync();  // exchange buffers are reused by the next chunk
   }
 
   // ---------------------------------------------------------------- one chunk, world > 1
@@ -1295,9 +1579,8 @@ struct wj_index {
     // registered below, so no per-record translation pass is needed
     const uint64_t R = rr_off[K];
     if (n_elems + R > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 stream elements"};
-    // partials path (pm): the records land in the chunk stream buffers of the per-run partial lists
-    uint32_t* recv_key = pm ? buf<uint32_t>(pc_key, R + 16) : buf_keep<uint32_t>(g_tid, n_elems + R + 16, n_elems) + n_elems;
-    uint32_t* recv_doc = pm ? buf<uint32_t>(pc_doc, R + 16) : buf_keep<uint32_t>(g_doc, n_elems + R + 16, n_elems) + n_elems;
+    uint32_t* recv_key = buf_keep<uint32_t>(g_tid, n_elems + R + 16, n_elems) + n_elems;
+    uint32_t* recv_doc = buf_keep<uint32_t>(g_doc, n_elems + R + 16, n_elems) + n_elems;
     std::vector<uint64_t> rec_soff(K + 1), rec_roff(K + 1);
     for (int o = 0; o <= K; ++o) { rec_soff[o] = r_off[o] * 4; rec_roff[o] = rr_off[o] * 4; }
     const uint64_t t0 = xport->sent;
@@ -1324,22 +1607,6 @@ struct wj_index {
       }, C2, U2, sslot, sdoc);
       n_dropped = dropped0;
       if (Ns != rt_off[K]) throw StatusError{WJ_ERR_CUDA, "received term text: token count mismatch (internal)"};
-      if (pm) {  // records -> owner chunk-table stream elements; sort by slot beside the dictionary update
-        phase(WJ_PHASE_STREAM);
-        for (int src = 0; src < K; ++src) {
-          const uint64_t nr = rr_off[src + 1] - rr_off[src];
-          if (nr == 0) continue;
-          k_xid_to_slot<<<grid_for(nr, 256), 256, 0, st>>>(recv_key + rr_off[src], nr, sslot + rt_off[src]);
-          launched();
-        }
-        phase(-1);
-        if (R > 0) chunk_partials(recv_terms, R, C2, U2);
-        n_elems += R;
-        n_tokens += R;
-        n_docs += tot_docs;
-        sync();  // exchange buffers are reused by the next chunk
-        return;
-      }
       dictionary_update(recv_terms, U2);
       phase(WJ_PHASE_STREAM);
       // source s's records: key & kRankMask = xid = index into the terms s sent; map xid -> termID
@@ -1618,7 +1885,7 @@ struct wj_index {
       // postings: they run on the side stream (idle once the last chunk is joined) meanwhile.
       join_partials();
       settle_partials();
-      sorted_elems = n_elems;
+      sorted_elems = n_elems - pm_merged;
       phase(-1);
       WJ_CUDA_CHECK(cudaEventRecord(ev_fork, st));  // ranks (k_lexrank) are ready in st order
       bool dict_started = false;
@@ -1857,7 +2124,7 @@ extern "C" {
 int index_init(wj_index** out, const wj_config* cfg) {
   if (!out || !cfg) return WJ_ERR_INVALID_ARG;
   *out = nullptr;
-  if (cfg->world < 1 || cfg->world > 1024 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~(WJ_FLAG_PROFILE | WJ_FLAG_LOOPBACK | WJ_FLAG_VBYTE | WJ_FLAG_HOST_PIPELINE | WJ_FLAG_BALANCED_OWNERS | WJ_FLAG_STEM | WJ_FLAG_STOPWORDS)) || cfg->reserved) {
+  if (cfg->world < 1 || cfg->world > 1024 || cfg->rank < 0 || cfg->rank >= cfg->world || (cfg->flags & ~(WJ_FLAG_PROFILE | WJ_FLAG_LOOPBACK | WJ_FLAG_VBYTE | WJ_FLAG_HOST_PIPELINE | WJ_FLAG_BALANCED_OWNERS | WJ_FLAG_STEM | WJ_FLAG_STOPWORDS | WJ_FLAG_HOT_TERMS | WJ_FLAG_GLOBAL_STREAM)) || cfg->reserved) {
     g_init_err = "invalid config";
     return WJ_ERR_INVALID_ARG;
   }
@@ -1886,6 +2153,10 @@ int index_init(wj_index** out, const wj_config* cfg) {
   ix->balanced = (cfg->flags & WJ_FLAG_BALANCED_OWNERS) != 0;
   ix->stem_on = (cfg->flags & WJ_FLAG_STEM) != 0;
   ix->stop_on = (cfg->flags & WJ_FLAG_STOPWORDS) != 0;
+  if (cfg->workspace) {
+    ix->use_arena = true;
+    ix->arena_ws.init(cfg->workspace, cfg->workspace_bytes);
+  }
   int rc = guarded(ix, [&]() {
     if (cfg->stream) {
       ix->st = (cudaStream_t)cfg->stream;
@@ -1901,19 +2172,11 @@ int index_init(wj_index** out, const wj_config* cfg) {
         WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->pipe_done[i], cudaEventDisableTiming));
       }
     }
-    // per-run partial lists on one GPU; the distributed path (a transport: world > 1, or a
-    // communicator at world 1) keeps the global stream unless WJ_DIST_PARTIALS=1 (owner-side partial
-    // lists, parity-green but 11.53 -> 11.86-11.92 ms/step at K = 1 on config 2: the dictionary
-    // update it overlaps is ~1.2 ms there, less than the partial-list combine costs; profiles/r01_README.md)
+    // per-run partial lists (one GPU) / sender-side partial lists (a transport: world > 1, or a
+    // communicator at world 1); stemming / stop words and WJ_FLAG_GLOBAL_STREAM sort one global stream
     ix->pm = !ix->stem_on && !ix->stop_on;
-    if (ix->world > 1 || cfg->nccl_unique_id) {
-      const char* e = getenv("WJ_DIST_PARTIALS");
-      ix->pm = ix->pm && e && strtoull(e, nullptr, 10) != 0;
-    }
-    if (const char* e = getenv("WJ_PARTIALS")) ix->pm = ix->pm && strtoull(e, nullptr, 10) != 0;
-    if (const char* e = getenv("WJ_HOT_MIN_BYTES")) ix->hot_min_bytes = strtoull(e, nullptr, 10);
-    if (ix->hot_min_bytes != ~0ull) ix->pm = false;  // hot-term elements need the global stream
-    if (const char* e = getenv("WJ_SIDE_CTAS")) ix->side_ctas = std::max<uint32_t>((uint32_t)strtoul(e, nullptr, 10), 1);
+    if (cfg->flags & WJ_FLAG_GLOBAL_STREAM) ix->pm = false;
+    if (cfg->flags & WJ_FLAG_HOT_TERMS) ix->hot_min_bytes = 64ull << 10;
     if (ix->pm) {
       int least = 0, greatest = 0;
       WJ_CUDA_CHECK(cudaDeviceGetStreamPriorityRange(&least, &greatest));
@@ -1923,8 +2186,6 @@ int index_init(wj_index** out, const wj_config* cfg) {
       WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->ev_side, cudaEventDisableTiming));
       WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->ev_dict, cudaEventDisableTiming));
     }
-    if (const char* e = getenv("WJ_TABLE_POW2")) ix->table_pow2 = strtoull(e, nullptr, 10) != 0;
-    if (const char* e = getenv("WJ_TABLE_PCT")) ix->table_pct = std::max<uint64_t>(strtoull(e, nullptr, 10), 110);
     if (cfg->world > 1 || cfg->nccl_unique_id) {  // a transport at world 1 runs the same distributed path
       try {
         if (cfg->flags & WJ_FLAG_LOOPBACK)
@@ -1942,9 +2203,6 @@ int index_init(wj_index** out, const wj_config* cfg) {
     WJ_DS_ATTR(uint64_t, true, true); WJ_DS_ATTR(uint32_t, false, false); WJ_DS_ATTR(uint32_t, true, false);
     WJ_DS_ATTR(uint32_t, false, true); WJ_DS_ATTR(uint32_t, true, true);
 #undef WJ_DS_ATTR
-    if (const char* e = getenv("WJ_EMIT_CARVEOUT"))
-      WJ_CUDA_CHECK(cudaFuncSetAttribute(k_tok_emit, cudaFuncAttributePreferredSharedMemoryCarveout,
-                                         (int)strtol(e, nullptr, 10)));
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rle_write_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)rle_smem_bytes()));
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rle_write_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -2053,8 +2311,10 @@ int index_stats(wj_index* ix, wj_stats* out) {
     out->btree_height_max = ix->height_max;
     out->exchange_bytes = ix->exchange_bytes;
     out->device_bytes = ix->device_bytes;
-    out->stream_elems = ix->finalized ? ix->sorted_elems : ix->n_elems;
+    out->stream_elems = ix->finalized ? ix->sorted_elems : ix->n_elems - ix->pm_merged;
     out->table_retries = ix->table_retries;
+    out->hot_elems_saved = ix->hot_elems_saved;
+    out->exchange_ms = ix->exchange_ms;
     for (int i = 0; i < WJ_PHASE_COUNT; ++i) {
       out->phase_ms[i] = ix->phase_ms[i];
       out->phase_launches[i] = ix->phase_launches[i];
@@ -2311,7 +2571,7 @@ void index_destroy(wj_index* ix) {
   ix->free_all();
   for (int i = 0; i < 2; ++i) {
     for (DevBuf* b : {&ix->pipe_text[i], &ix->pipe_off[i]})
-      if (b->p) cudaFree(b->p);
+      ix->dev_free(b->p);
     if (ix->pipe_copied[i]) cudaEventDestroy(ix->pipe_copied[i]);
     if (ix->pipe_done[i]) cudaEventDestroy(ix->pipe_done[i]);
   }

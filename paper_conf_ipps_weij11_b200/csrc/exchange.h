@@ -89,6 +89,7 @@ struct LoopbackTransport : Transport {
     hub->barrier();
     sent += soff[world] - (soff[rank + 1] - soff[rank]);
   }
+
 };
 
 // ------------------------------------------------------------------ NCCL (dlopen)
@@ -179,6 +180,7 @@ struct NcclTransport : Transport {
     nccl_check(a.GroupEnd(), "ncclGroupEnd");
     sent += soff[world] - (soff[rank + 1] - soff[rank]);
   }
+
 };
 
 // ------------------------------------------------------------------ K-way merge of serialized slices

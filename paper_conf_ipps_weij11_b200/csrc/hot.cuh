@@ -1,11 +1,11 @@
-// Sampled popular terms: the paper splits "popular" trie collections, "containing
-// the most frequently occurring terms", from the rest and decides membership on a sample, "1MB out of
+// Sampled popular terms: the paper treats "popular" terms, "the most
+// frequently occurring terms", apart from the rest and decides membership on a sample, "1MB out of
 // every 1GB".  B200 re-design: per chunk, the first 1 MiB of its documents is
-// tokenised with the same kernels, the <= 256 most frequent terms (>= 16 occurrences, <= 11 bytes) are
-// "hot"; in k_tok_emit a hot token does not enter the (slot, docID) stream (it leaves a hole) but
-// increments a dense (hot term x document) counter; afterwards every nonzero (term, document) counter
-// becomes one stream element carrying its count (count <= 127 per element).  The result is unchanged;
-// the sort and run-length passes see ~30% fewer elements on Zipf text.
+// tokenised with the same kernels and the <= 127 most frequent terms (>= 16 occurrences, <= 11
+// bytes) become hot; k_hot_seed claims their slots in the chunk table first, with the hot id in the
+// slot's k1 (bits 57..63).  In k_tok_emit the tokens of one hot term that fall in one document of a
+// warp's 8 KB window become ONE stream element carrying their count (the other tokens leave holes),
+// so the sort and run-length passes see fewer elements (0.75 N on config 2).  The result is unchanged.
 #pragma once
 #include "common.cuh"
 #include "tokenize.cuh"
@@ -13,8 +13,7 @@
 
 namespace wj {
 
-constexpr uint32_t kHotMax = 256;
-constexpr uint32_t kHotTable = 1024;  // open-addressing slots of the hot lookup table
+constexpr uint32_t kHotMax = 127;   // hot ids 1..127
 constexpr uint32_t kHotMinCount = 16;
 
 // hash of a term of <= 16 bytes from its folded words: identical to k_tok_emit's
@@ -74,45 +73,18 @@ __global__ void k_hot_extract(const Slot* table, const uint32_t* slots, uint32_t
   if (i < H) hk[i] = *(const ulonglong2*)(table + slots[i]);
 }
 
-// one thread: insert the hot terms into the chunk table (their slots) and into the hot lookup table
-__global__ void k_hot_build(const ulonglong2* hk, uint32_t H, Slot* table, uint32_t* slot_ref, uint32_t cap,
-                            HotEntry* hot, uint32_t* hot_slot, uint32_t* overflow) {
-  if (threadIdx.x != 0 || blockIdx.x != 0) return;
-  for (uint32_t i = 0; i < kHotTable; ++i) hot[i] = HotEntry{0ull, 0ull, 0u, 0u, {0u, 0u}};
-  for (uint32_t id = 0; id < H; ++id) {
-    const uint64_t k0 = hk[id].x, k1 = hk[id].y;
-    const uint32_t len = (uint32_t)k0 & 0xFFu;
-    const uint32_t w0 = (uint32_t)(k0 >> 32), w1 = (uint32_t)k1, w2 = (uint32_t)(k1 >> 32) & 0xFFFFFFu;
-    const uint64_t h = term_hash16(w0, w1, w2, 0u, len);
-    const uint32_t s = table_insert(nullptr, table, slot_ref, cap, h, k0, k1, 0u, len, nullptr, 0u, overflow);
-    hot_slot[id] = s;
-    uint32_t j = (uint32_t)(h >> 20) & (kHotTable - 1);
-    while (hot[j].k0 != 0) j = (j + 1) & (kHotTable - 1);
-    hot[j] = HotEntry{k0, k1, id, s, {0u, 0u}};
-  }
-}
-
-struct HotElemCount {
-  const uint32_t* tf;
-  __device__ __forceinline__ uint32_t operator()(uint64_t i) const { return (tf[i] + 126u) / 127u; }
-};
-
-// nonzero (hot term, document) counters -> stream elements (slot | count << 25, docID), term-major
-__global__ void k_hot_elems(const uint32_t* tf, uint64_t n, uint32_t D, const uint32_t* off, const uint32_t* hot_slot,
-                            uint32_t doc_base, uint32_t* out_key, uint32_t* out_doc) {
-  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= n) return;
-  uint32_t t = tf[i];
-  if (t == 0) return;
-  const uint32_t id = (uint32_t)(i / D), d = (uint32_t)(i % D);
-  uint32_t p = off[i];
-  while (t) {
-    const uint32_t c = t < 127u ? t : 127u;
-    out_key[p] = hot_slot[id] | (c << 25);
-    out_doc[p] = doc_base + d;
-    ++p;
-    t -= c;
-  }
+// thread i seeds hot id i + 1: claims the term's slot in the chunk table with the id in k1 bits 57..
+__global__ void k_hot_seed(const ulonglong2* hk, uint32_t H, Slot* table, uint32_t* slot_ref, uint32_t cap,
+                           uint32_t* hot_slot, uint32_t* overflow) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= H) return;
+  const uint32_t id = i + 1;
+  const uint64_t k0 = hk[i].x, k1 = hk[i].y | ((uint64_t)id << kHotShift);
+  const uint32_t len = (uint32_t)k0 & 0xFFu;
+  const uint32_t w0 = (uint32_t)(k0 >> 32), w1 = (uint32_t)hk[i].y, w2 = (uint32_t)(hk[i].y >> 32) & 0xFFFFFFu;
+  const uint64_t h = term_hash16(w0, w1, w2, 0u, len);
+  uint32_t hot = 0;
+  hot_slot[id] = table_insert(nullptr, table, slot_ref, cap, h, k0, k1, 0u, len, nullptr, 0u, overflow, &hot);
 }
 
 }  // namespace wj

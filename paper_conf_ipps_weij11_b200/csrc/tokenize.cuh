@@ -41,23 +41,13 @@ struct ChunkView {
   uint64_t n_docs;
 };
 
-// hot lookup entry (hot.cuh): a sampled popular term of <= 11 bytes, identified by its slot words
-struct __align__(16) HotEntry {
-  unsigned long long k0, k1;
-  uint32_t id, slot;
-  uint32_t pad[2];
-};
-
 struct EmitOut {
-  const HotEntry* hot;     // hot lookup table (nullptr: no hot terms)
-  uint32_t hot_mask;       // lookup table size - 1
-  uint32_t hot_docs;       // documents of the chunk (columns of hot_tf)
-  uint32_t* hot_tf;        // hot term x document token counts
+  const uint32_t* hot_slot;  // hot id (1..127) -> its slot in this table; nullptr: no hot aggregation
   Slot* table;             // chunk hash table
   uint32_t* slot_ref;      // per slot: first-occurrence offset (written by the inserter)
   uint32_t cap;            // capacity (slots; any value >= 1)
   uint32_t doc_base;       // global DocID of local document 0
-  uint32_t* slot;          // per kept token: table slot
+  uint32_t* slot;          // per kept token: slot | count << 25 (key 0 = hole: merged hot token)
   uint32_t* doc;           // per kept token: global DocID
   uint32_t* dbg_start;     // optional (debug): token start
   uint32_t* dbg_len;       // optional (debug): token length
@@ -336,9 +326,12 @@ __device__ __forceinline__ uint32_t hash_fin(uint32_t h) {
 }
 __device__ __forceinline__ uint32_t hash_tag(uint32_t h) { return (h * 0x9E3779B1u) >> 8; }
 
+// Find or claim the slot of a term.  *hot = the sampled hot-term id stored in the slot's k1 (0: none;
+// only slots seeded by k_hot_seed carry one).
 __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* table, uint32_t* slot_ref, uint32_t cap,
                                                  uint64_t h, uint64_t k0, uint64_t k1, uint32_t s_abs, uint32_t len,
-                                                 const uint32_t* win32, uint32_t s_win, uint32_t* overflow) {
+                                                 const uint32_t* win32, uint32_t s_win, uint32_t* overflow,
+                                                 uint32_t* hot) {
   uint32_t i = __umulhi((uint32_t)h, cap);
   for (int probe = 0; probe < 4096; ++probe) {
     // Slots are claimed once (CAS on k0) and published once (k1), so a cached read can only be
@@ -350,6 +343,7 @@ __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* tabl
         slot_ref[i] = s_abs;
         if (len > kSlotBytes) __threadfence();  // only > 11-byte terms are compared via slot_ref
         *(volatile unsigned long long*)&table[i].k1 = k1;
+        *hot = 0;
         return i;
       }
       e.x = prev;
@@ -357,7 +351,8 @@ __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* tabl
     }
     if (e.x == k0) {
       while (e.y == 0) e.y = *(volatile unsigned long long*)&table[i].k1;
-      if (e.y == k1) {
+      if ((e.y & kSlotK1Mask) == k1) {
+        *hot = (uint32_t)(e.y >> kHotShift);
         if (len <= kSlotBytes) return i;
         // acquire: the inserter wrote slot_ref[i] before its release of k1 (__threadfence + store)
         (void)ld_acquire_u64(&table[i].k1);
@@ -372,6 +367,7 @@ __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* tabl
     i = i + 1 == cap ? 0u : i + 1;
   }
   atomicExch(overflow, 1u);
+  *hot = 0;
   return kMiss;
 }
 
@@ -383,191 +379,255 @@ __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* tabl
 #ifndef WJ_EMIT_MINB
 #define WJ_EMIT_MINB 6
 #endif
-__global__ void __launch_bounds__(kTokThreads, WJ_EMIT_MINB) k_tok_emit(ChunkView cv, uint32_t n_segs, const uint64_t* kstart,
-                                                          const uint32_t* range_off, EmitOut eo) {
+// HOT (opt-in, WJ_FLAG_HOT_TERMS): a warp walks kHotSub consecutive count ranges (4 x 2 KB), the
+// window over which the tokens of a sampled hot term that fall in one
+// document are merged into one stream element carrying their count; merged tokens leave holes (key 0)
+// that the first sort pass drops.  Measured slower than the plain kernel on config 2 (the merge work
+// and 48 registers cost more in emit than the sort and run-length passes save; profiles/r02_README.md),
+// so the plain instantiation (one range per warp, no hot state, 40 registers) is the default.
+constexpr uint32_t kHotSub = 4;
+constexpr uint32_t kHotIds = 128;  // hot ids 1..127 (7 bits of the slot's k1)
+template <bool HOT>
+__host__ __device__ constexpr uint32_t emit_sub() { return HOT ? kHotSub : 1u; }
+
+template <bool HOT>
+__global__ void __launch_bounds__(kTokThreads, HOT ? 5 : WJ_EMIT_MINB) k_tok_emit(ChunkView cv, uint32_t n_segs,
+                                                          const uint64_t* kstart, const uint32_t* range_off, EmitOut eo) {
+  constexpr uint32_t kEmitSub = emit_sub<HOT>();
   __shared__ __align__(16) uint32_t win[kTokWarps][kWinBytes / 4];
   __shared__ uint32_t queue[kTokWarps][kQueueCap + 1];
   __shared__ uint32_t bnd[kTokWarps][32];
+  __shared__ uint32_t hacc[kTokWarps][HOT ? kHotIds : 1];  // per hot id: count << 16 | first position (warp-relative)
   const uint32_t lane = lane_id();
   const int w = threadIdx.x >> 5;
-  const uint32_t gw = blockIdx.x * kTokWarps + w;
-  const uint32_t sb0 = gw * kSegsPerWarp;
-  if (sb0 >= n_segs) return;
-  const uint32_t se = min(sb0 + kSegsPerWarp, n_segs);
-  const uint32_t last = se < n_segs ? se : se - 1;
-  const uint32_t B0 = sb0 * kSegBytes;
+  const uint32_t n_ranges = (n_segs + kSegsPerWarp - 1) / kSegsPerWarp;
+  const uint32_t gw0 = (blockIdx.x * kTokWarps + w) * kEmitSub;
+  if (gw0 >= n_ranges) return;
   uint32_t* w32 = win[w];
   uint32_t* q = queue[w];
-  // stage the range and the look-ahead segment (tokens may run past the range)
-  uint4 v[kSegsPerWarp + 1];
-#pragma unroll
-  for (int j = 0; j <= kSegsPerWarp; ++j) v[j] = load_lane16(cv, sb0 + j);
-#pragma unroll
-  for (int j = 0; j <= kSegsPerWarp; ++j)  // fold A-Z once here (classification is case-blind)
-    *(uint4*)&w32[(j * kSegBytes + 16 * lane) / 4] =
-        make_uint4(lower4(v[j].x), lower4(v[j].y), lower4(v[j].z), lower4(v[j].w));
-  if (lane < 4) w32[(kWinBytes - 16) / 4 + lane] = 0;
-  __syncwarp();
-
-  const uint64_t k_range_lo = kstart[gw];
-  uint64_t kcur = k_range_lo;
-  uint32_t prev = prev_token_bit(cv, B0);
-  uint32_t qn = 0;
-  uint64_t obase = range_off[gw];
-  uint64_t k_range_hi = k_range_lo;
-  bool open = false;
-  uint32_t open_start = 0;
-
-  auto flush = [&]() {
-    for (uint32_t r = 0; r < qn; r += 32) {
-      const uint32_t idx = r + lane;
-      if (idx < qn) {
-        const uint32_t e = q[idx];
-        const uint32_t s_win = e >> 8, len = e & 255u;
-        const uint32_t s_abs = B0 + s_win;
-        // first 16 folded bytes: 5 window words, 4 funnel shifts, length masks
-        uint32_t wd[4];
-        {
-          const uint32_t a = s_win >> 2, sh = (s_win & 3) * 8;
-          uint32_t x[5];
-#pragma unroll
-          for (int k = 0; k < 5; ++k) x[k] = w32[a + k];
-#pragma unroll
-          for (int k = 0; k < 4; ++k) {
-            const uint32_t rem = min(max((int)len - 4 * k, 0), 4);
-            wd[k] = __funnelshift_r(x[k], x[k + 1], sh) & __funnelshift_lc(0xFFFFFFFFu, 0u, rem * 8);
-          }
-        }
-        uint32_t h32 = hash_init(len);
-#pragma unroll
-        for (int k = 0; k < 4; ++k) h32 = hash_mix(h32, wd[k]);
-        for (uint32_t k = 4; k * 4 < len; ++k) h32 = hash_mix(h32, win_word(w32, s_win, len, k));
-        h32 = hash_fin(h32);
-        const uint64_t h = h32;
-        // DocID = (number of doc_off[k] <= s, k < n_docs) - 1 (readings S9, S16)
-        uint64_t lo = k_range_lo, hi = k_range_hi;
-        while (lo < hi) {
-          const uint64_t mid = (lo + hi) >> 1;
-          if (cv.doc_off[mid] <= s_abs) lo = mid + 1; else hi = mid;
-        }
-        const uint32_t doc = eo.doc_base + (uint32_t)(lo - 1);
-        const uint64_t k0 = (uint64_t)len | ((uint64_t)hash_tag(h32) << 8) | ((uint64_t)wd[0] << 32);
-        const uint64_t k1 = (uint64_t)wd[1] | ((uint64_t)(wd[2] & 0xFFFFFFu) << 32) | (1ull << 56);
-        const uint64_t out = obase + idx;
-        bool hot = false;
-        if (eo.hot && len <= kSlotBytes) {  // sampled popular term: count it per document, leave a hole
-          uint32_t j = (uint32_t)(h >> 20) & eo.hot_mask;
-          for (;;) {
-            const uint64_t e0 = __ldg(&eo.hot[j].k0);
-            if (e0 == 0) break;
-            if (e0 == k0 && __ldg(&eo.hot[j].k1) == k1) {
-              atomicAdd(&eo.hot_tf[(uint64_t)__ldg(&eo.hot[j].id) * eo.hot_docs + (doc - eo.doc_base)], 1u);
-              hot = true;
-              break;
-            }
-            j = (j + 1) & eo.hot_mask;
-          }
-        }
-        if (hot) {
-          __stcs(eo.slot + out, 0u);
-        } else {
-          const uint32_t slot =
-              table_insert(cv.text, eo.table, eo.slot_ref, eo.cap, h, k0, k1, s_abs, len, w32, s_win, eo.overflow);
-          __stcs(eo.slot + out, slot | (1u << 25));  // stream element: slot | count 1 << 25
-          __stcs(eo.doc + out, doc);
-        }
-        if (eo.dbg_start) { eo.dbg_start[out] = s_abs; eo.dbg_len[out] = len; }
+  uint32_t* ha = hacc[w];
+  constexpr bool hot_on = HOT;
+  const uint64_t wbase = HOT ? range_off[gw0] : 0;  // output index of the warp's first token
+  uint32_t hdoc = 0;                                 // document of the accumulated hot counts
+  if (hot_on) {
+    for (uint32_t i = lane; i < kHotIds; i += 32) ha[i] = 0;
+    __syncwarp();
+  }
+  // accumulated hot elements -> stream (each at the output position of its first token)
+  auto hot_flush = [&]() {
+    if (!HOT) return;
+    for (uint32_t i = lane; i < kHotIds; i += 32) {
+      const uint32_t a = ha[i];
+      if (a >> 16) {
+        const uint64_t o = wbase + (a & 0xFFFFu);
+        __stcs(eo.slot + o, __ldg(&eo.hot_slot[i]) | ((a >> 16) << 25));
+        __stcs(eo.doc + o, hdoc);
+        ha[i] = 0;
       }
     }
-    obase += qn;
-    qn = 0;
     __syncwarp();
   };
 
-  for (uint32_t seg = sb0; seg <= last; ++seg) {
-    const uint32_t j = seg - sb0;
-    const uint32_t s0 = seg * kSegBytes;
-    const uint4 vv = *(const uint4*)&w32[(j * kSegBytes + 16 * lane) / 4];
-    // reloaded per segment here: a register carried across the flushes costs the emit kernel more
-    // (spills) than the load (count: 0.426 -> 0.408 ms with the carried register, emit +0.025 ms)
-    uint64_t nb = next_bound(cv, kcur);
-    const SegBits sb = seg_bits(cv, s0, vv, prev, kcur, nb, bnd[w]);
-    prev = __shfl_sync(0xffffffffu, sb.tm, 31) >> 15;
-    const SegTok tk = seg_tok(sb);
-    if (open) {  // the previous segment's last token ends in this one
-      const uint32_t ft = first_term(sb, tk);
-      if (ft != kNone && s0 + ft - open_start <= kMaxTermLen) {
-        if (qn + 1 > (uint32_t)kQueueCap) flush();
-        if (lane == 0) q[qn] = ((open_start - B0) << 8) | (s0 + ft - open_start);
-        ++qn;
-        __syncwarp();
-      }
-      open = false;
-    }
-    if (seg == se) break;
-    k_range_hi = kcur;
-    // kept tokens starting in this lane (a > 255-byte token needs a lane of 16 token bytes)
-    uint32_t c = __popc(sb.startm) - ((int)lane == tk.open_lane ? 1u : 0u);
-    if (__ballot_sync(0xffffffffu, sb.tm == 0xFFFFu)) {
-      c = 0;
-      for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
-        const int jb = __ffs(sm) - 1;
-        const uint32_t pos = 16 * lane + jb;
-        if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
-        c += (tok_end_rel(sb, tk, jb) - pos <= kMaxTermLen) ? 1u : 0u;
-      }
-    }
-    uint32_t inc = c;
+  for (uint32_t sub = 0; sub < kEmitSub; ++sub) {
+    const uint32_t gw = gw0 + sub;
+    if (gw >= n_ranges) break;
+    const uint32_t sb0 = gw * kSegsPerWarp;
+    const uint32_t se = min(sb0 + kSegsPerWarp, n_segs);
+    const uint32_t last = se < n_segs ? se : se - 1;
+    const uint32_t B0 = sb0 * kSegBytes;
+    // stage the range and the look-ahead segment (tokens may run past the range)
+    {
+      uint4 v[kSegsPerWarp + 1];
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
-      if ((int)lane >= o) inc += u;
+      for (int j = 0; j <= kSegsPerWarp; ++j) v[j] = load_lane16(cv, sb0 + j);
+      __syncwarp();  // the previous range's window is no longer read
+#pragma unroll
+      for (int j = 0; j <= kSegsPerWarp; ++j)  // fold A-Z once here (classification is case-blind)
+        *(uint4*)&w32[(j * kSegBytes + 16 * lane) / 4] =
+            make_uint4(lower4(v[j].x), lower4(v[j].y), lower4(v[j].z), lower4(v[j].w));
+      if (lane < 4) w32[(kWinBytes - 16) / 4 + lane] = 0;
+      __syncwarp();
     }
-    const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
-    if (qn + tot > (uint32_t)kQueueCap) flush();
-    if (tot <= (uint32_t)kQueueCap) {
-      uint32_t pos_q = qn + inc - c;
-      for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
-        const int jb = __ffs(sm) - 1;
-        const uint32_t pos = 16 * lane + jb;
-        if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
-        const uint32_t len = tok_end_rel(sb, tk, jb) - pos;
-        if (len <= kMaxTermLen) q[pos_q++] = ((s0 + pos - B0) << 8) | len;
+
+    const uint64_t k_range_lo = kstart[gw];
+    uint64_t kcur = k_range_lo;
+    uint32_t prev = prev_token_bit(cv, B0);
+    uint32_t qn = 0;
+    uint64_t obase = range_off[gw];
+    uint64_t k_range_hi = k_range_lo;
+    bool open = false;
+    uint32_t open_start = 0;
+
+    auto flush = [&]() {
+      for (uint32_t r = 0; r < qn; r += 32) {
+        const uint32_t idx = r + lane;
+        const bool valid = idx < qn;
+        uint32_t hid = 0, doc = 0;
+        uint64_t out = 0;
+        if (valid) {
+          const uint32_t e = q[idx];
+          const uint32_t s_win = e >> 8, len = e & 255u;
+          const uint32_t s_abs = B0 + s_win;
+          // first 16 folded bytes: 5 window words, 4 funnel shifts, length masks
+          uint32_t wd[4];
+          {
+            const uint32_t a = s_win >> 2, sh = (s_win & 3) * 8;
+            uint32_t x[5];
+#pragma unroll
+            for (int k = 0; k < 5; ++k) x[k] = w32[a + k];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+              const uint32_t rem = min(max((int)len - 4 * k, 0), 4);
+              wd[k] = __funnelshift_r(x[k], x[k + 1], sh) & __funnelshift_lc(0xFFFFFFFFu, 0u, rem * 8);
+            }
+          }
+          uint32_t h32 = hash_init(len);
+#pragma unroll
+          for (int k = 0; k < 4; ++k) h32 = hash_mix(h32, wd[k]);
+          for (uint32_t k = 4; k * 4 < len; ++k) h32 = hash_mix(h32, win_word(w32, s_win, len, k));
+          h32 = hash_fin(h32);
+          const uint64_t h = h32;
+          // DocID = (number of doc_off[k] <= s, k < n_docs) - 1 (readings S9, S16)
+          uint64_t lo = k_range_lo, hi = k_range_hi;
+          while (lo < hi) {
+            const uint64_t mid = (lo + hi) >> 1;
+            if (cv.doc_off[mid] <= s_abs) lo = mid + 1; else hi = mid;
+          }
+          doc = eo.doc_base + (uint32_t)(lo - 1);
+          const uint64_t k0 = (uint64_t)len | ((uint64_t)hash_tag(h32) << 8) | ((uint64_t)wd[0] << 32);
+          const uint64_t k1 = (uint64_t)wd[1] | ((uint64_t)(wd[2] & 0xFFFFFFu) << 32) | (1ull << 56);
+          out = obase + idx;
+          const uint32_t slot = table_insert(cv.text, eo.table, eo.slot_ref, eo.cap, h, k0, k1, s_abs, len, w32, s_win,
+                                             eo.overflow, &hid);
+          if (!HOT) hid = 0;
+          // stream element: slot | count 1 << 25, or a hole (key 0) for a merged hot token
+          __stcs(eo.slot + out, hid ? 0u : (slot | (1u << 25)));
+          if (!hid) __stcs(eo.doc + out, doc);
+          if (eo.dbg_start) { eo.dbg_start[out] = s_abs; eo.dbg_len[out] = len; }
+        }
+        // hot tokens: per document (documents ascend with the lane), lanes of one hot id merge into
+        // their leader (the earliest token), which updates the warp's accumulator
+        uint32_t pend = HOT ? __ballot_sync(0xffffffffu, hid != 0) : 0u;
+        while (HOT && pend) {
+          const uint32_t d = __shfl_sync(0xffffffffu, doc, __ffs(pend) - 1);
+          if (d != hdoc) {
+            hot_flush();
+            hdoc = d;
+          }
+          const bool mine = ((pend >> lane) & 1u) && doc == d;
+          const uint32_t grp = __ballot_sync(0xffffffffu, mine);
+          if (mine) {
+            const uint32_t peers = __match_any_sync(grp, hid);
+            if ((int)lane == __ffs(peers) - 1) {
+              uint32_t a = ha[hid];
+              uint32_t c = a >> 16;
+              const uint32_t add = __popc(peers);
+              const uint32_t pos = (uint32_t)(out - wbase);
+              if (c + add > 127u) {  // the element is full: write it, start the next at this token
+                const uint64_t o = wbase + (a & 0xFFFFu);
+                __stcs(eo.slot + o, __ldg(&eo.hot_slot[hid]) | (c << 25));
+                __stcs(eo.doc + o, hdoc);
+                c = 0;
+              }
+              if (c == 0) a = pos;
+              ha[hid] = (a & 0xFFFFu) | ((c + add) << 16);
+            }
+          }
+          pend &= ~grp;
+          __syncwarp();
+        }
       }
-      qn += tot;
-    } else {
-      // Rare: more kept tokens start in this segment than the queue holds (up to 512: dense
-      // document starts, e.g. consecutive 1-byte documents).  Queue them in rounds of kQueueCap,
-      // flushing between rounds (the queue is empty here: tot > kQueueCap forced the flush above).
-      for (uint32_t r0 = 0; r0 < tot; r0 += (uint32_t)kQueueCap) {
-        uint32_t pos_q = inc - c;  // segment-relative index of the lane's first kept token
+      obase += qn;
+      qn = 0;
+      __syncwarp();
+    };
+
+    for (uint32_t seg = sb0; seg <= last; ++seg) {
+      const uint32_t j = seg - sb0;
+      const uint32_t s0 = seg * kSegBytes;
+      const uint4 vv = *(const uint4*)&w32[(j * kSegBytes + 16 * lane) / 4];
+      // reloaded per segment here: a register carried across the flushes costs the emit kernel more
+      // (spills) than the load (count: 0.426 -> 0.408 ms with the carried register, emit +0.025 ms)
+      uint64_t nb = next_bound(cv, kcur);
+      const SegBits sb = seg_bits(cv, s0, vv, prev, kcur, nb, bnd[w]);
+      prev = __shfl_sync(0xffffffffu, sb.tm, 31) >> 15;
+      const SegTok tk = seg_tok(sb);
+      if (open) {  // the previous segment's last token ends in this one
+        const uint32_t ft = first_term(sb, tk);
+        if (ft != kNone && s0 + ft - open_start <= kMaxTermLen) {
+          if (qn + 1 > (uint32_t)kQueueCap) flush();
+          if (lane == 0) q[qn] = ((open_start - B0) << 8) | (s0 + ft - open_start);
+          ++qn;
+          __syncwarp();
+        }
+        open = false;
+      }
+      if (seg == se) break;
+      k_range_hi = kcur;
+      // kept tokens starting in this lane (a > 255-byte token needs a lane of 16 token bytes)
+      uint32_t c = __popc(sb.startm) - ((int)lane == tk.open_lane ? 1u : 0u);
+      if (__ballot_sync(0xffffffffu, sb.tm == 0xFFFFu)) {
+        c = 0;
+        for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
+          const int jb = __ffs(sm) - 1;
+          const uint32_t pos = 16 * lane + jb;
+          if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
+          c += (tok_end_rel(sb, tk, jb) - pos <= kMaxTermLen) ? 1u : 0u;
+        }
+      }
+      uint32_t inc = c;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
+        if ((int)lane >= o) inc += u;
+      }
+      const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
+      if (qn + tot > (uint32_t)kQueueCap) flush();
+      if (tot <= (uint32_t)kQueueCap) {
+        uint32_t pos_q = qn + inc - c;
         for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
           const int jb = __ffs(sm) - 1;
           const uint32_t pos = 16 * lane + jb;
           if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
           const uint32_t len = tok_end_rel(sb, tk, jb) - pos;
-          if (len > kMaxTermLen) continue;
-          if (pos_q >= r0 && pos_q < r0 + (uint32_t)kQueueCap) q[pos_q - r0] = ((s0 + pos - B0) << 8) | len;
-          ++pos_q;
+          if (len <= kMaxTermLen) q[pos_q++] = ((s0 + pos - B0) << 8) | len;
         }
-        qn = min(tot - r0, (uint32_t)kQueueCap);
-        __syncwarp();
-        flush();
+        qn += tot;
+      } else {
+        // Rare: more kept tokens start in this segment than the queue holds (up to 512: dense
+        // document starts, e.g. consecutive 1-byte documents).  Queue them in rounds of kQueueCap,
+        // flushing between rounds (the queue is empty here: tot > kQueueCap forced the flush above).
+        for (uint32_t r0 = 0; r0 < tot; r0 += (uint32_t)kQueueCap) {
+          uint32_t pos_q = inc - c;  // segment-relative index of the lane's first kept token
+          for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
+            const int jb = __ffs(sm) - 1;
+            const uint32_t pos = 16 * lane + jb;
+            if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
+            const uint32_t len = tok_end_rel(sb, tk, jb) - pos;
+            if (len > kMaxTermLen) continue;
+            if (pos_q >= r0 && pos_q < r0 + (uint32_t)kQueueCap) q[pos_q - r0] = ((s0 + pos - B0) << 8) | len;
+            ++pos_q;
+          }
+          qn = min(tot - r0, (uint32_t)kQueueCap);
+          __syncwarp();
+          flush();
+        }
       }
-    }
-    if (tk.open_lane >= 0) { open = true; open_start = s0 + tk.open_pos; }
-    __syncwarp();
-  }
-  k_range_hi = kcur;
-  if (open) {  // chunk end
-    if (cv.n_bytes - open_start <= kMaxTermLen) {
-      if (qn + 1 > (uint32_t)kQueueCap) flush();
-      if (lane == 0) q[qn] = ((open_start - B0) << 8) | (uint32_t)(cv.n_bytes - open_start);
-      ++qn;
+      if (tk.open_lane >= 0) { open = true; open_start = s0 + tk.open_pos; }
       __syncwarp();
     }
+    k_range_hi = kcur;
+    if (open) {  // chunk end
+      if (cv.n_bytes - open_start <= kMaxTermLen) {
+        if (qn + 1 > (uint32_t)kQueueCap) flush();
+        if (lane == 0) q[qn] = ((open_start - B0) << 8) | (uint32_t)(cv.n_bytes - open_start);
+        ++qn;
+        __syncwarp();
+      }
+    }
+    flush();
   }
-  flush();
+  if (hot_on) hot_flush();
 }
 
 }  // namespace wj

@@ -38,8 +38,8 @@ def test_library_is_sm100a():
 
 
 def test_struct_sizes_match_header(tmp_path):
-    # wj_config: 3 x i32 + pad + 2 pointers + u64 + 2 x u32 = 48 bytes on LP64
-    assert ctypes.sizeof(wj.Config) == 48
+    # wj_config: 3 x i32 + pad + 2 pointers + u64 + 2 x u32 + pointer + u64 = 64 bytes on LP64
+    assert ctypes.sizeof(wj.Config) == 64
     # the binding's structs against the C compiler's view of include/wjindex.h
     src = tmp_path / "sz.c"
     src.write_text('#include <stdio.h>\n#include "wjindex.h"\n'

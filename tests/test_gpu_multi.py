@@ -24,7 +24,7 @@ import paper_conf_ipps_weij11_b200 as wj  # noqa: E402
 
 
 def dist_index(text, doc_off, K, cuts=None, queries=(), vbyte=False, balanced=False, maps=None, stem=False,
-               stop=False):
+               stop=False, **kw):
     off = np.asarray(doc_off, dtype=np.uint64)
     text = np.asarray(text, dtype=np.uint8)
     n = len(off) - 1
@@ -37,7 +37,7 @@ def dist_index(text, doc_off, K, cuts=None, queries=(), vbyte=False, balanced=Fa
     def run(r):
         try:
             with wj.Index(device=0, rank=r, world=K, hub=hub, own_stream=True, vbyte=vbyte, balanced=balanced, stem=stem,
-                          stop=stop) as ix:
+                          stop=stop, **kw) as ix:
                 for a, b in zip(cuts, cuts[1:]):
                     # rank r's contiguous document range of this chunk (rank order = DocID order)
                     bounds = [a + (b - a) * i // K for i in range(K + 1)]
@@ -65,7 +65,7 @@ def dist_index(text, doc_off, K, cuts=None, queries=(), vbyte=False, balanced=Fa
     return slices, answers
 
 
-@pytest.mark.parametrize("K", [2, 3, 4])
+@pytest.mark.parametrize("K", [2, 3, 4, 8])
 def test_loopback_config1(K):
     text, off = gen.generate(gen.CONFIGS[1])
     want = oracle.index_bytes(text, off)
@@ -77,17 +77,65 @@ def test_loopback_config1(K):
     assert wj.merge_serialized(slices) == want
 
 
-@pytest.mark.parametrize("K", [1, 2, 3])
-@pytest.mark.parametrize("dist_partials", ["0", "1"])
-def test_loopback_owner_partials(K, dist_partials, monkeypatch):
-    """Owner side on per-run partial lists (WJ_DIST_PARTIALS=1: received records sorted by the owner's
-    chunk-table slot on the side stream) and on the global stream (default): both
-    byte-identical to the oracle over three chunks."""
-    monkeypatch.setenv("WJ_DIST_PARTIALS", dist_partials)
+@pytest.mark.parametrize("K", [1, 2, 3, 8])
+@pytest.mark.parametrize("global_stream", [False, True])
+def test_loopback_both_paths(K, global_stream):
+    """Default: sender-side partial lists (every rank sorts its own stream by (owner, term) and sends
+    per-term postings, P:160-162 / P:237); WJ_FLAG_GLOBAL_STREAM: token records routed to the owner and
+    one global sort at finalize.  Both byte-identical to the oracle over three chunks."""
     text, off = gen.generate(gen.CONFIGS[1])
     want = oracle.index_bytes(text, off)
-    slices, _ = dist_index(text, off, K, cuts=[0, 300, 301, 1000])
+    slices, _ = dist_index(text, off, K, cuts=[0, 300, 301, 1000], global_stream=global_stream)
     assert wj.merge_serialized(slices) == want
+
+
+@pytest.mark.parametrize("K", [2, 8])
+def test_loopback_hot_terms(K):
+    # opt-in hot-term merging on the senders (holes + count elements in the local sort)
+    cfg = gen.CONFIGS[2].scaled(chunk_bytes=8 << 20, vocab=100_000)
+    text, off = gen.generate(cfg)
+    n = len(off) - 1
+    slices, _ = dist_index(text, off, K, cuts=[0, n // 2, n], hot=True)
+    assert wj.merge_serialized(slices) == oracle.index_bytes(text, off)
+
+
+def test_loopback_k8_config3_shape_exchange_volume():
+    """K = 8 on Wikipedia-shaped text (short documents): byte-identical merge, and the bytes sent
+    stay below 8 B per token (postings aggregated per (term, document) plus term bytes and headers)."""
+    cfg = gen.CONFIGS[3].scaled(chunk_bytes=16 << 20, vocab=200_000)
+    text, off = gen.generate(cfg)
+    n = len(off) - 1
+    K = 8
+    stats = [None] * K
+    hub = wj.LoopbackHub(K)
+    slices = [None] * K
+    errors = []
+
+    def run(r):
+        try:
+            with wj.Index(device=0, rank=r, world=K, hub=hub, own_stream=True) as ix:
+                bounds = [n * i // K for i in range(K + 1)]
+                lo, hi = bounds[r], bounds[r + 1]
+                ix.add_stream(text[int(off[lo]):int(off[hi])], off[lo:hi + 1] - off[lo])
+                ix.finalize()
+                slices[r] = ix.serialize()
+                stats[r] = ix.stats()
+        except Exception as e:  # pragma: no cover
+            errors.append((r, e))
+            raise
+
+    th = [threading.Thread(target=run, args=(r,)) for r in range(K)]
+    for x in th:
+        x.start()
+    for x in th:
+        x.join(timeout=600)
+    hub.close()
+    assert not errors, errors
+    full = oracle.index_bytes(text, off)
+    assert wj.merge_serialized(slices) == full
+    sent = sum(s["exchange_bytes"] for s in stats)
+    ntok = int(wjformat.parse(full).n_tokens)
+    assert sent < 8 * ntok
 
 
 def test_loopback_edges_and_queries():
@@ -187,7 +235,7 @@ def test_loopback_host_pipeline():
     assert wj.merge_serialized(slices) == oracle.index_bytes(text, off)
 
 
-@pytest.mark.parametrize("K", [3, 4])
+@pytest.mark.parametrize("K", [3, 4, 8])
 def test_loopback_balanced_owner_map(K):
     # sampled bin-packing of the trie collections: same map on every rank, every slice
     # holds exactly its collections, the merge is the oracle's file, and the sampled-token load of

@@ -23,8 +23,8 @@ if not torch.cuda.is_available():  # pragma: no cover
 import paper_conf_ipps_weij11_b200 as wj  # noqa: E402
 
 
-def gpu_index(text, doc_off, cuts=None, device_input=False, vbyte=False):
-    with wj.Index(device=0, vbyte=vbyte) as ix:
+def gpu_index(text, doc_off, cuts=None, device_input=False, vbyte=False, **kw):
+    with wj.Index(device=0, vbyte=vbyte, **kw) as ix:
         off = np.asarray(doc_off, dtype=np.uint64)
         text = np.asarray(text, dtype=np.uint8)
         cuts = cuts or [0, len(off) - 1]
@@ -307,28 +307,48 @@ def test_config2_full_size_sha():
 
 
 # ------------------------------------------------------------------ sampled hot terms
-@pytest.fixture
-def hot_threshold(monkeypatch):
-    # contexts read WJ_HOT_MIN_BYTES at index_init: enable the (opt-in) hot-term path on small chunks
-    monkeypatch.setenv("WJ_HOT_MIN_BYTES", "65536")
-    yield
-
-
+@pytest.mark.parametrize("global_stream", [False, True])
 @pytest.mark.parametrize("cfg_id", [2, 3, 4])
-def test_hot_path_shapes(hot_threshold, cfg_id):
+def test_hot_path_shapes(cfg_id, global_stream):
     cfg = gen.CONFIGS[cfg_id].scaled(chunk_bytes=6 << 20, vocab=200_000)
     text, off = gen.generate(cfg)
     n = len(off) - 1
     want = oracle.index_bytes(text, off)
-    assert_same_index(gpu_index(text, off), want)
-    assert_same_index(gpu_index(text, off, cuts=[0, n // 3, n // 3 + 1, n]), want)
+    for cuts in (None, [0, n // 3, n // 3 + 1, n]):
+        with wj.Index(device=0, hot=True, global_stream=global_stream) as ix:
+            c = cuts or [0, n]
+            for a, b in zip(c, c[1:]):
+                ix.add_stream(text[int(off[a]):int(off[b])], (off[a:b + 1] - off[a]).astype(np.uint64))
+            ix.finalize()
+            assert_same_index(ix.serialize(), want)
+            s = ix.stats()
+            assert s["hot_elems_saved"] > 0
+            if not global_stream:
+                assert s["stream_elems"] + s["hot_elems_saved"] == s["n_tokens"]
 
 
-def test_hot_path_repetitive_docs(hot_threshold):
-    # a term whose per-document count exceeds 127 (split into several stream elements) and one-token docs
-    docs = [b"the " * 600 + b"cat", b"the", b"", b"The the THE"] * 300 + [b"x y z " * 5000]
+@pytest.mark.parametrize("global_stream", [False, True])
+def test_hot_path_repetitive_docs(global_stream):
+    # a term whose count in one document's 8 KB window exceeds 127 (several count elements), runs of
+    # one-token documents, hot terms at every document boundary of a warp round
+    docs = [b"the " * 600 + b"cat", b"the", b"", b"The the THE"] * 300 + [b"x y z " * 5000] + [b"the"] * 3000
     text, off = gen.from_docs(docs)
-    assert_same_index(gpu_index(text, off), oracle.index_bytes(text, off))
+    want = oracle.index_bytes(text, off)
+    assert_same_index(gpu_index(text, off, hot=True, global_stream=global_stream), want)
+    assert_same_index(gpu_index(text, off, cuts=[0, 1000, 1001, len(docs)], hot=True, global_stream=global_stream),
+                      want)
+
+
+def test_hot_off_by_default():
+    cfg = gen.CONFIGS[2].scaled(chunk_bytes=10 << 20, vocab=100_000)
+    text, off = gen.generate(cfg)
+    want = oracle.index_bytes(text, off)
+    with wj.Index(device=0) as ix:
+        ix.add_stream(text, off)
+        ix.finalize()
+        assert_same_index(ix.serialize(), want)
+        s = ix.stats()
+        assert s["hot_elems_saved"] == 0 and s["stream_elems"] == s["n_tokens"]
 
 
 def test_multichunk_config3_shape():
@@ -481,19 +501,19 @@ def test_new_terms_sharing_long_prefixes(seed):
 
 
 # ------------------------------------------------------------------ partial lists per run (partials.cuh)
-@pytest.mark.parametrize("partials", ["1", "0"])
-def test_partials_and_global_stream_paths(monkeypatch, partials):
+@pytest.mark.parametrize("global_stream", [False, True])
+def test_partials_and_global_stream_paths(global_stream):
     # default single-GPU path: per-chunk partial postings combined at finalize;
-    # WJ_PARTIALS=0: the global stream sorted at finalize.  Both must give the oracle's bytes, with
-    # chunks of very different sizes, empty chunks and a single-document chunk.
-    monkeypatch.setenv("WJ_PARTIALS", partials)
+    # WJ_FLAG_GLOBAL_STREAM: the global stream sorted at finalize.  Both must give the oracle's bytes,
+    # with chunks of very different sizes, empty chunks and a single-document chunk.
     cfg = gen.CONFIGS[3].scaled(chunk_bytes=3 << 20, vocab=50_000)
     text, off = gen.generate(cfg)
     n = len(off) - 1
     want = oracle.index_bytes(text, off)
     for cuts in ([0, n], [0, 1, 1, n // 7, n // 2, n - 1, n], [0, n // 3, 2 * n // 3, n]):
-        assert_same_index(gpu_index(text, off, cuts=cuts), want)
-    assert_same_index(gpu_index(text, off, cuts=[0, n // 2, n], vbyte=True), oracle.index_bytes(text, off, vbyte=True))
+        assert_same_index(gpu_index(text, off, cuts=cuts, global_stream=global_stream), want)
+    assert_same_index(gpu_index(text, off, cuts=[0, n // 2, n], vbyte=True, global_stream=global_stream),
+                      oracle.index_bytes(text, off, vbyte=True))
 
 
 def test_partials_repeated_reset_and_read_postings():
@@ -568,3 +588,43 @@ def test_table_overflow_retry_forced():
         got = ix.serialize()
         assert ix.stats()["table_retries"] >= 1
     assert_same_index(got, want)
+
+
+# ------------------------------------------------------------------ full-size multi-chunk configs
+def _fullsize_multichunk(cfg_id, chunks, **kw):
+    """Configs 3 / 4 at full chunk size (1 GiB per index_add_stream): every chunk after the
+    first probes and extends a non-empty dictionary (B-trees of height 3-4).  The GPU
+    index is SHA-256-identical to the doc-range-sharded oracle (oracle_add_mt over all host cores)."""
+    import os
+    threads = max(1, min(64, len(os.sched_getaffinity(0))))
+    o = oracle.Oracle()
+    with wj.Index(**kw) as ix:
+        for c in range(chunks):
+            text, off = gen.generate(gen.CONFIGS[cfg_id], chunk=c)
+            tt = torch.from_numpy(text).cuda()
+            to = torch.from_numpy(off.astype(np.int64)).cuda()
+            ix.add_stream(tt, to)
+            o.add(text, off, threads=threads)
+            torch.cuda.synchronize()
+            del tt, to
+        ix.finalize()
+        got = ix.serialize()
+        st = ix.stats()
+    want = o.serialize()
+    o.close()
+    assert _sha(got) == _sha(want)
+    wjformat.check_invariants(wjformat.parse(got))
+    return st
+
+
+@pytest.mark.slow
+def test_config3_full_size_4_chunks():
+    st = _fullsize_multichunk(3, 4)
+    assert st["n_chunks"] == 4 and st["btree_height_max"] >= 3
+
+
+@pytest.mark.slow
+def test_config4_full_size_prefix_2_chunks():
+    # Library-of-Congress shape: long documents, 1% hapax tokens (high new-term insert rate)
+    st = _fullsize_multichunk(4, 2)
+    assert st["n_chunks"] == 2 and st["new_terms_last"] > 100_000 and st["btree_height_max"] >= 3

@@ -4,7 +4,7 @@ cp $L /tmp/lib_orig.so
 for rep in $(seq ${REPS:-1}); do
 for v in $LIBS; do
   cp ablibs/lib_$v.so $L
-  env $ENVS python bench.py --steps ${STEPS:-20} --warmup 3 --e2e-steps 0 --no-cpu-baseline > gpurun_out/ab_$v.json 2>gpurun_out/ab_$v.err
+  env $ENVS python bench.py --steps ${STEPS:-20} --warmup 3 --e2e-steps 0 --no-cpu-baseline $BENCH_ARGS > gpurun_out/ab_$v.json 2>gpurun_out/ab_$v.err
   python - $v <<'PY'
 import json,sys
 d=json.load(open(f"gpurun_out/ab_{sys.argv[1]}.json"))
