@@ -406,23 +406,31 @@ def main():
             traffic = None
 
     phases = {k: (s1["phase_ms"][k] - s0["phase_ms"][k]) / args.steps for k in wj.PHASES}
+    # all-to-all-v rounds of the multi-rank path: bytes this rank sent per step, device-
+    # synchronised wall time of the rounds, fraction of 900 GB/s per direction (NVLink 5), max over ranks
+    xb = (s1["exchange_bytes"] - s0["exchange_bytes"]) / args.steps
+    xms = (s1["exchange_ms"] - s0["exchange_ms"]) / args.steps
+    if world > 1:
+        t = torch.tensor([xb, xms], device="cuda", dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        xb, xms = float(t[0].item()), float(t[1].item())
+    exchange = {"bytes_per_step": xb, "ms_per_step": xms,
+                "nvlink_frac": (xb / (xms / 1e3) / 900e9) if xms > 0 and xb > 0 else None,
+                "bytes_per_gib_text": xb / (T / 2**30)}
     kernels = {k: {"ms_per_step": kms[k] / args.steps, "launches_per_step": kcnt[k] / args.steps} for k in wj.KERNELS}
 
     # e2e through the public API with host buffers: H2D of the chunk inside, D2H of the whole index.
     # --e2e-chunks S > 1 feeds the step's text as S pinned host chunks to a context with the host
     # pipeline (Fig. 9: the copy of chunk c+1 overlaps the indexing of chunk c).
-    e2e = None
-    if args.e2e_steps > 0:
+    def e2e_leg(vbyte):
         S = max(1, args.e2e_chunks)
-        ixe = ix
-        if S > 1:
-            nid2 = [None]
-            if world > 1 or force_dist:  # a fresh communicator for the second context
-                nid2 = [wj.nccl_unique_id() if rank == 0 else None]
-                if world > 1:
-                    dist.broadcast_object_list(nid2, src=0)
-            ixe = wj.Index(device=local, rank=rank, world=world, vbyte=args.vbyte, pipeline=True, nccl_id=nid2[0],
-                           balanced=world > 1)
+        nid2 = [None]
+        if world > 1 or force_dist:  # a fresh communicator for the second context
+            nid2 = [wj.nccl_unique_id() if rank == 0 else None]
+            if world > 1:
+                dist.broadcast_object_list(nid2, src=0)
+        ixe = wj.Index(device=local, rank=rank, world=world, vbyte=vbyte, pipeline=S > 1, nccl_id=nid2[0],
+                       balanced=world > 1)
         nd = len(doc_off) - 1
         cuts = sorted({0, nd} | {int(np.searchsorted(doc_off, T * k // S)) for k in range(1, S)})
         parts = []
@@ -455,13 +463,19 @@ def main():
             t = torch.tensor([ems], device="cuda")
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ems = float(t.item())
-        e2e = {"value": total_bytes / (ems / 1e3) / 1e6, "unit": "MB/s", "ms_per_step": ems,
-               "h2d_bytes_per_step": T + 8 * (nd + len(parts)), "d2h_bytes_per_step": out_bytes,
-               "host_chunks": len(parts),
-               "what": ("index_add_stream(pinned host text + doc_off%s) + index_finalize + index_serialize to pinned host"
-                        % (f", {len(parts)} chunks, WJ_FLAG_HOST_PIPELINE" if len(parts) > 1 else ""))}
-        if ixe is not ix:
-            ixe.close()
+        ixe.close()
+        return {"value": total_bytes / (ems / 1e3) / 1e6, "unit": "MB/s", "ms_per_step": ems,
+                "h2d_bytes_per_step": T + 8 * (nd + len(parts)), "d2h_bytes_per_step": out_bytes,
+                "host_chunks": len(parts),
+                "what": ("index_add_stream(pinned host text + doc_off%s) + index_finalize + index_serialize (%s) to "
+                         "pinned host" % (f", {len(parts)} chunks, WJ_FLAG_HOST_PIPELINE" if len(parts) > 1 else "",
+                                          "WJINV002 d-gap + vbyte postings" if vbyte else "WJINV001"))}
+
+    e2e = e2e_vbyte = None
+    if args.e2e_steps > 0:
+        e2e = e2e_leg(args.vbyte)
+        if not args.vbyte:  # the compressed output format: less than half the D2H bytes
+            e2e_vbyte = e2e_leg(True)
 
     steady = None
     if args.steady_chunks > 0 and world == 1 and not force_dist:
@@ -482,7 +496,7 @@ def main():
                        "postings_format": "vbyte d-gaps (WJINV002)" if args.vbyte else "u32 docid + u32 tf (WJINV001)",
                        "parallelism": "single GPU" if world == 1 else
                        f"{world} ranks: document ranges, trie collections bin-packed by sampled load (P:212), NCCL all-to-all-v"},
-            "exchange_bytes_per_step": (s1["exchange_bytes"]),
+            "exchange": exchange,
             "mib_per_s": total_bytes / (ms / 1e3) / 2**20,
             "tokens_per_s": N * world / (ms / 1e3),
             "roofline": {"bound": "hbm", "scope": "whole step (SURVEY 8(d) compulsory bytes)", "achieved": step_gbs,
@@ -499,6 +513,7 @@ def main():
                                   "def": "implementation bytes of DESIGN.md section 7 (design evidence, not the headline)"},
             "cpu_baseline": cpu,
             "e2e": e2e,
+            "e2e_vbyte": e2e_vbyte,
             "steady_state": steady,
             "gpu_launches": int(round(launches * args.steps)),
             "gpu_launches_per_step": launches,

@@ -225,9 +225,9 @@ struct wj_index {
 
   Transport* xport = nullptr;  // world > 1
   // sampled hot terms of the current chunk (hot.cuh): hot_slotb = hot id -> chunk-table slot
-  DevBuf hot_samp, hot_slotb, hot_kb, samp_off, samp_slot, samp_doc, samp_cnt, samp_ck, samp_cv,
+  DevBuf hot_samp, hot_slotb, hot_kb, hot_matb, hot_posb, hot_cfb, hot_nhb, samp_off, samp_slot, samp_doc, samp_cnt, samp_ck, samp_cv,
       samp_ck2, samp_cv2, samp_n;
-  uint32_t hot_H = 0;
+  uint32_t hot_H = 0, hot_D = 0;  // hot terms of the current chunk (matrix rows), its documents
   bool stream_has_hot = false;  // some chunk appended hot-term elements (holes + counts > 1)
   // Partial postings per chunk (partials.cuh; single GPU, no stemming / stop words / hot terms): the
   // chunk's stream is sorted by slot and run-length encoded on side_st while the dictionary update
@@ -244,7 +244,9 @@ struct wj_index {
   uint32_t side_ctas = kRsCtas;      // ... for the side stream's sort (148 / 222 measured slower)
   bool pc_pending = false;           // the last chunk's posting count is still on the device (dscal[13])
   bool pc_join = false;              // the last chunk's side-stream work is not joined yet
-  uint64_t pc_U = 0, pc_Nc = 0;
+  uint64_t pc_U = 0, pc_Nc = 0, Ns_last = 0;  // pc_Nc: stream tokens of the pending chunk
+  bool pc_hot = false;                         // the pending chunk has hot-term lists
+  uint32_t doc_base_cur = 0;                   // first DocID of the chunk being indexed
   std::vector<uint64_t> rec_end;     // end of each chunk's records
   uint64_t sorted_elems = 0;    // stream elements the last finalize sorted (after hole compaction)
   // Sampled hot terms (hot.cuh) merged per document in the emit kernel: opt-in
@@ -361,7 +363,7 @@ struct wj_index {
       b->p = nullptr;
       b->cap = 0;
     }
-    DevBuf* hs[] = {&hot_samp, &hot_slotb, &hot_kb, &samp_off, &samp_slot, &samp_doc, &samp_cnt,
+    DevBuf* hs[] = {&hot_samp, &hot_slotb, &hot_kb, &hot_matb, &hot_posb, &hot_cfb, &hot_nhb, &samp_off, &samp_slot, &samp_doc, &samp_cnt,
                     &samp_ck, &samp_cv, &samp_ck2, &samp_cv2, &samp_n};
     for (DevBuf* b : hs) { dev_free(b->p); *b = DevBuf{}; }
     DevBuf* xs[] = {&x_owner, &x_iota, &x_sorted, &x_sorted2, &x_owner2, &x_xid, &x_cnt, &x_toff, &x_boff, &x_send,
@@ -568,7 +570,8 @@ struct wj_index {
     if (clear_table) WJ_CUDA_CHECK(cudaMemsetAsync(tab, 0, C * sizeof(Slot), st));
     WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 5, 0, 8, st));
     EmitOut eo;
-    eo.hot_slot = (use_hot && hot_H) ? (const uint32_t*)hot_slotb.p : nullptr;
+    eo.hot_mat = (use_hot && hot_H) ? (uint32_t*)hot_matb.p : nullptr;
+    eo.hot_docs = hot_D;
     eo.table = tab;
     eo.slot_ref = sref;
     eo.cap = (uint32_t)C;
@@ -579,11 +582,9 @@ struct wj_index {
     eo.dbg_len = dlen;
     eo.overflow = (uint32_t*)(dscal() + 5);
     const uint64_t ranges = (n_segs + kSegsPerWarp - 1) / kSegsPerWarp;
-    const uint32_t sub = eo.hot_slot ? emit_sub<true>() : emit_sub<false>();
-    const uint64_t warps = (ranges + sub - 1) / sub;  // a warp walks `sub` ranges
-    const unsigned grid = (unsigned)((warps + kTokWarps - 1) / kTokWarps);
+    const unsigned grid = (unsigned)((ranges + kTokWarps - 1) / kTokWarps);
     ktime(WJ_KERNEL_TOKENIZE_EMIT, [&] {
-      if (eo.hot_slot)
+      if (eo.hot_mat)
         k_tok_emit<true><<<grid, kTokThreads, 0, st>>>(cv, (uint32_t)n_segs, (const uint64_t*)kstart.p,
                                                        (const uint32_t*)seg_cnt.p, eo);
       else
@@ -742,7 +743,11 @@ struct wj_index {
     U = 0;
     phase(WJ_PHASE_TOKENIZE);
     hot_H = 0;
-    if (allow_hot && cv.n_bytes >= hot_min_bytes && cv.n_docs > 0) hot_H = select_hot(cv);
+    hot_D = (uint32_t)cv.n_docs;
+    if (allow_hot && cv.n_bytes >= hot_min_bytes && cv.n_docs > 0) {
+      hot_H = select_hot(cv);
+      hot_H = (uint32_t)std::min<uint64_t>(hot_H, (64ull << 20) / cv.n_docs);  // matrix <= 256 MB
+    }
     const uint64_t Nc = count_tokens(cv, n_segs);
     n_dropped += h_scal[1];
     out_alloc(Nc, slot_out, doc_out);
@@ -760,6 +765,8 @@ struct wj_index {
       uint32_t* sref = buf<uint32_t>(slotref, C);
       WJ_CUDA_CHECK(cudaMemsetAsync(tab, 0, C * sizeof(Slot), st));
       if (hot_H) {  // hot terms first: their slots in this table carry their hot ids
+        uint32_t* mat = buf<uint32_t>(hot_matb, (uint64_t)hot_H * hot_D);
+        WJ_CUDA_CHECK(cudaMemsetAsync(mat, 0, (uint64_t)hot_H * hot_D * 4, st));
         WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 5, 0, 8, st));
         k_hot_seed<<<1, 128, 0, st>>>((const ulonglong2*)hot_kb.p, hot_H, tab, sref, (uint32_t)C,
                                       (uint32_t*)hot_slotb.p, (uint32_t*)(dscal() + 5));
@@ -963,6 +970,10 @@ struct wj_index {
   // term's key (key & kRankMask); the posting count is left in dscal[8] (u32, no host round trip)
   void rle(const uint32_t* key, const uint32_t* docs, uint64_t N, bool counts, uint32_t* od, uint32_t* of, uint64_t* po,
            uint64_t* csp) {
+    if (N == 0) {  // e.g. every token of the chunk was a hot term
+      WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 8, 0, 8, st));
+      return;
+    }
     uint64_t per = (N + 148 * 2 - 1) / (148 * 2);
     per = (per + kRleTile - 1) / kRleTile * kRleTile;
     const uint32_t G = (uint32_t)((N + per - 1) / per);
@@ -1019,10 +1030,23 @@ struct wj_index {
       // holes (merged hot tokens, key 0) are dropped by the first pass: Ns elements remain
       uint64_t Ns = Nc;
       const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, bits, nullptr, true, nullptr, kRankMask, hot, &Ns);
+      Ns_last = Ns;
       hot_elems_saved += Nc - Ns;
       pm_merged += Nc - Ns;
       phase(WJ_PHASE_POSTINGS);
-      rle(in1 ? k1 : kt, in1 ? v1 : dt, Ns, hot, od + pbase, of + pbase, po, cs);
+      rle(in1 ? k1 : kt, in1 ? v1 : dt, Ns, false, od + pbase, of + pbase, po, cs);
+      if (hot) {  // the hot matrix rows -> the hot terms' partial lists, after the run-length postings
+        const uint64_t HD = (uint64_t)hot_H * hot_D;
+        uint32_t* hp = buf<uint32_t>(hot_posb, HD + 1);
+        uint32_t* hcf = buf<uint32_t>(hot_cfb, hot_H);
+        const uint32_t* mat = (const uint32_t*)hot_matb.p;
+        scan<uint32_t>(NonZeroU32{mat}, HD, hp, hp + HD);
+        k_hot_scatter<<<grid_for(HD, 256), 256, 0, st>>>(mat, HD, hot_D, hp, (const uint32_t*)(dscal() + 8),
+                                                         doc_base_cur, od + pbase, of + pbase);
+        k_hot_rowsum<<<hot_H, 256, 0, st>>>(mat, hot_D, hcf);
+        k_hot_total<<<1, 1, 0, st>>>(hp + HD, (uint32_t*)(dscal() + 8), (uint32_t*)(dscal() + 12));
+        launched(3);
+      }
       phase(-1);
       WJ_CUDA_CHECK(cudaEventRecord(ev_side, st));
     } catch (...) {
@@ -1046,7 +1070,8 @@ struct wj_index {
     WJ_CUDA_CHECK(cudaStreamWaitEvent(st, ev_dict, 0));
     pc_join = true;
     pc_U = U;
-    pc_Nc = Nc;
+    pc_Nc = Ns_last;
+    pc_hot = hot;
   }
 
   // Join the last chunk's side-stream work and write its records; runs before the next chunk's
@@ -1063,9 +1088,16 @@ struct wj_index {
     uint64_t* rs = buf_keep<uint64_t>(rec_start, nrec + U, nrec);
     uint32_t* rd = buf_keep<uint32_t>(rec_df, nrec + U, nrec);
     uint32_t* rc = buf_keep<uint32_t>(rec_cf, nrec + U, nrec);
-    k_chunk_records<<<grid_for(U, 256), 256, 0, st>>>((const uint32_t*)u_slot.p, (uint32_t)U, po, cs,
-                                                      (const uint32_t*)(dscal() + 8), Nc, (const uint32_t*)u_tid.p, pbase,
-                                                      rt + nrec, rs + nrec, rd + nrec, rc + nrec);
+    const uint32_t* nh = nullptr;
+    if (pc_hot) {  // records in partial-list order: non-hot terms (slot order), then the hot terms
+      uint32_t* p = buf<uint32_t>(hot_nhb, U + 1);
+      scan<uint32_t>(NotHotSlot{(const uint32_t*)u_slot.p, (const Slot*)table.p}, U, p, p + U);
+      nh = p;
+    }
+    k_chunk_records<<<grid_for(U, 256), 256, 0, st>>>(
+        (const uint32_t*)u_slot.p, (uint32_t)U, po, cs, (const uint32_t*)(dscal() + (pc_hot ? 12 : 8)), Nc,
+        (const uint32_t*)u_tid.p, pbase, rt + nrec, rs + nrec, rd + nrec, rc + nrec, (const Slot*)table.p,
+        pc_hot ? (const uint32_t*)hot_posb.p : nullptr, (const uint32_t*)hot_cfb.p, hot_D, nh, pc_hot ? hot_H : 0u);
     launched();
     WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 13, dscal() + 8, 8, cudaMemcpyDeviceToHost, st));
     pc_pending = true;
@@ -1149,6 +1181,7 @@ struct wj_index {
     }
     if (n_docs + nd > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 documents"};
     const uint32_t doc_base = (uint32_t)n_docs;
+    doc_base_cur = doc_base;
     if (nd == 0 || n_bytes == 0) {
       n_docs += nd;
       phase(-1);
@@ -1168,7 +1201,7 @@ struct wj_index {
       if (n_elems + nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 stream elements"};
       sp = buf_keep<uint32_t>(g_tid, n_elems + nc + 16, n_elems) + n_elems;  // +16: TMA round-up reads
       dp = buf_keep<uint32_t>(g_doc, n_elems + nc + 16, n_elems) + n_elems;
-    }, C, U, so, dout, !norm);
+    }, C, U, so, dout, pm && !norm);
     if (Nc > 0 && norm) {  // f4: stems / stop words
       uint64_t U2 = 0;
       const uint8_t* ntext = nullptr;
@@ -1204,13 +1237,13 @@ struct wj_index {
 
   // ---------------------------------------------------------------- one chunk, world > 1
   // Sender-side partial lists: every rank tokenises its own documents,
-  // groups its unique terms by owner (collection b -> b mod K, or the balanced map),
-  // sorts + run-length encodes its stream by (owner, term) into (docID, tf) postings written straight
-  // into its partial-list buffer, and sends each owner its terms (folded bytes), a (df, cf) header per
-  // term and that term's postings in one all-to-all-v round.  The owner deduplicates the received
-  // terms, updates its exclusive dictionary slice and appends one partial-list record per
-  // (source, term), in source-rank order = docID order; its own postings never move.  Finalize
-  // is the single-GPU partial-list combine.
+  // groups its unique terms by owner (collection b -> b mod K, or the balanced map) and
+  // sends each owner its terms (folded bytes) first; then, overlapped, it sorts + run-length encodes its
+  // stream by (owner, term) into (docID, tf) postings on the side stream while, as an owner, it
+  // deduplicates the received terms and updates its exclusive dictionary slice on the
+  // dictionary stream.  A second all-to-all-v moves a (df, cf) header per term and the postings grouped
+  // per term; the owner appends one partial-list record per (source, term) in source-rank
+  // order = docID order, and finalize is the single-GPU partial-list combine.
   void add_chunk_dist_pl(const uint8_t* text, uint64_t n_bytes, const uint64_t* off, uint64_t nd) {
     const int K = world;
     phase(WJ_PHASE_EXCHANGE);
@@ -1237,12 +1270,11 @@ struct wj_index {
         if (nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 tokens in one chunk"};
         sp = buf<uint32_t>(pc_key, nc + 16);
         dp = buf<uint32_t>(pc_doc, nc + 16);
-      }, C, U, lslot, ldoc, true);
+      }, C, U, lslot, ldoc, false);
     }
-    const bool hot = hot_H > 0;
     std::vector<uint64_t> t_off(K + 1, 0), b_off(K + 1, 0), p_off(K + 1, 0), c_off(K + 1, 0);
     uint8_t* send_terms = (uint8_t*)grow(x_send, 16);
-    uint64_t P_local = 0;
+    uint64_t* toff_d = buf<uint64_t>(x_toff, K + 1);
     // the chunk's postings: K == 1 straight into the partial-list buffer; K > 1 into scratch, from where
     // every owner's range (the own one by a device copy) lands in the owners' partial-list buffers in
     // source-rank order, so each chunk's partial lists are back to back in record order
@@ -1254,12 +1286,14 @@ struct wj_index {
       od = buf<uint32_t>(x_rkey, Nc + 16);
       of = buf<uint32_t>(x_rdoc, Nc + 16);
     }
+    uint32_t* hdf = buf<uint32_t>(x_hdf, U + 1);
+    uint32_t* hcf = buf<uint32_t>(x_hcf, U + 1);
+    uint64_t* bnd = buf<uint64_t>(x_bnd, 2 * (K + 1));
+    uint32_t* km = nullptr;
     if (U > 0) {
       // 2. unique terms grouped by owner (stable): t_off, xid, gpos map, packed term bytes
       uint32_t* own = buf<uint32_t>(x_owner, U + 16);
       uint32_t* iota = buf<uint32_t>(x_iota, U + 16);
-      uint32_t* own2 = buf<uint32_t>(x_owner2, U + 16);
-      uint32_t* srt2 = buf<uint32_t>(x_sorted2, U + 16);
       uint32_t* oc = buf<uint32_t>(x_cnt, 2 * K);
       WJ_CUDA_CHECK(cudaMemsetAsync(oc, 0, 2 * K * 4, st));
       k_owner<<<grid_for(U, 256), 256, 0, st>>>((const uint32_t*)u_bucket.p, (uint32_t)U, (uint32_t)K,
@@ -1267,6 +1301,8 @@ struct wj_index {
       launched();
       const uint32_t* sorted_u = iota;
       if (K > 1) {
+        uint32_t* own2 = buf<uint32_t>(x_owner2, U + 16);
+        uint32_t* srt2 = buf<uint32_t>(x_sorted2, U + 16);
         WJ_CUDA_CHECK(cudaMemcpyAsync(own2, own, U * 4, cudaMemcpyDeviceToDevice, st));
         int obits = 0;
         while ((1 << obits) < K) ++obits;
@@ -1277,19 +1313,55 @@ struct wj_index {
       WJ_CUDA_CHECK(cudaMemcpyAsync(oc_h.data(), oc, K * 4, cudaMemcpyDeviceToHost, st));
       sync();
       for (int o = 0; o < K; ++o) t_off[o + 1] = t_off[o] + oc_h[o];
-      uint64_t* toff_d = buf<uint64_t>(x_toff, K + 1);
       WJ_CUDA_CHECK(cudaMemcpyAsync(toff_d, t_off.data(), (K + 1) * 8, cudaMemcpyHostToDevice, st));
       uint32_t* xid = buf<uint32_t>(x_xid, U);
       k_xid<<<grid_for(U, 256), 256, 0, st>>>(sorted_u, (uint32_t)U, own, toff_d, xid);
       launched();
-      uint32_t* km = buf<uint32_t>(x_keymap, C);
+      km = buf<uint32_t>(x_keymap, C);
       k_slot_gpos<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, (uint32_t)C, (const uint32_t*)uid.p, own, xid,
                                                     toff_d, km);
       launched();
       uint64_t* boff = buf<uint64_t>(x_boff, U + 1);
       scan<uint64_t>(PackTermSize{sorted_u, (const uint32_t*)u_len.p}, U, boff, boff + U);
-      // 3. the stream sorted by gpos (map applied by the first pass; holes of merged hot tokens dropped),
-      //    run-length encoded into this rank's partial-list buffer
+      for (int o = 0; o <= K; ++o)
+        WJ_CUDA_CHECK(cudaMemcpyAsync(&b_off[o], boff + t_off[o], 8, cudaMemcpyDeviceToHost, st));
+      sync();
+      send_terms = (uint8_t*)grow(x_send, b_off[K] + 16);
+      k_pack_terms<<<grid_for(U, 256), 256, 0, st>>>(sorted_u, (uint32_t)U, boff, (const uint4*)u_w.p, text,
+                                                    (const uint32_t*)u_ref.p, (const uint32_t*)u_len.p, send_terms);
+      launched();
+    }
+    // 3. first exchange: the terms (folded bytes) to their owners
+    std::vector<uint64_t> cnt(2 * K, 0), all(2 * K * K);
+    for (int o = 0; o < K; ++o) {
+      cnt[o] = t_off[o + 1] - t_off[o];
+      cnt[K + o] = b_off[o + 1] - b_off[o];
+    }
+    xport->allgather(cnt.data(), 2 * K, all.data(), st);
+    std::vector<uint64_t> rt(K + 1, 0), rb(K + 1, 0);
+    for (int s = 0; s < K; ++s) {
+      const uint64_t* c = all.data() + (size_t)s * 2 * K;
+      rt[s + 1] = rt[s] + c[rank];
+      rb[s + 1] = rb[s] + c[K + rank];
+    }
+    const uint64_t RT = rt[K];
+    uint8_t* recv_terms = (uint8_t*)grow(x_recv_terms, rb[K] + 32);
+    const uint64_t t0 = xport->sent;
+    double xms = 0;
+    auto exchange = [&](auto&& f) {
+      const auto tx = std::chrono::steady_clock::now();
+      try {
+        f();
+      } catch (const ExchangeError& e) {
+        throw StatusError{WJ_ERR_NCCL, e.msg};
+      }
+      WJ_CUDA_CHECK(cudaStreamSynchronize(st));
+      xms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - tx).count();
+    };
+    exchange([&] { xport->alltoallv(send_terms, b_off.data(), recv_terms, rb.data(), st); });
+    // 4. overlapped: side stream = the local stream sorted by gpos (map applied by the first pass) and
+    //    run-length encoded, headers, per-owner bounds; dictionary stream = the owner's dictionary
+    if (U > 0) {
       int bits = 0;
       while (bits < 32 && ((uint64_t)1 << bits) < U) ++bits;
       uint32_t* kt = (uint32_t*)pc_key.p;
@@ -1298,110 +1370,110 @@ struct wj_index {
       uint32_t* v1 = buf<uint32_t>(sv1, Nc + 16);
       uint64_t* po = buf<uint64_t>(pc_po, U + 1);
       uint64_t* cs = buf<uint64_t>(pc_cs, U + 1);
-      phase(WJ_PHASE_SORT);
-      std::vector<std::pair<uint64_t, const uint32_t*>> segs{{0, km}};
-      uint64_t Ns = Nc;
-      bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, std::max(bits, 1), nullptr, true, &segs, kRankMask, hot,
-                                      &Ns);
-      hot_elems_saved += Nc - Ns;
-      phase(WJ_PHASE_POSTINGS);
-      rle(in1 ? k1 : kt, in1 ? v1 : dt, Ns, hot, od, of, po, cs);
-      phase(WJ_PHASE_EXCHANGE);
-      uint32_t* hdf = buf<uint32_t>(x_hdf, U);
-      uint32_t* hcf = buf<uint32_t>(x_hcf, U);
-      k_term_hdr<<<grid_for(U, 256), 256, 0, st>>>(po, cs, (uint32_t)U, (const uint32_t*)(dscal() + 8), Nc, hdf, hcf);
-      launched();
-      uint64_t* bnd = buf<uint64_t>(x_bnd, 2 * (K + 1));
-      k_owner_bounds<<<grid_for(K + 1, 256), 256, 0, st>>>(po, cs, toff_d, (uint32_t)K, (uint32_t)U,
-                                                          (const uint32_t*)(dscal() + 8), Nc, bnd, bnd + K + 1);
-      launched();
-      std::vector<uint64_t> hb(2 * (K + 1));
-      WJ_CUDA_CHECK(cudaMemcpyAsync(hb.data(), bnd, hb.size() * 8, cudaMemcpyDeviceToHost, st));
-      for (int o = 0; o <= K; ++o)
-        WJ_CUDA_CHECK(cudaMemcpyAsync(&b_off[o], boff + t_off[o], 8, cudaMemcpyDeviceToHost, st));
-      sync();
-      for (int o = 0; o <= K; ++o) {
-        p_off[o] = hb[o];
-        c_off[o] = hb[K + 1 + o];
+      phase(-1);
+      WJ_CUDA_CHECK(cudaEventRecord(ev_fork, st));
+      WJ_CUDA_CHECK(cudaStreamWaitEvent(side_st, ev_fork, 0));
+      swap_side();
+      try {
+        phase(WJ_PHASE_SORT);
+        std::vector<std::pair<uint64_t, const uint32_t*>> segs{{0, km}};
+        const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, std::max(bits, 1), nullptr, true, &segs, kRankMask);
+        phase(WJ_PHASE_POSTINGS);
+        rle(in1 ? k1 : kt, in1 ? v1 : dt, Nc, false, od, of, po, cs);
+        k_term_hdr<<<grid_for(U, 256), 256, 0, st>>>(po, cs, (uint32_t)U, (const uint32_t*)(dscal() + 8), Nc, hdf, hcf);
+        k_owner_bounds<<<grid_for(K + 1, 256), 256, 0, st>>>(po, cs, toff_d, (uint32_t)K, (uint32_t)U,
+                                                            (const uint32_t*)(dscal() + 8), Nc, bnd, bnd + K + 1);
+        launched(2);
+        phase(-1);
+        WJ_CUDA_CHECK(cudaEventRecord(ev_side, st));
+      } catch (...) {
+        swap_side();
+        throw;
       }
-      P_local = p_off[K];
-      send_terms = (uint8_t*)grow(x_send, b_off[K] + 16);
-      k_pack_terms<<<grid_for(U, 256), 256, 0, st>>>(sorted_u, (uint32_t)U, boff, (const uint4*)u_w.p, text,
-                                                    (const uint32_t*)u_ref.p, (const uint32_t*)u_len.p, send_terms);
-      launched();
+      swap_side();
+    } else {
+      WJ_CUDA_CHECK(cudaMemsetAsync(bnd, 0, 2 * (K + 1) * 8, st));
+      WJ_CUDA_CHECK(cudaEventRecord(ev_side, st));
     }
-    // 4. exchange: per owner [terms, term bytes, postings, tokens]; then the term bytes, the headers and
-    //    the postings (own postings stay in place: zero-size self segment)
-    std::vector<uint64_t> cnt(4 * K, 0), all(4 * K * K);
+    uint32_t* sslot = nullptr;
+    if (RT > 0) {  // the owner's dictionary on the high-priority stream
+      WJ_CUDA_CHECK(cudaEventRecord(ev_fork, st));
+      WJ_CUDA_CHECK(cudaStreamWaitEvent(hp_st, ev_fork, 0));
+      std::swap(st, hp_st);
+      try {
+        uint64_t* so = buf<uint64_t>(x_syn_off, 2);
+        const uint64_t h2[2] = {0, rb[K]};
+        WJ_CUDA_CHECK(cudaMemcpyAsync(so, h2, 16, cudaMemcpyHostToDevice, st));
+        ChunkView sv{recv_terms, rb[K], so, 1};
+        uint64_t C2 = 0, U2 = 0;
+        uint32_t* sdoc = nullptr;
+        const uint64_t dropped0 = n_dropped;
+        const uint64_t Ns2 = tokenize_dedup(sv, 0, [&](uint64_t nc, uint32_t*& sp2, uint32_t*& dp2) {
+          sp2 = buf<uint32_t>(x_syn_slot, nc + 16);
+          dp2 = buf<uint32_t>(x_syn_doc, nc + 16);
+        }, C2, U2, sslot, sdoc);
+        n_dropped = dropped0;
+        if (Ns2 != RT) throw StatusError{WJ_ERR_CUDA, "received term text: token count mismatch (internal)"};
+        dictionary_update(recv_terms, U2);
+        phase(-1);
+        WJ_CUDA_CHECK(cudaEventRecord(ev_dict, st));
+      } catch (...) {
+        std::swap(st, hp_st);
+        throw;
+      }
+      std::swap(st, hp_st);
+      WJ_CUDA_CHECK(cudaStreamWaitEvent(st, ev_dict, 0));
+    }
+    WJ_CUDA_CHECK(cudaStreamWaitEvent(st, ev_side, 0));
+    phase(WJ_PHASE_EXCHANGE);
+    std::vector<uint64_t> hb(2 * (K + 1));
+    WJ_CUDA_CHECK(cudaMemcpyAsync(hb.data(), bnd, hb.size() * 8, cudaMemcpyDeviceToHost, st));
+    sync();
+    for (int o = 0; o <= K; ++o) {
+      p_off[o] = hb[o];
+      c_off[o] = hb[K + 1 + o];
+    }
+    // 5. second exchange: per owner [postings, tokens]; then the headers and the postings
+    std::vector<uint64_t> cnt2(2 * K, 0), all2(2 * K * K);
     for (int o = 0; o < K; ++o) {
-      cnt[o] = t_off[o + 1] - t_off[o];
-      cnt[K + o] = b_off[o + 1] - b_off[o];
-      cnt[2 * K + o] = p_off[o + 1] - p_off[o];
-      cnt[3 * K + o] = c_off[o + 1] - c_off[o];
+      cnt2[o] = p_off[o + 1] - p_off[o];
+      cnt2[K + o] = c_off[o + 1] - c_off[o];
     }
-    xport->allgather(cnt.data(), 4 * K, all.data(), st);
-    std::vector<uint64_t> rt(K + 1, 0), rb(K + 1, 0), rp(K + 1, 0);
+    xport->allgather(cnt2.data(), 2 * K, all2.data(), st);
+    std::vector<uint64_t> rp(K + 1, 0);
     uint64_t my_tokens = 0;
     for (int s = 0; s < K; ++s) {
-      const uint64_t* c = all.data() + (size_t)s * 4 * K;
-      rt[s + 1] = rt[s] + c[rank];
-      rb[s + 1] = rb[s] + c[K + rank];
-      rp[s + 1] = rp[s] + c[2 * K + rank];
-      my_tokens += c[3 * K + rank];
+      const uint64_t* c = all2.data() + (size_t)s * 2 * K;
+      rp[s + 1] = rp[s] + c[rank];
+      my_tokens += c[K + rank];
     }
-    const uint64_t RT = rt[K], RP = rp[K];  // RP: postings of this owner's terms over all sources
-    uint8_t* recv_terms = (uint8_t*)grow(x_recv_terms, rb[K] + 32);
+    const uint64_t RP = rp[K];  // postings of this owner's terms over all sources
     uint32_t* rhdf = buf<uint32_t>(x_rhdf, RT + 1);
     uint32_t* rhcf = buf<uint32_t>(x_rhcf, RT + 1);
-    uint32_t* hdf = buf<uint32_t>(x_hdf, std::max<uint64_t>(U, 1));
-    uint32_t* hcf = buf<uint32_t>(x_hcf, std::max<uint64_t>(U, 1));
-    std::vector<uint64_t> s4(K + 1), r4(K + 1), rpb(K + 1);
+    std::vector<uint64_t> s4(K + 1), r4(K + 1);
     for (int o = 0; o <= K; ++o) {
       s4[o] = t_off[o] * 4;
       r4[o] = rt[o] * 4;
     }
-    const uint64_t t0 = xport->sent;
-    {
-      const auto tx = std::chrono::steady_clock::now();
-      try {
-        xport->alltoallv(send_terms, b_off.data(), recv_terms, rb.data(), st);
-        xport->alltoallv(hdf, s4.data(), rhdf, r4.data(), st);
-        xport->alltoallv(hcf, s4.data(), rhcf, r4.data(), st);
-        if (K > 1) {  // postings: owner o's range of the scratch -> o's partial-list buffer
-          uint32_t* pd = buf_keep<uint32_t>(pp_doc, pbase + RP + 16, pbase) + pbase;
-          uint32_t* pt = buf_keep<uint32_t>(pp_tf, pbase + RP + 16, pbase) + pbase;
-          std::vector<uint64_t> spb(K + 1);
-          for (int o = 0; o <= K; ++o) {
-            spb[o] = p_off[o] * 4;
-            rpb[o] = rp[o] * 4;
-          }
-          xport->alltoallv(od, spb.data(), pd, rpb.data(), st);
-          xport->alltoallv(of, spb.data(), pt, rpb.data(), st);
+    exchange([&] {
+      xport->alltoallv(hdf, s4.data(), rhdf, r4.data(), st);
+      xport->alltoallv(hcf, s4.data(), rhcf, r4.data(), st);
+      if (K > 1) {  // postings: owner o's range of the scratch -> o's partial-list buffer
+        uint32_t* pd = buf_keep<uint32_t>(pp_doc, pbase + RP + 16, pbase) + pbase;
+        uint32_t* pt = buf_keep<uint32_t>(pp_tf, pbase + RP + 16, pbase) + pbase;
+        std::vector<uint64_t> spb(K + 1), rpb(K + 1);
+        for (int o = 0; o <= K; ++o) {
+          spb[o] = p_off[o] * 4;
+          rpb[o] = rp[o] * 4;
         }
-      } catch (const ExchangeError& e) {
-        throw StatusError{WJ_ERR_NCCL, e.msg};
+        xport->alltoallv(od, spb.data(), pd, rpb.data(), st);
+        xport->alltoallv(of, spb.data(), pt, rpb.data(), st);
       }
-      WJ_CUDA_CHECK(cudaStreamSynchronize(st));
-      exchange_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - tx).count();
-    }
+    });
+    exchange_ms += xms;
     exchange_bytes += xport->sent - t0;
-    // 5. owner side: the received terms through the tokenizer / dedup / dictionary, then one record
-    //    per (source, term) in source-rank order
+    // 6. owner side: one record per (source, term) in source-rank order
     if (RT > 0) {
-      uint64_t* so = buf<uint64_t>(x_syn_off, 2);
-      const uint64_t h2[2] = {0, rb[K]};
-      WJ_CUDA_CHECK(cudaMemcpyAsync(so, h2, 16, cudaMemcpyHostToDevice, st));
-      ChunkView sv{recv_terms, rb[K], so, 1};
-      uint64_t C2 = 0, U2 = 0;
-      uint32_t *sslot = nullptr, *sdoc = nullptr;
-      const uint64_t dropped0 = n_dropped;
-      const uint64_t Ns2 = tokenize_dedup(sv, 0, [&](uint64_t nc, uint32_t*& sp2, uint32_t*& dp2) {
-        sp2 = buf<uint32_t>(x_syn_slot, nc + 16);
-        dp2 = buf<uint32_t>(x_syn_doc, nc + 16);
-      }, C2, U2, sslot, sdoc);
-      n_dropped = dropped0;
-      if (Ns2 != RT) throw StatusError{WJ_ERR_CUDA, "received term text: token count mismatch (internal)"};
-      dictionary_update(recv_terms, U2);
       phase(WJ_PHASE_STREAM);
       uint64_t* pre = buf<uint64_t>(x_rpre, RT + 1);
       uint32_t* rtid = buf_keep<uint32_t>(rec_tid, nrec + RT, nrec);
@@ -1412,10 +1484,9 @@ struct wj_index {
         const uint64_t nt = rt[s + 1] - rt[s];
         if (nt == 0) continue;
         scan<uint64_t>(U32AsU64{rhdf + rt[s]}, nt, pre + rt[s], (uint64_t*)nullptr);
-        const uint64_t pb = pbase + rp[s];
         k_recv_records<<<grid_for(nt, 256), 256, 0, st>>>(sslot + rt[s], (uint32_t)nt, (const Slot*)table.p,
                                                           (const uint32_t*)uid.p, (const uint32_t*)u_tid.p, rhdf + rt[s],
-                                                          rhcf + rt[s], pre + rt[s], pb, rtid + nrec + rt[s],
+                                                          rhcf + rt[s], pre + rt[s], pbase + rp[s], rtid + nrec + rt[s],
                                                           rst + nrec + rt[s], rdf + nrec + rt[s], rcf + nrec + rt[s]);
         launched();
         rec_end.push_back(nrec + rt[s + 1]);
@@ -1429,7 +1500,8 @@ struct wj_index {
     sync();  // exchange buffers are reused by the next chunk
   }
 
-  // ---------------------------------------------------------------- one chunk, world > 1
+  // ---------------------------------------------------------------- one chunk, world > 1, global stream
+  // (stemming / stop words / WJ_FLAG_GLOBAL_STREAM): token records routed to the owners
   void add_chunk_dist(const uint8_t* text, uint64_t n_bytes, const uint64_t* off, uint64_t nd) {
     const int K = world;
     // DocID base = documents of earlier chunks + of lower ranks in this chunk
@@ -1781,6 +1853,7 @@ struct wj_index {
     bool in1 = false;
     uint64_t cur_n = n;
     for (int p = 0; p < passes; ++p) {
+      if (cur_n == 0) break;  // every element was a hole
       uint64_t per = (cur_n + rs_ctas - 1) / rs_ctas;
       per = (per + kOsTile - 1) / kOsTile * kOsTile;
       const uint32_t G = (uint32_t)((cur_n + per - 1) / per);

@@ -1,19 +1,21 @@
 // Sampled popular terms: the paper treats "popular" terms, "the most
 // frequently occurring terms", apart from the rest and decides membership on a sample, "1MB out of
-// every 1GB".  B200 re-design: per chunk, the first 1 MiB of its documents is
-// tokenised with the same kernels and the <= 127 most frequent terms (>= 16 occurrences, <= 11
-// bytes) become hot; k_hot_seed claims their slots in the chunk table first, with the hot id in the
-// slot's k1 (bits 57..63).  In k_tok_emit the tokens of one hot term that fall in one document of a
-// warp's 8 KB window become ONE stream element carrying their count (the other tokens leave holes),
-// so the sort and run-length passes see fewer elements (0.75 N on config 2).  The result is unchanged.
+// every 1GB".  B200 re-design (opt-in, WJ_FLAG_HOT_TERMS): per chunk, the first
+// 1 MiB of its documents is tokenised with the same kernels and the <= 64 most frequent terms
+// (>= 16 occurrences, <= 11 bytes) become hot; k_hot_seed claims their slots in the chunk table first,
+// with the hot id in the slot's k1 (bits 57..63).  k_tok_emit counts hot tokens in a dense (hot term x
+// document) matrix instead of the (slot, docID) stream (they leave holes there), so the sort and
+// run-length passes never see them; k_hot_scatter turns each matrix row into the term's partial
+// list (docIDs ascending by construction).  The result is unchanged.
 #pragma once
 #include "common.cuh"
 #include "tokenize.cuh"
 #include "dict.cuh"
+#include "scan.cuh"
 
 namespace wj {
 
-constexpr uint32_t kHotMax = 127;   // hot ids 1..127
+constexpr uint32_t kHotMax = kHotMaxH;  // hot ids 1..64 (tokenize.cuh)
 constexpr uint32_t kHotMinCount = 16;
 
 // hash of a term of <= 16 bytes from its folded words: identical to k_tok_emit's
@@ -85,6 +87,40 @@ __global__ void k_hot_seed(const ulonglong2* hk, uint32_t H, Slot* table, uint32
   const uint64_t h = term_hash16(w0, w1, w2, 0u, len);
   uint32_t hot = 0;
   hot_slot[id] = table_insert(nullptr, table, slot_ref, cap, h, k0, k1, 0u, len, nullptr, 0u, overflow, &hot);
+}
+
+struct NonZeroU32 {
+  const uint32_t* p;
+  __device__ __forceinline__ uint32_t operator()(uint64_t i) const { return p[i] != 0u ? 1u : 0u; }
+};
+
+// nonzero matrix entries -> the hot terms' partial lists, appended after the chunk's run-length
+// postings (*P_rle of them); pos = exclusive scan of the nonzero flags (row-major: term, document)
+__global__ void k_hot_scatter(const uint32_t* mat, uint64_t n, uint32_t D, const uint32_t* pos, const uint32_t* P_rle,
+                              uint32_t doc_base, uint32_t* od, uint32_t* of) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const uint32_t c = mat[i];
+  if (c == 0) return;
+  const uint64_t p = (uint64_t)*P_rle + pos[i];
+  od[p] = doc_base + (uint32_t)(i % D);
+  of[p] = c;
+}
+
+// tokens of each hot term (its cf): one block per matrix row
+__global__ void k_hot_rowsum(const uint32_t* mat, uint32_t D, uint32_t* cf) {
+  const uint32_t* row = mat + (uint64_t)blockIdx.x * D;
+  uint32_t s = 0;
+  for (uint32_t d = threadIdx.x; d < D; d += blockDim.x) s += row[d];
+  uint32_t tot;
+  block_exclusive_sum<uint32_t>(s, tot);
+  if (threadIdx.x == 0) cf[blockIdx.x] = tot;
+}
+
+// P_rle (run-length postings of the stream) is kept in *p_rle; *P becomes the chunk's total postings
+__global__ void k_hot_total(const uint32_t* hot_total, uint32_t* P, uint32_t* p_rle) {
+  *p_rle = *P;
+  *P += *hot_total;
 }
 
 }  // namespace wj

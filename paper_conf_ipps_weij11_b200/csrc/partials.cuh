@@ -16,28 +16,54 @@ namespace wj {
 
 // Per unique term u of a chunk (u ascending = slot ascending = the order of the sorted runs):
 // start / df / cf of its partial list from the run-length output (post_off / cstart indexed by slot).
+// With hot terms (hot_pos != nullptr) a hot slot (k1 hot id) has no stream elements: its list is row
+// h of the hot matrix, appended after the *P_rle run-length postings; a non-hot term's list ends where
+// the next non-hot term's begins (at most kHotMax hot terms lie in between).  NT = stream tokens.
+// With hot terms the records are ordered like the partial lists: non-hot terms in slot order at their
+// rank among the non-hot ones (nh_pos), then the H hot terms in hot-id order.
 __global__ void k_chunk_records(const uint32_t* __restrict__ u_slot, uint32_t U, const uint64_t* __restrict__ post_off,
-                                const uint64_t* __restrict__ cstart, const uint32_t* __restrict__ P_dev, uint64_t Nc,
+                                const uint64_t* __restrict__ cstart, const uint32_t* __restrict__ P_rle, uint64_t NT,
                                 const uint32_t* __restrict__ u_tid, uint64_t pbase, uint32_t* rec_tid,
-                                uint64_t* rec_start, uint32_t* rec_df, uint32_t* rec_cf) {
+                                uint64_t* rec_start, uint32_t* rec_df, uint32_t* rec_cf, const Slot* __restrict__ table,
+                                const uint32_t* __restrict__ hot_pos, const uint32_t* __restrict__ hot_cf, uint32_t D,
+                                const uint32_t* __restrict__ nh_pos, uint32_t H) {
   const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
   if (u >= U) return;
+  auto hot_of = [&](uint32_t slot) -> uint32_t {
+    return hot_pos ? (uint32_t)(table[slot].k1 >> kHotShift) : 0u;
+  };
   const uint32_t s = u_slot[u];
+  const uint32_t h = hot_of(s);
+  const uint32_t r = h ? U - H + (h - 1) : (hot_pos ? nh_pos[u] : u);
+  rec_tid[r] = u_tid[u];
+  if (h) {
+    const uint64_t a = hot_pos[(uint64_t)(h - 1) * D], b = hot_pos[(uint64_t)h * D];
+    rec_start[r] = pbase + *P_rle + a;
+    rec_df[r] = (uint32_t)(b - a);
+    rec_cf[r] = hot_cf[h - 1];
+    return;
+  }
   const uint64_t a = post_off[s], ta = cstart[s];
-  uint64_t b, tb;
-  if (u + 1 < U) {
-    const uint32_t s2 = u_slot[u + 1];
+  uint64_t b = *P_rle, tb = NT;
+  for (uint32_t v = u + 1; v < U; ++v) {
+    const uint32_t s2 = u_slot[v];
+    if (hot_of(s2)) continue;
     b = post_off[s2];
     tb = cstart[s2];
-  } else {
-    b = *P_dev;
-    tb = Nc;
+    break;
   }
-  rec_tid[u] = u_tid[u];
-  rec_start[u] = pbase + a;
-  rec_df[u] = (uint32_t)(b - a);
-  rec_cf[u] = (uint32_t)(tb - ta);
+  rec_start[r] = pbase + a;
+  rec_df[r] = (uint32_t)(b - a);
+  rec_cf[r] = (uint32_t)(tb - ta);
 }
+
+struct NotHotSlot {  // 1 for a unique term whose slot carries no hot id
+  const uint32_t* u_slot;
+  const Slot* table;
+  __device__ __forceinline__ uint32_t operator()(uint64_t u) const {
+    return (table[u_slot[u]].k1 >> kHotShift) ? 0u : 1u;
+  }
+};
 
 // One chunk's records, in chunk order: offset of the partial inside its term's list = postings of
 // the term in earlier chunks; termIDs are distinct within a chunk, so there is no conflict.

@@ -42,12 +42,13 @@ struct ChunkView {
 };
 
 struct EmitOut {
-  const uint32_t* hot_slot;  // hot id (1..127) -> its slot in this table; nullptr: no hot aggregation
+  uint32_t* hot_mat;       // HOT: (hot term x chunk document) token counts, hot_docs columns
+  uint32_t hot_docs;       // documents of the chunk
   Slot* table;             // chunk hash table
   uint32_t* slot_ref;      // per slot: first-occurrence offset (written by the inserter)
   uint32_t cap;            // capacity (slots; any value >= 1)
   uint32_t doc_base;       // global DocID of local document 0
-  uint32_t* slot;          // per kept token: slot | count << 25 (key 0 = hole: merged hot token)
+  uint32_t* slot;          // per kept token: slot | 1 << 25 (key 0 = hole: a hot token, HOT only)
   uint32_t* doc;           // per kept token: global DocID
   uint32_t* dbg_start;     // optional (debug): token start
   uint32_t* dbg_len;       // optional (debug): token length
@@ -379,255 +380,206 @@ __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* tabl
 #ifndef WJ_EMIT_MINB
 #define WJ_EMIT_MINB 6
 #endif
-// HOT (opt-in, WJ_FLAG_HOT_TERMS): a warp walks kHotSub consecutive count ranges (4 x 2 KB), the
-// window over which the tokens of a sampled hot term that fall in one
-// document are merged into one stream element carrying their count; merged tokens leave holes (key 0)
-// that the first sort pass drops.  Measured slower than the plain kernel on config 2 (the merge work
-// and 48 registers cost more in emit than the sort and run-length passes save; profiles/r02_README.md),
-// so the plain instantiation (one range per warp, no hot state, 40 registers) is the default.
-constexpr uint32_t kHotSub = 4;
-constexpr uint32_t kHotIds = 128;  // hot ids 1..127 (7 bits of the slot's k1)
-template <bool HOT>
-__host__ __device__ constexpr uint32_t emit_sub() { return HOT ? kHotSub : 1u; }
+// HOT (WJ_FLAG_HOT_TERMS): the <= kHotMaxH sampled hot terms of the chunk (SURVEY 8(f2)(ii),
+// P:202-208) do not enter the (slot, docID) stream: their tokens leave holes (key 0, dropped by the
+// first sort pass) and are counted in the dense (hot term x document) matrix eo.hot_mat, through
+// per-warp shared-memory counters for the first kHotDocs documents of the warp's range (flushed with
+// one global add per nonzero counter at the range's end); the matrix rows become the hot terms'
+// partial lists (k_hot_rows).
+constexpr uint32_t kHotMaxH = 64;
+constexpr uint32_t kHotDocs = 4;
+constexpr uint32_t kHotWords = kHotDocs * kHotMaxH / 2;  // u16 counter pairs per warp
 
 template <bool HOT>
-__global__ void __launch_bounds__(kTokThreads, HOT ? 5 : WJ_EMIT_MINB) k_tok_emit(ChunkView cv, uint32_t n_segs,
+__global__ void __launch_bounds__(kTokThreads, WJ_EMIT_MINB) k_tok_emit(ChunkView cv, uint32_t n_segs,
                                                           const uint64_t* kstart, const uint32_t* range_off, EmitOut eo) {
-  constexpr uint32_t kEmitSub = emit_sub<HOT>();
   __shared__ __align__(16) uint32_t win[kTokWarps][kWinBytes / 4];
   __shared__ uint32_t queue[kTokWarps][kQueueCap + 1];
   __shared__ uint32_t bnd[kTokWarps][32];
-  __shared__ uint32_t hacc[kTokWarps][HOT ? kHotIds : 1];  // per hot id: count << 16 | first position (warp-relative)
+  __shared__ uint32_t hcnt[kTokWarps][HOT ? kHotWords : 1];
   const uint32_t lane = lane_id();
   const int w = threadIdx.x >> 5;
-  const uint32_t n_ranges = (n_segs + kSegsPerWarp - 1) / kSegsPerWarp;
-  const uint32_t gw0 = (blockIdx.x * kTokWarps + w) * kEmitSub;
-  if (gw0 >= n_ranges) return;
+  const uint32_t gw = blockIdx.x * kTokWarps + w;
+  const uint32_t sb0 = gw * kSegsPerWarp;
+  if (sb0 >= n_segs) return;
+  const uint32_t se = min(sb0 + kSegsPerWarp, n_segs);
+  const uint32_t last = se < n_segs ? se : se - 1;
+  const uint32_t B0 = sb0 * kSegBytes;
   uint32_t* w32 = win[w];
   uint32_t* q = queue[w];
-  uint32_t* ha = hacc[w];
-  constexpr bool hot_on = HOT;
-  const uint64_t wbase = HOT ? range_off[gw0] : 0;  // output index of the warp's first token
-  uint32_t hdoc = 0;                                 // document of the accumulated hot counts
-  if (hot_on) {
-    for (uint32_t i = lane; i < kHotIds; i += 32) ha[i] = 0;
-    __syncwarp();
-  }
-  // accumulated hot elements -> stream (each at the output position of its first token)
-  auto hot_flush = [&]() {
-    if (!HOT) return;
-    for (uint32_t i = lane; i < kHotIds; i += 32) {
-      const uint32_t a = ha[i];
-      if (a >> 16) {
-        const uint64_t o = wbase + (a & 0xFFFFu);
-        __stcs(eo.slot + o, __ldg(&eo.hot_slot[i]) | ((a >> 16) << 25));
-        __stcs(eo.doc + o, hdoc);
-        ha[i] = 0;
+  uint32_t* hc = hcnt[w];
+  // stage the range and the look-ahead segment (tokens may run past the range)
+  uint4 v[kSegsPerWarp + 1];
+#pragma unroll
+  for (int j = 0; j <= kSegsPerWarp; ++j) v[j] = load_lane16(cv, sb0 + j);
+#pragma unroll
+  for (int j = 0; j <= kSegsPerWarp; ++j)  // fold A-Z once here (classification is case-blind)
+    *(uint4*)&w32[(j * kSegBytes + 16 * lane) / 4] =
+        make_uint4(lower4(v[j].x), lower4(v[j].y), lower4(v[j].z), lower4(v[j].w));
+  if (lane < 4) w32[(kWinBytes - 16) / 4 + lane] = 0;
+  if (HOT)
+    for (uint32_t i = lane; i < kHotWords; i += 32) hc[i] = 0;
+  __syncwarp();
+
+  const uint64_t k_range_lo = kstart[gw];
+  uint64_t kcur = k_range_lo;
+  uint32_t prev = prev_token_bit(cv, B0);
+  uint32_t qn = 0;
+  uint64_t obase = range_off[gw];
+  uint64_t k_range_hi = k_range_lo;
+  bool open = false;
+  uint32_t open_start = 0;
+
+  auto flush = [&]() {
+    for (uint32_t r = 0; r < qn; r += 32) {
+      const uint32_t idx = r + lane;
+      if (idx < qn) {
+        const uint32_t e = q[idx];
+        const uint32_t s_win = e >> 8, len = e & 255u;
+        const uint32_t s_abs = B0 + s_win;
+        // first 16 folded bytes: 5 window words, 4 funnel shifts, length masks
+        uint32_t wd[4];
+        {
+          const uint32_t a = s_win >> 2, sh = (s_win & 3) * 8;
+          uint32_t x[5];
+#pragma unroll
+          for (int k = 0; k < 5; ++k) x[k] = w32[a + k];
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const uint32_t rem = min(max((int)len - 4 * k, 0), 4);
+            wd[k] = __funnelshift_r(x[k], x[k + 1], sh) & __funnelshift_lc(0xFFFFFFFFu, 0u, rem * 8);
+          }
+        }
+        uint32_t h32 = hash_init(len);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) h32 = hash_mix(h32, wd[k]);
+        for (uint32_t k = 4; k * 4 < len; ++k) h32 = hash_mix(h32, win_word(w32, s_win, len, k));
+        h32 = hash_fin(h32);
+        const uint64_t h = h32;
+        // DocID = (number of doc_off[k] <= s, k < n_docs) - 1 (readings S9, S16)
+        uint64_t lo = k_range_lo, hi = k_range_hi;
+        while (lo < hi) {
+          const uint64_t mid = (lo + hi) >> 1;
+          if (cv.doc_off[mid] <= s_abs) lo = mid + 1; else hi = mid;
+        }
+        const uint32_t ldoc = (uint32_t)(lo - 1);  // chunk-local document
+        const uint64_t k0 = (uint64_t)len | ((uint64_t)hash_tag(h32) << 8) | ((uint64_t)wd[0] << 32);
+        const uint64_t k1 = (uint64_t)wd[1] | ((uint64_t)(wd[2] & 0xFFFFFFu) << 32) | (1ull << 56);
+        const uint64_t out = obase + idx;
+        uint32_t hid = 0;
+        const uint32_t slot =
+            table_insert(cv.text, eo.table, eo.slot_ref, eo.cap, h, k0, k1, s_abs, len, w32, s_win, eo.overflow, &hid);
+        if (HOT && hid) {  // hot term: count it, leave a hole
+          const uint32_t dd = ldoc - (uint32_t)(k_range_lo - 1), hh = hid - 1;
+          if (dd < kHotDocs) atomicAdd(&hc[dd * (kHotMaxH / 2) + (hh >> 1)], 1u << (16 * (hh & 1)));
+          else atomicAdd(&eo.hot_mat[(uint64_t)hh * eo.hot_docs + ldoc], 1u);
+          __stcs(eo.slot + out, 0u);
+        } else {
+          __stcs(eo.slot + out, slot | (1u << 25));  // stream element: slot | count 1 << 25
+          __stcs(eo.doc + out, eo.doc_base + ldoc);
+        }
+        if (eo.dbg_start) { eo.dbg_start[out] = s_abs; eo.dbg_len[out] = len; }
       }
     }
+    obase += qn;
+    qn = 0;
     __syncwarp();
   };
 
-  for (uint32_t sub = 0; sub < kEmitSub; ++sub) {
-    const uint32_t gw = gw0 + sub;
-    if (gw >= n_ranges) break;
-    const uint32_t sb0 = gw * kSegsPerWarp;
-    const uint32_t se = min(sb0 + kSegsPerWarp, n_segs);
-    const uint32_t last = se < n_segs ? se : se - 1;
-    const uint32_t B0 = sb0 * kSegBytes;
-    // stage the range and the look-ahead segment (tokens may run past the range)
-    {
-      uint4 v[kSegsPerWarp + 1];
-#pragma unroll
-      for (int j = 0; j <= kSegsPerWarp; ++j) v[j] = load_lane16(cv, sb0 + j);
-      __syncwarp();  // the previous range's window is no longer read
-#pragma unroll
-      for (int j = 0; j <= kSegsPerWarp; ++j)  // fold A-Z once here (classification is case-blind)
-        *(uint4*)&w32[(j * kSegBytes + 16 * lane) / 4] =
-            make_uint4(lower4(v[j].x), lower4(v[j].y), lower4(v[j].z), lower4(v[j].w));
-      if (lane < 4) w32[(kWinBytes - 16) / 4 + lane] = 0;
-      __syncwarp();
+  for (uint32_t seg = sb0; seg <= last; ++seg) {
+    const uint32_t j = seg - sb0;
+    const uint32_t s0 = seg * kSegBytes;
+    const uint4 vv = *(const uint4*)&w32[(j * kSegBytes + 16 * lane) / 4];
+    // reloaded per segment here: a register carried across the flushes costs the emit kernel more
+    // (spills) than the load (count: 0.426 -> 0.408 ms with the carried register, emit +0.025 ms)
+    uint64_t nb = next_bound(cv, kcur);
+    const SegBits sb = seg_bits(cv, s0, vv, prev, kcur, nb, bnd[w]);
+    prev = __shfl_sync(0xffffffffu, sb.tm, 31) >> 15;
+    const SegTok tk = seg_tok(sb);
+    if (open) {  // the previous segment's last token ends in this one
+      const uint32_t ft = first_term(sb, tk);
+      if (ft != kNone && s0 + ft - open_start <= kMaxTermLen) {
+        if (qn + 1 > (uint32_t)kQueueCap) flush();
+        if (lane == 0) q[qn] = ((open_start - B0) << 8) | (s0 + ft - open_start);
+        ++qn;
+        __syncwarp();
+      }
+      open = false;
     }
-
-    const uint64_t k_range_lo = kstart[gw];
-    uint64_t kcur = k_range_lo;
-    uint32_t prev = prev_token_bit(cv, B0);
-    uint32_t qn = 0;
-    uint64_t obase = range_off[gw];
-    uint64_t k_range_hi = k_range_lo;
-    bool open = false;
-    uint32_t open_start = 0;
-
-    auto flush = [&]() {
-      for (uint32_t r = 0; r < qn; r += 32) {
-        const uint32_t idx = r + lane;
-        const bool valid = idx < qn;
-        uint32_t hid = 0, doc = 0;
-        uint64_t out = 0;
-        if (valid) {
-          const uint32_t e = q[idx];
-          const uint32_t s_win = e >> 8, len = e & 255u;
-          const uint32_t s_abs = B0 + s_win;
-          // first 16 folded bytes: 5 window words, 4 funnel shifts, length masks
-          uint32_t wd[4];
-          {
-            const uint32_t a = s_win >> 2, sh = (s_win & 3) * 8;
-            uint32_t x[5];
-#pragma unroll
-            for (int k = 0; k < 5; ++k) x[k] = w32[a + k];
-#pragma unroll
-            for (int k = 0; k < 4; ++k) {
-              const uint32_t rem = min(max((int)len - 4 * k, 0), 4);
-              wd[k] = __funnelshift_r(x[k], x[k + 1], sh) & __funnelshift_lc(0xFFFFFFFFu, 0u, rem * 8);
-            }
-          }
-          uint32_t h32 = hash_init(len);
-#pragma unroll
-          for (int k = 0; k < 4; ++k) h32 = hash_mix(h32, wd[k]);
-          for (uint32_t k = 4; k * 4 < len; ++k) h32 = hash_mix(h32, win_word(w32, s_win, len, k));
-          h32 = hash_fin(h32);
-          const uint64_t h = h32;
-          // DocID = (number of doc_off[k] <= s, k < n_docs) - 1 (readings S9, S16)
-          uint64_t lo = k_range_lo, hi = k_range_hi;
-          while (lo < hi) {
-            const uint64_t mid = (lo + hi) >> 1;
-            if (cv.doc_off[mid] <= s_abs) lo = mid + 1; else hi = mid;
-          }
-          doc = eo.doc_base + (uint32_t)(lo - 1);
-          const uint64_t k0 = (uint64_t)len | ((uint64_t)hash_tag(h32) << 8) | ((uint64_t)wd[0] << 32);
-          const uint64_t k1 = (uint64_t)wd[1] | ((uint64_t)(wd[2] & 0xFFFFFFu) << 32) | (1ull << 56);
-          out = obase + idx;
-          const uint32_t slot = table_insert(cv.text, eo.table, eo.slot_ref, eo.cap, h, k0, k1, s_abs, len, w32, s_win,
-                                             eo.overflow, &hid);
-          if (!HOT) hid = 0;
-          // stream element: slot | count 1 << 25, or a hole (key 0) for a merged hot token
-          __stcs(eo.slot + out, hid ? 0u : (slot | (1u << 25)));
-          if (!hid) __stcs(eo.doc + out, doc);
-          if (eo.dbg_start) { eo.dbg_start[out] = s_abs; eo.dbg_len[out] = len; }
-        }
-        // hot tokens: per document (documents ascend with the lane), lanes of one hot id merge into
-        // their leader (the earliest token), which updates the warp's accumulator
-        uint32_t pend = HOT ? __ballot_sync(0xffffffffu, hid != 0) : 0u;
-        while (HOT && pend) {
-          const uint32_t d = __shfl_sync(0xffffffffu, doc, __ffs(pend) - 1);
-          if (d != hdoc) {
-            hot_flush();
-            hdoc = d;
-          }
-          const bool mine = ((pend >> lane) & 1u) && doc == d;
-          const uint32_t grp = __ballot_sync(0xffffffffu, mine);
-          if (mine) {
-            const uint32_t peers = __match_any_sync(grp, hid);
-            if ((int)lane == __ffs(peers) - 1) {
-              uint32_t a = ha[hid];
-              uint32_t c = a >> 16;
-              const uint32_t add = __popc(peers);
-              const uint32_t pos = (uint32_t)(out - wbase);
-              if (c + add > 127u) {  // the element is full: write it, start the next at this token
-                const uint64_t o = wbase + (a & 0xFFFFu);
-                __stcs(eo.slot + o, __ldg(&eo.hot_slot[hid]) | (c << 25));
-                __stcs(eo.doc + o, hdoc);
-                c = 0;
-              }
-              if (c == 0) a = pos;
-              ha[hid] = (a & 0xFFFFu) | ((c + add) << 16);
-            }
-          }
-          pend &= ~grp;
-          __syncwarp();
-        }
+    if (seg == se) break;
+    k_range_hi = kcur;
+    // kept tokens starting in this lane (a > 255-byte token needs a lane of 16 token bytes)
+    uint32_t c = __popc(sb.startm) - ((int)lane == tk.open_lane ? 1u : 0u);
+    if (__ballot_sync(0xffffffffu, sb.tm == 0xFFFFu)) {
+      c = 0;
+      for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
+        const int jb = __ffs(sm) - 1;
+        const uint32_t pos = 16 * lane + jb;
+        if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
+        c += (tok_end_rel(sb, tk, jb) - pos <= kMaxTermLen) ? 1u : 0u;
       }
-      obase += qn;
-      qn = 0;
-      __syncwarp();
-    };
-
-    for (uint32_t seg = sb0; seg <= last; ++seg) {
-      const uint32_t j = seg - sb0;
-      const uint32_t s0 = seg * kSegBytes;
-      const uint4 vv = *(const uint4*)&w32[(j * kSegBytes + 16 * lane) / 4];
-      // reloaded per segment here: a register carried across the flushes costs the emit kernel more
-      // (spills) than the load (count: 0.426 -> 0.408 ms with the carried register, emit +0.025 ms)
-      uint64_t nb = next_bound(cv, kcur);
-      const SegBits sb = seg_bits(cv, s0, vv, prev, kcur, nb, bnd[w]);
-      prev = __shfl_sync(0xffffffffu, sb.tm, 31) >> 15;
-      const SegTok tk = seg_tok(sb);
-      if (open) {  // the previous segment's last token ends in this one
-        const uint32_t ft = first_term(sb, tk);
-        if (ft != kNone && s0 + ft - open_start <= kMaxTermLen) {
-          if (qn + 1 > (uint32_t)kQueueCap) flush();
-          if (lane == 0) q[qn] = ((open_start - B0) << 8) | (s0 + ft - open_start);
-          ++qn;
-          __syncwarp();
-        }
-        open = false;
-      }
-      if (seg == se) break;
-      k_range_hi = kcur;
-      // kept tokens starting in this lane (a > 255-byte token needs a lane of 16 token bytes)
-      uint32_t c = __popc(sb.startm) - ((int)lane == tk.open_lane ? 1u : 0u);
-      if (__ballot_sync(0xffffffffu, sb.tm == 0xFFFFu)) {
-        c = 0;
-        for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
-          const int jb = __ffs(sm) - 1;
-          const uint32_t pos = 16 * lane + jb;
-          if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
-          c += (tok_end_rel(sb, tk, jb) - pos <= kMaxTermLen) ? 1u : 0u;
-        }
-      }
-      uint32_t inc = c;
+    }
+    uint32_t inc = c;
 #pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
-        if ((int)lane >= o) inc += u;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
+      if ((int)lane >= o) inc += u;
+    }
+    const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
+    if (qn + tot > (uint32_t)kQueueCap) flush();
+    if (tot <= (uint32_t)kQueueCap) {
+      uint32_t pos_q = qn + inc - c;
+      for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
+        const int jb = __ffs(sm) - 1;
+        const uint32_t pos = 16 * lane + jb;
+        if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
+        const uint32_t len = tok_end_rel(sb, tk, jb) - pos;
+        if (len <= kMaxTermLen) q[pos_q++] = ((s0 + pos - B0) << 8) | len;
       }
-      const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
-      if (qn + tot > (uint32_t)kQueueCap) flush();
-      if (tot <= (uint32_t)kQueueCap) {
-        uint32_t pos_q = qn + inc - c;
+      qn += tot;
+    } else {
+      // Rare: more kept tokens start in this segment than the queue holds (up to 512: dense
+      // document starts, e.g. consecutive 1-byte documents).  Queue them in rounds of kQueueCap,
+      // flushing between rounds (the queue is empty here: tot > kQueueCap forced the flush above).
+      for (uint32_t r0 = 0; r0 < tot; r0 += (uint32_t)kQueueCap) {
+        uint32_t pos_q = inc - c;  // segment-relative index of the lane's first kept token
         for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
           const int jb = __ffs(sm) - 1;
           const uint32_t pos = 16 * lane + jb;
           if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
           const uint32_t len = tok_end_rel(sb, tk, jb) - pos;
-          if (len <= kMaxTermLen) q[pos_q++] = ((s0 + pos - B0) << 8) | len;
+          if (len > kMaxTermLen) continue;
+          if (pos_q >= r0 && pos_q < r0 + (uint32_t)kQueueCap) q[pos_q - r0] = ((s0 + pos - B0) << 8) | len;
+          ++pos_q;
         }
-        qn += tot;
-      } else {
-        // Rare: more kept tokens start in this segment than the queue holds (up to 512: dense
-        // document starts, e.g. consecutive 1-byte documents).  Queue them in rounds of kQueueCap,
-        // flushing between rounds (the queue is empty here: tot > kQueueCap forced the flush above).
-        for (uint32_t r0 = 0; r0 < tot; r0 += (uint32_t)kQueueCap) {
-          uint32_t pos_q = inc - c;  // segment-relative index of the lane's first kept token
-          for (uint32_t sm = sb.startm; sm; sm &= sm - 1) {
-            const int jb = __ffs(sm) - 1;
-            const uint32_t pos = 16 * lane + jb;
-            if (tk.open_lane >= 0 && pos == tk.open_pos) continue;
-            const uint32_t len = tok_end_rel(sb, tk, jb) - pos;
-            if (len > kMaxTermLen) continue;
-            if (pos_q >= r0 && pos_q < r0 + (uint32_t)kQueueCap) q[pos_q - r0] = ((s0 + pos - B0) << 8) | len;
-            ++pos_q;
-          }
-          qn = min(tot - r0, (uint32_t)kQueueCap);
-          __syncwarp();
-          flush();
-        }
+        qn = min(tot - r0, (uint32_t)kQueueCap);
+        __syncwarp();
+        flush();
       }
-      if (tk.open_lane >= 0) { open = true; open_start = s0 + tk.open_pos; }
+    }
+    if (tk.open_lane >= 0) { open = true; open_start = s0 + tk.open_pos; }
+    __syncwarp();
+  }
+  k_range_hi = kcur;
+  if (open) {  // chunk end
+    if (cv.n_bytes - open_start <= kMaxTermLen) {
+      if (qn + 1 > (uint32_t)kQueueCap) flush();
+      if (lane == 0) q[qn] = ((open_start - B0) << 8) | (uint32_t)(cv.n_bytes - open_start);
+      ++qn;
       __syncwarp();
     }
-    k_range_hi = kcur;
-    if (open) {  // chunk end
-      if (cv.n_bytes - open_start <= kMaxTermLen) {
-        if (qn + 1 > (uint32_t)kQueueCap) flush();
-        if (lane == 0) q[qn] = ((open_start - B0) << 8) | (uint32_t)(cv.n_bytes - open_start);
-        ++qn;
-        __syncwarp();
-      }
-    }
-    flush();
   }
-  if (hot_on) hot_flush();
+  flush();
+  if (HOT) {  // the range's hot counters -> the (hot term x document) matrix
+    const uint32_t d0 = (uint32_t)(k_range_lo - 1);
+    for (uint32_t i = lane; i < kHotWords; i += 32) {
+      const uint32_t x = hc[i];
+      if (x == 0) continue;
+      const uint32_t dd = i / (kHotMaxH / 2), hh = 2 * (i % (kHotMaxH / 2));
+      if (x & 0xFFFFu) atomicAdd(&eo.hot_mat[(uint64_t)hh * eo.hot_docs + d0 + dd], x & 0xFFFFu);
+      if (x >> 16) atomicAdd(&eo.hot_mat[(uint64_t)(hh + 1) * eo.hot_docs + d0 + dd], x >> 16);
+    }
+  }
 }
 
 }  // namespace wj
