@@ -1989,7 +1989,7 @@ struct wj_index {
         const uint32_t* rd = (const uint32_t*)rec_df.p;
         if (rec_end.size() == 1) {  // one run: every partial list is its term's whole list
           k_rank_scatter_rec<<<grid_for(nrec, 256), 256, 0, st>>>(rt, rd, (const uint32_t*)rec_cf.p, nrec, ro, dfp, cfp,
-                                                                  bef);
+                                                                  (const uint64_t*)rec_start.p, cft);
           launched();
         } else {
           WJ_CUDA_CHECK(cudaMemsetAsync(dft, 0, (size_t)V * 4, st));
@@ -2013,9 +2013,9 @@ struct wj_index {
         uint32_t* od = buf<uint32_t>(out_doc, P + 1);
         uint32_t* of = buf<uint32_t>(out_tf, P + 1);
         ktime(WJ_KERNEL_COPY_PARTIALS, [&] {
-          if (rec_end.size() == 1) {  // one run: bef holds the record of each rank
+          if (rec_end.size() == 1) {  // one run: cft holds the list start of each rank
             k_copy_by_rank<<<grid_for((P + kCopyChunk - 1) / kCopyChunk * 32, 256), 256, 0, st>>>(
-                bef, (const uint64_t*)rec_start.p, V, P, po, (const uint32_t*)pp_doc.p, (const uint32_t*)pp_tf.p, od, of);
+                cft, V, P, po, (const uint32_t*)pp_doc.p, (const uint32_t*)pp_tf.p, od, of);
             launched();
             return;
           }

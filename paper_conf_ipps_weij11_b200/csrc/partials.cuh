@@ -88,23 +88,23 @@ __global__ void k_rank_scatter(const uint32_t* __restrict__ rank_of, uint32_t V,
   cf[r] = cf_tot[t];
 }
 
-// a single run: the records are the terms, df / cf straight to rank order, and the record of each rank
+// a single run: the records are the terms, df / cf straight to rank order, and the start of each rank's list
 __global__ void k_rank_scatter_rec(const uint32_t* __restrict__ rec_tid, const uint32_t* __restrict__ rec_df,
                                    const uint32_t* __restrict__ rec_cf, uint64_t R, const uint32_t* __restrict__ rank_of,
-                                   uint32_t* df, uint64_t* cf, uint32_t* rec_of_rank) {
+                                   uint32_t* df, uint64_t* cf, const uint64_t* __restrict__ rec_start,
+                                   uint64_t* src_of_rank) {
   const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= R) return;
   const uint32_t r = rank_of[rec_tid[i]];
   df[r] = rec_df[i];
   cf[r] = rec_cf[i];
-  rec_of_rank[r] = (uint32_t)i;
+  src_of_rank[r] = rec_start[i];  // sequential read here, so the copy reads its sources in rank order
 }
 
 // Single run: the same copy walked in destination (rank) order -- warp w writes the final postings
 // [w * kCopyChunk, (w + 1) * kCopyChunk) coalesced and gathers them from the partial lists (each
 // term's list is contiguous in both).
-__global__ void __launch_bounds__(256) k_copy_by_rank(const uint32_t* __restrict__ rec_of_rank,
-                                                      const uint64_t* __restrict__ rec_start, uint32_t V, uint64_t P,
+__global__ void __launch_bounds__(256) k_copy_by_rank(const uint64_t* __restrict__ src_of_rank, uint32_t V, uint64_t P,
                                                       const uint64_t* __restrict__ post_off,
                                                       const uint32_t* __restrict__ pdoc, const uint32_t* __restrict__ ptf,
                                                       uint32_t* __restrict__ out_doc, uint32_t* __restrict__ out_tf);
@@ -192,8 +192,7 @@ __global__ void __launch_bounds__(256) k_copy_partials(const uint32_t* __restric
   }
 }
 
-__global__ void __launch_bounds__(256) k_copy_by_rank(const uint32_t* __restrict__ rec_of_rank,
-                                                      const uint64_t* __restrict__ rec_start, uint32_t V, uint64_t P,
+__global__ void __launch_bounds__(256) k_copy_by_rank(const uint64_t* __restrict__ src_of_rank, uint32_t V, uint64_t P,
                                                       const uint64_t* __restrict__ post_off,
                                                       const uint32_t* __restrict__ pdoc, const uint32_t* __restrict__ ptf,
                                                       uint32_t* __restrict__ out_doc, uint32_t* __restrict__ out_tf) {
@@ -216,7 +215,7 @@ __global__ void __launch_bounds__(256) k_copy_by_rank(const uint32_t* __restrict
     const uint64_t i = r + lane;
     const bool v = i < V;
     const uint64_t d0 = v ? post_off[i] : ~0ull;
-    const uint64_t src = v ? rec_start[rec_of_rank[i]] : 0ull;
+    const uint64_t src = v ? src_of_rank[i] : 0ull;
     const uint64_t wend = (r + 32 < V) ? post_off[r + 32] : P;  // first posting after the window
     const uint64_t e = wend < hi ? wend : hi;
     const uint64_t ws = __shfl_sync(0xffffffffu, d0, 0);
