@@ -140,8 +140,9 @@ typedef struct {
   uint64_t host_syncs;             /* stream synchronisations since index_init (cumulative)          */
   uint64_t unique_terms_last;      /* unique terms of the last chunk                                 */
   uint64_t new_terms_last;         /* terms inserted by the last chunk                               */
-  uint64_t btree_nodes;            /* 512-byte B-tree nodes in the dictionary                        */
-  uint64_t btree_height_max;       /* tallest trie-collection B-tree                                 */
+  uint64_t btree_nodes;            /* 512-byte B-tree nodes in the dictionary, and the tallest trie- */
+  uint64_t btree_height_max;       /* collection B-tree, as of the last re-layout (done lazily before */
+                                   /* the next chunk's probe or a retrieval)                          */
   uint64_t exchange_bytes;         /* world > 1: bytes this rank sent                                */
   uint64_t device_bytes;           /* device memory held by the context                              */
   uint64_t stream_elems;           /* (term, docID) stream elements of the index so far (tokens, and  */

@@ -481,6 +481,7 @@ struct wj_index {
     pc_pending = pc_join = false;
     rec_end.clear();
     unique_last = new_last = n_nodes = height_max = 0;
+    btree_dirty = false;
     exchange_bytes = 0;
     V = 0;
     arena_used = 0;
@@ -919,10 +920,24 @@ struct wj_index {
     sync();
   }
 
-  // K3 probe + K4 insert/rebuild of the chunk's unique terms (u_* arrays) -> u_tid
+  // The B-trees are re-laid lazily: an insert only marks them stale; the next probe (the next chunk's
+  // dictionary update) or a retrieval rebuilds them first, so the last chunk of an index never pays
+  // for a rebuild that nothing reads (finalize ranks terms from E and the arena, not from the nodes).
+  bool btree_dirty = false;
+  void ensure_btrees() {
+    if (!btree_dirty) return;
+    btree_dirty = false;
+    const int open = cur_phase;
+    phase(WJ_PHASE_REBUILD);
+    rebuild();
+    phase(open);
+  }
+
+  // K3 probe + K4 insert of the chunk's unique terms (u_* arrays) -> u_tid
   void dictionary_update(const uint8_t* text, uint64_t U) {
     uint32_t* ut = buf<uint32_t>(u_tid, U);
     uint32_t* urk = buf<uint32_t>(u_rank, U);
+    if (V > 0) ensure_btrees();
     phase(WJ_PHASE_PROBE);
     DictView dv{(const Node*)nodes.p, (const uint32_t*)coll_root.p, (const uint32_t*)coll_n.p, (const uint8_t*)arena.p};
     if (V > 0) {
@@ -952,8 +967,7 @@ struct wj_index {
       if ((uint64_t)V + Nn > vmax)
         throw StatusError{WJ_ERR_CAPACITY, pm ? "more than 2^32-2 terms" : "more than 2^25 terms in one dictionary slice"};
       insert_new(text, U, Nn);
-      phase(WJ_PHASE_REBUILD);
-      rebuild();
+      btree_dirty = true;
     }
   }
 
@@ -2326,6 +2340,7 @@ int index_read_postings(wj_index* ix, const uint8_t* term, uint32_t len, uint32_
       const bool tok = (c >= '0' && c <= '9') || (c >= 'A' && c <= 'Z') || (c >= 'a' && c <= 'z') || c >= 0x80;
       if (!tok) return (int)WJ_NOT_FOUND;
     }
+    ix->ensure_btrees();
     uint8_t* q = (uint8_t*)ix->grow(ix->qbuf, 512);
     QueryResult* r = (QueryResult*)ix->grow(ix->qres, sizeof(QueryResult));
     WJ_CUDA_CHECK(cudaMemcpyAsync(q, term, len, cudaMemcpyHostToDevice, ix->st));
@@ -2449,6 +2464,7 @@ int index_debug_btree(wj_index* ix, void* nodes, uint64_t node_cap, uint64_t* n_
                       uint8_t* arena, uint64_t arena_cap, uint64_t* arena_bytes) {
   if (!ix || !n_nodes || !arena_bytes) return WJ_ERR_INVALID_ARG;
   return guarded(ix, [&]() {
+    ix->ensure_btrees();
     ix->sync();
     *n_nodes = ix->n_nodes;
     *arena_bytes = ix->arena_used;

@@ -381,13 +381,14 @@ __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* tabl
 #define WJ_EMIT_MINB 6
 #endif
 // HOT (WJ_FLAG_HOT_TERMS): the <= kHotMaxH sampled hot terms of the chunk (SURVEY 8(f2)(ii),
-// P:202-208) do not enter the (slot, docID) stream: their tokens leave holes (key 0, dropped by the
-// first sort pass) and are counted in the dense (hot term x document) matrix eo.hot_mat, through
+// P:202-208), recognised by the hot id k_hot_seed stored in their table slot, do not enter the
+// (slot, docID) stream (their tokens leave holes, key 0, dropped by the first sort pass) and are
+// counted in the dense (hot term x document) matrix eo.hot_mat, through
 // per-warp shared-memory counters for the first kHotDocs documents of the warp's range (flushed with
 // one global add per nonzero counter at the range's end); the matrix rows become the hot terms'
-// partial lists (k_hot_rows).
+// partial lists (k_hot_scatter).
 constexpr uint32_t kHotMaxH = 64;
-constexpr uint32_t kHotDocs = 4;
+constexpr uint32_t kHotDocs = 2;
 constexpr uint32_t kHotWords = kHotDocs * kHotMaxH / 2;  // u16 counter pairs per warp
 
 template <bool HOT>
@@ -467,17 +468,19 @@ __global__ void __launch_bounds__(kTokThreads, WJ_EMIT_MINB) k_tok_emit(ChunkVie
         const uint64_t k1 = (uint64_t)wd[1] | ((uint64_t)(wd[2] & 0xFFFFFFu) << 32) | (1ull << 56);
         const uint64_t out = obase + idx;
         uint32_t hid = 0;
+        // a hot term's slot was seeded with its hot id in k1 (k_hot_seed): table_insert returns it
         const uint32_t slot =
             table_insert(cv.text, eo.table, eo.slot_ref, eo.cap, h, k0, k1, s_abs, len, w32, s_win, eo.overflow, &hid);
-        if (HOT && hid) {  // hot term: count it, leave a hole
+#ifndef WJ_HOT_NO_ATOMIC
+        if (HOT && hid) {  // hot term: count it (the stream keeps a hole, key 0)
           const uint32_t dd = ldoc - (uint32_t)(k_range_lo - 1), hh = hid - 1;
           if (dd < kHotDocs) atomicAdd(&hc[dd * (kHotMaxH / 2) + (hh >> 1)], 1u << (16 * (hh & 1)));
           else atomicAdd(&eo.hot_mat[(uint64_t)hh * eo.hot_docs + ldoc], 1u);
-          __stcs(eo.slot + out, 0u);
-        } else {
-          __stcs(eo.slot + out, slot | (1u << 25));  // stream element: slot | count 1 << 25
-          __stcs(eo.doc + out, eo.doc_base + ldoc);
         }
+#endif
+        // branch-free stores: stream element slot | count 1 << 25, or a hole (the docID is not read)
+        __stcs(eo.slot + out, (HOT && hid) ? 0u : (slot | (1u << 25)));
+        __stcs(eo.doc + out, eo.doc_base + ldoc);
         if (eo.dbg_start) { eo.dbg_start[out] = s_abs; eo.dbg_len[out] = len; }
       }
     }
@@ -570,6 +573,7 @@ __global__ void __launch_bounds__(kTokThreads, WJ_EMIT_MINB) k_tok_emit(ChunkVie
     }
   }
   flush();
+#ifndef WJ_HOT_NO_FLUSH
   if (HOT) {  // the range's hot counters -> the (hot term x document) matrix
     const uint32_t d0 = (uint32_t)(k_range_lo - 1);
     for (uint32_t i = lane; i < kHotWords; i += 32) {
@@ -580,6 +584,7 @@ __global__ void __launch_bounds__(kTokThreads, WJ_EMIT_MINB) k_tok_emit(ChunkVie
       if (x >> 16) atomicAdd(&eo.hot_mat[(uint64_t)(hh + 1) * eo.hot_docs + d0 + dd], x >> 16);
     }
   }
+#endif
 }
 
 }  // namespace wj
