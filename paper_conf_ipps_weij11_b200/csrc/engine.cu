@@ -244,8 +244,10 @@ struct wj_index {
   uint32_t side_ctas = kRsCtas;      // ... for the side stream's sort (148 / 222 measured slower)
   bool pc_pending = false;           // the last chunk's posting count is still on the device (dscal[13])
   bool pc_join = false;              // the last chunk's side-stream work is not joined yet
-  uint64_t pc_U = 0, pc_Nc = 0, Ns_last = 0;  // pc_Nc: stream tokens of the pending chunk
+  uint64_t pc_U = 0, pc_Nc = 0;  // pc_Nc: tokens of the pending chunk
   bool pc_hot = false;                         // the pending chunk has hot-term lists
+  bool pc_settle_hot = false;                  // ... the joined, unsettled chunk
+  uint64_t pc_settle_tokens = 0;
   uint32_t doc_base_cur = 0;                   // first DocID of the chunk being indexed
   std::vector<uint64_t> rec_end;     // end of each chunk's records
   uint64_t sorted_elems = 0;    // stream elements the last finalize sorted (after hole compaction)
@@ -663,40 +665,47 @@ struct wj_index {
     owner_ready = true;
   }
 
-  uint32_t select_hot(const ChunkView& cv) {
-    uint64_t Cs = 0;
-    const uint64_t Ns = sample_counts(cv, Cs, 1024);
-    if (Ns == 0) return 0;
-    const uint32_t* cnt = (const uint32_t*)samp_cnt.p;
+  // Sampled hot terms of a chunk ("1MB out of every 1GB"), without a host round trip:
+  // the first 1 MiB of the chunk is tokenised into a scratch table (documents past it are never
+  // reached; a token cut at the edge occurs once and cannot reach kHotMinCount), tokens are counted per
+  // slot, (count, slot) pairs sorted, and k_hot_pick keeps the <= Hmax most frequent terms with
+  // >= kHotMinCount occurrences (<= 11 bytes) in hot_kb, their number in *hot_Hdev().
+  uint32_t* hot_Hdev() { return (uint32_t*)(dscal() + 14) + 1; }
+  void select_hot(const ChunkView& cv, uint32_t Hmax) {
+    const uint64_t S = std::min<uint64_t>(cv.n_bytes, 1ull << 20);
+    ChunkView sv{cv.text, S, cv.doc_off, cv.n_docs};
+    const uint64_t n_segs = (S + kSegBytes - 1) / kSegBytes;
+    const uint64_t ranges = (n_segs + kSegsPerWarp - 1) / kSegsPerWarp;
+    uint32_t* cnt = buf<uint32_t>(seg_cnt, ranges + 1);
+    uint64_t* ks = buf<uint64_t>(kstart, ranges);
+    k_warp_kstart<<<grid_for(ranges, 256), 256, 0, st>>>(sv, ranges, ks);
+    k_tok_count<<<(unsigned)((ranges + kTokWarps - 1) / kTokWarps), kTokThreads, 0, st>>>(
+        sv, (uint32_t)n_segs, ks, cnt, (unsigned long long*)(dscal() + 15));  // (its dropped count is ignored)
+    launched(2);
+    uint32_t* ns = (uint32_t*)(dscal() + 14);  // sample tokens
+    scan<uint32_t>(ArrayIn<uint32_t>{cnt}, ranges, cnt, ns);
+    const uint64_t Nmax = S + 16;  // a kept token takes >= 1 byte
+    uint32_t* ss = buf<uint32_t>(samp_slot, Nmax);
+    uint32_t* sd = buf<uint32_t>(samp_doc, Nmax);
+    const uint64_t Cs = pow2_at_least(2 * Nmax);  // at most half full: no probe overflow
+    emit_tokens(sv, n_segs, ss, sd, 0, Cs, nullptr, nullptr, false, true);
+    uint32_t* sc = buf<uint32_t>(samp_cnt, Cs);
+    WJ_CUDA_CHECK(cudaMemsetAsync(sc, 0, Cs * 4, st));
+    k_sample_count_dev<<<grid_for(Nmax, 256), 256, 0, st>>>(ss, ns, sc);
     uint32_t* ck = buf<uint32_t>(samp_ck, Cs + 16);
     uint32_t* cv2 = buf<uint32_t>(samp_cv, Cs + 16);
     uint32_t* ck2 = buf<uint32_t>(samp_ck2, Cs + 16);
     uint32_t* cvb = buf<uint32_t>(samp_cv2, Cs + 16);
-    k_sample_cand<<<grid_for(Cs, 256), 256, 0, st>>>((const Slot*)table.p, cnt, (uint32_t)Cs, ck, cv2);
-    launched();
+    k_sample_cand<<<grid_for(Cs, 256), 256, 0, st>>>((const Slot*)table.p, sc, (uint32_t)Cs, ck, cv2);
+    launched(2);
     int bits = 0;
-    while ((1ull << bits) <= Ns) ++bits;
+    while ((1ull << bits) <= Nmax) ++bits;
     const bool in1 = sort_pairs<uint32_t>(ck, cv2, ck2, cvb, Cs, 0, bits, nullptr, false);
-    const uint32_t* sk = in1 ? ck2 : ck;
-    const uint32_t* sv_ = in1 ? cvb : cv2;
-    const uint32_t take = (uint32_t)std::min<uint64_t>(kHotMax, Cs);
-    std::vector<uint32_t> tk(take), tv(take);
-    WJ_CUDA_CHECK(cudaMemcpyAsync(tk.data(), sk + (Cs - take), take * 4, cudaMemcpyDeviceToHost, st));
-    WJ_CUDA_CHECK(cudaMemcpyAsync(tv.data(), sv_ + (Cs - take), take * 4, cudaMemcpyDeviceToHost, st));
-    sync();
-    std::vector<uint32_t> hot_slots;
-    for (int i = (int)take - 1; i >= 0; --i)
-      if (tk[i] >= kHotMinCount) hot_slots.push_back(tv[i]);
-    const uint32_t H = (uint32_t)hot_slots.size();
-    if (H == 0) return 0;
-    uint32_t* hs = buf<uint32_t>(hot_samp, kHotMax);
-    WJ_CUDA_CHECK(cudaMemcpyAsync(hs, hot_slots.data(), H * 4, cudaMemcpyHostToDevice, st));
     ulonglong2* hk = (ulonglong2*)grow(hot_kb, kHotMax * sizeof(ulonglong2));
-    k_hot_extract<<<1, kHotMax, 0, st>>>((const Slot*)table.p, hs, H, hk);
+    k_hot_pick<<<1, kHotMax, 0, st>>>(in1 ? ck2 : ck, in1 ? cvb : cv2, (uint32_t)Cs, (const Slot*)table.p, Hmax, hk,
+                                      hot_Hdev());
     launched();
     buf<uint32_t>(hot_slotb, kHotMax + 1);  // written by k_hot_seed
-    sync();  // hot_slots (host) is read by the copy above
-    return H;
   }
 
   // L2 persisting access-policy window on the context stream (best effort; cleared with bytes == 0)
@@ -746,8 +755,9 @@ struct wj_index {
     hot_H = 0;
     hot_D = (uint32_t)cv.n_docs;
     if (allow_hot && cv.n_bytes >= hot_min_bytes && cv.n_docs > 0) {
-      hot_H = select_hot(cv);
-      hot_H = (uint32_t)std::min<uint64_t>(hot_H, (64ull << 20) / cv.n_docs);  // matrix <= 256 MB
+      // hot_H = rows of the (hot term x document) matrix (<= 256 MB); the picked count is on the device
+      hot_H = (uint32_t)std::min<uint64_t>(kHotMax, (64ull << 20) / cv.n_docs);
+      if (hot_H) select_hot(cv, hot_H);
     }
     const uint64_t Nc = count_tokens(cv, n_segs);
     n_dropped += h_scal[1];
@@ -769,7 +779,7 @@ struct wj_index {
         uint32_t* mat = buf<uint32_t>(hot_matb, (uint64_t)hot_H * hot_D);
         WJ_CUDA_CHECK(cudaMemsetAsync(mat, 0, (uint64_t)hot_H * hot_D * 4, st));
         WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 5, 0, 8, st));
-        k_hot_seed<<<1, 128, 0, st>>>((const ulonglong2*)hot_kb.p, hot_H, tab, sref, (uint32_t)C,
+        k_hot_seed<<<1, 128, 0, st>>>((const ulonglong2*)hot_kb.p, hot_Hdev(), tab, sref, (uint32_t)C,
                                       (uint32_t*)hot_slotb.p, (uint32_t*)(dscal() + 5));
         launched();
       }
@@ -982,8 +992,9 @@ struct wj_index {
 
   // run-length pass over a sorted stream (postings.cuh): docid/tf into od/of, post_off / cstart at each
   // term's key (key & kRankMask); the posting count is left in dscal[8] (u32, no host round trip)
+  // n_dev (optional): the actual element count on the device, N being an upper bound
   void rle(const uint32_t* key, const uint32_t* docs, uint64_t N, bool counts, uint32_t* od, uint32_t* of, uint64_t* po,
-           uint64_t* csp) {
+           uint64_t* csp, const uint32_t* n_dev = nullptr) {
     if (N == 0) {  // e.g. every token of the chunk was a hot term
       WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 8, 0, 8, st));
       return;
@@ -995,15 +1006,17 @@ struct wj_index {
     uint32_t* rl = buf<uint32_t>(rle_lead, (uint64_t)G + 1);
     uint64_t* rt = buf<uint64_t>(rle_tok, (uint64_t)G + 1);
     ktime(WJ_KERNEL_RLE_EMIT, [&] {
-      if (counts) k_rle_count<true><<<G, kRleThreads, 0, st>>>(key, docs, N, per, rc, rt);
-      else k_rle_count<false><<<G, kRleThreads, 0, st>>>(key, docs, N, per, rc, rt);
+      if (counts) k_rle_count<true><<<G, kRleThreads, 0, st>>>(key, docs, N, per, rc, rt, n_dev);
+      else k_rle_count<false><<<G, kRleThreads, 0, st>>>(key, docs, N, per, rc, rt, n_dev);
       launched();
       scan<uint32_t>(ArrayIn<uint32_t>{rc}, G, rc, (uint32_t*)(dscal() + 8));
       scan<uint64_t>(ArrayIn<uint64_t>{rt}, G, rt, (uint64_t*)(dscal() + 11));
       if (counts)
-        k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(key, docs, N, per, rc, rt, od, of, po, csp, rl);
+        k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(key, docs, N, per, rc, rt, od, of, po, csp, rl,
+                                                                        n_dev);
       else
-        k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(false), st>>>(key, docs, N, per, rc, rt, od, of, po, csp, rl);
+        k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(false), st>>>(key, docs, N, per, rc, rt, od, of, po, csp,
+                                                                          rl, n_dev);
       launched();
     });
     k_rle_fixup<<<grid_for(G, 256), 256, 0, st>>>(rc, rl, G, of);
@@ -1016,6 +1029,11 @@ struct wj_index {
     if (!pc_pending) return;
     sync();
     pbase += (uint32_t)h_scal[13];
+    if (pc_settle_hot) {  // stream elements left after the hot tokens' holes were dropped
+      const uint64_t left = (uint32_t)h_scal[14];
+      hot_elems_saved += pc_settle_tokens - left;
+      pm_merged += pc_settle_tokens - left;
+    }
     pc_pending = false;
   }
 
@@ -1041,14 +1059,13 @@ struct wj_index {
     swap_side();
     try {
       phase(WJ_PHASE_SORT);
-      // holes (merged hot tokens, key 0) are dropped by the first pass: Ns elements remain
-      uint64_t Ns = Nc;
-      const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, bits, nullptr, true, nullptr, kRankMask, hot, &Ns);
-      Ns_last = Ns;
-      hot_elems_saved += Nc - Ns;
-      pm_merged += Nc - Ns;
+      // holes (hot tokens, key 0) are dropped by the first pass; the count left stays on the device
+      // (*ns_dev) and the later passes and the run-length pass are launched for the upper bound Nc
+      uint32_t* ns_dev = hot ? (uint32_t*)(dscal() + 13) : nullptr;
+      const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, bits, nullptr, true, nullptr, kRankMask, hot, nullptr,
+                                            true, nullptr, ns_dev);
       phase(WJ_PHASE_POSTINGS);
-      rle(in1 ? k1 : kt, in1 ? v1 : dt, Ns, false, od + pbase, of + pbase, po, cs);
+      rle(in1 ? k1 : kt, in1 ? v1 : dt, Nc, false, od + pbase, of + pbase, po, cs, ns_dev);
       if (hot) {  // the hot matrix rows -> the hot terms' partial lists, after the run-length postings
         const uint64_t HD = (uint64_t)hot_H * hot_D;
         uint32_t* hp = buf<uint32_t>(hot_posb, HD + 1);
@@ -1084,7 +1101,7 @@ struct wj_index {
     WJ_CUDA_CHECK(cudaStreamWaitEvent(st, ev_dict, 0));
     pc_join = true;
     pc_U = U;
-    pc_Nc = Ns_last;
+    pc_Nc = Nc;
     pc_hot = hot;
   }
 
@@ -1110,11 +1127,15 @@ struct wj_index {
     }
     k_chunk_records<<<grid_for(U, 256), 256, 0, st>>>(
         (const uint32_t*)u_slot.p, (uint32_t)U, po, cs, (const uint32_t*)(dscal() + (pc_hot ? 12 : 8)), Nc,
+        pc_hot ? (const uint32_t*)(dscal() + 13) : nullptr,
         (const uint32_t*)u_tid.p, pbase, rt + nrec, rs + nrec, rd + nrec, rc + nrec, (const Slot*)table.p,
-        pc_hot ? (const uint32_t*)hot_posb.p : nullptr, (const uint32_t*)hot_cfb.p, hot_D, nh, pc_hot ? hot_H : 0u);
+        pc_hot ? (const uint32_t*)hot_posb.p : nullptr, (const uint32_t*)hot_cfb.p, hot_D, nh, hot_Hdev());
     launched();
     WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 13, dscal() + 8, 8, cudaMemcpyDeviceToHost, st));
+    if (pc_hot) WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 14, dscal() + 13, 8, cudaMemcpyDeviceToHost, st));
     pc_pending = true;
+    pc_settle_hot = pc_hot;
+    pc_settle_tokens = Nc;
     nrec += U;
     rec_end.push_back(nrec);
     phase(-1);
@@ -1837,7 +1858,7 @@ struct wj_index {
                   const uint32_t* rank_of, bool timed,
                   const std::vector<std::pair<uint64_t, const uint32_t*>>* segs = nullptr, K kmask = ~K(0),
                   bool skip0 = false, uint64_t* n_out = nullptr, bool mask_digits = true,
-                  std::vector<uint64_t>* digit_start = nullptr) {
+                  std::vector<uint64_t>* digit_start = nullptr, uint32_t* holes_n_dev = nullptr) {
     if (n_out) *n_out = n;
     if (n == 0) return false;
     int passes = end_bit > begin_bit ? (end_bit - begin_bit + 7) / 8 : 0;
@@ -1866,6 +1887,9 @@ struct wj_index {
     const uint32_t* first_map = (segs && !multi_map) ? (*segs)[0].second : rank_of;
     bool in1 = false;
     uint64_t cur_n = n;
+    // with holes_n_dev the count left by the first (hole-compacting) pass stays on the device: the
+    // later passes are launched for the upper bound and read the count (no host round trip)
+    const uint32_t* n_dev = nullptr;
     for (int p = 0; p < passes; ++p) {
       if (cur_n == 0) break;  // every element was a hole
       uint64_t per = (cur_n + rs_ctas - 1) / rs_ctas;
@@ -1885,20 +1909,20 @@ struct wj_index {
       auto up = [&] {
         WJ_CUDA_CHECK(cudaMemsetAsync(h1, 0, (size_t)256 * G * 4, st));
         const uint32_t GU = G * kRsUpSplit;
-        if (holes && masked) k_rs_up<K, true, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
-        else if (holes) k_rs_up<K, true, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
-        else if (masked) k_rs_up<K, false, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
-        else k_rs_up<K, false, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask);
+        if (holes && masked) k_rs_up<K, true, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, n_dev);
+        else if (holes) k_rs_up<K, true, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, n_dev);
+        else if (masked) k_rs_up<K, false, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, n_dev);
+        else k_rs_up<K, false, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, n_dev);
         launched();
       };
       if (timed) ktime(WJ_KERNEL_SORT_HIST, up); else up();
       scan<uint32_t>(ArrayIn<uint32_t>{h1}, (uint64_t)256 * G, h2, h2 + (uint64_t)256 * G);
       auto down = [&] {
         const size_t sm = ds_smem_bytes<K>();
-        if (holes && masked) k_rs_down2<K, true, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
-        else if (holes) k_rs_down2<K, true, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
-        else if (masked) k_rs_down2<K, false, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
-        else k_rs_down2<K, false, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask);
+        if (holes && masked) k_rs_down2<K, true, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
+        else if (holes) k_rs_down2<K, true, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
+        else if (masked) k_rs_down2<K, false, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
+        else k_rs_down2<K, false, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
         launched();
       };
       if (timed) ktime(WJ_KERNEL_SORT_SCATTER, down); else down();
@@ -1909,7 +1933,10 @@ struct wj_index {
         sync();
         digit_start->assign(ds.begin(), ds.end());
       }
-      if (holes) {  // elements that survive the compaction
+      if (holes && holes_n_dev) {
+        WJ_CUDA_CHECK(cudaMemcpyAsync(holes_n_dev, h2 + (uint64_t)256 * G, 4, cudaMemcpyDeviceToDevice, st));
+        n_dev = holes_n_dev;
+      } else if (holes) {  // elements that survive the compaction
         uint32_t tot = 0;
         WJ_CUDA_CHECK(cudaMemcpyAsync(&tot, h2 + (uint64_t)256 * G, 4, cudaMemcpyDeviceToHost, st));
         sync();
@@ -2081,16 +2108,18 @@ struct wj_index {
       uint32_t* of = buf<uint32_t>(out_tf, N);
       ktime(WJ_KERNEL_RLE_EMIT, [&] {
         if (stream_has_hot)
-          k_rle_count<true><<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc, rt);
+          k_rle_count<true><<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc, rt, nullptr);
         else
-          k_rle_count<false><<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc, rt);
+          k_rle_count<false><<<G, kRleThreads, 0, st>>>(f_key, f_doc, N, per, rc, rt, nullptr);
         launched();
         scan<uint32_t>(ArrayIn<uint32_t>{rc}, G, rc, (uint32_t*)(dscal() + 8));
         scan<uint64_t>(ArrayIn<uint64_t>{rt}, G, rt, (uint64_t*)(dscal() + 11));
         if (stream_has_hot)
-          k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl);
+          k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl,
+                                                                          nullptr);
         else
-          k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(false), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl);
+          k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(false), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po,
+                                                                            csp, rl, nullptr);
         launched();
       });
       k_rle_fixup<<<grid_for(G, 256), 256, 0, st>>>(rc, rl, G, of);

@@ -76,10 +76,10 @@ __global__ void k_hot_extract(const Slot* table, const uint32_t* slots, uint32_t
 }
 
 // thread i seeds hot id i + 1: claims the term's slot in the chunk table with the id in k1 bits 57..
-__global__ void k_hot_seed(const ulonglong2* hk, uint32_t H, Slot* table, uint32_t* slot_ref, uint32_t cap,
+__global__ void k_hot_seed(const ulonglong2* hk, const uint32_t* H, Slot* table, uint32_t* slot_ref, uint32_t cap,
                            uint32_t* hot_slot, uint32_t* overflow) {
   const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= H) return;
+  if (i >= *H) return;
   const uint32_t id = i + 1;
   const uint64_t k0 = hk[i].x, k1 = hk[i].y | ((uint64_t)id << kHotShift);
   const uint32_t len = (uint32_t)k0 & 0xFFu;
@@ -87,6 +87,24 @@ __global__ void k_hot_seed(const ulonglong2* hk, uint32_t H, Slot* table, uint32
   const uint64_t h = term_hash16(w0, w1, w2, 0u, len);
   uint32_t hot = 0;
   hot_slot[id] = table_insert(nullptr, table, slot_ref, cap, h, k0, k1, 0u, len, nullptr, 0u, overflow, &hot);
+}
+
+// sample token counts per slot; the sample's token count is on the device (*n)
+__global__ void k_sample_count_dev(const uint32_t* key, const uint32_t* n, uint32_t* cnt) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < *n) atomicAdd(&cnt[key[i] & ((1u << 25) - 1u)], 1u);
+}
+
+// the <= Hmax most frequent sampled terms with >= kHotMinCount occurrences: from the end of the
+// (count, slot) pairs sorted by count, in descending count order (ties: descending slot); their slot
+// words -> hk[0..H), H -> *H_out.  One block of kHotMax threads.
+__global__ void k_hot_pick(const uint32_t* sk, const uint32_t* sv, uint32_t Cs, const Slot* table, uint32_t Hmax,
+                           ulonglong2* hk, uint32_t* H_out) {
+  const uint32_t i = threadIdx.x;
+  const bool ok = i < Hmax && i < Cs && sk[Cs - 1 - i] >= kHotMinCount;
+  const uint32_t n = __syncthreads_count(ok);  // counts are non-increasing in i: the kept ones are a prefix
+  if (ok) hk[i] = *(const ulonglong2*)(table + sv[Cs - 1 - i]);
+  if (i == 0) *H_out = n;
 }
 
 struct NonZeroU32 {

@@ -23,10 +23,11 @@ namespace wj {
 // rank among the non-hot ones (nh_pos), then the H hot terms in hot-id order.
 __global__ void k_chunk_records(const uint32_t* __restrict__ u_slot, uint32_t U, const uint64_t* __restrict__ post_off,
                                 const uint64_t* __restrict__ cstart, const uint32_t* __restrict__ P_rle, uint64_t NT,
-                                const uint32_t* __restrict__ u_tid, uint64_t pbase, uint32_t* rec_tid,
+                                const uint32_t* __restrict__ NT_dev, const uint32_t* __restrict__ u_tid, uint64_t pbase,
+                                uint32_t* rec_tid,
                                 uint64_t* rec_start, uint32_t* rec_df, uint32_t* rec_cf, const Slot* __restrict__ table,
                                 const uint32_t* __restrict__ hot_pos, const uint32_t* __restrict__ hot_cf, uint32_t D,
-                                const uint32_t* __restrict__ nh_pos, uint32_t H) {
+                                const uint32_t* __restrict__ nh_pos, const uint32_t* __restrict__ H_dev) {
   const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
   if (u >= U) return;
   auto hot_of = [&](uint32_t slot) -> uint32_t {
@@ -34,7 +35,7 @@ __global__ void k_chunk_records(const uint32_t* __restrict__ u_slot, uint32_t U,
   };
   const uint32_t s = u_slot[u];
   const uint32_t h = hot_of(s);
-  const uint32_t r = h ? U - H + (h - 1) : (hot_pos ? nh_pos[u] : u);
+  const uint32_t r = h ? U - *H_dev + (h - 1) : (hot_pos ? nh_pos[u] : u);
   rec_tid[r] = u_tid[u];
   if (h) {
     const uint64_t a = hot_pos[(uint64_t)(h - 1) * D], b = hot_pos[(uint64_t)h * D];
@@ -44,7 +45,7 @@ __global__ void k_chunk_records(const uint32_t* __restrict__ u_slot, uint32_t U,
     return;
   }
   const uint64_t a = post_off[s], ta = cstart[s];
-  uint64_t b = *P_rle, tb = NT;
+  uint64_t b = *P_rle, tb = NT_dev ? *NT_dev : NT;  // NT_dev: stream tokens left after the hot holes
   for (uint32_t v = u + 1; v < U; ++v) {
     const uint32_t s2 = u_slot[v];
     if (hot_of(s2)) continue;

@@ -81,6 +81,12 @@ __device__ __forceinline__ uint32_t block_min_after(uint32_t v, uint32_t* sm /* 
 // across tiles and writes docid, tf = sum of counts (coalesced through shared memory), post_off[rank]
 // and the token offset cstart[rank] of the term's first element (cf = difference).  Runs that continue
 // across ranges are completed by k_rle_fixup (range_lead = tokens before the range's first posting).
+// elements per CTA range of the run-length pass (a multiple of its tile); engine.cu rle() cuts the same
+__host__ __device__ __forceinline__ uint64_t rle_per(uint64_t N, uint64_t G) {
+  const uint64_t per = (N + G - 1) / G;
+  return (per + kRleTile - 1) / kRleTile * kRleTile;
+}
+
 constexpr uint32_t kCountShift = 25;
 constexpr uint32_t kRankMask = (1u << kCountShift) - 1u;
 
@@ -129,7 +135,11 @@ __device__ __forceinline__ void rle_flags(const uint32_t* k, const uint32_t* d, 
 template <bool COUNTS>
 __global__ void __launch_bounds__(kRleThreads) k_rle_count(const uint32_t* __restrict__ key, const uint32_t* __restrict__ doc,
                                                            uint64_t N, uint64_t per, uint32_t* range_cnt,
-                                                           uint64_t* range_tok) {
+                                                           uint64_t* range_tok, const uint32_t* __restrict__ n_dev) {
+  if (n_dev) {  // the actual length (N is an upper bound): ranges re-cut for it
+    N = min(N, (uint64_t)*n_dev);
+    per = rle_per(N, gridDim.x);
+  }
   const uint64_t lo = (uint64_t)blockIdx.x * per;
   const uint64_t hi = lo + per < N ? lo + per : N;
   uint32_t c = 0;
@@ -174,7 +184,12 @@ __global__ void WJ_RLE_BOUNDS k_rle_write_tma(const uint32_t* __restrict__ key,
                                                                uint64_t per, const uint32_t* __restrict__ range_off,
                                                                const uint64_t* __restrict__ range_tok_off,
                                                                uint32_t* out_doc, uint32_t* out_tf, uint64_t* post_off,
-                                                               uint64_t* cstart, uint32_t* range_lead) {
+                                                               uint64_t* cstart, uint32_t* range_lead,
+                                                               const uint32_t* __restrict__ n_dev) {
+  if (n_dev) {
+    N = min(N, (uint64_t)*n_dev);
+    per = rle_per(N, gridDim.x);
+  }
   extern __shared__ __align__(128) uint32_t rsm[];
   __shared__ __align__(8) uint64_t bar[2];
   __shared__ uint32_t sm[16];
@@ -187,7 +202,10 @@ __global__ void WJ_RLE_BOUNDS k_rle_write_tma(const uint32_t* __restrict__ key,
   uint32_t* cpi = rsm + 6 * kRleTile;  // exclusive token-count prefix of each tile item (+ total)
   const uint64_t lo = (uint64_t)blockIdx.x * per;
   const uint64_t hi = lo + per < N ? lo + per : N;
-  if (lo >= hi) return;
+  if (lo >= hi) {  // an empty range (N shrank below the launch's upper bound)
+    if (threadIdx.x == 0) range_lead[blockIdx.x] = 0;
+    return;
+  }
   auto issue = [&](int s, uint64_t base) {  // thread 0
     const uint32_t cnt = (uint32_t)min((uint64_t)kRleTile, hi - base);
     const uint32_t b = (cnt * 4 + 15) & ~15u;

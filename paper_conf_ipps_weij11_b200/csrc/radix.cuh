@@ -66,9 +66,21 @@ __device__ __forceinline__ K rs_dkey(K k, K kmask) { return MASK ? (k & kmask) :
 // the map gather of the first pass, which is L2-latency bound at 2 CTAs/SM.
 constexpr int kRsUpSplit = 4;
 
+// elements per CTA range for n elements over G ranges (a multiple of the 4096-element tile); the
+// host uses the same cut (engine.cu sort_pairs)
+__host__ __device__ __forceinline__ uint64_t rs_per(uint64_t n, uint64_t G) {
+  const uint64_t per = (n + G - 1) / G;
+  return (per + kOsTile - 1) / kOsTile * kOsTile;
+}
+
 template <typename K, bool HOLES, bool MASK>
 __global__ void __launch_bounds__(256) k_rs_up(K* keys, uint64_t n, uint64_t per, int shift,
-                                               const uint32_t* __restrict__ map, uint32_t* hist, K kmask) {
+                                               const uint32_t* __restrict__ map, uint32_t* hist, K kmask,
+                                               const uint32_t* __restrict__ n_dev) {
+  if (n_dev) {  // elements left by an earlier hole-compacting pass: ranges re-cut for that count
+    n = min(n, (uint64_t)*n_dev);
+    per = rs_per(n, gridDim.x / kRsUpSplit);
+  }
   __shared__ uint32_t h[kOsWarps][256];
   const int w = threadIdx.x >> 5;
   for (int x = 0; x < kOsWarps; ++x) h[x][threadIdx.x] = 0;
@@ -167,7 +179,11 @@ template <typename K, bool HOLES, bool MASK>
 __global__ void WJ_DS_BOUNDS k_rs_down2(const K* __restrict__ kin, const uint32_t* __restrict__ vin,
                                                          K* __restrict__ kout, uint32_t* __restrict__ vout, uint64_t n,
                                                          uint64_t per, int shift, const uint32_t* __restrict__ offs,
-                                                         K kmask) {
+                                                         K kmask, const uint32_t* __restrict__ n_dev) {
+  if (n_dev) {
+    n = min(n, (uint64_t)*n_dev);
+    per = rs_per(n, gridDim.x);
+  }
   extern __shared__ __align__(128) unsigned char os_smem[];
   __shared__ __align__(8) uint64_t bar[2];
   __shared__ uint32_t wcnt[kDsWarps][256];

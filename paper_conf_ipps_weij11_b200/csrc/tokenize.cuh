@@ -384,15 +384,18 @@ __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* tabl
 // P:202-208), recognised by the hot id k_hot_seed stored in their table slot, do not enter the
 // (slot, docID) stream (their tokens leave holes, key 0, dropped by the first sort pass) and are
 // counted in the dense (hot term x document) matrix eo.hot_mat, through
-// per-warp shared-memory counters for the first kHotDocs documents of the warp's range (flushed with
-// one global add per nonzero counter at the range's end); the matrix rows become the hot terms'
-// partial lists (k_hot_scatter).
+// per-warp shared-memory counters for the first kHotDocs documents of the warp's range (one global add
+// per nonzero counter at the range's end); the matrix rows become the hot terms' partial lists
+// (k_hot_scatter).
 constexpr uint32_t kHotMaxH = 64;
 constexpr uint32_t kHotDocs = 2;
-constexpr uint32_t kHotWords = kHotDocs * kHotMaxH / 2;  // u16 counter pairs per warp
+constexpr uint32_t kHotWords = kHotDocs * kHotMaxH;  // u32 counters per warp: [document][hot id]
+#ifndef WJ_EMIT_HOT_MINB
+#define WJ_EMIT_HOT_MINB 5  // 48 registers: at 40 the hot instance spills (emit 3.84 vs 2.74 ms)
+#endif
 
 template <bool HOT>
-__global__ void __launch_bounds__(kTokThreads, WJ_EMIT_MINB) k_tok_emit(ChunkView cv, uint32_t n_segs,
+__global__ void __launch_bounds__(kTokThreads, HOT ? WJ_EMIT_HOT_MINB : WJ_EMIT_MINB) k_tok_emit(ChunkView cv, uint32_t n_segs,
                                                           const uint64_t* kstart, const uint32_t* range_off, EmitOut eo) {
   __shared__ __align__(16) uint32_t win[kTokWarps][kWinBytes / 4];
   __shared__ uint32_t queue[kTokWarps][kQueueCap + 1];
@@ -434,6 +437,7 @@ __global__ void __launch_bounds__(kTokThreads, WJ_EMIT_MINB) k_tok_emit(ChunkVie
   auto flush = [&]() {
     for (uint32_t r = 0; r < qn; r += 32) {
       const uint32_t idx = r + lane;
+      uint32_t hkey = 0xFFFFFFFFu;  // HOT: [document][hot id] counter of this lane's hot token
       if (idx < qn) {
         const uint32_t e = q[idx];
         const uint32_t s_win = e >> 8, len = e & 255u;
@@ -471,18 +475,17 @@ __global__ void __launch_bounds__(kTokThreads, WJ_EMIT_MINB) k_tok_emit(ChunkVie
         // a hot term's slot was seeded with its hot id in k1 (k_hot_seed): table_insert returns it
         const uint32_t slot =
             table_insert(cv.text, eo.table, eo.slot_ref, eo.cap, h, k0, k1, s_abs, len, w32, s_win, eo.overflow, &hid);
-#ifndef WJ_HOT_NO_ATOMIC
-        if (HOT && hid) {  // hot term: count it (the stream keeps a hole, key 0)
+        if (HOT && hid) {  // hot term: counted below (the stream keeps a hole, key 0)
           const uint32_t dd = ldoc - (uint32_t)(k_range_lo - 1), hh = hid - 1;
-          if (dd < kHotDocs) atomicAdd(&hc[dd * (kHotMaxH / 2) + (hh >> 1)], 1u << (16 * (hh & 1)));
+          if (dd < kHotDocs) hkey = dd * kHotMaxH + hh;
           else atomicAdd(&eo.hot_mat[(uint64_t)hh * eo.hot_docs + ldoc], 1u);
         }
-#endif
         // branch-free stores: stream element slot | count 1 << 25, or a hole (the docID is not read)
         __stcs(eo.slot + out, (HOT && hid) ? 0u : (slot | (1u << 25)));
         __stcs(eo.doc + out, eo.doc_base + ldoc);
         if (eo.dbg_start) { eo.dbg_start[out] = s_abs; eo.dbg_len[out] = len; }
       }
+      if (HOT && hkey != 0xFFFFFFFFu) atomicAdd(&hc[hkey], 1u);  // (a warp match first was slower)
     }
     obase += qn;
     qn = 0;
@@ -573,18 +576,13 @@ __global__ void __launch_bounds__(kTokThreads, WJ_EMIT_MINB) k_tok_emit(ChunkVie
     }
   }
   flush();
-#ifndef WJ_HOT_NO_FLUSH
   if (HOT) {  // the range's hot counters -> the (hot term x document) matrix
     const uint32_t d0 = (uint32_t)(k_range_lo - 1);
     for (uint32_t i = lane; i < kHotWords; i += 32) {
       const uint32_t x = hc[i];
-      if (x == 0) continue;
-      const uint32_t dd = i / (kHotMaxH / 2), hh = 2 * (i % (kHotMaxH / 2));
-      if (x & 0xFFFFu) atomicAdd(&eo.hot_mat[(uint64_t)hh * eo.hot_docs + d0 + dd], x & 0xFFFFu);
-      if (x >> 16) atomicAdd(&eo.hot_mat[(uint64_t)(hh + 1) * eo.hot_docs + d0 + dd], x >> 16);
+      if (x) atomicAdd(&eo.hot_mat[(uint64_t)(i % kHotMaxH) * eo.hot_docs + d0 + i / kHotMaxH], x);
     }
   }
-#endif
 }
 
 }  // namespace wj
