@@ -201,7 +201,8 @@ struct UniqueView {
   const uint32_t* cache;
 };
 
-// Warp-cooperative descent for one key.  Returns termID (tid) or kMiss with *ins_rank set.
+// Warp-cooperative descent for one key (retrieval, k_query).  Returns termID (tid) or kMiss with
+// *ins_rank set.
 __device__ __forceinline__ uint32_t probe_key(const DictView& dv, const uint4& w, const uint8_t* text, uint32_t ref,
                                               uint32_t len, uint32_t bucket, uint32_t cache, uint32_t* ins_rank) {
   const uint32_t lane = lane_id();
@@ -233,13 +234,92 @@ __device__ __forceinline__ uint32_t probe_key(const DictView& dv, const uint4& w
   }
 }
 
-// probe every unique term of the chunk: warp per term, grid-stride
-__global__ void k_probe(DictView dv, UniqueView uv, uint32_t U, uint32_t* tid_out, uint32_t* rank_out) {
+// Probe with four keys per warp (8 lanes per key): a descent is a chain of dependent loads, so the
+// probe is latency-bound; four independent descents per warp and the node's key line (caches) and
+// child line loaded together halve the dependent loads per level and quadruple the keys in flight.
+// Lane gl of a group holds words 4gl..4gl+3 of each line (word 0 of line 0 = count, word j >= 1 =
+// cache j-1; line 3 = children).  Same result as probe_key.
+constexpr int kProbeKeysPerWarp = 4;
+__global__ void __launch_bounds__(256) k_probe4(DictView dv, UniqueView uv, uint32_t U, uint32_t* tid_out,
+                                                uint32_t* rank_out) {
+  const uint32_t lane = lane_id(), g = lane >> 3, gl = lane & 7;
   const uint32_t warps = gridDim.x * (blockDim.x >> 5);
-  for (uint32_t u = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); u < U; u += warps) {
-    uint32_t r = 0;
-    const uint32_t t = probe_key(dv, uv.w[u], uv.text, uv.ref[u], uv.len[u], uv.bucket[u], uv.cache[u], &r);
-    if (lane_id() == 0) { tid_out[u] = t; rank_out[u] = r; }
+  for (uint32_t base = (blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * kProbeKeysPerWarp; base < U;
+       base += warps * kProbeKeysPerWarp) {
+    const uint32_t u = base + g;
+    const bool active0 = u < U;
+    uint32_t bucket = 0, cache = 0, len = 0, ref = 0, n = 0;
+    uint4 w = make_uint4(0, 0, 0, 0);
+    if (active0) {
+      bucket = uv.bucket[u];
+      cache = uv.cache[u];
+      len = uv.len[u];
+      ref = uv.ref[u];
+      w = uv.w[u];
+      n = dv.coll_n[bucket];
+    }
+    const uint32_t plen = bucket_plen(bucket), slen = len - plen;
+    uint32_t node = active0 && n ? dv.coll_root[bucket] : 0u, lo = 0, m = n, h = height_of(n);
+    bool done = !active0 || n == 0;
+    uint32_t res_tid = kMiss, res_rank = 0;
+    // every lane of the warp runs the loop until all four descents are done (warp-synchronous ballots)
+    while (__any_sync(0xffffffffu, !done)) {
+      uint4 c4 = make_uint4(0, 0, 0, 0), ch4 = make_uint4(0, 0, 0, 0);
+      const Node* nd = dv.nodes + node;
+      if (!done) {
+        c4 = __ldg((const uint4*)nd + gl);                 // line 0: count, caches
+        if (h > 1) ch4 = __ldg((const uint4*)nd->child + gl);  // line 3: children (same round trip)
+      }
+      const uint32_t cnt = __shfl_sync(0xffffffffu, c4.x, lane & ~7u);
+      const uint32_t cw[4] = {c4.x, c4.y, c4.z, c4.w};
+      uint32_t ltm = 0, eqm = 0;  // per lane, bit t: entry 4gl+t-1 is < key / == key
+#pragma unroll
+      for (int t = 0; t < 4; ++t) {
+        const uint32_t j = 4 * gl + t;  // word j = cache j-1
+        const bool valid = !done && j >= 1 && j - 1 < cnt;
+        int cmp = 0;
+        if (valid) {
+          if (cache != cw[t]) cmp = cache < cw[t] ? -1 : 1;
+          else if (slen >= 4) cmp = cmp_sfx_arena(w, uv.text, ref, plen, slen, dv.arena, __ldg(&nd->str[j - 1]));
+        }
+        ltm |= (valid && cmp > 0 ? 1u : 0u) << t;
+        eqm |= (valid && cmp == 0 ? 1u : 0u) << t;
+      }
+      // group-wide: number of entries below the key, and the first equal entry
+      uint32_t pos = __popc(ltm), eqj = eqm ? 4 * gl + __ffs(eqm) - 2 : 0xFFFFFFFFu;
+#pragma unroll
+      for (int o = 1; o < 8; o <<= 1) {
+        pos += __shfl_xor_sync(0xffffffffu, pos, o);
+        eqj = min(eqj, __shfl_xor_sync(0xffffffffu, eqj, o));
+      }
+      if (!done) {
+        if (eqj != 0xFFFFFFFFu) {  // hit
+          res_tid = __ldg(&nd->post[eqj]);
+          done = true;
+        } else if (h == 1) {       // miss at a leaf: insertion rank
+          res_rank = lo + pos;
+          done = true;
+        }
+      }
+      // child[pos]: word pos of line 3 is in group lane pos / 4, component pos % 4
+      const uint32_t chw[4] = {ch4.x, ch4.y, ch4.z, ch4.w};
+      uint32_t mine = 0;
+#pragma unroll
+      for (int t = 0; t < 4; ++t)
+        if ((pos & 3u) == (uint32_t)t) mine = chw[t];
+      const uint32_t child = __shfl_sync(0xffffffffu, mine, (lane & ~7u) + ((pos >> 2) & 7u));
+      if (!done) {
+        const Split sp = split_of(m, h);
+        lo = child_lo(sp, lo, pos);
+        m = child_m(sp, pos);
+        node = child;
+        --h;
+      }
+    }
+    if (active0 && gl == 0) {
+      tid_out[u] = res_tid;
+      rank_out[u] = res_rank;
+    }
   }
 }
 

@@ -953,9 +953,10 @@ struct wj_index {
     if (V > 0) {
       UniqueView uv{text, (const uint4*)u_w.p, (const uint32_t*)u_ref.p, (const uint32_t*)u_len.p,
                     (const uint32_t*)u_bucket.p, (const uint32_t*)u_cache.p};
-      const unsigned blocks = (unsigned)std::min<uint64_t>((U + 7) / 8, 148ull * 64);
+      const unsigned blocks = (unsigned)std::min<uint64_t>((U + 8 * kProbeKeysPerWarp - 1) / (8 * kProbeKeysPerWarp),
+                                                          148ull * 64);
       ktime(WJ_KERNEL_PROBE, [&] {
-        k_probe<<<blocks, 256, 0, st>>>(dv, uv, (uint32_t)U, ut, urk);
+        k_probe4<<<blocks, 256, 0, st>>>(dv, uv, (uint32_t)U, ut, urk);
         launched();
       });
     } else {

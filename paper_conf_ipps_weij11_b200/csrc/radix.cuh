@@ -243,7 +243,10 @@ __global__ void WJ_DS_BOUNDS k_rs_down2(const K* __restrict__ kin, const uint32_
       dg[k] = (uint32_t)((rs_dkey<K, MASK>(kv, kmask) >> shift) & 255u);
       // 64-bit keys (all distinct: new-term sort): shared-memory masks; 32-bit keys (Zipf-skewed
       // ranks, many equal digits per warp -> atomic conflicts): ballots
-      rank[k] = sizeof(K) == 8 ? digit_peers_smem(wbins[w], dg[k], valid) : digit_peers(dg[k], valid);
+#ifndef WJ_DS_SMEM_PEERS
+#define WJ_DS_SMEM_PEERS 0
+#endif
+      rank[k] = (sizeof(K) == 8 || WJ_DS_SMEM_PEERS) ? digit_peers_smem(wbins[w], dg[k], valid) : digit_peers(dg[k], valid);
     }
 #pragma unroll
     for (int k = 0; k < kDsItems; ++k) {
