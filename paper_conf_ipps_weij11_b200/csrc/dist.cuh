@@ -50,16 +50,18 @@ __global__ void k_xid(const uint32_t* sorted_u, uint32_t U, const uint32_t* u_ow
 }
 
 struct PackTermSize {
-  const uint32_t* sorted_u;
+  const uint32_t* sorted_u;  // nullptr: identity (unique terms already in owner order)
   const uint32_t* u_len;
-  __device__ __forceinline__ uint64_t operator()(uint64_t j) const { return (uint64_t)u_len[sorted_u[j]] + 1; }
+  __device__ __forceinline__ uint64_t operator()(uint64_t j) const {
+    return (uint64_t)u_len[sorted_u ? sorted_u[j] : (uint32_t)j] + 1;
+  }
 };
 
 __global__ void k_pack_terms(const uint32_t* sorted_u, uint32_t U, const uint64_t* boff, const uint4* u_w,
                              const uint8_t* text, const uint32_t* u_ref, const uint32_t* u_len, uint8_t* out) {
   const uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
   if (j >= U) return;
-  const uint32_t u = sorted_u[j];
+  const uint32_t u = sorted_u ? sorted_u[j] : j;
   const uint4 w = u_w[u];
   const uint32_t len = u_len[u], ref = u_ref[u];
   uint8_t* o = out + boff[j];
@@ -119,40 +121,41 @@ __global__ void k_xid_map(const uint32_t* syn_slot, uint32_t n, const Slot* tabl
 }
 
 // ------------------------------------------------------------------ sender-side partial lists
-// (SURVEY 8(e)): every rank sorts and run-length encodes its own documents' stream by
-// gpos = (owner's first term index + xid), so the postings it sends to owner o are one contiguous range
+// (SURVEY 8(e)): every rank's chunk table is partitioned by owner, so sorting and
+// run-length encoding its stream by slot makes the postings it sends to owner o one contiguous range
 // of (docID, tf) pairs, grouped per term (P:160-162's per-term grouping, aggregated to one posting per
 // (term, document)); a header (df, cf) per term and the folded term bytes go with them.
 
-// slot -> gpos of its unique term (the stream sort key)
-__global__ void k_slot_gpos(const Slot* table, uint32_t C, const uint32_t* slot_uid, const uint32_t* u_owner,
-                            const uint32_t* xid, const uint64_t* t_off, uint32_t* km) {
-  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= C || table[i].k0 == 0) return;
-  const uint32_t u = slot_uid[i];
-  km[i] = (uint32_t)t_off[u_owner[u]] + xid[u];
+// per unique term u (slot order = owner order: the chunk table is partitioned by owner): df, cf of
+// its local partial list from the run-length output (post_off / cstart indexed by slot; every unique
+// term occurs); P_dev = postings of the chunk, NT = its tokens
+__global__ void k_term_hdr(const uint32_t* u_slot, uint32_t U, const uint64_t* post_off, const uint64_t* cstart,
+                           const uint32_t* P_dev, uint64_t NT, uint32_t* df, uint32_t* cf) {
+  const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
+  if (u >= U) return;
+  const uint32_t s = u_slot[u];
+  const uint64_t b = u + 1 < U ? post_off[u_slot[u + 1]] : (uint64_t)*P_dev;
+  const uint64_t tb = u + 1 < U ? cstart[u_slot[u + 1]] : NT;
+  df[u] = (uint32_t)(b - post_off[s]);
+  cf[u] = (uint32_t)(tb - cstart[s]);
 }
 
-// per term (gpos g): df, cf of its local partial list from the run-length output (post_off / cstart
-// indexed by gpos; every gpos occurs); P_dev = postings of the chunk, NT = its tokens
-__global__ void k_term_hdr(const uint64_t* post_off, const uint64_t* cstart, uint32_t U, const uint32_t* P_dev, uint64_t NT,
-                           uint32_t* df, uint32_t* cf) {
-  const uint32_t g = blockIdx.x * blockDim.x + threadIdx.x;
-  if (g >= U) return;
-  const uint64_t b = g + 1 < U ? post_off[g + 1] : (uint64_t)*P_dev;
-  const uint64_t tb = g + 1 < U ? cstart[g + 1] : NT;
-  df[g] = (uint32_t)(b - post_off[g]);
-  cf[g] = (uint32_t)(tb - cstart[g]);
-}
-
-// per owner o (o <= K): postings / tokens before its first term; bounds[o] = t_off[o] (U: the end)
-__global__ void k_owner_bounds(const uint64_t* post_off, const uint64_t* cstart, const uint64_t* t_off, uint32_t K,
-                               uint32_t U, const uint32_t* P_dev, uint64_t NT, uint64_t* p_off, uint64_t* c_off) {
+// per owner o (o <= K): postings / tokens before its first term (t_off[o] = its first unique term)
+__global__ void k_owner_bounds(const uint32_t* u_slot, const uint64_t* post_off, const uint64_t* cstart,
+                               const uint64_t* t_off, uint32_t K, uint32_t U, const uint32_t* P_dev, uint64_t NT,
+                               uint64_t* p_off, uint64_t* c_off) {
   const uint32_t o = blockIdx.x * blockDim.x + threadIdx.x;
   if (o > K) return;
-  const uint64_t g = t_off[o];
-  p_off[o] = g < U ? post_off[g] : (uint64_t)*P_dev;
-  c_off[o] = g < U ? cstart[g] : NT;
+  const uint64_t u = t_off[o];
+  p_off[o] = u < U ? post_off[u_slot[u]] : (uint64_t)*P_dev;
+  c_off[o] = u < U ? cstart[u_slot[u]] : NT;
+}
+
+// first unique term of each table partition: t_off[o] = uid of slot o * Cp (exclusive scan), t_off[K] = U
+__global__ void k_part_bounds(const uint32_t* uid, uint32_t K, uint64_t Cp, const uint32_t* U_dev, uint64_t* t_off) {
+  const uint32_t o = blockIdx.x * blockDim.x + threadIdx.x;
+  if (o > K) return;
+  t_off[o] = o < K ? uid[(uint64_t)o * Cp] : *U_dev;
 }
 
 // owner side: the records of source s's terms (xid order = the order s sent them): termID from the

@@ -578,6 +578,9 @@ struct wj_index {
     eo.table = tab;
     eo.slot_ref = sref;
     eo.cap = (uint32_t)C;
+    eo.parts = tab_parts;
+    eo.part_cap = (uint32_t)(C / tab_parts);
+    eo.owner_tab = owner_ready ? (const uint32_t*)owner_tab.p : nullptr;
     eo.doc_base = doc_base;
     eo.slot = slot_out;
     eo.doc = doc_out;
@@ -587,12 +590,14 @@ struct wj_index {
     const uint64_t ranges = (n_segs + kSegsPerWarp - 1) / kSegsPerWarp;
     const unsigned grid = (unsigned)((ranges + kTokWarps - 1) / kTokWarps);
     ktime(WJ_KERNEL_TOKENIZE_EMIT, [&] {
-      if (eo.hot_mat)
-        k_tok_emit<true><<<grid, kTokThreads, 0, st>>>(cv, (uint32_t)n_segs, (const uint64_t*)kstart.p,
-                                                       (const uint32_t*)seg_cnt.p, eo);
+      const uint64_t* ks = (const uint64_t*)kstart.p;
+      const uint32_t* ro = (const uint32_t*)seg_cnt.p;
+      if (eo.parts > 1)
+        k_tok_emit<false, true><<<grid, kTokThreads, 0, st>>>(cv, (uint32_t)n_segs, ks, ro, eo);
+      else if (eo.hot_mat)
+        k_tok_emit<true, false><<<grid, kTokThreads, 0, st>>>(cv, (uint32_t)n_segs, ks, ro, eo);
       else
-        k_tok_emit<false><<<grid, kTokThreads, 0, st>>>(cv, (uint32_t)n_segs, (const uint64_t*)kstart.p,
-                                                        (const uint32_t*)seg_cnt.p, eo);
+        k_tok_emit<false, false><<<grid, kTokThreads, 0, st>>>(cv, (uint32_t)n_segs, ks, ro, eo);
       launched();
     });
   }
@@ -745,9 +750,13 @@ struct wj_index {
   // ---------------------------------------------------------------- one chunk
   // K1 (count + emit + dedup): tokens of cv into (slot, docID) arrays given by out_alloc(Nc); unique
   // terms of the chunk into the u_* arrays.  Returns Nc; sets C (table capacity), U.
+  // parts > 1 (multi-rank): the table is cut into `parts` equal partitions, partition o holding the
+  // terms whose trie collection rank o owns, so slot order groups the unique terms and
+  // the sorted stream by owner
+  uint32_t tab_parts = 1;  // partitions of the table emit_tokens fills
   template <class F>
   uint64_t tokenize_dedup(const ChunkView& cv, uint32_t doc_base, F&& out_alloc, uint64_t& C, uint64_t& U,
-                          uint32_t*& slot_out, uint32_t*& doc_out, bool allow_hot = false) {
+                          uint32_t*& slot_out, uint32_t*& doc_out, bool allow_hot = false, uint32_t parts = 1) {
     const uint64_t n_segs = (cv.n_bytes + kSegBytes - 1) / kSegBytes;
     C = 0;
     U = 0;
@@ -769,7 +778,9 @@ struct wj_index {
     est = std::min<uint64_t>(est, Nc + 16);
     // stream elements carry the slot below the count bits (slot | count << kCountShift): C <= 2^25
     constexpr uint64_t kMaxC = (uint64_t)kRankMask + 1;
-    C = std::min<uint64_t>(table_cap(est * table_pct / 100), kMaxC);
+    uint64_t Cp = table_cap(est * table_pct / 100 / parts);  // slots per partition
+    C = std::min<uint64_t>(Cp * parts, kMaxC / parts * parts);
+    tab_parts = parts;
     uint32_t* slot_uid = nullptr;
     for (;;) {
       Slot* tab = buf<Slot>(table, C);
@@ -792,12 +803,15 @@ struct wj_index {
       U = (uint32_t)h_scal[2];
       if (((uint32_t)h_scal[5]) == 0) break;
       // probe sequence overflow: retry with a larger table
-      if (C >= kMaxC)
+      if (C >= kMaxC / parts * parts) {
+        tab_parts = 1;
         throw StatusError{WJ_ERR_CAPACITY, "more than ~2^25 distinct terms in one index_add_stream call: pass smaller chunks"};
-      C = std::min<uint64_t>(C * 2, kMaxC);
+      }
+      C = std::min<uint64_t>(C * 2, kMaxC / parts * parts);
       ++table_retries;
       phase(WJ_PHASE_TOKENIZE);
     }
+    tab_parts = 1;
     unique_last = U;
     table_est = (U * 5) / 4;
     // unique terms: first occurrence, folded bytes, Table I bucket, stripped-suffix cache, sort key
@@ -1306,7 +1320,7 @@ struct wj_index {
         if (nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 tokens in one chunk"};
         sp = buf<uint32_t>(pc_key, nc + 16);
         dp = buf<uint32_t>(pc_doc, nc + 16);
-      }, C, U, lslot, ldoc, false);
+      }, C, U, lslot, ldoc, false, (uint32_t)K);  // table partitioned by owner (slot order = owner order)
     }
     std::vector<uint64_t> t_off(K + 1, 0), b_off(K + 1, 0), p_off(K + 1, 0), c_off(K + 1, 0);
     uint8_t* send_terms = (uint8_t*)grow(x_send, 16);
@@ -1325,45 +1339,24 @@ struct wj_index {
     uint32_t* hdf = buf<uint32_t>(x_hdf, U + 1);
     uint32_t* hcf = buf<uint32_t>(x_hcf, U + 1);
     uint64_t* bnd = buf<uint64_t>(x_bnd, 2 * (K + 1));
-    uint32_t* km = nullptr;
-    if (U > 0) {
-      // 2. unique terms grouped by owner (stable): t_off, xid, gpos map, packed term bytes
-      uint32_t* own = buf<uint32_t>(x_owner, U + 16);
-      uint32_t* iota = buf<uint32_t>(x_iota, U + 16);
-      uint32_t* oc = buf<uint32_t>(x_cnt, 2 * K);
-      WJ_CUDA_CHECK(cudaMemsetAsync(oc, 0, 2 * K * 4, st));
-      k_owner<<<grid_for(U, 256), 256, 0, st>>>((const uint32_t*)u_bucket.p, (uint32_t)U, (uint32_t)K,
-                                                owner_ready ? (const uint32_t*)owner_tab.p : nullptr, own, iota, oc);
-      launched();
-      const uint32_t* sorted_u = iota;
-      if (K > 1) {
-        uint32_t* own2 = buf<uint32_t>(x_owner2, U + 16);
-        uint32_t* srt2 = buf<uint32_t>(x_sorted2, U + 16);
-        WJ_CUDA_CHECK(cudaMemcpyAsync(own2, own, U * 4, cudaMemcpyDeviceToDevice, st));
-        int obits = 0;
-        while ((1 << obits) < K) ++obits;
-        uint32_t* srt1 = (uint32_t*)grow(x_sorted, (U + 16) * 4);
-        sorted_u = sort_pairs<uint32_t>(own2, iota, srt1, srt2, U, 0, obits, nullptr, false) ? srt2 : iota;
-      }
-      std::vector<uint32_t> oc_h(K);
-      WJ_CUDA_CHECK(cudaMemcpyAsync(oc_h.data(), oc, K * 4, cudaMemcpyDeviceToHost, st));
-      sync();
-      for (int o = 0; o < K; ++o) t_off[o + 1] = t_off[o] + oc_h[o];
-      WJ_CUDA_CHECK(cudaMemcpyAsync(toff_d, t_off.data(), (K + 1) * 8, cudaMemcpyHostToDevice, st));
-      uint32_t* xid = buf<uint32_t>(x_xid, U);
-      k_xid<<<grid_for(U, 256), 256, 0, st>>>(sorted_u, (uint32_t)U, own, toff_d, xid);
-      launched();
-      km = buf<uint32_t>(x_keymap, C);
-      k_slot_gpos<<<grid_for(C, 256), 256, 0, st>>>((const Slot*)table.p, (uint32_t)C, (const uint32_t*)uid.p, own, xid,
-                                                    toff_d, km);
+    const bool solo = K == 1;  // one rank owns everything: no exchange, the local terms are the owner's
+    if (U > 0 && solo) {
+      t_off[1] = U;
+      WJ_CUDA_CHECK(cudaMemcpyAsync(toff_d, t_off.data(), 2 * 8, cudaMemcpyHostToDevice, st));
+    } else if (U > 0) {
+      // 2. the unique terms are in owner order already: t_off = first unique term of each partition
+      k_part_bounds<<<grid_for(K + 1, 256), 256, 0, st>>>((const uint32_t*)uid.p, (uint32_t)K, C / K,
+                                                          (const uint32_t*)(dscal() + 2), toff_d);
       launched();
       uint64_t* boff = buf<uint64_t>(x_boff, U + 1);
-      scan<uint64_t>(PackTermSize{sorted_u, (const uint32_t*)u_len.p}, U, boff, boff + U);
+      scan<uint64_t>(PackTermSize{nullptr, (const uint32_t*)u_len.p}, U, boff, boff + U);
+      WJ_CUDA_CHECK(cudaMemcpyAsync(t_off.data(), toff_d, (K + 1) * 8, cudaMemcpyDeviceToHost, st));
+      sync();
       for (int o = 0; o <= K; ++o)
         WJ_CUDA_CHECK(cudaMemcpyAsync(&b_off[o], boff + t_off[o], 8, cudaMemcpyDeviceToHost, st));
       sync();
       send_terms = (uint8_t*)grow(x_send, b_off[K] + 16);
-      k_pack_terms<<<grid_for(U, 256), 256, 0, st>>>(sorted_u, (uint32_t)U, boff, (const uint4*)u_w.p, text,
+      k_pack_terms<<<grid_for(U, 256), 256, 0, st>>>(nullptr, (uint32_t)U, boff, (const uint4*)u_w.p, text,
                                                     (const uint32_t*)u_ref.p, (const uint32_t*)u_len.p, send_terms);
       launched();
     }
@@ -1373,7 +1366,8 @@ struct wj_index {
       cnt[o] = t_off[o + 1] - t_off[o];
       cnt[K + o] = b_off[o + 1] - b_off[o];
     }
-    xport->allgather(cnt.data(), 2 * K, all.data(), st);
+    if (!solo) xport->allgather(cnt.data(), 2 * K, all.data(), st);
+    else all = cnt;
     std::vector<uint64_t> rt(K + 1, 0), rb(K + 1, 0);
     for (int s = 0; s < K; ++s) {
       const uint64_t* c = all.data() + (size_t)s * 2 * K;
@@ -1394,30 +1388,31 @@ struct wj_index {
       WJ_CUDA_CHECK(cudaStreamSynchronize(st));
       xms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - tx).count();
     };
-    exchange([&] { xport->alltoallv(send_terms, b_off.data(), recv_terms, rb.data(), st); });
-    // 4. overlapped: side stream = the local stream sorted by gpos (map applied by the first pass) and
+    if (!solo) exchange([&] { xport->alltoallv(send_terms, b_off.data(), recv_terms, rb.data(), st); });
+    uint32_t* us = buf<uint32_t>(x_xid, U + 1);  // the local unique terms' slots (u_slot is reused by the owner)
+    // 4. overlapped: side stream = the local stream sorted by slot (= by owner, then term) and
     //    run-length encoded, headers, per-owner bounds; dictionary stream = the owner's dictionary
     if (U > 0) {
       int bits = 0;
-      while (bits < 32 && ((uint64_t)1 << bits) < U) ++bits;
+      while (bits < 32 && ((uint64_t)1 << bits) < C) ++bits;
       uint32_t* kt = (uint32_t*)pc_key.p;
       uint32_t* dt = (uint32_t*)pc_doc.p;
       uint32_t* k1 = buf<uint32_t>(sk1, Nc + 16);
       uint32_t* v1 = buf<uint32_t>(sv1, Nc + 16);
-      uint64_t* po = buf<uint64_t>(pc_po, U + 1);
-      uint64_t* cs = buf<uint64_t>(pc_cs, U + 1);
+      uint64_t* po = buf<uint64_t>(pc_po, C + 1);
+      uint64_t* cs = buf<uint64_t>(pc_cs, C + 1);
+      WJ_CUDA_CHECK(cudaMemcpyAsync(us, u_slot.p, U * 4, cudaMemcpyDeviceToDevice, st));
       phase(-1);
       WJ_CUDA_CHECK(cudaEventRecord(ev_fork, st));
       WJ_CUDA_CHECK(cudaStreamWaitEvent(side_st, ev_fork, 0));
       swap_side();
       try {
         phase(WJ_PHASE_SORT);
-        std::vector<std::pair<uint64_t, const uint32_t*>> segs{{0, km}};
-        const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, std::max(bits, 1), nullptr, true, &segs, kRankMask);
+        const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, std::max(bits, 1), nullptr, true);
         phase(WJ_PHASE_POSTINGS);
         rle(in1 ? k1 : kt, in1 ? v1 : dt, Nc, false, od, of, po, cs);
-        k_term_hdr<<<grid_for(U, 256), 256, 0, st>>>(po, cs, (uint32_t)U, (const uint32_t*)(dscal() + 8), Nc, hdf, hcf);
-        k_owner_bounds<<<grid_for(K + 1, 256), 256, 0, st>>>(po, cs, toff_d, (uint32_t)K, (uint32_t)U,
+        k_term_hdr<<<grid_for(U, 256), 256, 0, st>>>(us, (uint32_t)U, po, cs, (const uint32_t*)(dscal() + 8), Nc, hdf, hcf);
+        k_owner_bounds<<<grid_for(K + 1, 256), 256, 0, st>>>(us, po, cs, toff_d, (uint32_t)K, (uint32_t)U,
                                                             (const uint32_t*)(dscal() + 8), Nc, bnd, bnd + K + 1);
         launched(2);
         phase(-1);
@@ -1437,6 +1432,10 @@ struct wj_index {
       WJ_CUDA_CHECK(cudaStreamWaitEvent(hp_st, ev_fork, 0));
       std::swap(st, hp_st);
       try {
+        if (solo) {  // the owner's terms are the local unique terms: no re-tokenisation
+          dictionary_update(text, U);
+          sslot = us;
+        } else {
         uint64_t* so = buf<uint64_t>(x_syn_off, 2);
         const uint64_t h2[2] = {0, rb[K]};
         WJ_CUDA_CHECK(cudaMemcpyAsync(so, h2, 16, cudaMemcpyHostToDevice, st));
@@ -1451,6 +1450,7 @@ struct wj_index {
         n_dropped = dropped0;
         if (Ns2 != RT) throw StatusError{WJ_ERR_CUDA, "received term text: token count mismatch (internal)"};
         dictionary_update(recv_terms, U2);
+        }
         phase(-1);
         WJ_CUDA_CHECK(cudaEventRecord(ev_dict, st));
       } catch (...) {
@@ -1475,7 +1475,8 @@ struct wj_index {
       cnt2[o] = p_off[o + 1] - p_off[o];
       cnt2[K + o] = c_off[o + 1] - c_off[o];
     }
-    xport->allgather(cnt2.data(), 2 * K, all2.data(), st);
+    if (!solo) xport->allgather(cnt2.data(), 2 * K, all2.data(), st);
+    else all2 = cnt2;
     std::vector<uint64_t> rp(K + 1, 0);
     uint64_t my_tokens = 0;
     for (int s = 0; s < K; ++s) {
@@ -1484,14 +1485,14 @@ struct wj_index {
       my_tokens += c[K + rank];
     }
     const uint64_t RP = rp[K];  // postings of this owner's terms over all sources
-    uint32_t* rhdf = buf<uint32_t>(x_rhdf, RT + 1);
-    uint32_t* rhcf = buf<uint32_t>(x_rhcf, RT + 1);
+    uint32_t* rhdf = solo ? hdf : buf<uint32_t>(x_rhdf, RT + 1);
+    uint32_t* rhcf = solo ? hcf : buf<uint32_t>(x_rhcf, RT + 1);
     std::vector<uint64_t> s4(K + 1), r4(K + 1);
     for (int o = 0; o <= K; ++o) {
       s4[o] = t_off[o] * 4;
       r4[o] = rt[o] * 4;
     }
-    exchange([&] {
+    if (!solo) exchange([&] {
       xport->alltoallv(hdf, s4.data(), rhdf, r4.data(), st);
       xport->alltoallv(hcf, s4.data(), rhcf, r4.data(), st);
       if (K > 1) {  // postings: owner o's range of the scratch -> o's partial-list buffer

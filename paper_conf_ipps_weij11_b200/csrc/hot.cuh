@@ -86,7 +86,7 @@ __global__ void k_hot_seed(const ulonglong2* hk, const uint32_t* H, Slot* table,
   const uint32_t w0 = (uint32_t)(k0 >> 32), w1 = (uint32_t)hk[i].y, w2 = (uint32_t)(hk[i].y >> 32) & 0xFFFFFFu;
   const uint64_t h = term_hash16(w0, w1, w2, 0u, len);
   uint32_t hot = 0;
-  hot_slot[id] = table_insert(nullptr, table, slot_ref, cap, h, k0, k1, 0u, len, nullptr, 0u, overflow, &hot);
+  hot_slot[id] = table_insert(nullptr, table, slot_ref, 0u, cap, h, k0, k1, 0u, len, nullptr, 0u, overflow, &hot);
 }
 
 // sample token counts per slot; the sample's token count is on the device (*n)

@@ -164,12 +164,11 @@ template <typename K>
 inline size_t ds_smem_bytes() { return 2 * (size_t)kOsTile * (sizeof(K) + sizeof(uint32_t)) + kOsTile * 2; }
 
 template <typename K, bool HOLES, bool MASK>
-// 48 registers (no spills): two CTAs use 48K of the 64K registers and 183 KB of shared memory, so
-// small CTAs of another stream (the dictionary update next to the partials path's side-stream sort)
-// can run beside the persistent downsweep: step 9.36 -> 9.27 ms on config 2, although the pass
-// itself is ~4% slower than at 64 registers (WJ_DS_MAXREG=0: __launch_bounds__(512, 2) only)
+// 64 registers (__launch_bounds__(512, 2)): with the lazy B-tree re-layout the dictionary stream
+// no longer needs room beside the persistent downsweep; the earlier 48-register cap
+// (WJ_DS_MAXREG=48) is 2.93 -> 3.09 ms for the three passes, step 8.98 vs 9.00-9.02 ms (A/B x2)
 #ifndef WJ_DS_MAXREG
-#define WJ_DS_MAXREG 48
+#define WJ_DS_MAXREG 0
 #endif
 #if WJ_DS_MAXREG > 0
 #define WJ_DS_BOUNDS __maxnreg__(WJ_DS_MAXREG)
@@ -243,10 +242,8 @@ __global__ void WJ_DS_BOUNDS k_rs_down2(const K* __restrict__ kin, const uint32_
       dg[k] = (uint32_t)((rs_dkey<K, MASK>(kv, kmask) >> shift) & 255u);
       // 64-bit keys (all distinct: new-term sort): shared-memory masks; 32-bit keys (Zipf-skewed
       // ranks, many equal digits per warp -> atomic conflicts): ballots
-#ifndef WJ_DS_SMEM_PEERS
-#define WJ_DS_SMEM_PEERS 0
-#endif
-      rank[k] = (sizeof(K) == 8 || WJ_DS_SMEM_PEERS) ? digit_peers_smem(wbins[w], dg[k], valid) : digit_peers(dg[k], valid);
+      // (shared-memory masks for the 32-bit stream keys too: 3.31 vs 3.09 ms for the three passes)
+      rank[k] = sizeof(K) == 8 ? digit_peers_smem(wbins[w], dg[k], valid) : digit_peers(dg[k], valid);
     }
 #pragma unroll
     for (int k = 0; k < kDsItems; ++k) {

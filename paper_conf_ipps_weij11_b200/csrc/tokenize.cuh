@@ -47,6 +47,9 @@ struct EmitOut {
   Slot* table;             // chunk hash table
   uint32_t* slot_ref;      // per slot: first-occurrence offset (written by the inserter)
   uint32_t cap;            // capacity (slots; any value >= 1)
+  uint32_t parts;          // multi-rank: the table is cut into `parts` partitions of part_cap slots,
+  uint32_t part_cap;       // partition o holding the terms whose trie collection rank o owns
+  const uint32_t* owner_tab;  // collection -> owner (balanced map), or nullptr: b mod parts
   uint32_t doc_base;       // global DocID of local document 0
   uint32_t* slot;          // per kept token: slot | 1 << 25 (key 0 = hole: a hot token, HOT only)
   uint32_t* doc;           // per kept token: global DocID
@@ -329,11 +332,13 @@ __device__ __forceinline__ uint32_t hash_tag(uint32_t h) { return (h * 0x9E3779B
 
 // Find or claim the slot of a term.  *hot = the sampled hot-term id stored in the slot's k1 (0: none;
 // only slots seeded by k_hot_seed carry one).
-__device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* table, uint32_t* slot_ref, uint32_t cap,
-                                                 uint64_t h, uint64_t k0, uint64_t k1, uint32_t s_abs, uint32_t len,
-                                                 const uint32_t* win32, uint32_t s_win, uint32_t* overflow,
+// The probe sequence stays inside the partition [base, base + cap) (base = 0, cap = capacity for an
+// unpartitioned table).
+__device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* table, uint32_t* slot_ref, uint32_t base,
+                                                 uint32_t cap, uint64_t h, uint64_t k0, uint64_t k1, uint32_t s_abs,
+                                                 uint32_t len, const uint32_t* win32, uint32_t s_win, uint32_t* overflow,
                                                  uint32_t* hot) {
-  uint32_t i = __umulhi((uint32_t)h, cap);
+  uint32_t i = base + __umulhi((uint32_t)h, cap);
   for (int probe = 0; probe < 4096; ++probe) {
     // Slots are claimed once (CAS on k0) and published once (k1), so a cached read can only be
     // stale-empty: the CAS or the volatile re-read below resolves it.
@@ -365,11 +370,37 @@ __device__ __forceinline__ uint32_t table_insert(const uint8_t* text, Slot* tabl
         if (eq) return i;
       }
     }
-    i = i + 1 == cap ? 0u : i + 1;
+    i = i + 1 == base + cap ? base : i + 1;
   }
   atomicExch(overflow, 1u);
   *hot = 0;
   return kMiss;
+}
+
+// Table I index (readings S5, S8) of a folded term from its first 16 bytes (wd, zero
+// padded) and, past 16 bytes, the staged window (only the all-digits test reads them)
+__device__ __forceinline__ uint32_t term_bucket_w(const uint32_t (&wd)[4], uint32_t len, const uint32_t* w32,
+                                                  uint32_t s_win) {
+  bool digits = true;
+#pragma unroll
+  for (uint32_t k = 0; k < 4; ++k) {
+    if (4 * k >= len) break;
+    const uint32_t rem = len - 4 * k;
+    const uint32_t valid = rem >= 4 ? 0x80808080u : (0x80808080u & ((1u << (8 * rem)) - 1u));
+    if ((digit4(wd[k]) & valid) != valid) digits = false;
+  }
+  for (uint32_t k = 4; 4 * k < len && digits; ++k) {
+    const uint32_t rem = len - 4 * k;
+    const uint32_t valid = rem >= 4 ? 0x80808080u : (0x80808080u & ((1u << (8 * rem)) - 1u));
+    if ((digit4(win_word(w32, s_win, len, k)) & valid) != valid) digits = false;
+  }
+  const uint32_t b0 = wd[0] & 0xFFu, b1 = (wd[0] >> 8) & 0xFFu, b2 = (wd[0] >> 16) & 0xFFu;
+  if (digits) return 1 + (b0 - '0');
+  if (b0 - 'a' < 26u) {
+    if (len > 3 && b1 - 'a' < 26u && b2 - 'a' < 26u) return 37 + 676 * (b0 - 'a') + 26 * (b1 - 'a') + (b2 - 'a');
+    return 11 + (b0 - 'a');
+  }
+  return 0;
 }
 
 // Launch bounds for 6 CTAs/SM (40 registers) with 320-entry token queues (31 KB of shared memory per
@@ -394,7 +425,9 @@ constexpr uint32_t kHotWords = kHotDocs * kHotMaxH;  // u32 counters per warp: [
 #define WJ_EMIT_HOT_MINB 5  // 48 registers: at 40 the hot instance spills (emit 3.84 vs 2.74 ms)
 #endif
 
-template <bool HOT>
+// PARTS: the table is partitioned by owner rank (multi-rank path); HOT / PARTS are compile-time so that
+// the one-GPU instantiation carries neither
+template <bool HOT, bool PARTS>
 __global__ void __launch_bounds__(kTokThreads, HOT ? WJ_EMIT_HOT_MINB : WJ_EMIT_MINB) k_tok_emit(ChunkView cv, uint32_t n_segs,
                                                           const uint64_t* kstart, const uint32_t* range_off, EmitOut eo) {
   __shared__ __align__(16) uint32_t win[kTokWarps][kWinBytes / 4];
@@ -471,10 +504,15 @@ __global__ void __launch_bounds__(kTokThreads, HOT ? WJ_EMIT_HOT_MINB : WJ_EMIT_
         const uint64_t k0 = (uint64_t)len | ((uint64_t)hash_tag(h32) << 8) | ((uint64_t)wd[0] << 32);
         const uint64_t k1 = (uint64_t)wd[1] | ((uint64_t)(wd[2] & 0xFFFFFFu) << 32) | (1ull << 56);
         const uint64_t out = obase + idx;
-        uint32_t hid = 0;
+        uint32_t hid = 0, tbase = 0, tcap = eo.cap;
+        if (PARTS) {  // multi-rank: the partition of the rank that owns the term's collection
+          const uint32_t b = term_bucket_w(wd, len, w32, s_win);
+          tbase = (eo.owner_tab ? __ldg(&eo.owner_tab[b]) : b % eo.parts) * eo.part_cap;
+          tcap = eo.part_cap;
+        }
         // a hot term's slot was seeded with its hot id in k1 (k_hot_seed): table_insert returns it
-        const uint32_t slot =
-            table_insert(cv.text, eo.table, eo.slot_ref, eo.cap, h, k0, k1, s_abs, len, w32, s_win, eo.overflow, &hid);
+        const uint32_t slot = table_insert(cv.text, eo.table, eo.slot_ref, tbase, tcap, h, k0, k1, s_abs, len, w32, s_win,
+                                           eo.overflow, &hid);
         if (HOT && hid) {  // hot term: counted below (the stream keeps a hole, key 0)
           const uint32_t dd = ldoc - (uint32_t)(k_range_lo - 1), hh = hid - 1;
           if (dd < kHotDocs) hkey = dd * kHotMaxH + hh;
