@@ -237,7 +237,7 @@ struct wj_index {
   cudaStream_t side_st = nullptr, hp_st = nullptr;  // side: lowest priority; hp: dictionary, highest
   cudaEvent_t ev_fork = nullptr, ev_side = nullptr, ev_dict = nullptr;
   DevBuf side_scan, side_hist, side_hist_scan;
-  DevBuf pc_key, pc_doc, pc_po, pc_cs, u_slot, pp_doc, pp_tf, rec_tid, rec_start, rec_df, rec_cf, rec_before, df_totb,
+  DevBuf pc_key, pc_doc, pc_po, pc_cs, u_slot, pp_pair, x_pair, rec_tid, rec_start, rec_df, rec_cf, rec_before, df_totb,
       cf_totb;
   uint64_t pbase = 0, nrec = 0;      // partial postings / records of the chunks so far
   uint32_t rs_ctas = kRsCtas;        // radix downsweep CTAs (ranges) of sort_pairs
@@ -358,7 +358,7 @@ struct wj_index {
                      &post_off, &df, &cf, &term_off, &term_bytes, &vb_first, &vb_tiles, &vb_code, &vb_boff, &samp_hist, &owner_tab,
                      &table_s, &uid_s, &st_off, &st_text, &st_keep, &st_tidx, &st_m1, &st_slot, &st_doc, &st_tiles,
                      &st_doff, &stop_keys, &side_scan, &side_hist, &side_hist_scan, &pc_key, &pc_doc, &pc_po,
-                     &pc_cs, &u_slot, &pp_doc, &pp_tf, &rec_tid, &rec_start, &rec_df, &rec_cf, &rec_before, &df_totb,
+                     &pc_cs, &u_slot, &pp_pair, &x_pair, &rec_tid, &rec_start, &rec_df, &rec_cf, &rec_before, &df_totb,
                      &cf_totb};
     for (DevBuf* b : all) {
       dev_free(b->p);
@@ -560,8 +560,7 @@ struct wj_index {
       launched();
     });
     scan<uint32_t>(ArrayIn<uint32_t>{cnt}, ranges, cnt, (uint32_t*)(dscal() + 0));
-    readback(0, 2);
-    readback(10, 1);
+    readback(0, 11);  // kept tokens [0], dropped [1], doc_off check [10]: one round trip
     if ((uint32_t)h_scal[10]) throw StatusError{WJ_ERR_INVALID_ARG, "doc_off must start at 0, be non-decreasing and end at n_bytes"};
     return (uint32_t)h_scal[0];
   }
@@ -1008,8 +1007,14 @@ struct wj_index {
   // run-length pass over a sorted stream (postings.cuh): docid/tf into od/of, post_off / cstart at each
   // term's key (key & kRankMask); the posting count is left in dscal[8] (u32, no host round trip)
   // n_dev (optional): the actual element count on the device, N being an upper bound
+  // pairs != nullptr: the postings go there as interleaved (docID, tf) pairs (per-run partial lists)
   void rle(const uint32_t* key, const uint32_t* docs, uint64_t N, bool counts, uint32_t* od, uint32_t* of, uint64_t* po,
-           uint64_t* csp, const uint32_t* n_dev = nullptr) {
+           uint64_t* csp, const uint32_t* n_dev = nullptr, uint2* pairs = nullptr) {
+    const uint32_t ostride = pairs ? 2u : 1u;
+    if (pairs) {
+      od = (uint32_t*)pairs;
+      of = (uint32_t*)pairs + 1;
+    }
     if (N == 0) {  // e.g. every token of the chunk was a hot term
       WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 8, 0, 8, st));
       return;
@@ -1027,14 +1032,14 @@ struct wj_index {
       scan<uint32_t>(ArrayIn<uint32_t>{rc}, G, rc, (uint32_t*)(dscal() + 8));
       scan<uint64_t>(ArrayIn<uint64_t>{rt}, G, rt, (uint64_t*)(dscal() + 11));
       if (counts)
-        k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(key, docs, N, per, rc, rt, od, of, po, csp, rl,
-                                                                        n_dev);
+        k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(key, docs, N, per, rc, rt, od, of, ostride, po,
+                                                                        csp, rl, n_dev);
       else
-        k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(false), st>>>(key, docs, N, per, rc, rt, od, of, po, csp,
-                                                                          rl, n_dev);
+        k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(false), st>>>(key, docs, N, per, rc, rt, od, of, ostride,
+                                                                          po, csp, rl, n_dev);
       launched();
     });
-    k_rle_fixup<<<grid_for(G, 256), 256, 0, st>>>(rc, rl, G, of);
+    k_rle_fixup<<<grid_for(G, 256), 256, 0, st>>>(rc, rl, G, of, ostride);
     launched();
     WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 8) + 1, 0, 4, st));
   }
@@ -1062,8 +1067,7 @@ struct wj_index {
     uint32_t* dt = (uint32_t*)pc_doc.p;
     uint32_t* k1 = buf<uint32_t>(sk1, Nc + 16);
     uint32_t* v1 = buf<uint32_t>(sv1, Nc + 16);
-    uint32_t* od = buf_keep<uint32_t>(pp_doc, pbase + Nc + 16, pbase);  // P_c <= N_c
-    uint32_t* of = buf_keep<uint32_t>(pp_tf, pbase + Nc + 16, pbase);
+    uint2* pp = buf_keep<uint2>(pp_pair, pbase + Nc + 16, pbase);  // P_c <= N_c
     uint64_t* po = buf<uint64_t>(pc_po, C + 1);
     uint64_t* cs = buf<uint64_t>(pc_cs, C + 1);
     int bits = 0;
@@ -1080,7 +1084,7 @@ struct wj_index {
       const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, bits, nullptr, true, nullptr, kRankMask, hot, nullptr,
                                             true, nullptr, ns_dev);
       phase(WJ_PHASE_POSTINGS);
-      rle(in1 ? k1 : kt, in1 ? v1 : dt, Nc, false, od + pbase, of + pbase, po, cs, ns_dev);
+      rle(in1 ? k1 : kt, in1 ? v1 : dt, Nc, false, nullptr, nullptr, po, cs, ns_dev, pp + pbase);
       if (hot) {  // the hot matrix rows -> the hot terms' partial lists, after the run-length postings
         const uint64_t HD = (uint64_t)hot_H * hot_D;
         uint32_t* hp = buf<uint32_t>(hot_posb, HD + 1);
@@ -1088,7 +1092,7 @@ struct wj_index {
         const uint32_t* mat = (const uint32_t*)hot_matb.p;
         scan<uint32_t>(NonZeroU32{mat}, HD, hp, hp + HD);
         k_hot_scatter<<<grid_for(HD, 256), 256, 0, st>>>(mat, HD, hot_D, hp, (const uint32_t*)(dscal() + 8),
-                                                         doc_base_cur, od + pbase, of + pbase);
+                                                         doc_base_cur, pp + pbase);
         k_hot_rowsum<<<hot_H, 256, 0, st>>>(mat, hot_D, hcf);
         k_hot_total<<<1, 1, 0, st>>>(hp + HD, (uint32_t*)(dscal() + 8), (uint32_t*)(dscal() + 12));
         launched(3);
@@ -1328,14 +1332,7 @@ struct wj_index {
     // the chunk's postings: K == 1 straight into the partial-list buffer; K > 1 into scratch, from where
     // every owner's range (the own one by a device copy) lands in the owners' partial-list buffers in
     // source-rank order, so each chunk's partial lists are back to back in record order
-    uint32_t *od = nullptr, *of = nullptr;
-    if (K == 1) {
-      od = buf_keep<uint32_t>(pp_doc, pbase + Nc + 16, pbase) + pbase;
-      of = buf_keep<uint32_t>(pp_tf, pbase + Nc + 16, pbase) + pbase;
-    } else {
-      od = buf<uint32_t>(x_rkey, Nc + 16);
-      of = buf<uint32_t>(x_rdoc, Nc + 16);
-    }
+    uint2* opp = K == 1 ? buf_keep<uint2>(pp_pair, pbase + Nc + 16, pbase) + pbase : buf<uint2>(x_pair, Nc + 16);
     uint32_t* hdf = buf<uint32_t>(x_hdf, U + 1);
     uint32_t* hcf = buf<uint32_t>(x_hcf, U + 1);
     uint64_t* bnd = buf<uint64_t>(x_bnd, 2 * (K + 1));
@@ -1410,7 +1407,7 @@ struct wj_index {
         phase(WJ_PHASE_SORT);
         const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, std::max(bits, 1), nullptr, true);
         phase(WJ_PHASE_POSTINGS);
-        rle(in1 ? k1 : kt, in1 ? v1 : dt, Nc, false, od, of, po, cs);
+        rle(in1 ? k1 : kt, in1 ? v1 : dt, Nc, false, nullptr, nullptr, po, cs, nullptr, opp);
         k_term_hdr<<<grid_for(U, 256), 256, 0, st>>>(us, (uint32_t)U, po, cs, (const uint32_t*)(dscal() + 8), Nc, hdf, hcf);
         k_owner_bounds<<<grid_for(K + 1, 256), 256, 0, st>>>(us, po, cs, toff_d, (uint32_t)K, (uint32_t)U,
                                                             (const uint32_t*)(dscal() + 8), Nc, bnd, bnd + K + 1);
@@ -1496,15 +1493,13 @@ struct wj_index {
       xport->alltoallv(hdf, s4.data(), rhdf, r4.data(), st);
       xport->alltoallv(hcf, s4.data(), rhcf, r4.data(), st);
       if (K > 1) {  // postings: owner o's range of the scratch -> o's partial-list buffer
-        uint32_t* pd = buf_keep<uint32_t>(pp_doc, pbase + RP + 16, pbase) + pbase;
-        uint32_t* pt = buf_keep<uint32_t>(pp_tf, pbase + RP + 16, pbase) + pbase;
+        uint2* pd = buf_keep<uint2>(pp_pair, pbase + RP + 16, pbase) + pbase;
         std::vector<uint64_t> spb(K + 1), rpb(K + 1);
         for (int o = 0; o <= K; ++o) {
-          spb[o] = p_off[o] * 4;
-          rpb[o] = rp[o] * 4;
+          spb[o] = p_off[o] * 8;
+          rpb[o] = rp[o] * 8;
         }
-        xport->alltoallv(od, spb.data(), pd, rpb.data(), st);
-        xport->alltoallv(of, spb.data(), pt, rpb.data(), st);
+        xport->alltoallv(opp, spb.data(), pd, rpb.data(), st);
       }
     });
     exchange_ms += xms;
@@ -2058,14 +2053,13 @@ struct wj_index {
         ktime(WJ_KERNEL_COPY_PARTIALS, [&] {
           if (rec_end.size() == 1) {  // one run: cft holds the list start of each rank
             k_copy_by_rank<<<grid_for((P + kCopyChunk - 1) / kCopyChunk * 32, 256), 256, 0, st>>>(
-                cft, V, P, po, (const uint32_t*)pp_doc.p, (const uint32_t*)pp_tf.p, od, of);
+                cft, V, P, po, (const uint2*)pp_pair.p, od, of);
             launched();
             return;
           }
           k_copy_partials<<<grid_for((P + kCopyChunk - 1) / kCopyChunk * 32, 256), 256, 0, st>>>(
               rt, (const uint64_t*)rec_start.p, rd, bef, nrec, P, ro, po,
-                                                                   (const uint32_t*)pp_doc.p, (const uint32_t*)pp_tf.p,
-                                                                   od, of);
+                                                                   (const uint2*)pp_pair.p, od, of);
           launched();
         });
       } else {
@@ -2117,14 +2111,14 @@ struct wj_index {
         scan<uint32_t>(ArrayIn<uint32_t>{rc}, G, rc, (uint32_t*)(dscal() + 8));
         scan<uint64_t>(ArrayIn<uint64_t>{rt}, G, rt, (uint64_t*)(dscal() + 11));
         if (stream_has_hot)
-          k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po, csp, rl,
-                                                                          nullptr);
+          k_rle_write_tma<true><<<G, kRleThreads, rle_smem_bytes(), st>>>(f_key, f_doc, N, per, rc, rt, od, of, 1u, po,
+                                                                          csp, rl, nullptr);
         else
-          k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(false), st>>>(f_key, f_doc, N, per, rc, rt, od, of, po,
-                                                                            csp, rl, nullptr);
+          k_rle_write_tma<false><<<G, kRleThreads, rle_smem_bytes(false), st>>>(f_key, f_doc, N, per, rc, rt, od, of, 1u,
+                                                                            po, csp, rl, nullptr);
         launched();
       });
-      k_rle_fixup<<<grid_for(G, 256), 256, 0, st>>>(rc, rl, G, of);
+      k_rle_fixup<<<grid_for(G, 256), 256, 0, st>>>(rc, rl, G, of, 1u);
       launched();
       WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 8) + 1, 0, 4, st));
       readback(8, 1);

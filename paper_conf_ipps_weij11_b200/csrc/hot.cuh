@@ -70,10 +70,6 @@ __global__ void k_sample_cand(const Slot* table, const uint32_t* cnt, uint32_t C
   cval[i] = i;
 }
 
-__global__ void k_hot_extract(const Slot* table, const uint32_t* slots, uint32_t H, ulonglong2* hk) {
-  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i < H) hk[i] = *(const ulonglong2*)(table + slots[i]);
-}
 
 // thread i seeds hot id i + 1: claims the term's slot in the chunk table with the id in k1 bits 57..
 __global__ void k_hot_seed(const ulonglong2* hk, const uint32_t* H, Slot* table, uint32_t* slot_ref, uint32_t cap,
@@ -115,14 +111,13 @@ struct NonZeroU32 {
 // nonzero matrix entries -> the hot terms' partial lists, appended after the chunk's run-length
 // postings (*P_rle of them); pos = exclusive scan of the nonzero flags (row-major: term, document)
 __global__ void k_hot_scatter(const uint32_t* mat, uint64_t n, uint32_t D, const uint32_t* pos, const uint32_t* P_rle,
-                              uint32_t doc_base, uint32_t* od, uint32_t* of) {
+                              uint32_t doc_base, uint2* pp) {
   const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   const uint32_t c = mat[i];
   if (c == 0) return;
   const uint64_t p = (uint64_t)*P_rle + pos[i];
-  od[p] = doc_base + (uint32_t)(i % D);
-  of[p] = c;
+  pp[p] = make_uint2(doc_base + (uint32_t)(i % D), c);
 }
 
 // tokens of each hot term (its cf): one block per matrix row

@@ -107,7 +107,7 @@ __global__ void k_rank_scatter_rec(const uint32_t* __restrict__ rec_tid, const u
 // term's list is contiguous in both).
 __global__ void __launch_bounds__(256) k_copy_by_rank(const uint64_t* __restrict__ src_of_rank, uint32_t V, uint64_t P,
                                                       const uint64_t* __restrict__ post_off,
-                                                      const uint32_t* __restrict__ pdoc, const uint32_t* __restrict__ ptf,
+                                                      const uint2* __restrict__ pp,
                                                       uint32_t* __restrict__ out_doc, uint32_t* __restrict__ out_tf);
 
 struct U32AsU64 {
@@ -129,7 +129,7 @@ __global__ void __launch_bounds__(256) k_copy_partials(const uint32_t* __restric
                                                        const uint32_t* __restrict__ before, uint64_t R, uint64_t P,
                                                        const uint32_t* __restrict__ rank_of,
                                                        const uint64_t* __restrict__ post_off,
-                                                       const uint32_t* __restrict__ pdoc, const uint32_t* __restrict__ ptf,
+                                                       const uint2* __restrict__ pp,
                                                        uint32_t* __restrict__ out_doc, uint32_t* __restrict__ out_tf) {
   const uint64_t w = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint32_t lane = threadIdx.x & 31;
@@ -175,8 +175,9 @@ __global__ void __launch_bounds__(256) k_copy_partials(const uint32_t* __restric
         const uint32_t sj = __shfl_sync(0xffffffffu, srel, j);
         dd[q] = __shfl_sync(0xffffffffu, dst, j) + (pr - sj);
         if (p < e) {
-          dv[q] = __ldcs(pdoc + p);
-          tv[q] = __ldcs(ptf + p);
+          const uint2 x = __ldcs(pp + p);  // interleaved (docID, tf): one sector for a short list
+          dv[q] = x.x;
+          tv[q] = x.y;
         }
       }
 #pragma unroll
@@ -195,7 +196,7 @@ __global__ void __launch_bounds__(256) k_copy_partials(const uint32_t* __restric
 
 __global__ void __launch_bounds__(256) k_copy_by_rank(const uint64_t* __restrict__ src_of_rank, uint32_t V, uint64_t P,
                                                       const uint64_t* __restrict__ post_off,
-                                                      const uint32_t* __restrict__ pdoc, const uint32_t* __restrict__ ptf,
+                                                      const uint2* __restrict__ pp,
                                                       uint32_t* __restrict__ out_doc, uint32_t* __restrict__ out_tf) {
   const uint64_t w = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint32_t lane = threadIdx.x & 31;
@@ -236,8 +237,9 @@ __global__ void __launch_bounds__(256) k_copy_by_rank(const uint64_t* __restrict
         const uint32_t dj = __shfl_sync(0xffffffffu, drel, j);
         const uint64_t sp = __shfl_sync(0xffffffffu, src, j) + (pr - dj);
         if (p < e) {
-          dv[q] = __ldg(pdoc + sp);
-          tv[q] = __ldg(ptf + sp);
+          const uint2 x = __ldg(pp + sp);
+          dv[q] = x.x;
+          tv[q] = x.y;
         }
       }
 #pragma unroll

@@ -78,7 +78,8 @@ __device__ __forceinline__ uint32_t block_min_after(uint32_t v, uint32_t* sm /* 
 // docID.  CTA c owns the contiguous element range [c*per, min(N,(c+1)*per)).  k_rle_count counts
 // posting starts and tokens per range; scans give each range's first posting index and token offset;
 // k_rle_write_tma walks its range tile by tile (TMA-prefetched 2-stage ring), carries the open run
-// across tiles and writes docid, tf = sum of counts (coalesced through shared memory), post_off[rank]
+// across tiles and writes docid, tf = sum of counts (coalesced through shared memory; ostride 2 =
+// interleaved (docID, tf) pairs, the per-run partial lists), post_off[rank]
 // and the token offset cstart[rank] of the term's first element (cf = difference).  Runs that continue
 // across ranges are completed by k_rle_fixup (range_lead = tokens before the range's first posting).
 // elements per CTA range of the run-length pass (a multiple of its tile); engine.cu rle() cuts the same
@@ -183,7 +184,8 @@ __global__ void WJ_RLE_BOUNDS k_rle_write_tma(const uint32_t* __restrict__ key,
                                                                const uint32_t* __restrict__ doc, uint64_t N,
                                                                uint64_t per, const uint32_t* __restrict__ range_off,
                                                                const uint64_t* __restrict__ range_tok_off,
-                                                               uint32_t* out_doc, uint32_t* out_tf, uint64_t* post_off,
+                                                               uint32_t* out_doc, uint32_t* out_tf, uint32_t ostride,
+                                                               uint64_t* post_off,
                                                                uint64_t* cstart, uint32_t* range_lead,
                                                                const uint32_t* __restrict__ n_dev) {
   if (n_dev) {
@@ -281,7 +283,7 @@ __global__ void WJ_RLE_BOUNDS k_rle_write_tma(const uint32_t* __restrict__ key,
       }
       if (have_open) {
         s_open_len += lead;
-        if (first_all != 0xFFFFFFFFu) out_tf[open_p] = s_open_len;
+        if (first_all != 0xFFFFFFFFu) out_tf[(uint64_t)ostride * open_p] = s_open_len;
       }
     }
     uint32_t lp = ex;
@@ -303,8 +305,12 @@ __global__ void WJ_RLE_BOUNDS k_rle_write_tma(const uint32_t* __restrict__ key,
     }
     __syncthreads();
     for (uint32_t x = threadIdx.x; x < tot; x += kRleThreads) {
-      __stcs(out_doc + p0 + x, st_doc[x]);
-      __stcs(out_tf + p0 + x, st_tf[x]);
+      if (ostride == 2) {  // interleaved (docID, tf) pairs (per-run partial lists)
+        __stcs((uint2*)out_doc + p0 + x, make_uint2(st_doc[x], st_tf[x]));
+      } else {
+        __stcs(out_doc + p0 + x, st_doc[x]);
+        __stcs(out_tf + p0 + x, st_tf[x]);
+      }
     }
     if (threadIdx.x == 0) {
       if (tot) s_open_len = st_tf[tot - 1];
@@ -321,17 +327,18 @@ __global__ void WJ_RLE_BOUNDS k_rle_write_tma(const uint32_t* __restrict__ key,
     s ^= 1;
   }
   if (threadIdx.x == 0) {
-    if (have_open) out_tf[open_p] = s_open_len;
+    if (have_open) out_tf[(uint64_t)ostride * open_p] = s_open_len;
     range_lead[blockIdx.x] = s_lead;
   }
 }
 
 // runs that continue across tiles: add each tile's leading items to the preceding posting
-__global__ void k_rle_fixup(const uint32_t* tile_p0, const uint32_t* tile_lead, uint32_t tiles, uint32_t* out_tf) {
+__global__ void k_rle_fixup(const uint32_t* tile_p0, const uint32_t* tile_lead, uint32_t tiles, uint32_t* out_tf,
+                            uint32_t ostride) {
   const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
   if (t == 0 || t >= tiles) return;
   const uint32_t lead = tile_lead[t];
-  if (lead) atomicAdd(&out_tf[tile_p0[t] - 1], lead);
+  if (lead) atomicAdd(&out_tf[(uint64_t)ostride * (tile_p0[t] - 1)], lead);
 }
 
 __global__ void k_df_cf(uint64_t* post_off, const uint64_t* cstart, uint32_t V, uint64_t P, uint64_t NT, uint32_t* df,

@@ -104,3 +104,48 @@ def test_balance_owners_lpt_properties():
     # hand example: counts 5,4,3,3,3 over 2 ranks -> 5->r0, 4->r1, 3->r1 (4<5), 3->r0 (8>7? r0=5<7), 3->r1
     own = wj.balance_owners(np.array([5, 4, 3, 3, 3], dtype=np.uint64), 2)
     assert own.tolist() == [0, 1, 1, 0, 1]
+
+
+def _gloo_owner_map_worker(rank, world, port, q):
+    """The balanced owner map protocol of the multi-rank path (engine.cu build_owner_map):
+    each rank counts the tokens per trie collection of its own document range (the oracle's token dump
+    stands in for the device sample), the counts are all-gathered (gloo here, NCCL in the library), and
+    every rank bin-packs the summed counts with the library's host LPT (index_balance_owners)."""
+    import torch.distributed as dist
+
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    text, off = gen.generate(gen.CONFIGS[1].scaled(vocab=3000))
+    n = len(off) - 1
+    lo, hi = n * rank // world, n * (rank + 1) // world
+    t = text[int(off[lo]):int(off[hi])]
+    o = (np.asarray(off[lo:hi + 1], dtype=np.uint64) - off[lo]).astype(np.uint64)
+    counts = np.zeros(wj.N_COLLECTIONS, dtype=np.uint64)
+    for _, b, _ in oracle.dump_tokens(t, o):
+        counts[b] += 1
+    allc = [None] * world
+    dist.all_gather_object(allc, counts)
+    own = wj.balance_owners(np.sum(allc, axis=0).astype(np.uint64), world)
+    maps = [None] * world
+    dist.all_gather_object(maps, own)
+    full = oracle.index_bytes(text, off)
+    mine = wjformat.split_by_owner(full, world, lambda term: int(own[oracle.bucket(term)]))[rank]
+    got = [None] * world
+    dist.all_gather_object(got, mine)
+    if rank == 0:
+        q.put(all(np.array_equal(maps[0], m) for m in maps) and wj.merge_serialized(got) == full
+              and not np.array_equal(own, np.arange(wj.N_COLLECTIONS) % world))
+    dist.destroy_process_group()
+
+
+def test_gloo_world2_balanced_owner_map_protocol():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_gloo_owner_map_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    ok = q.get(timeout=180)
+    for p in ps:
+        p.join(timeout=60)
+    assert ok
