@@ -237,6 +237,7 @@ struct wj_index {
   cudaStream_t side_st = nullptr, hp_st = nullptr;  // side: lowest priority; hp: dictionary, highest
   cudaEvent_t ev_fork = nullptr, ev_side = nullptr, ev_dict = nullptr;
   DevBuf side_scan, side_hist, side_hist_scan;
+  DevBuf mr_key, mr_idx, mr_key2, mr_idx2, mr_dst, mr_src;  // several runs: records in destination order
   DevBuf pc_key, pc_doc, pc_po, pc_cs, u_slot, pp_pair, x_pair, rec_tid, rec_start, rec_df, rec_cf, rec_before, df_totb,
       cf_totb;
   uint64_t pbase = 0, nrec = 0;      // partial postings / records of the chunks so far
@@ -358,7 +359,7 @@ struct wj_index {
                      &post_off, &df, &cf, &term_off, &term_bytes, &vb_first, &vb_tiles, &vb_code, &vb_boff, &samp_hist, &owner_tab,
                      &table_s, &uid_s, &st_off, &st_text, &st_keep, &st_tidx, &st_m1, &st_slot, &st_doc, &st_tiles,
                      &st_doff, &stop_keys, &side_scan, &side_hist, &side_hist_scan, &pc_key, &pc_doc, &pc_po,
-                     &pc_cs, &u_slot, &pp_pair, &x_pair, &rec_tid, &rec_start, &rec_df, &rec_cf, &rec_before, &df_totb,
+                     &pc_cs, &u_slot, &pp_pair, &x_pair, &mr_key, &mr_idx, &mr_key2, &mr_idx2, &mr_dst, &mr_src, &rec_tid, &rec_start, &rec_df, &rec_cf, &rec_before, &df_totb,
                      &cf_totb};
     for (DevBuf* b : all) {
       dev_free(b->p);
@@ -2057,10 +2058,25 @@ struct wj_index {
             launched();
             return;
           }
-          k_copy_partials<<<grid_for((P + kCopyChunk - 1) / kCopyChunk * 32, 256), 256, 0, st>>>(
-              rt, (const uint64_t*)rec_start.p, rd, bef, nrec, P, ro, po,
-                                                                   (const uint2*)pp_pair.p, od, of);
+          // several runs: the records sorted into destination order (rank, then run: a stable sort by
+          // rank), then the same rank-order copy (coalesced writes, each partial list one gathered read)
+          uint32_t* rk = buf<uint32_t>(mr_key, nrec + 16);
+          uint32_t* ri = buf<uint32_t>(mr_idx, nrec + 16);
+          uint32_t* rk2 = buf<uint32_t>(mr_key2, nrec + 16);
+          uint32_t* ri2 = buf<uint32_t>(mr_idx2, nrec + 16);
+          k_rec_rank_key<<<grid_for(nrec, 256), 256, 0, st>>>(rt, nrec, ro, rk, ri);
           launched();
+          int rbits = 0;
+          while (rbits < 32 && ((uint64_t)1 << rbits) < V) ++rbits;
+          const uint32_t* sorted = sort_pairs<uint32_t>(rk, ri, rk2, ri2, nrec, 0, std::max(rbits, 1), nullptr, false)
+                                       ? ri2 : ri;
+          uint64_t* dst = buf<uint64_t>(mr_dst, nrec + 1);
+          uint64_t* src = buf<uint64_t>(mr_src, nrec + 1);
+          k_rec_dest<<<grid_for(nrec, 256), 256, 0, st>>>(sorted, nrec, rt, bef, (const uint64_t*)rec_start.p, ro, po,
+                                                          dst, src);
+          k_copy_by_rank<<<grid_for((P + kCopyChunk - 1) / kCopyChunk * 32, 256), 256, 0, st>>>(
+              src, nrec, P, dst, (const uint2*)pp_pair.p, od, of);
+          launched(2);
         });
       } else {
         WJ_CUDA_CHECK(cudaMemsetAsync(po, 0, 8, st));

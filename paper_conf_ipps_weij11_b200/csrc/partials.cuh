@@ -110,89 +110,35 @@ __global__ void __launch_bounds__(256) k_copy_by_rank(const uint64_t* __restrict
                                                       const uint2* __restrict__ pp,
                                                       uint32_t* __restrict__ out_doc, uint32_t* __restrict__ out_tf);
 
+// several runs: each record's (rank of its term) as the key of a stable sort that puts the records in
+// destination order (rank, then run), and its index as the value
+__global__ void k_rec_rank_key(const uint32_t* __restrict__ rec_tid, uint64_t R, const uint32_t* __restrict__ rank_of,
+                               uint32_t* key, uint32_t* idx) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= R) return;
+  key[i] = rank_of[rec_tid[i]];
+  idx[i] = (uint32_t)i;
+}
+
+// records in destination order -> (destination start, source start) of each partial list; the
+// destination starts increase strictly (df >= 1), so k_copy_by_rank copies them like one run's lists
+__global__ void k_rec_dest(const uint32_t* __restrict__ sorted, uint64_t R, const uint32_t* __restrict__ rec_tid,
+                           const uint32_t* __restrict__ before, const uint64_t* __restrict__ rec_start,
+                           const uint32_t* __restrict__ rank_of, const uint64_t* __restrict__ post_off,
+                           uint64_t* dst_start, uint64_t* src_start) {
+  const uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= R) return;
+  const uint32_t i = sorted[j];
+  dst_start[j] = post_off[rank_of[rec_tid[i]]] + before[i];
+  src_start[j] = rec_start[i];
+}
+
 struct U32AsU64 {
   const uint32_t* p;
   __device__ __forceinline__ uint64_t operator()(uint64_t i) const { return p[i]; }
 };
 
-// Copy every partial list to post_off[rank(term)] + before.  The partial lists lie back to back in
-// record order, so warp w copies the source postings [w * kCopyChunk, (w + 1) * kCopyChunk): it finds
-// the record holding its first posting (binary search on rec_start), then walks windows of 32
-// records, 32 postings at a time (coalesced reads; each lane finds its record in the window with a
-// 5-step shuffle search); writes are contiguous within each record's list.  Long lists (the Zipf
-// head) are spread over many warps.
-constexpr uint32_t kCopyChunk = 1024;
-
-__global__ void __launch_bounds__(256) k_copy_partials(const uint32_t* __restrict__ rec_tid,
-                                                       const uint64_t* __restrict__ rec_start,
-                                                       const uint32_t* __restrict__ rec_df,
-                                                       const uint32_t* __restrict__ before, uint64_t R, uint64_t P,
-                                                       const uint32_t* __restrict__ rank_of,
-                                                       const uint64_t* __restrict__ post_off,
-                                                       const uint2* __restrict__ pp,
-                                                       uint32_t* __restrict__ out_doc, uint32_t* __restrict__ out_tf) {
-  const uint64_t w = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const uint32_t lane = threadIdx.x & 31;
-  uint64_t lo = w * kCopyChunk;
-  if (lo >= P) return;
-  const uint64_t hi = lo + kCopyChunk < P ? lo + kCopyChunk : P;
-  // first record: the last one with rec_start <= lo (rec_start is increasing; record 0 starts at 0)
-  uint64_t r = 0;
-  if (lane == 0) {
-    uint64_t a = 0, b = R;  // invariant: rec_start[a] <= lo, answer in [a, b)
-    while (b - a > 1) {
-      const uint64_t m = (a + b) >> 1;
-      if (rec_start[m] <= lo) a = m; else b = m;
-    }
-    r = a;
-  }
-  r = __shfl_sync(0xffffffffu, r, 0);
-  for (;;) {
-    const uint64_t i = r + lane;
-    const bool v = i < R;
-    const uint64_t st = v ? rec_start[i] : ~0ull;
-    const uint32_t n = v ? rec_df[i] : 0u;
-    const uint64_t dst = v ? post_off[rank_of[rec_tid[i]]] + before[i] : 0ull;
-    const uint64_t wend = __shfl_sync(0xffffffffu, v ? st + n : 0ull, 31);  // end of the window
-    const uint64_t last = (r + 31 < R) ? wend : P;
-    const uint64_t e = last < hi ? last : hi;
-    // window-relative starts (u32) for cheaper shuffles; 4 x 32 postings per step, loads before stores
-    const uint64_t ws = __shfl_sync(0xffffffffu, st, 0);
-    const uint32_t srel = v ? (uint32_t)(st - ws) : 0xFFFFFFFFu;
-    for (uint64_t base = lo; base < e; base += 128) {  // warp-uniform trip count
-      uint32_t dv[4], tv[4];
-      uint64_t dd[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const uint64_t p = base + 32 * q + lane;
-        const uint32_t pr = (uint32_t)(p - ws);
-        uint32_t j = 0;  // last lane of the window with start <= p
-#pragma unroll
-        for (int b = 16; b > 0; b >>= 1) {
-          const uint32_t sj = __shfl_sync(0xffffffffu, srel, j + b);
-          if (sj <= pr) j += b;
-        }
-        const uint32_t sj = __shfl_sync(0xffffffffu, srel, j);
-        dd[q] = __shfl_sync(0xffffffffu, dst, j) + (pr - sj);
-        if (p < e) {
-          const uint2 x = __ldcs(pp + p);  // interleaved (docID, tf): one sector for a short list
-          dv[q] = x.x;
-          tv[q] = x.y;
-        }
-      }
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        if (base + 32 * q + lane < e) {
-          __stcs(out_doc + dd[q], dv[q]);
-          __stcs(out_tf + dd[q], tv[q]);
-        }
-      }
-    }
-    if (e >= hi) break;
-    lo = e;
-    r += 32;
-  }
-}
+constexpr uint32_t kCopyChunk = 1024;  // postings per warp of the copy
 
 __global__ void __launch_bounds__(256) k_copy_by_rank(const uint64_t* __restrict__ src_of_rank, uint32_t V, uint64_t P,
                                                       const uint64_t* __restrict__ post_off,
