@@ -273,7 +273,7 @@ struct wj_index {
   // chunk scratch
   DevBuf text_stage, doc_stage, seg_cnt, table, uid, u_w, u_ref, u_len, u_bucket, u_cache, u_key, u_tid, u_rank, midx, nk_key,
       nk_val, nk_key2, nk_val2, aoff, ns_tid, ns_bucket, ns_rank, nlo, nhi, nbase, lvA[4], lvB[4], child_off, root_idx,
-      scan_scr, hist, hist_scan, os_hist, os_look, os_ctr, kstart, slotref, dbg_start, dbg_len, dbg_off, dbg_out, dbg_slot, dbg_doc, lexg, qbuf, qres;
+      scan_scr, hist, hist_scan, kstart, slotref, dbg_start, dbg_len, dbg_off, dbg_out, dbg_slot, dbg_doc, lexg, qbuf, qres;
   // finalize
   DevBuf rank_of, term_at, sk1, sv1, pidx, out_doc, out_tf, post_off, df, cf, term_off, term_bytes;
   DevBuf vb_first, vb_tiles, vb_code, vb_boff;  // f1 (WJ_FLAG_VBYTE)
@@ -354,7 +354,7 @@ struct wj_index {
                      &t_arena, &t_cache, &t_bucket, &scal, &g_tid, &g_doc, &text_stage, &doc_stage, &seg_cnt, &table,
                      &uid, &u_w, &u_ref, &u_len, &u_bucket, &u_cache, &u_key, &u_tid, &u_rank, &midx, &nk_key, &nk_val,
                      &nk_key2, &nk_val2, &aoff, &ns_tid, &ns_bucket, &ns_rank, &nlo, &nhi, &nbase, &child_off,
-                     &root_idx, &scan_scr, &hist, &hist_scan, &os_hist, &os_look, &os_ctr, &kstart, &slotref, &dbg_start, &dbg_len, &dbg_off, &dbg_out, &dbg_slot,
+                     &root_idx, &scan_scr, &hist, &hist_scan, &kstart, &slotref, &dbg_start, &dbg_len, &dbg_off, &dbg_out, &dbg_slot,
                      &dbg_doc, &lexg, &qbuf, &qres, &rank_of, &term_at, &sk1, &sv1, &pidx, &out_doc, &out_tf,
                      &post_off, &df, &cf, &term_off, &term_bytes, &vb_first, &vb_tiles, &vb_code, &vb_boff, &samp_hist, &owner_tab,
                      &table_s, &uid_s, &st_off, &st_text, &st_keep, &st_tidx, &st_m1, &st_slot, &st_doc, &st_tiles,
