@@ -383,24 +383,18 @@ __global__ void k_tie_fix(const uint64_t* key, uint32_t* val, uint32_t N, const 
   }
 }
 
-// New terms, in unique order (coalesced column reads): termIDs by warp-aggregated atomics (the
-// paper's GPU indexer assigns postings pointers as it inserts), arena append <len><suffix>
-// (Fig. 6) at the scanned offset, per-term columns.  The sorted-order lists for the merge are filled
-// afterwards by k_ns_fill.
+// New terms, in unique order (coalesced column reads): the next termIDs in unique order (V0 + the
+// term's index among the chunk's misses; the paper's GPU indexer assigns postings pointers as it
+// inserts), arena append <len><suffix> (Fig. 6) at the scanned offset, per-term columns
+// (coalesced: consecutive misses get consecutive termIDs).  The sorted-order lists for the merge are
+// filled afterwards by k_ns_fill.
 __global__ void k_new_terms(uint32_t U, const uint32_t* aoff, uint64_t arena_base, const uint8_t* text,
                             const uint4* u_w, const uint32_t* u_ref, const uint32_t* u_len, const uint32_t* u_bucket,
-                            const uint32_t* u_cache, uint32_t* u_tid, uint32_t* tid_counter, uint8_t* arena,
-                            uint32_t* t_arena, uint32_t* t_cache, uint32_t* t_bucket) {
+                            const uint32_t* u_cache, uint32_t* u_tid, const uint32_t* miss_idx, uint32_t V0,
+                            uint8_t* arena, uint32_t* t_arena, uint32_t* t_cache, uint32_t* t_bucket) {
   const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
-  const bool active = u < U && u_tid[u] == kMiss;
-  const uint32_t lane = lane_id();
-  const uint32_t am = __ballot_sync(0xffffffffu, active);
-  if (!am) return;
-  uint32_t base = 0;
-  if (lane == 0) base = atomicAdd(tid_counter, (uint32_t)__popc(am));
-  base = __shfl_sync(0xffffffffu, base, 0);
-  if (!active) return;
-  const uint32_t tid = base + __popc(am & ((1u << lane) - 1u));
+  if (u >= U || u_tid[u] != kMiss) return;
+  const uint32_t tid = V0 + miss_idx[u];
   const uint32_t b = u_bucket[u], plen = bucket_plen(b), ref = u_ref[u], slen = u_len[u] - plen;
   const uint64_t off = arena_base + aoff[u];
   arena[off] = (uint8_t)slen;
@@ -566,22 +560,34 @@ struct LexGroups {
   uint32_t gbase[37];
 };
 
+// 11 warps (kLexGroupThreads): warp k finds the first bucket-0 index whose first byte is >= '0'+k
+// (k = 10: >= 0x80) by a 32-way search (each round probes 32 evenly spaced entries: ~5 dependent rounds
+// instead of ~22 for a binary search on one lane); thread 0 then accumulates the group bases.
+constexpr int kLexGroupThreads = 11 * 32;
 __global__ void k_lex_groups(const uint32_t* e_tid, const uint32_t* coll_base, const uint32_t* coll_n,
                              const uint32_t* t_cache, LexGroups* g) {
-  // lanes 0..10: first bucket-0 index whose first byte is >= '0'+k (k = 10: >= 0x80), in parallel
-  const uint32_t k = threadIdx.x;
+  const uint32_t k = threadIdx.x >> 5, lane = lane_id();
   const uint32_t b0 = coll_base[0], n0 = coll_n[0];
   if (k <= 10) {
     const uint32_t target = k < 10 ? '0' + k : 0x80;
-    uint32_t lo = 0, hi = n0;
+    uint32_t lo = 0, hi = n0;  // the answer is in [lo, hi]
     while (lo < hi) {
-      const uint32_t mid = (lo + hi) >> 1;
-      if ((t_cache[e_tid[b0 + mid]] >> 24) < target) lo = mid + 1; else hi = mid;
+      const uint32_t pos = lo + (uint32_t)((uint64_t)(hi - lo) * lane / 32u);
+      const uint32_t ge = __ballot_sync(0xffffffffu, (t_cache[e_tid[b0 + pos]] >> 24) >= target);
+      if (!ge) {
+        lo = __shfl_sync(0xffffffffu, pos, 31) + 1;
+      } else {
+        const int f = __ffs(ge) - 1;
+        const uint32_t pf = __shfl_sync(0xffffffffu, pos, f);
+        const uint32_t pb = __shfl_sync(0xffffffffu, pos, f > 0 ? f - 1 : 0);
+        hi = pf;
+        if (f > 0) lo = pb + 1;
+      }
     }
-    g->zlo[k] = lo;
+    if (lane == 0) g->zlo[k] = lo;
   }
-  __syncwarp();
-  if (k != 0) return;
+  __syncthreads();
+  if (threadIdx.x != 0) return;
   uint32_t acc = 0;
   for (int q = 0; q < 10; ++q) {
     g->gbase[q] = acc;
@@ -608,9 +614,47 @@ __device__ __forceinline__ uint32_t count_less(const uint32_t* e_tid, uint32_t l
   return lo - first;
 }
 
+// term x vs the byte string s[0..sl): <0, 0, >0
+__device__ __forceinline__ int cmp_full_str(const uint8_t* arena, const uint32_t* t_arena, const uint32_t* t_bucket,
+                                            uint32_t x, const uint8_t* s, uint32_t sl) {
+  const uint32_t bx = t_bucket[x], ax = t_arena[x], px = bucket_plen(bx), lx = px + arena[ax];
+  const uint32_t m = lx < sl ? lx : sl;
+  for (uint32_t i = 0; i < m; ++i) {
+    const uint32_t cx = full_byte(arena, ax, bx, px, i);
+    if (cx != s[i]) return cx < s[i] ? -1 : 1;
+  }
+  return lx == sl ? 0 : (lx < sl ? -1 : 1);
+}
+
+// Per 3-letter collection b = 37 + 676 k + 26 i + j (prefix c0 c1 c2, terms longer than 3 bytes):
+// short_le[b - 37] = terms of the short bucket 11 + k (first letter c0, not in a 3-letter collection)
+// that are <= "c0c1c2".  Every term T of collection b compares with a short-bucket term s as
+// "c0c1c2" does: s either differs from c0c1c2 within its first min(|s|, 3) bytes, or is a prefix of it
+// (< T), and a longer s starting with c0c1c2 would be in collection b itself.  So k_lexrank's count of
+// short terms below T is this per-collection constant instead of a binary search per term.
+__global__ void k_lex_short(const uint32_t* e_tid, const uint32_t* coll_base, const uint32_t* coll_n,
+                            const uint8_t* arena, const uint32_t* t_arena, const uint32_t* t_bucket, uint32_t* short_le) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= 17576u) return;
+  const uint32_t k = i / 676u;
+  const uint8_t key[3] = {(uint8_t)('a' + k), (uint8_t)('a' + (i / 26u) % 26u), (uint8_t)('a' + i % 26u)};
+  const uint32_t first = coll_base[11 + k];
+  uint32_t lo = first, hi = first + coll_n[11 + k];
+  while (lo < hi) {  // first entry > key
+    const uint32_t mid = (lo + hi) >> 1;
+    if (cmp_full_str(arena, t_arena, t_bucket, e_tid[mid], key, 3) <= 0) lo = mid + 1; else hi = mid;
+  }
+  short_le[i] = lo - first;
+}
+
+// Ranks of all terms (rank_of by termID, rank_info by rank).  With rec_df != nullptr (one run whose
+// records are indexed by termID, engine.cu finalize) the run's df / cf / partial-list start are
+// gathered here and written by rank (coalesced) instead of scattered by a separate pass.
 __global__ void k_lexrank(const uint32_t* e_tid, const uint32_t* e_bkt, uint32_t V, const uint32_t* coll_base,
                           const uint32_t* coll_n, const LexGroups* g, const uint8_t* arena, const uint32_t* t_arena,
-                          const uint32_t* t_bucket, const uint32_t* t_cache, uint32_t* rank_of, uint2* rank_info) {
+                          const uint32_t* t_bucket, const uint32_t* t_cache, const uint32_t* short_le, uint32_t* rank_of,
+                          uint2* rank_info, const uint32_t* rec_df, const uint32_t* rec_cf, const uint64_t* rec_start,
+                          uint32_t* df_r, uint64_t* cf_r, uint64_t* start_r) {
   const uint32_t p = blockIdx.x * blockDim.x + threadIdx.x;
   if (p >= V) return;
   const uint32_t tid = e_tid[p], b = e_bkt[p];
@@ -638,13 +682,17 @@ __global__ void k_lexrank(const uint32_t* e_tid, const uint32_t* e_bkt, uint32_t
   } else {
     const uint32_t k = (b - 37) / 676;
     const uint32_t j = p - coll_base[37 + 676 * k];
-    rank = g->gbase[10 + k] + j +
-           count_less(e_tid, coll_base[11 + k], coll_base[11 + k] + coll_n[11 + k], arena, t_arena, t_bucket, tid);
+    rank = g->gbase[10 + k] + j + short_le[b - 37];
   }
   rank_of[tid] = rank;
   // by rank, for the final dictionary bytes: arena offset, Table I index | full term length << 16
   const uint32_t a = t_arena[tid];
   rank_info[rank] = make_uint2(a, b | ((bucket_plen(b) + arena[a]) << 16));
+  if (rec_df) {
+    df_r[rank] = rec_df[tid];
+    cf_r[rank] = rec_cf[tid];
+    start_r[rank] = rec_start[tid];
+  }
 }
 
 }  // namespace wj

@@ -210,6 +210,7 @@ struct wj_index {
   uint32_t V = 0;
   uint64_t arena_used = 0;
   uint64_t table_est = 0;
+  bool recs_by_tid = false;     // the records of run 0 are indexed by termID (chunk_partials)
   uint64_t table_retries = 0;  // chunk-table probe overflows retried with a larger table (cumulative)
   // chunk table capacity = table_pct% of the expected unique terms, any multiple of 4096 slots
   // (mulhi indexing).  On config 2 the emit kernel gets faster with capacity (2.82 / 2.45 /
@@ -265,7 +266,7 @@ struct wj_index {
   DevBuf nodes, coll_root, coll_n, coll_base, coll_base2, e_tid, e_bkt, e_tid2, e_bkt2, arena, t_arena, t_cache,
       t_bucket;
   // device scalars: [0] tokens, [1] dropped, [2] U, [3] Nnew, [4] arena total, [5] overflow|bad,
-  // [6] tid counter (u32 view), [7] level count, [8] P, [9] TB, [10] bad doc_off, [11] rle tokens,
+  // [6] unused, [7] level count, [8] P, [9] TB, [10] bad doc_off, [11] rle tokens,
   DevBuf scal;
   uint64_t* h_scal = nullptr;  // pinned
   // token stream (termID, docID) of all chunks
@@ -273,7 +274,7 @@ struct wj_index {
   // chunk scratch
   DevBuf text_stage, doc_stage, seg_cnt, table, uid, u_w, u_ref, u_len, u_bucket, u_cache, u_key, u_tid, u_rank, midx, nk_key,
       nk_val, nk_key2, nk_val2, aoff, ns_tid, ns_bucket, ns_rank, nlo, nhi, nbase, lvA[4], lvB[4], child_off, root_idx,
-      scan_scr, hist, hist_scan, kstart, slotref, dbg_start, dbg_len, dbg_off, dbg_out, dbg_slot, dbg_doc, lexg, qbuf, qres;
+      scan_scr, hist, hist_scan, kstart, slotref, dbg_start, dbg_len, dbg_off, dbg_out, dbg_slot, dbg_doc, lexg, lex_short, qbuf, qres;
   // finalize
   DevBuf rank_of, term_at, sk1, sv1, pidx, out_doc, out_tf, post_off, df, cf, term_off, term_bytes;
   DevBuf vb_first, vb_tiles, vb_code, vb_boff;  // f1 (WJ_FLAG_VBYTE)
@@ -355,7 +356,7 @@ struct wj_index {
                      &uid, &u_w, &u_ref, &u_len, &u_bucket, &u_cache, &u_key, &u_tid, &u_rank, &midx, &nk_key, &nk_val,
                      &nk_key2, &nk_val2, &aoff, &ns_tid, &ns_bucket, &ns_rank, &nlo, &nhi, &nbase, &child_off,
                      &root_idx, &scan_scr, &hist, &hist_scan, &kstart, &slotref, &dbg_start, &dbg_len, &dbg_off, &dbg_out, &dbg_slot,
-                     &dbg_doc, &lexg, &qbuf, &qres, &rank_of, &term_at, &sk1, &sv1, &pidx, &out_doc, &out_tf,
+                     &dbg_doc, &lexg, &lex_short, &qbuf, &qres, &rank_of, &term_at, &sk1, &sv1, &pidx, &out_doc, &out_tf,
                      &post_off, &df, &cf, &term_off, &term_bytes, &vb_first, &vb_tiles, &vb_code, &vb_boff, &samp_hist, &owner_tab,
                      &table_s, &uid_s, &st_off, &st_text, &st_keep, &st_tidx, &st_m1, &st_slot, &st_doc, &st_tiles,
                      &st_doff, &stop_keys, &side_scan, &side_hist, &side_hist_scan, &pc_key, &pc_doc, &pc_po,
@@ -1064,6 +1065,9 @@ struct wj_index {
   // hot: the stream holds merged hot-term elements (counts) and holes (hot.cuh)
   void chunk_partials(const uint8_t* text, uint64_t Nc, uint64_t C, uint64_t U, bool hot) {
     settle_partials();  // the previous chunk is joined (add_chunk), its posting count read here
+    // the first chunk into an empty dictionary: every unique term is new and takes termID = its unique
+    // index (k_new_terms), so its records (k_chunk_records, record u = unique term u) are indexed by termID
+    recs_by_tid = nrec == 0 && V == 0 && !hot;
     uint32_t* kt = (uint32_t*)pc_key.p;
     uint32_t* dt = (uint32_t*)pc_doc.p;
     uint32_t* k1 = buf<uint32_t>(sk1, Nc + 16);
@@ -1300,6 +1304,7 @@ struct wj_index {
   // per term; the owner appends one partial-list record per (source, term) in source-rank
   // order = docID order, and finalize is the single-GPU partial-list combine.
   void add_chunk_dist_pl(const uint8_t* text, uint64_t n_bytes, const uint64_t* off, uint64_t nd) {
+    recs_by_tid = false;  // records per (source rank, term): not indexed by termID
     const int K = world;
     phase(WJ_PHASE_EXCHANGE);
     std::vector<uint64_t> ndall(K);
@@ -1765,13 +1770,10 @@ struct wj_index {
     uint32_t* nt = buf<uint32_t>(ns_tid, Nn);
     uint32_t* nb = buf<uint32_t>(ns_bucket, Nn);
     uint32_t* nr = buf<uint32_t>(ns_rank, Nn);
-    uint32_t* counter = (uint32_t*)(dscal() + 6);
-    k_fill<uint32_t><<<1, 1, 0, st>>>(counter, 1, V);
-    launched();
     k_new_terms<<<grid_for(U, 256), 256, 0, st>>>((uint32_t)U, ao, arena_used, text, (const uint4*)u_w.p,
                                                   (const uint32_t*)u_ref.p, (const uint32_t*)u_len.p,
                                                   (const uint32_t*)u_bucket.p, (const uint32_t*)u_cache.p,
-                                                  (uint32_t*)u_tid.p, counter, ar, ta, tc, tb);
+                                                  (uint32_t*)u_tid.p, (const uint32_t*)midx.p, V, ar, ta, tc, tb);
     launched();
     k_ns_fill<<<grid_for(Nn, 256), 256, 0, st>>>(sv, (uint32_t)Nn, (const uint32_t*)u_tid.p,
                                                  (const uint32_t*)u_bucket.p, (const uint32_t*)u_rank.p, nt, nb, nr);
@@ -1974,28 +1976,36 @@ struct wj_index {
     uint2* ta = buf<uint2>(term_at, V);  // rank_info
     if (!pm && (uint64_t)V > (uint64_t)kRankMask + 1)  // enforced at insert already (dictionary_update)
       throw StatusError{WJ_ERR_CAPACITY, "more than 2^25 terms in one dictionary slice"};
-    if (V > 0) {
-      phase(WJ_PHASE_LEXRANK);
-      LexGroups* g = (LexGroups*)grow(lexg, sizeof(LexGroups));
-      k_lex_groups<<<1, 32, 0, st>>>((const uint32_t*)e_tid.p, (const uint32_t*)coll_base.p,
-                                     (const uint32_t*)coll_n.p, (const uint32_t*)t_cache.p, g);
-      launched();
-      k_lexrank<<<grid_for(V, 256), 256, 0, st>>>((const uint32_t*)e_tid.p, (const uint32_t*)e_bkt.p, V,
-                                                  (const uint32_t*)coll_base.p, (const uint32_t*)coll_n.p, g,
-                                                  (const uint8_t*)arena.p, (const uint32_t*)t_arena.p,
-                                                  (const uint32_t*)t_bucket.p, (const uint32_t*)t_cache.p, ro, ta);
-      launched();
-    }
+    if (pm) join_partials();  // the last run's records (on st)
+    // one run whose records are indexed by termID (the first chunk into an empty dictionary, chunk_partials):
+    // k_lexrank gathers df / cf / list start per term and writes them by rank
+    const bool by_tid = pm && recs_by_tid && rec_end.size() == 1 && nrec == V && V > 0;
     uint64_t* po = buf<uint64_t>(post_off, (uint64_t)V + 1);
     uint32_t* dfp = buf<uint32_t>(df, V);
     uint64_t* cfp = buf<uint64_t>(cf, V);
     uint64_t* csp = buf<uint64_t>(cstart_b, (uint64_t)V + 1);
+    uint64_t* src_r = by_tid ? buf<uint64_t>(cf_totb, V) : nullptr;  // list start by rank (k_copy_by_rank)
+    if (V > 0) {
+      phase(WJ_PHASE_LEXRANK);
+      LexGroups* g = (LexGroups*)grow(lexg, sizeof(LexGroups));
+      k_lex_groups<<<1, kLexGroupThreads, 0, st>>>((const uint32_t*)e_tid.p, (const uint32_t*)coll_base.p,
+                                     (const uint32_t*)coll_n.p, (const uint32_t*)t_cache.p, g);
+      uint32_t* sle = buf<uint32_t>(lex_short, 17576);
+      k_lex_short<<<grid_for(17576, 256), 256, 0, st>>>((const uint32_t*)e_tid.p, (const uint32_t*)coll_base.p,
+                                                        (const uint32_t*)coll_n.p, (const uint8_t*)arena.p,
+                                                        (const uint32_t*)t_arena.p, (const uint32_t*)t_bucket.p, sle);
+      k_lexrank<<<grid_for(V, 256), 256, 0, st>>>(
+          (const uint32_t*)e_tid.p, (const uint32_t*)e_bkt.p, V, (const uint32_t*)coll_base.p, (const uint32_t*)coll_n.p, g,
+          (const uint8_t*)arena.p, (const uint32_t*)t_arena.p, (const uint32_t*)t_bucket.p, (const uint32_t*)t_cache.p, sle,
+          ro, ta, by_tid ? (const uint32_t*)rec_df.p : nullptr, (const uint32_t*)rec_cf.p, (const uint64_t*)rec_start.p,
+          dfp, cfp, src_r);
+      launched(3);
+    }
     P = 0;
     if (pm) {
       // combine the chunks' partial lists (partials.cuh): totals per term in chunk order, post_off in
       // rank order, one copy of every partial list to its place.  The dictionary bytes need no
       // postings: they run on the side stream (idle once the last chunk is joined) meanwhile.
-      join_partials();
       settle_partials();
       sorted_elems = n_elems - pm_merged;
       phase(-1);
@@ -2027,9 +2037,11 @@ struct wj_index {
         const uint32_t* rt = (const uint32_t*)rec_tid.p;
         const uint32_t* rd = (const uint32_t*)rec_df.p;
         if (rec_end.size() == 1) {  // one run: every partial list is its term's whole list
-          k_rank_scatter_rec<<<grid_for(nrec, 256), 256, 0, st>>>(rt, rd, (const uint32_t*)rec_cf.p, nrec, ro, dfp, cfp,
-                                                                  (const uint64_t*)rec_start.p, cft);
-          launched();
+          if (!by_tid) {  // (by_tid: k_lexrank wrote df, cf and the list starts by rank already)
+            k_rank_scatter_rec<<<grid_for(nrec, 256), 256, 0, st>>>(rt, rd, (const uint32_t*)rec_cf.p, nrec, ro, dfp, cfp,
+                                                                    (const uint64_t*)rec_start.p, cft);
+            launched();
+          }
         } else {
           WJ_CUDA_CHECK(cudaMemsetAsync(dft, 0, (size_t)V * 4, st));
           WJ_CUDA_CHECK(cudaMemsetAsync(cft, 0, (size_t)V * 8, st));

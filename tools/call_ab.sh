@@ -16,4 +16,5 @@ for v in $VARIANTS; do
   bash tools/build_variant.sh $n $(echo $d | tr ',' ' ')
   names="$names $n"
 done
-[ -z "$names" ] || LIBS="$names" bash tools/ab_libs.sh
+names="$PREBUILT $names"  # PREBUILT: ablibs/lib_<name>.so built here from another commit
+[ -z "${names// }" ] || LIBS="$names" bash tools/ab_libs.sh
