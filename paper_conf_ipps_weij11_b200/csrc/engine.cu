@@ -1021,6 +1021,26 @@ struct wj_index {
       WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 8, 0, 8, st));
       return;
     }
+    if (!counts && !n_dev) {  // plain stream: one warp per range (k_rlw_*)
+      const uint64_t W = 148ull * 3 * kRlwWarps;  // one wave at 3 CTAs per SM
+      const uint64_t per = rlw_per(N, W);
+      const uint32_t Wn = (uint32_t)((N + per - 1) / per);
+      const unsigned grid = (Wn + kRlwWarps - 1) / kRlwWarps;
+      const uint32_t Wg = grid * kRlwWarps;  // warps launched (ranges past N count 0)
+      uint32_t* rc = buf<uint32_t>(rle_p0, (uint64_t)Wg + 1);
+      uint32_t* rl = buf<uint32_t>(rle_lead, (uint64_t)Wg + 1);
+      ktime(WJ_KERNEL_RLE_EMIT, [&] {
+        k_rlw_count<<<grid, kRlwThreads, 0, st>>>(key, docs, N, per, rc);
+        launched();
+        scan<uint32_t>(ArrayIn<uint32_t>{rc}, Wg, rc, (uint32_t*)(dscal() + 8));
+        k_rlw_write<<<grid, kRlwThreads, 0, st>>>(key, docs, N, per, rc, od, of, ostride, po, csp, rl);
+        launched();
+      });
+      k_rle_fixup<<<grid_for(Wg, 256), 256, 0, st>>>(rc, rl, Wg, of, ostride);
+      launched();
+      WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 8) + 1, 0, 4, st));
+      return;
+    }
     uint64_t per = (N + 148 * 2 - 1) / (148 * 2);
     per = (per + kRleTile - 1) / kRleTile * kRleTile;
     const uint32_t G = (uint32_t)((N + per - 1) / per);

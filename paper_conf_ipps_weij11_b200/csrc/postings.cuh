@@ -332,6 +332,202 @@ __global__ void WJ_RLE_BOUNDS k_rle_write_tma(const uint32_t* __restrict__ key,
   }
 }
 
+// ------------------------------------------------------------------ run-length, one warp per range
+// Plain streams (every element one token, the element count known on the host): each warp owns a
+// contiguous range of `per` elements (a multiple of kRlwStep) and walks it 512 elements per step,
+// 16 per lane from registers; head flags, the warp scan of posting counts, the next head after each
+// lane (suffix min over lanes) and the staging of (docID, tf) pairs for a coalesced write-out all stay
+// inside the warp: no block barriers (the block version stalled ~20% on them at 2 CTAs/SM, 96
+// registers).  Posting offsets per warp range come from k_rlw_count + a scan; runs continuing across
+// ranges are completed by k_rle_fixup (range_lead = elements before the range's first head).
+constexpr int kRlwItems = 16;
+constexpr int kRlwStep = 32 * kRlwItems;  // 512
+constexpr int kRlwThreads = 256;
+constexpr int kRlwWarps = kRlwThreads / 32;
+
+__host__ __device__ __forceinline__ uint64_t rlw_per(uint64_t N, uint64_t W) {
+  const uint64_t per = (N + W - 1) / W;
+  return (per + kRlwStep - 1) / kRlwStep * kRlwStep;
+}
+
+// the lane's 16 elements of the step at i0 (past hi: key 0, doc ~0) and the element before them
+__device__ __forceinline__ void rlw_load(const uint32_t* key, const uint32_t* doc, uint64_t i0, uint64_t hi,
+                                         uint32_t (&k)[kRlwItems], uint32_t (&d)[kRlwItems]) {
+  const uint64_t b = i0 + (uint64_t)kRlwItems * lane_id();
+  if (b + kRlwItems <= hi) {
+#pragma unroll
+    for (int q = 0; q < kRlwItems / 4; ++q) {
+      const uint4 x = __ldcs((const uint4*)(key + b) + q);
+      const uint4 y = __ldcs((const uint4*)(doc + b) + q);
+      k[4 * q] = x.x; k[4 * q + 1] = x.y; k[4 * q + 2] = x.z; k[4 * q + 3] = x.w;
+      d[4 * q] = y.x; d[4 * q + 1] = y.y; d[4 * q + 2] = y.z; d[4 * q + 3] = y.w;
+    }
+  } else {
+#pragma unroll
+    for (int j = 0; j < kRlwItems; ++j) {
+      const bool v = b + j < hi;
+      k[j] = v ? key[b + j] : 0u;
+      d[j] = v ? doc[b + j] : 0xFFFFFFFFu;
+    }
+  }
+}
+
+// head (new term or new document) and term-start masks of the lane's items; (pk, pd) = the element
+// before the step, carried by the caller (pk = 0xFFFFFFFF before the stream's first element)
+__device__ __forceinline__ void rlw_flags(const uint32_t (&k)[kRlwItems], const uint32_t (&d)[kRlwItems], uint32_t pk,
+                                          uint32_t pd, uint32_t nvalid, uint32_t& npm, uint32_t& ntm) {
+  const uint32_t lane = lane_id();
+  uint32_t qk = __shfl_up_sync(0xffffffffu, k[kRlwItems - 1], 1);
+  uint32_t qd = __shfl_up_sync(0xffffffffu, d[kRlwItems - 1], 1);
+  if (lane == 0) { qk = pk; qd = pd; }
+  npm = 0;
+  ntm = 0;
+  uint32_t pr = qk & kRankMask;
+  const uint32_t first = lane * kRlwItems;
+#pragma unroll
+  for (int j = 0; j < kRlwItems; ++j) {
+    const bool valid = first + j < nvalid;
+    const uint32_t r = k[j] & kRankMask;
+    const bool nt = valid && (qk == 0xFFFFFFFFu || r != pr);
+    const bool np = valid && (nt || d[j] != qd);
+    npm |= (np ? 1u : 0u) << j;
+    ntm |= (nt ? 1u : 0u) << j;
+    pr = r;
+    qd = d[j];
+    qk = 0;
+  }
+}
+
+__global__ void __launch_bounds__(kRlwThreads) k_rlw_count(const uint32_t* __restrict__ key,
+                                                           const uint32_t* __restrict__ doc, uint64_t N, uint64_t per,
+                                                           uint32_t* wcnt) {
+  const uint32_t gw = blockIdx.x * kRlwWarps + (threadIdx.x >> 5);
+  const uint64_t lo = (uint64_t)gw * per;
+  const uint64_t hi = lo + per < N ? lo + per : N;
+  uint32_t c = 0;
+  if (lo < hi) {
+    uint32_t pk = lo > 0 ? key[lo - 1] : 0xFFFFFFFFu, pd = lo > 0 ? doc[lo - 1] : 0xFFFFFFFFu;
+    for (uint64_t i0 = lo; i0 < hi; i0 += kRlwStep) {
+      uint32_t k[kRlwItems], d[kRlwItems], npm, ntm;
+      rlw_load(key, doc, i0, hi, k, d);
+      const uint32_t nvalid = (uint32_t)min((uint64_t)kRlwStep, hi - i0);
+      rlw_flags(k, d, pk, pd, nvalid, npm, ntm);
+      c += __popc(npm);
+      pk = __shfl_sync(0xffffffffu, k[kRlwItems - 1], 31);
+      pd = __shfl_sync(0xffffffffu, d[kRlwItems - 1], 31);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+  }
+  if (lane_id() == 0) wcnt[gw] = c;
+}
+
+// woff: exclusive posting offset of each warp range (scan of k_rlw_count); writes (docID, tf) at
+// out_doc / out_tf [ostride * posting] (ostride 2: interleaved pairs), post_off / cstart at each term's
+// key, range_lead[gw] = elements of the range before its first head
+__global__ void __launch_bounds__(kRlwThreads, 3) k_rlw_write(const uint32_t* __restrict__ key,
+                                                              const uint32_t* __restrict__ doc, uint64_t N, uint64_t per,
+                                                              const uint32_t* __restrict__ woff, uint32_t* out_doc,
+                                                              uint32_t* out_tf, uint32_t ostride, uint64_t* post_off,
+                                                              uint64_t* cstart, uint32_t* range_lead) {
+  __shared__ uint2 stage[kRlwWarps][kRlwStep];
+  const uint32_t lane = lane_id();
+  const int w = threadIdx.x >> 5;
+  const uint32_t gw = blockIdx.x * kRlwWarps + w;
+  const uint64_t lo = (uint64_t)gw * per;
+  const uint64_t hi = lo + per < N ? lo + per : N;
+  if (lo >= hi) {
+    if (lane == 0) range_lead[gw] = 0;
+    return;
+  }
+  uint2* sg = stage[w];
+  uint32_t pk = lo > 0 ? key[lo - 1] : 0xFFFFFFFFu, pd = lo > 0 ? doc[lo - 1] : 0xFFFFFFFFu;
+  uint32_t p = woff[gw];
+  uint32_t lead = 0, open_len = 0, open_p = 0;
+  bool lead_done = false, have_open = false;
+  const uint32_t lt = (1u << lane) - 1u;
+  for (uint64_t i0 = lo; i0 < hi; i0 += kRlwStep) {
+    uint32_t k[kRlwItems], d[kRlwItems], npm, ntm;
+    rlw_load(key, doc, i0, hi, k, d);
+    const uint32_t nvalid = (uint32_t)min((uint64_t)kRlwStep, hi - i0);
+    rlw_flags(k, d, pk, pd, nvalid, npm, ntm);
+    const uint32_t c = __popc(npm);
+    uint32_t inc = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
+      if ((int)lane >= o) inc += u;
+    }
+    const uint32_t T = __shfl_sync(0xffffffffu, inc, 31);
+    const uint32_t base = lane * kRlwItems;
+    // first head of each lane; next head after each lane (suffix min over later lanes)
+    const uint32_t mine = npm ? base + __ffs(npm) - 1 : 0xFFFFFFFFu;
+    uint32_t after = mine;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t u = __shfl_down_sync(0xffffffffu, after, o);
+      if (lane + o < 32) after = min(after, u);
+    }
+    uint32_t next_after = __shfl_down_sync(0xffffffffu, after, 1);
+    if (lane == 31) next_after = 0xFFFFFFFFu;
+    const uint32_t first_all = __shfl_sync(0xffffffffu, after, 0);
+    const uint32_t before = first_all == 0xFFFFFFFFu ? nvalid : first_all;  // elements before the step's first head
+    if (!lead_done) {
+      lead += before;
+      lead_done = first_all != 0xFFFFFFFFu;
+    }
+    if (have_open) {  // the previous step's last posting runs into this step
+      open_len += before;
+      if (first_all != 0xFFFFFFFFu) {
+        if (lane == 0) out_tf[(uint64_t)ostride * open_p] = open_len;
+        have_open = false;
+      }
+    }
+    uint32_t lp = inc - c;
+    uint32_t last_tf = 0;
+#pragma unroll
+    for (int j = 0; j < kRlwItems; ++j) {
+      if ((npm >> j) & 1u) {
+        const uint32_t pos = base + j;
+        const uint32_t rest = npm & ~((2u << j) - 1u);
+        const uint32_t end = rest ? base + __ffs(rest) - 1 : min(next_after, nvalid);
+        last_tf = end - pos;
+        sg[lp] = make_uint2(d[j], last_tf);
+        if ((ntm >> j) & 1u) {
+          const uint32_t r = k[j] & kRankMask;
+          post_off[r] = p + lp;
+          cstart[r] = i0 + pos;
+        }
+        ++lp;
+      }
+    }
+    __syncwarp();
+    if (ostride == 2) {
+      for (uint32_t x = lane; x < T; x += 32) __stcs((uint2*)out_doc + p + x, sg[x]);
+    } else {
+      for (uint32_t x = lane; x < T; x += 32) {
+        const uint2 v = sg[x];
+        __stcs(out_doc + p + x, v.x);
+        __stcs(out_tf + p + x, v.y);
+      }
+    }
+    if (T) {  // the step's last posting may continue into the next step
+      const uint32_t hl = 31 - __clz(__ballot_sync(0xffffffffu, c != 0));  // lane holding it
+      open_len = __shfl_sync(0xffffffffu, last_tf, hl);
+      open_p = p + T - 1;
+      have_open = true;
+    }
+    p += T;
+    pk = __shfl_sync(0xffffffffu, k[kRlwItems - 1], 31);
+    pd = __shfl_sync(0xffffffffu, d[kRlwItems - 1], 31);
+    __syncwarp();
+  }
+  if (lane == 0) {
+    if (have_open) out_tf[(uint64_t)ostride * open_p] = open_len;
+    range_lead[gw] = lead;
+  }
+}
+
 // runs that continue across tiles: add each tile's leading items to the preceding posting
 __global__ void k_rle_fixup(const uint32_t* tile_p0, const uint32_t* tile_lead, uint32_t tiles, uint32_t* out_tf,
                             uint32_t ostride) {

@@ -340,6 +340,18 @@ def test_hot_path_repetitive_docs(global_stream):
                       want)
 
 
+def test_long_runs_across_run_length_ranges():
+    """(term, doc) runs far longer than a run-length warp range (k_rlw_write walks 512-element steps;
+    a range with no posting start adds all its elements to the previous range's open posting through
+    k_rle_fixup), next to single-token documents and a new document at every step boundary."""
+    docs = [b"w " * 70000 + b"end", b"w", b"v w"] + [b"w " * 511 + b"q"] * 40 + [b"a " * 1024] * 3 + [b"x"] * 2000
+    text, off = gen.from_docs(docs)
+    want = oracle.index_bytes(text, off)
+    assert_same_index(gpu_index(text, off), want)
+    assert_same_index(gpu_index(text, off, cuts=[0, 1, 40, len(docs)]), want)
+    assert_same_index(gpu_index(text, off, global_stream=True), want)
+
+
 def test_hot_off_by_default():
     cfg = gen.CONFIGS[2].scaled(chunk_bytes=10 << 20, vocab=100_000)
     text, off = gen.generate(cfg)
