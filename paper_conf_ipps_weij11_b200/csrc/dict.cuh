@@ -406,14 +406,23 @@ __global__ void k_new_terms(uint32_t U, const uint32_t* aoff, uint64_t arena_bas
   u_tid[u] = tid;
 }
 
+// E (the per-collection sorted key order) carries, besides termIDs, each term's arena offset and
+// "info" = Table I index | full length << 16, so that finalize reads them in E order (k_lexrank)
+__host__ __device__ __forceinline__ uint32_t e_info(uint32_t bucket, uint32_t full_len) { return bucket | full_len << 16; }
+__host__ __device__ __forceinline__ uint32_t e_info_bucket(uint32_t info) { return info & 0xFFFFu; }
+
 __global__ void k_ns_fill(const uint32_t* sorted_u, uint32_t N, const uint32_t* u_tid, const uint32_t* u_bucket,
-                          const uint32_t* u_rank, uint32_t* ns_tid, uint32_t* ns_bucket, uint32_t* ns_rank) {
+                          const uint32_t* u_rank, const uint32_t* u_len, const uint32_t* aoff, uint64_t arena_base,
+                          uint32_t* ns_tid, uint32_t* ns_bucket, uint32_t* ns_rank, uint32_t* ns_info, uint32_t* ns_arena) {
   const uint32_t k = blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= N) return;
   const uint32_t u = sorted_u[k];
   ns_tid[k] = u_tid[u];
-  ns_bucket[k] = u_bucket[u];
+  const uint32_t b = u_bucket[u];
+  ns_bucket[k] = b;
   ns_rank[k] = u_rank[u];
+  ns_info[k] = e_info(b, u_len[u]);
+  ns_arena[k] = (uint32_t)(arena_base + aoff[u]);
 }
 
 // per-collection [lo, hi) of the sorted new terms
@@ -432,22 +441,24 @@ struct NewCount {
   __device__ __forceinline__ uint32_t operator()(uint64_t b) const { return coll_n[b] + (nhi[b] - nlo[b]); }
 };
 
-__global__ void k_place_new(const uint32_t* ns_tid, const uint32_t* ns_bucket, const uint32_t* ns_rank, uint32_t N,
-                            const uint32_t* nlo, const uint32_t* nbase, uint32_t* e_tid, uint32_t* e_bkt) {
+__global__ void k_place_new(const uint32_t* ns_tid, const uint32_t* ns_info, const uint32_t* ns_arena,
+                            const uint32_t* ns_rank, uint32_t N, const uint32_t* nlo, const uint32_t* nbase, uint32_t* e_tid,
+                            uint32_t* e_inf, uint32_t* e_ar) {
   const uint32_t k = blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= N) return;
-  const uint32_t b = ns_bucket[k];
+  const uint32_t inf = ns_info[k], b = e_info_bucket(inf);
   const uint32_t pos = nbase[b] + ns_rank[k] + (k - nlo[b]);
   e_tid[pos] = ns_tid[k];
-  e_bkt[pos] = b;
+  e_inf[pos] = inf;
+  e_ar[pos] = ns_arena[k];
 }
 
-__global__ void k_place_old(const uint32_t* o_tid, const uint32_t* o_bkt, uint32_t V, const uint32_t* obase,
-                            const uint32_t* ns_rank, const uint32_t* nlo, const uint32_t* nhi, const uint32_t* nbase,
-                            uint32_t* e_tid, uint32_t* e_bkt) {
+__global__ void k_place_old(const uint32_t* o_tid, const uint32_t* o_inf, const uint32_t* o_ar, uint32_t V,
+                            const uint32_t* obase, const uint32_t* ns_rank, const uint32_t* nlo, const uint32_t* nhi,
+                            const uint32_t* nbase, uint32_t* e_tid, uint32_t* e_inf, uint32_t* e_ar) {
   const uint32_t p = blockIdx.x * blockDim.x + threadIdx.x;
   if (p >= V) return;
-  const uint32_t b = o_bkt[p];
+  const uint32_t inf = o_inf[p], b = e_info_bucket(inf);
   const uint32_t i = p - obase[b];
   // number of new keys of b with insertion rank <= i
   uint32_t lo = nlo[b], hi = nhi[b];
@@ -458,7 +469,8 @@ __global__ void k_place_old(const uint32_t* o_tid, const uint32_t* o_bkt, uint32
   }
   const uint32_t pos = nbase[b] + i + (lo - first);
   e_tid[pos] = o_tid[p];
-  e_bkt[pos] = b;
+  e_inf[pos] = inf;
+  e_ar[pos] = o_ar[p];
 }
 
 // ------------------------------------------------------------------ bulk rebuild, level by level
@@ -647,17 +659,18 @@ __global__ void k_lex_short(const uint32_t* e_tid, const uint32_t* coll_base, co
   short_le[i] = lo - first;
 }
 
-// Ranks of all terms (rank_of by termID, rank_info by rank).  With rec_df != nullptr (one run whose
-// records are indexed by termID, engine.cu finalize) the run's df / cf / partial-list start are
-// gathered here and written by rank (coalesced) instead of scattered by a separate pass.
-__global__ void k_lexrank(const uint32_t* e_tid, const uint32_t* e_bkt, uint32_t V, const uint32_t* coll_base,
-                          const uint32_t* coll_n, const LexGroups* g, const uint8_t* arena, const uint32_t* t_arena,
-                          const uint32_t* t_bucket, const uint32_t* t_cache, const uint32_t* short_le, uint32_t* rank_of,
-                          uint2* rank_info, const uint32_t* rec_df, const uint32_t* rec_cf, const uint64_t* rec_start,
-                          uint32_t* df_r, uint64_t* cf_r, uint64_t* start_r) {
+// Ranks of all terms (rank_of by termID, rank_info by rank), reading E, its arena offsets and infos in
+// order.  With rec != nullptr (one run whose records are indexed by termID, engine.cu finalize) the
+// run's (list start, df, cf) are gathered here (one 16-byte record per term) and written by rank
+// (coalesced) instead of scattered by a separate pass.
+__global__ void k_lexrank(const uint32_t* e_tid, const uint32_t* e_inf, const uint32_t* e_ar, uint32_t V,
+                          const uint32_t* coll_base, const uint32_t* coll_n, const LexGroups* g, const uint8_t* arena,
+                          const uint32_t* t_arena, const uint32_t* t_bucket, const uint32_t* t_cache,
+                          const uint32_t* short_le, uint32_t* rank_of, uint2* rank_info, const uint4* rec, uint32_t* df_r,
+                          uint64_t* cf_r, uint64_t* start_r) {
   const uint32_t p = blockIdx.x * blockDim.x + threadIdx.x;
   if (p >= V) return;
-  const uint32_t tid = e_tid[p], b = e_bkt[p];
+  const uint32_t tid = e_tid[p], inf = e_inf[p], b = e_info_bucket(inf);
   uint32_t rank;
   if (b == 0) {
     const uint32_t i = p - coll_base[0];
@@ -686,12 +699,12 @@ __global__ void k_lexrank(const uint32_t* e_tid, const uint32_t* e_bkt, uint32_t
   }
   rank_of[tid] = rank;
   // by rank, for the final dictionary bytes: arena offset, Table I index | full term length << 16
-  const uint32_t a = t_arena[tid];
-  rank_info[rank] = make_uint2(a, b | ((bucket_plen(b) + arena[a]) << 16));
-  if (rec_df) {
-    df_r[rank] = rec_df[tid];
-    cf_r[rank] = rec_cf[tid];
-    start_r[rank] = rec_start[tid];
+  rank_info[rank] = make_uint2(e_ar[p], inf);
+  if (rec) {
+    const uint4 r = rec[tid];  // list start (lo, hi), df, cf
+    df_r[rank] = r.z;
+    cf_r[rank] = r.w;
+    start_r[rank] = (uint64_t)r.x | (uint64_t)r.y << 32;
   }
 }
 

@@ -239,7 +239,7 @@ struct wj_index {
   cudaEvent_t ev_fork = nullptr, ev_side = nullptr, ev_dict = nullptr;
   DevBuf side_scan, side_hist, side_hist_scan;
   DevBuf mr_key, mr_idx, mr_key2, mr_idx2, mr_dst, mr_src;  // several runs: records in destination order
-  DevBuf pc_key, pc_doc, pc_po, pc_cs, u_slot, pp_pair, x_pair, rec_tid, rec_start, rec_df, rec_cf, rec_before, df_totb,
+  DevBuf pc_key, pc_doc, pc_po, pc_cs, u_slot, pp_pair, x_pair, rec_tid, rec_start, rec_df, rec_cf, rec_aos, rec_before, df_totb,
       cf_totb;
   uint64_t pbase = 0, nrec = 0;      // partial postings / records of the chunks so far
   uint32_t rs_ctas = kRsCtas;        // radix downsweep CTAs (ranges) of sort_pairs
@@ -263,7 +263,8 @@ struct wj_index {
       x_hdf, x_hcf, x_rhdf, x_rhcf, x_rpre, x_bnd;
   double exchange_ms = 0;  // host wall time inside the all-to-all-v calls (cumulative)
   // persistent dictionary
-  DevBuf nodes, coll_root, coll_n, coll_base, coll_base2, e_tid, e_bkt, e_tid2, e_bkt2, arena, t_arena, t_cache,
+  // E = per-collection sorted key order: termID, info (Table I index | full length << 16), arena offset
+  DevBuf nodes, coll_root, coll_n, coll_base, coll_base2, e_tid, e_bkt, e_tid2, e_bkt2, e_ar, e_ar2, arena, t_arena, t_cache,
       t_bucket;
   // device scalars: [0] tokens, [1] dropped, [2] U, [3] Nnew, [4] arena total, [5] overflow|bad,
   // [6] unused, [7] level count, [8] P, [9] TB, [10] bad doc_off, [11] rle tokens,
@@ -273,7 +274,7 @@ struct wj_index {
   DevBuf g_tid, g_doc;
   // chunk scratch
   DevBuf text_stage, doc_stage, seg_cnt, table, uid, u_w, u_ref, u_len, u_bucket, u_cache, u_key, u_tid, u_rank, midx, nk_key,
-      nk_val, nk_key2, nk_val2, aoff, ns_tid, ns_bucket, ns_rank, nlo, nhi, nbase, lvA[4], lvB[4], child_off, root_idx,
+      nk_val, nk_key2, nk_val2, aoff, ns_tid, ns_bucket, ns_rank, ns_info, ns_arena, nlo, nhi, nbase, lvA[4], lvB[4], child_off, root_idx,
       scan_scr, hist, hist_scan, kstart, slotref, dbg_start, dbg_len, dbg_off, dbg_out, dbg_slot, dbg_doc, lexg, lex_short, qbuf, qres;
   // finalize
   DevBuf rank_of, term_at, sk1, sv1, pidx, out_doc, out_tf, post_off, df, cf, term_off, term_bytes;
@@ -351,16 +352,16 @@ struct wj_index {
     return (T*)grow(b, std::max<uint64_t>(n, 1) * sizeof(T), true, used * sizeof(T));
   }
   void free_all() {
-    DevBuf* all[] = {&nodes, &coll_root, &coll_n, &coll_base, &coll_base2, &e_tid, &e_bkt, &e_tid2, &e_bkt2, &arena,
+    DevBuf* all[] = {&nodes, &coll_root, &coll_n, &coll_base, &coll_base2, &e_tid, &e_bkt, &e_tid2, &e_bkt2, &e_ar, &e_ar2, &arena,
                      &t_arena, &t_cache, &t_bucket, &scal, &g_tid, &g_doc, &text_stage, &doc_stage, &seg_cnt, &table,
                      &uid, &u_w, &u_ref, &u_len, &u_bucket, &u_cache, &u_key, &u_tid, &u_rank, &midx, &nk_key, &nk_val,
-                     &nk_key2, &nk_val2, &aoff, &ns_tid, &ns_bucket, &ns_rank, &nlo, &nhi, &nbase, &child_off,
+                     &nk_key2, &nk_val2, &aoff, &ns_tid, &ns_bucket, &ns_rank, &ns_info, &ns_arena, &nlo, &nhi, &nbase, &child_off,
                      &root_idx, &scan_scr, &hist, &hist_scan, &kstart, &slotref, &dbg_start, &dbg_len, &dbg_off, &dbg_out, &dbg_slot,
                      &dbg_doc, &lexg, &lex_short, &qbuf, &qres, &rank_of, &term_at, &sk1, &sv1, &pidx, &out_doc, &out_tf,
                      &post_off, &df, &cf, &term_off, &term_bytes, &vb_first, &vb_tiles, &vb_code, &vb_boff, &samp_hist, &owner_tab,
                      &table_s, &uid_s, &st_off, &st_text, &st_keep, &st_tidx, &st_m1, &st_slot, &st_doc, &st_tiles,
                      &st_doff, &stop_keys, &side_scan, &side_hist, &side_hist_scan, &pc_key, &pc_doc, &pc_po,
-                     &pc_cs, &u_slot, &pp_pair, &x_pair, &mr_key, &mr_idx, &mr_key2, &mr_idx2, &mr_dst, &mr_src, &rec_tid, &rec_start, &rec_df, &rec_cf, &rec_before, &df_totb,
+                     &pc_cs, &u_slot, &pp_pair, &x_pair, &mr_key, &mr_idx, &mr_key2, &mr_idx2, &mr_dst, &mr_src, &rec_tid, &rec_start, &rec_df, &rec_cf, &rec_aos, &rec_before, &df_totb,
                      &cf_totb};
     for (DevBuf* b : all) {
       dev_free(b->p);
@@ -1173,7 +1174,8 @@ struct wj_index {
         (const uint32_t*)u_slot.p, (uint32_t)U, po, cs, (const uint32_t*)(dscal() + (pc_hot ? 12 : 8)), Nc,
         pc_hot ? (const uint32_t*)(dscal() + 13) : nullptr,
         (const uint32_t*)u_tid.p, pbase, rt + nrec, rs + nrec, rd + nrec, rc + nrec, (const Slot*)table.p,
-        pc_hot ? (const uint32_t*)hot_posb.p : nullptr, (const uint32_t*)hot_cfb.p, hot_D, nh, hot_Hdev());
+        pc_hot ? (const uint32_t*)hot_posb.p : nullptr, (const uint32_t*)hot_cfb.p, hot_D, nh, hot_Hdev(),
+        recs_by_tid ? buf<uint4>(rec_aos, U) : nullptr);
     launched();
     WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 13, dscal() + 8, 8, cudaMemcpyDeviceToHost, st));
     if (pc_hot) WJ_CUDA_CHECK(cudaMemcpyAsync(h_scal + 14, dscal() + 13, 8, cudaMemcpyDeviceToHost, st));
@@ -1795,8 +1797,11 @@ struct wj_index {
                                                   (const uint32_t*)u_bucket.p, (const uint32_t*)u_cache.p,
                                                   (uint32_t*)u_tid.p, (const uint32_t*)midx.p, V, ar, ta, tc, tb);
     launched();
+    uint32_t* ni = buf<uint32_t>(ns_info, Nn);
+    uint32_t* na = buf<uint32_t>(ns_arena, Nn);
     k_ns_fill<<<grid_for(Nn, 256), 256, 0, st>>>(sv, (uint32_t)Nn, (const uint32_t*)u_tid.p,
-                                                 (const uint32_t*)u_bucket.p, (const uint32_t*)u_rank.p, nt, nb, nr);
+                                                 (const uint32_t*)u_bucket.p, (const uint32_t*)u_rank.p,
+                                                 (const uint32_t*)u_len.p, ao, arena_used, nt, nb, nr, ni, na);
     launched();
     arena_used += A;
     // merge into the sorted key order E of every collection
@@ -1810,17 +1815,20 @@ struct wj_index {
     scan<uint32_t>(NewCount{(const uint32_t*)coll_n.p, lo, hi}, kCollections, cb2, cb2 + kCollections);
     uint32_t* et2 = buf<uint32_t>(e_tid2, Vn);
     uint32_t* eb2 = buf<uint32_t>(e_bkt2, Vn);
-    k_place_new<<<grid_for(Nn, 256), 256, 0, st>>>(nt, nb, nr, (uint32_t)Nn, lo, cb2, et2, eb2);
+    uint32_t* ea2 = buf<uint32_t>(e_ar2, Vn);
+    k_place_new<<<grid_for(Nn, 256), 256, 0, st>>>(nt, ni, na, nr, (uint32_t)Nn, lo, cb2, et2, eb2, ea2);
     launched();
     if (V > 0) {
-      k_place_old<<<grid_for(V, 256), 256, 0, st>>>((const uint32_t*)e_tid.p, (const uint32_t*)e_bkt.p, V,
-                                                    (const uint32_t*)coll_base.p, nr, lo, hi, cb2, et2, eb2);
+      k_place_old<<<grid_for(V, 256), 256, 0, st>>>((const uint32_t*)e_tid.p, (const uint32_t*)e_bkt.p,
+                                                    (const uint32_t*)e_ar.p, V, (const uint32_t*)coll_base.p, nr, lo, hi,
+                                                    cb2, et2, eb2, ea2);
       launched();
     }
     k_update_counts<<<grid_for(kCollections, 256), 256, 0, st>>>((uint32_t*)coll_n.p, lo, hi);
     launched();
     std::swap(e_tid, e_tid2);
     std::swap(e_bkt, e_bkt2);
+    std::swap(e_ar, e_ar2);
     std::swap(coll_base, coll_base2);
     V = (uint32_t)Vn;
   }
@@ -2015,10 +2023,9 @@ struct wj_index {
                                                         (const uint32_t*)coll_n.p, (const uint8_t*)arena.p,
                                                         (const uint32_t*)t_arena.p, (const uint32_t*)t_bucket.p, sle);
       k_lexrank<<<grid_for(V, 256), 256, 0, st>>>(
-          (const uint32_t*)e_tid.p, (const uint32_t*)e_bkt.p, V, (const uint32_t*)coll_base.p, (const uint32_t*)coll_n.p, g,
-          (const uint8_t*)arena.p, (const uint32_t*)t_arena.p, (const uint32_t*)t_bucket.p, (const uint32_t*)t_cache.p, sle,
-          ro, ta, by_tid ? (const uint32_t*)rec_df.p : nullptr, (const uint32_t*)rec_cf.p, (const uint64_t*)rec_start.p,
-          dfp, cfp, src_r);
+          (const uint32_t*)e_tid.p, (const uint32_t*)e_bkt.p, (const uint32_t*)e_ar.p, V, (const uint32_t*)coll_base.p,
+          (const uint32_t*)coll_n.p, g, (const uint8_t*)arena.p, (const uint32_t*)t_arena.p, (const uint32_t*)t_bucket.p,
+          (const uint32_t*)t_cache.p, sle, ro, ta, by_tid ? (const uint4*)rec_aos.p : nullptr, dfp, cfp, src_r);
       launched(3);
     }
     P = 0;

@@ -27,7 +27,8 @@ __global__ void k_chunk_records(const uint32_t* __restrict__ u_slot, uint32_t U,
                                 uint32_t* rec_tid,
                                 uint64_t* rec_start, uint32_t* rec_df, uint32_t* rec_cf, const Slot* __restrict__ table,
                                 const uint32_t* __restrict__ hot_pos, const uint32_t* __restrict__ hot_cf, uint32_t D,
-                                const uint32_t* __restrict__ nh_pos, const uint32_t* __restrict__ H_dev) {
+                                const uint32_t* __restrict__ nh_pos, const uint32_t* __restrict__ H_dev,
+                                uint4* rec_aos) {
   const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
   if (u >= U) return;
   auto hot_of = [&](uint32_t slot) -> uint32_t {
@@ -56,6 +57,8 @@ __global__ void k_chunk_records(const uint32_t* __restrict__ u_slot, uint32_t U,
   rec_start[r] = pbase + a;
   rec_df[r] = (uint32_t)(b - a);
   rec_cf[r] = (uint32_t)(tb - ta);
+  if (rec_aos)  // the same record as one 16-byte line (finalize of a run indexed by termID, k_lexrank)
+    rec_aos[r] = make_uint4((uint32_t)(pbase + a), (uint32_t)((pbase + a) >> 32), (uint32_t)(b - a), (uint32_t)(tb - ta));
 }
 
 struct NotHotSlot {  // 1 for a unique term whose slot carries no hot id
