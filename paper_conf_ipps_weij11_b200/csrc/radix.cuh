@@ -20,14 +20,39 @@ constexpr int kOsTile = kOsThreads * kOsItems;  // 4096
 
 // Lanes holding the same 8-bit digit (a warp-wide multi-split with 8 ballots: cheaper than
 // MATCH.ANY on sm_100a); `valid` lanes only.
+#ifndef WJ_PEERS_ASM
+#define WJ_PEERS_ASM 1
+#endif
 __device__ __forceinline__ uint32_t digit_peers(uint32_t d, bool valid) {
   uint32_t peers = __ballot_sync(0xffffffffu, valid);
+#if WJ_PEERS_ASM
+  // The integer ALU pipe issues one warp instruction every 2 cycles per SMSP (B300_MICROARCH.md
+  // "fma vs alu split") and this loop is ~45% of the downsweep's instructions: one predicate test, the
+  // ballot and one predicated LOP3 per bit (the C form compiles to shift, test, a second compare, ballot,
+  // select and LOP3).
+  uint32_t m[8];
+#pragma unroll
+  for (int b = 0; b < 8; ++b)  // m[b] = lanes whose bit b equals this lane's
+    asm("{\n\t.reg .pred p;\n\t.reg .b32 t;\n\t"
+        "and.b32 t, %1, %2;\n\t"
+        "setp.ne.u32 p, t, 0;\n\t"
+        "vote.sync.ballot.b32 %0, p, 0xffffffff;\n\t"
+        "@!p not.b32 %0, %0;\n\t}"
+        : "=r"(m[b])
+        : "r"(d), "r"(1u << b));
+  uint32_t a, b2, c;  // the AND of 9 masks as 4 three-input LOP3s (ptxas keeps 2-input ANDs otherwise)
+  asm("lop3.b32 %0, %1, %2, %3, 0x80;" : "=r"(a) : "r"(peers), "r"(m[0]), "r"(m[1]));
+  asm("lop3.b32 %0, %1, %2, %3, 0x80;" : "=r"(b2) : "r"(m[2]), "r"(m[3]), "r"(m[4]));
+  asm("lop3.b32 %0, %1, %2, %3, 0x80;" : "=r"(c) : "r"(m[5]), "r"(m[6]), "r"(m[7]));
+  asm("lop3.b32 %0, %1, %2, %3, 0x80;" : "=r"(peers) : "r"(a), "r"(b2), "r"(c));
+#else
 #pragma unroll
   for (int b = 0; b < 8; ++b) {
     const bool bit = (d >> b) & 1u;
     const uint32_t m = __ballot_sync(0xffffffffu, bit);
     peers &= bit ? m : ~m;
   }
+#endif
   return peers;
 }
 
