@@ -106,6 +106,10 @@ __global__ void k_update_counts(uint32_t* coll_n, const uint32_t* nlo, const uin
   const uint32_t b = blockIdx.x * blockDim.x + threadIdx.x;
   if (b < kCollections) coll_n[b] += nhi[b] - nlo[b];
 }
+__global__ void k_iota_u32(uint32_t* p, uint32_t n) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) p[i] = i;
+}
 
 // doc_off validation: doc_off[0]==0, non-decreasing, doc_off[n]==n_bytes
 __global__ void k_check_docoff(const uint64_t* d, uint64_t n_docs, uint64_t n_bytes, uint32_t* bad) {
@@ -209,6 +213,11 @@ struct wj_index {
   uint64_t unique_last = 0, new_last = 0, n_nodes = 0, height_max = 0;
   uint32_t V = 0;
   uint64_t arena_used = 0;
+  // The first insert into an empty dictionary takes its arena size A from a bound (the chunk's text
+  // bytes + U, set in dict_text_bytes by the caller; 0 = no bound) instead of a host round trip on the
+  // dictionary stream; A stays on the device (dscal[4]) until settle_arena() reads it.
+  uint64_t dict_text_bytes = 0;
+  bool arena_pending = false;
   uint64_t table_est = 0;
   bool recs_by_tid = false;     // the records of run 0 are indexed by termID (chunk_partials)
   uint64_t table_retries = 0;  // chunk-table probe overflows retried with a larger table (cumulative)
@@ -235,6 +244,11 @@ struct wj_index {
   // runs on st; finalize combines the partial lists.  WJ_PARTIALS=0: global stream
   // sorted at finalize instead.
   bool pm = false;
+  // packed chunk stream (partials path without hot terms): the emit kernel writes one u64 per token,
+  // slot << 32 | docID, into pc_key; the sort moves it as a value-less 64-bit key and the run-length
+  // pass reads it back (one 8-byte access per element everywhere instead of two 4-byte ones)
+  unsigned long long* emit_elem = nullptr;
+  bool pc_packed = false;
   cudaStream_t side_st = nullptr, hp_st = nullptr;  // side: lowest priority; hp: dictionary, highest
   cudaEvent_t ev_fork = nullptr, ev_side = nullptr, ev_dict = nullptr;
   DevBuf side_scan, side_hist, side_hist_scan;
@@ -243,7 +257,10 @@ struct wj_index {
       cf_totb;
   uint64_t pbase = 0, nrec = 0;      // partial postings / records of the chunks so far
   uint32_t rs_ctas = kRsCtas;        // radix downsweep CTAs (ranges) of sort_pairs
-  uint32_t side_ctas = kRsCtas;      // ... for the side stream's sort (148 / 222 measured slower)
+#ifndef WJ_SIDE_CTAS
+#define WJ_SIDE_CTAS kRsCtas
+#endif
+  uint32_t side_ctas = WJ_SIDE_CTAS;  // ... for the side stream's sort (148 / 222 measured slower)
   bool pc_pending = false;           // the last chunk's posting count is still on the device (dscal[13])
   bool pc_join = false;              // the last chunk's side-stream work is not joined yet
   uint64_t pc_U = 0, pc_Nc = 0;  // pc_Nc: tokens of the pending chunk
@@ -490,6 +507,8 @@ struct wj_index {
     exchange_bytes = 0;
     V = 0;
     arena_used = 0;
+    arena_pending = false;
+    dict_text_bytes = 0;
     P = TB = PB = 0;
     finalized = false;
     f_key = f_doc = nullptr;
@@ -586,6 +605,7 @@ struct wj_index {
     eo.doc_base = doc_base;
     eo.slot = slot_out;
     eo.doc = doc_out;
+    eo.elem = use_hot ? nullptr : emit_elem;
     eo.dbg_start = dstart;
     eo.dbg_len = dlen;
     eo.overflow = (uint32_t*)(dscal() + 5);
@@ -982,10 +1002,16 @@ struct wj_index {
     }
     phase(WJ_PHASE_INSERT);
     uint32_t* mi = buf<uint32_t>(midx, U);
-    scan<uint32_t>(IsMiss{ut}, U, mi, (uint32_t*)(dscal() + 3));
-    WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 3) + 1, 0, 4, st));
-    readback(3, 1);
-    const uint64_t Nn = (uint32_t)h_scal[3];
+    uint64_t Nn = U;
+    if (V > 0) {
+      scan<uint32_t>(IsMiss{ut}, U, mi, (uint32_t*)(dscal() + 3));
+      WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 3) + 1, 0, 4, st));
+      readback(3, 1);
+      Nn = (uint32_t)h_scal[3];
+    } else {  // an empty dictionary: every unique term is new, miss index = unique index (no round trip)
+      k_iota_u32<<<grid_for(U, 256), 256, 0, st>>>(mi, (uint32_t)U);
+      launched();
+    }
     new_last = Nn;
     if (Nn > 0) {
       // the per-run partial lists carry u32 termIDs; the global-stream path (multi-rank, stemming)
@@ -1012,7 +1038,8 @@ struct wj_index {
   // n_dev (optional): the actual element count on the device, N being an upper bound
   // pairs != nullptr: the postings go there as interleaved (docID, tf) pairs (per-run partial lists)
   void rle(const uint32_t* key, const uint32_t* docs, uint64_t N, bool counts, uint32_t* od, uint32_t* of, uint64_t* po,
-           uint64_t* csp, const uint32_t* n_dev = nullptr, uint2* pairs = nullptr) {
+           uint64_t* csp, const uint32_t* n_dev = nullptr, uint2* pairs = nullptr,
+           const unsigned long long* elem = nullptr) {
     const uint32_t ostride = pairs ? 2u : 1u;
     if (pairs) {
       od = (uint32_t*)pairs;
@@ -1022,8 +1049,12 @@ struct wj_index {
       WJ_CUDA_CHECK(cudaMemsetAsync(dscal() + 8, 0, 8, st));
       return;
     }
+    if (elem && (counts || n_dev)) throw StatusError{WJ_ERR_STATE, "packed stream with counts"};
     if (!counts && !n_dev) {  // plain stream: one warp per range (k_rlw_*)
-      const uint64_t W = 148ull * 3 * kRlwWarps;  // one wave at 3 CTAs per SM
+#ifndef WJ_RLW_WAVES
+#define WJ_RLW_WAVES 1
+#endif
+      const uint64_t W = 148ull * 3 * kRlwWarps * WJ_RLW_WAVES;  // one wave at 3 CTAs per SM
       const uint64_t per = rlw_per(N, W);
       const uint32_t Wn = (uint32_t)((N + per - 1) / per);
       const unsigned grid = (Wn + kRlwWarps - 1) / kRlwWarps;
@@ -1031,10 +1062,12 @@ struct wj_index {
       uint32_t* rc = buf<uint32_t>(rle_p0, (uint64_t)Wg + 1);
       uint32_t* rl = buf<uint32_t>(rle_lead, (uint64_t)Wg + 1);
       ktime(WJ_KERNEL_RLE_EMIT, [&] {
-        k_rlw_count<<<grid, kRlwThreads, 0, st>>>(key, docs, N, per, rc);
+        if (elem) k_rlw_count<true><<<grid, kRlwThreads, 0, st>>>(key, docs, elem, N, per, rc);
+        else k_rlw_count<false><<<grid, kRlwThreads, 0, st>>>(key, docs, elem, N, per, rc);
         launched();
         scan<uint32_t>(ArrayIn<uint32_t>{rc}, Wg, rc, (uint32_t*)(dscal() + 8));
-        k_rlw_write<<<grid, kRlwThreads, 0, st>>>(key, docs, N, per, rc, od, of, ostride, po, csp, rl);
+        if (elem) k_rlw_write<true><<<grid, kRlwThreads, 0, st>>>(key, docs, elem, N, per, rc, od, of, ostride, po, csp, rl);
+        else k_rlw_write<false><<<grid, kRlwThreads, 0, st>>>(key, docs, elem, N, per, rc, od, of, ostride, po, csp, rl);
         launched();
       });
       k_rle_fixup<<<grid_for(Wg, 256), 256, 0, st>>>(rc, rl, Wg, of, ostride);
@@ -1089,10 +1122,12 @@ struct wj_index {
     // the first chunk into an empty dictionary: every unique term is new and takes termID = its unique
     // index (k_new_terms), so its records (k_chunk_records, record u = unique term u) are indexed by termID
     recs_by_tid = nrec == 0 && V == 0 && !hot;
+    const bool packed = pc_packed;
     uint32_t* kt = (uint32_t*)pc_key.p;
     uint32_t* dt = (uint32_t*)pc_doc.p;
-    uint32_t* k1 = buf<uint32_t>(sk1, Nc + 16);
-    uint32_t* v1 = buf<uint32_t>(sv1, Nc + 16);
+    uint32_t* k1 = packed ? nullptr : buf<uint32_t>(sk1, Nc + 16);
+    uint32_t* v1 = packed ? nullptr : buf<uint32_t>(sv1, Nc + 16);
+    unsigned long long* e1 = packed ? buf<unsigned long long>(sk1, Nc + 16) : nullptr;
     uint2* pp = buf_keep<uint2>(pp_pair, pbase + Nc + 16, pbase);  // P_c <= N_c
     uint64_t* po = buf<uint64_t>(pc_po, C + 1);
     uint64_t* cs = buf<uint64_t>(pc_cs, C + 1);
@@ -1107,10 +1142,18 @@ struct wj_index {
       // holes (hot tokens, key 0) are dropped by the first pass; the count left stays on the device
       // (*ns_dev) and the later passes and the run-length pass are launched for the upper bound Nc
       uint32_t* ns_dev = hot ? (uint32_t*)(dscal() + 13) : nullptr;
-      const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, bits, nullptr, true, nullptr, kRankMask, hot, nullptr,
-                                            true, nullptr, ns_dev);
-      phase(WJ_PHASE_POSTINGS);
-      rle(in1 ? k1 : kt, in1 ? v1 : dt, Nc, false, nullptr, nullptr, po, cs, ns_dev, pp + pbase);
+      if (packed) {  // value-less 64-bit keys, digits from the slot bits (32 ..)
+        unsigned long long* e0 = (unsigned long long*)pc_key.p;
+        const bool in1 = sort_pairs<uint64_t>((uint64_t*)e0, nullptr, (uint64_t*)e1, nullptr, Nc, 32,
+                                              32 + std::max(bits, 1), nullptr, true);
+        phase(WJ_PHASE_POSTINGS);
+        rle(nullptr, nullptr, Nc, false, nullptr, nullptr, po, cs, nullptr, pp + pbase, in1 ? e1 : e0);
+      } else {
+        const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, bits, nullptr, true, nullptr, kRankMask, hot, nullptr,
+                                              true, nullptr, ns_dev);
+        phase(WJ_PHASE_POSTINGS);
+        rle(in1 ? k1 : kt, in1 ? v1 : dt, Nc, false, nullptr, nullptr, po, cs, ns_dev, pp + pbase);
+      }
       if (hot) {  // the hot matrix rows -> the hot terms' partial lists, after the run-length postings
         const uint64_t HD = (uint64_t)hot_H * hot_D;
         uint32_t* hp = buf<uint32_t>(hot_posb, HD + 1);
@@ -1133,6 +1176,9 @@ struct wj_index {
     // the dictionary update (latency-bound small kernels with host round trips) on a high-priority
     // stream, so its CTAs are scheduled ahead of the side stream's whenever SMs free up
     WJ_CUDA_CHECK(cudaStreamWaitEvent(hp_st, ev_fork, 0));
+#ifdef WJ_SERIAL_FORK  // experiment: the dictionary update after the side stream (no overlap)
+    WJ_CUDA_CHECK(cudaStreamWaitEvent(hp_st, ev_side, 0));
+#endif
     std::swap(st, hp_st);
     try {
       dictionary_update(text, U);
@@ -1272,9 +1318,17 @@ struct wj_index {
     uint64_t C = 0, U = 0;
     uint32_t *so = nullptr, *dout = nullptr;
     const bool norm = stem_on || stop_on;
+    emit_elem = nullptr;
+    pc_packed = false;
     const uint64_t Nc = tokenize_dedup(cv, doc_base, [&](uint64_t nc, uint32_t*& sp, uint32_t*& dp) {
       if (pm) {  // the chunk's own stream; the previous chunk's side work is joined on st already
         if (nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 tokens in one chunk"};
+        pc_packed = !norm && hot_H == 0;
+        if (pc_packed) {
+          emit_elem = buf<unsigned long long>(pc_key, nc + 16);
+          sp = dp = nullptr;
+          return;
+        }
         sp = buf<uint32_t>(pc_key, nc + 16);  // +16: TMA round-up reads
         dp = buf<uint32_t>(pc_doc, nc + 16);
         return;
@@ -1283,6 +1337,7 @@ struct wj_index {
       sp = buf_keep<uint32_t>(g_tid, n_elems + nc + 16, n_elems) + n_elems;  // +16: TMA round-up reads
       dp = buf_keep<uint32_t>(g_doc, n_elems + nc + 16, n_elems) + n_elems;
     }, C, U, so, dout, pm && !norm);
+    emit_elem = nullptr;
     if (Nc > 0 && norm) {  // f4: stems / stop words
       uint64_t U2 = 0;
       const uint8_t* ntext = nullptr;
@@ -1302,7 +1357,9 @@ struct wj_index {
         n_tokens += kept;
       }
     } else if (Nc > 0 && pm) {
+      dict_text_bytes = n_bytes;
       chunk_partials(text, Nc, C, U, hot_H > 0);
+      dict_text_bytes = 0;
       n_elems += Nc;
       n_tokens += Nc;
     } else if (Nc > 0) {
@@ -1761,7 +1818,16 @@ struct wj_index {
     sync();  // exchange buffers are reused by the next chunk
   }
 
+  // the arena size of a deferred first insert (dscal[4], written by its ArenaSizeU scan)
+  void settle_arena() {
+    if (!arena_pending) return;
+    readback(4, 1);
+    arena_used = (uint32_t)h_scal[4];
+    arena_pending = false;
+  }
+
   void insert_new(const uint8_t* text, uint64_t U, uint64_t Nn) {
+    settle_arena();
     uint64_t* kk = buf<uint64_t>(nk_key, Nn + 16);
     uint32_t* kv = buf<uint32_t>(nk_val, Nn + 16);
     uint64_t* kk2 = buf<uint64_t>(nk_key2, Nn + 16);
@@ -1781,10 +1847,17 @@ struct wj_index {
     scan<uint32_t>(ArenaSizeU{(const uint32_t*)u_tid.p, (const uint32_t*)u_len.p, (const uint32_t*)u_bucket.p}, U, ao,
                    (uint32_t*)(dscal() + 4));
     WJ_CUDA_CHECK(cudaMemsetAsync((uint32_t*)(dscal() + 4) + 1, 0, 4, st));
-    readback(4, 1);
-    const uint64_t A = (uint32_t)h_scal[4];
-    if (arena_used + A >= 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "string arena exceeds 4 GiB"};
-    uint8_t* ar = buf_keep<uint8_t>(arena, arena_used + A, arena_used);
+    uint64_t A = 0;
+    uint8_t* ar = nullptr;
+    const bool defer = V == 0 && arena_used == 0 && dict_text_bytes > 0 && dict_text_bytes + U < 0xFFFFFFFFull;
+    if (defer) {  // A <= sum over the unique terms of (1 + length) <= text bytes + U
+      ar = buf_keep<uint8_t>(arena, dict_text_bytes + U, 0);
+    } else {
+      readback(4, 1);
+      A = (uint32_t)h_scal[4];
+      if (arena_used + A >= 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "string arena exceeds 4 GiB"};
+      ar = buf_keep<uint8_t>(arena, arena_used + A, arena_used);
+    }
     const uint64_t Vn = (uint64_t)V + Nn;
     uint32_t* ta = buf_keep<uint32_t>(t_arena, Vn, V);
     uint32_t* tc = buf_keep<uint32_t>(t_cache, Vn, V);
@@ -1803,7 +1876,8 @@ struct wj_index {
                                                  (const uint32_t*)u_bucket.p, (const uint32_t*)u_rank.p,
                                                  (const uint32_t*)u_len.p, ao, arena_used, nt, nb, nr, ni, na);
     launched();
-    arena_used += A;
+    if (defer) arena_pending = true;
+    else arena_used += A;
     // merge into the sorted key order E of every collection
     uint32_t* lo = buf<uint32_t>(nlo, kCollections + 1);
     uint32_t* hi = buf<uint32_t>(nhi, kCollections + 1);
@@ -1946,8 +2020,11 @@ struct wj_index {
       if (timed) ktime(WJ_KERNEL_SORT_HIST, up); else up();
       scan<uint32_t>(ArrayIn<uint32_t>{h1}, (uint64_t)256 * G, h2, h2 + (uint64_t)256 * G);
       auto down = [&] {
-        const size_t sm = ds_smem_bytes<K>();
-        if (holes && masked) k_rs_down2<K, true, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
+        const size_t sm = v0 ? ds_smem_bytes<K>() : ds_smem_bytes<K, true>();
+        if (!v0) {  // value-less keys (the packed stream): no holes, no masked digits
+          if (holes || masked) throw StatusError{WJ_ERR_STATE, "value-less sort with holes / masked digits"};
+          k_rs_down2<K, false, false, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
+        } else if (holes && masked) k_rs_down2<K, true, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
         else if (holes) k_rs_down2<K, true, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
         else if (masked) k_rs_down2<K, false, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
         else k_rs_down2<K, false, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
@@ -2370,6 +2447,8 @@ int index_init(wj_index** out, const wj_config* cfg) {
     WJ_DS_ATTR(uint64_t, true, true); WJ_DS_ATTR(uint32_t, false, false); WJ_DS_ATTR(uint32_t, true, false);
     WJ_DS_ATTR(uint32_t, false, true); WJ_DS_ATTR(uint32_t, true, true);
 #undef WJ_DS_ATTR
+    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rs_down2<uint64_t, false, false, true>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ds_smem_bytes<uint64_t, true>()));
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rle_write_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)rle_smem_bytes()));
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rle_write_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -2545,6 +2624,7 @@ int index_debug_btree(wj_index* ix, void* nodes, uint64_t node_cap, uint64_t* n_
   if (!ix || !n_nodes || !arena_bytes) return WJ_ERR_INVALID_ARG;
   return guarded(ix, [&]() {
     ix->ensure_btrees();
+    ix->settle_arena();
     ix->sync();
     *n_nodes = ix->n_nodes;
     *arena_bytes = ix->arena_used;

@@ -350,25 +350,56 @@ __host__ __device__ __forceinline__ uint64_t rlw_per(uint64_t N, uint64_t W) {
   return (per + kRlwStep - 1) / kRlwStep * kRlwStep;
 }
 
-// the lane's 16 elements of the step at i0 (past hi: key 0, doc ~0) and the element before them
-__device__ __forceinline__ void rlw_load(const uint32_t* key, const uint32_t* doc, uint64_t i0, uint64_t hi,
-                                         uint32_t (&k)[kRlwItems], uint32_t (&d)[kRlwItems]) {
+// the lane's 16 elements of the step at i0 (past hi: key 0, doc ~0) and the element before them.
+// PACKED: the stream is one u64 array (slot << 32 | docID, the emit kernel's packed output); else
+// key[] / doc[] (SoA).
+template <bool PACKED>
+__device__ __forceinline__ void rlw_load(const uint32_t* key, const uint32_t* doc, const unsigned long long* elem,
+                                         uint64_t i0, uint64_t hi, uint32_t (&k)[kRlwItems], uint32_t (&d)[kRlwItems]) {
   const uint64_t b = i0 + (uint64_t)kRlwItems * lane_id();
   if (b + kRlwItems <= hi) {
+    if (PACKED) {
 #pragma unroll
-    for (int q = 0; q < kRlwItems / 4; ++q) {
-      const uint4 x = __ldcs((const uint4*)(key + b) + q);
-      const uint4 y = __ldcs((const uint4*)(doc + b) + q);
-      k[4 * q] = x.x; k[4 * q + 1] = x.y; k[4 * q + 2] = x.z; k[4 * q + 3] = x.w;
-      d[4 * q] = y.x; d[4 * q + 1] = y.y; d[4 * q + 2] = y.z; d[4 * q + 3] = y.w;
+      for (int q = 0; q < kRlwItems / 2; ++q) {
+        const uint4 x = __ldcs((const uint4*)(elem + b) + q);
+        d[2 * q] = x.x; k[2 * q] = x.y; d[2 * q + 1] = x.z; k[2 * q + 1] = x.w;
+      }
+    } else {
+#pragma unroll
+      for (int q = 0; q < kRlwItems / 4; ++q) {
+        const uint4 x = __ldcs((const uint4*)(key + b) + q);
+        const uint4 y = __ldcs((const uint4*)(doc + b) + q);
+        k[4 * q] = x.x; k[4 * q + 1] = x.y; k[4 * q + 2] = x.z; k[4 * q + 3] = x.w;
+        d[4 * q] = y.x; d[4 * q + 1] = y.y; d[4 * q + 2] = y.z; d[4 * q + 3] = y.w;
+      }
     }
   } else {
 #pragma unroll
     for (int j = 0; j < kRlwItems; ++j) {
       const bool v = b + j < hi;
-      k[j] = v ? key[b + j] : 0u;
-      d[j] = v ? doc[b + j] : 0xFFFFFFFFu;
+      if (PACKED) {
+        const unsigned long long e = v ? elem[b + j] : 0xFFFFFFFFull;
+        k[j] = (uint32_t)(e >> 32);
+        d[j] = (uint32_t)e;
+      } else {
+        k[j] = v ? key[b + j] : 0u;
+        d[j] = v ? doc[b + j] : 0xFFFFFFFFu;
+      }
     }
+  }
+}
+
+// (key, doc) of element i
+template <bool PACKED>
+__device__ __forceinline__ void rlw_at(const uint32_t* key, const uint32_t* doc, const unsigned long long* elem, uint64_t i,
+                                       uint32_t& k, uint32_t& d) {
+  if (PACKED) {
+    const unsigned long long e = elem[i];
+    k = (uint32_t)(e >> 32);
+    d = (uint32_t)e;
+  } else {
+    k = key[i];
+    d = doc[i];
   }
 }
 
@@ -398,18 +429,21 @@ __device__ __forceinline__ void rlw_flags(const uint32_t (&k)[kRlwItems], const 
   }
 }
 
+template <bool PACKED>
 __global__ void __launch_bounds__(kRlwThreads) k_rlw_count(const uint32_t* __restrict__ key,
-                                                           const uint32_t* __restrict__ doc, uint64_t N, uint64_t per,
-                                                           uint32_t* wcnt) {
+                                                           const uint32_t* __restrict__ doc,
+                                                           const unsigned long long* __restrict__ elem, uint64_t N,
+                                                           uint64_t per, uint32_t* wcnt) {
   const uint32_t gw = blockIdx.x * kRlwWarps + (threadIdx.x >> 5);
   const uint64_t lo = (uint64_t)gw * per;
   const uint64_t hi = lo + per < N ? lo + per : N;
   uint32_t c = 0;
   if (lo < hi) {
-    uint32_t pk = lo > 0 ? key[lo - 1] : 0xFFFFFFFFu, pd = lo > 0 ? doc[lo - 1] : 0xFFFFFFFFu;
+    uint32_t pk = 0xFFFFFFFFu, pd = 0xFFFFFFFFu;
+    if (lo > 0) rlw_at<PACKED>(key, doc, elem, lo - 1, pk, pd);
     for (uint64_t i0 = lo; i0 < hi; i0 += kRlwStep) {
       uint32_t k[kRlwItems], d[kRlwItems], npm, ntm;
-      rlw_load(key, doc, i0, hi, k, d);
+      rlw_load<PACKED>(key, doc, elem, i0, hi, k, d);
       const uint32_t nvalid = (uint32_t)min((uint64_t)kRlwStep, hi - i0);
       rlw_flags(k, d, pk, pd, nvalid, npm, ntm);
       c += __popc(npm);
@@ -425,8 +459,11 @@ __global__ void __launch_bounds__(kRlwThreads) k_rlw_count(const uint32_t* __res
 // woff: exclusive posting offset of each warp range (scan of k_rlw_count); writes (docID, tf) at
 // out_doc / out_tf [ostride * posting] (ostride 2: interleaved pairs), post_off / cstart at each term's
 // key, range_lead[gw] = elements of the range before its first head
+template <bool PACKED>
 __global__ void __launch_bounds__(kRlwThreads, 3) k_rlw_write(const uint32_t* __restrict__ key,
-                                                              const uint32_t* __restrict__ doc, uint64_t N, uint64_t per,
+                                                              const uint32_t* __restrict__ doc,
+                                                              const unsigned long long* __restrict__ elem, uint64_t N,
+                                                              uint64_t per,
                                                               const uint32_t* __restrict__ woff, uint32_t* out_doc,
                                                               uint32_t* out_tf, uint32_t ostride, uint64_t* post_off,
                                                               uint64_t* cstart, uint32_t* range_lead) {
@@ -441,14 +478,15 @@ __global__ void __launch_bounds__(kRlwThreads, 3) k_rlw_write(const uint32_t* __
     return;
   }
   uint2* sg = stage[w];
-  uint32_t pk = lo > 0 ? key[lo - 1] : 0xFFFFFFFFu, pd = lo > 0 ? doc[lo - 1] : 0xFFFFFFFFu;
+  uint32_t pk = 0xFFFFFFFFu, pd = 0xFFFFFFFFu;
+  if (lo > 0) rlw_at<PACKED>(key, doc, elem, lo - 1, pk, pd);
   uint32_t p = woff[gw];
   uint32_t lead = 0, open_len = 0, open_p = 0;
   bool lead_done = false, have_open = false;
   const uint32_t lt = (1u << lane) - 1u;
   for (uint64_t i0 = lo; i0 < hi; i0 += kRlwStep) {
     uint32_t k[kRlwItems], d[kRlwItems], npm, ntm;
-    rlw_load(key, doc, i0, hi, k, d);
+    rlw_load<PACKED>(key, doc, elem, i0, hi, k, d);
     const uint32_t nvalid = (uint32_t)min((uint64_t)kRlwStep, hi - i0);
     rlw_flags(k, d, pk, pd, nvalid, npm, ntm);
     const uint32_t c = __popc(npm);

@@ -185,10 +185,12 @@ constexpr int kDsWarps = kDsThreads / 32;
 constexpr int kDsItems = 8;
 static_assert(kDsThreads * kDsItems == kOsTile, "tile");
 
-template <typename K>
-inline size_t ds_smem_bytes() { return 2 * (size_t)kOsTile * (sizeof(K) + sizeof(uint32_t)) + kOsTile * 2; }
+template <typename K, bool NOVAL = false>
+inline size_t ds_smem_bytes() { return 2 * (size_t)kOsTile * (sizeof(K) + (NOVAL ? 0 : sizeof(uint32_t))) + kOsTile * 2; }
 
-template <typename K, bool HOLES, bool MASK>
+// NOVAL: keys only (the packed stream: u64 slot << 32 | docID, digits from the slot bits), one TMA load,
+// one shared-memory gather and one 8-byte store per element instead of two of each
+template <typename K, bool HOLES, bool MASK, bool NOVAL = false>
 // 64 registers (__launch_bounds__(512, 2)): with the lazy B-tree re-layout the dictionary stream
 // no longer needs room beside the persistent downsweep; the earlier 48-register cap
 // (WJ_DS_MAXREG=48) is 2.93 -> 3.09 ms for the three passes, step 8.98 vs 9.00-9.02 ms (A/B x2)
@@ -211,13 +213,14 @@ __global__ void WJ_DS_BOUNDS k_rs_down2(const K* __restrict__ kin, const uint32_
   extern __shared__ __align__(128) unsigned char os_smem[];
   __shared__ __align__(8) uint64_t bar[2];
   __shared__ uint32_t wcnt[kDsWarps][256];
-  __shared__ uint32_t wbins[kDsWarps][256];
+  constexpr bool kSmemPeers = sizeof(K) == 8 && !NOVAL;  // 64-bit (all distinct) keys: shared-memory masks
+  __shared__ uint32_t wbins[kSmemPeers ? kDsWarps : 1][256];
   __shared__ uint32_t dig_off[256];
   __shared__ uint32_t dig_glob[256];
   __shared__ uint32_t run_base[256];
   __shared__ uint32_t wtot[8];
   __shared__ uint32_t s_tvalid;
-  const size_t stage_bytes = (size_t)kOsTile * (sizeof(K) + sizeof(uint32_t));
+  const size_t stage_bytes = (size_t)kOsTile * (sizeof(K) + (NOVAL ? 0 : sizeof(uint32_t)));
   auto skey = [&](int s) { return (K*)(os_smem + s * stage_bytes); };
   auto sval = [&](int s) { return (uint32_t*)(os_smem + s * stage_bytes + (size_t)kOsTile * sizeof(K)); };
   uint16_t* inv = (uint16_t*)(os_smem + 2 * stage_bytes);
@@ -233,9 +236,9 @@ __global__ void WJ_DS_BOUNDS k_rs_down2(const K* __restrict__ kin, const uint32_
     const uint32_t bk = (uint32_t)((cnt * sizeof(K) + 15) & ~(size_t)15);
     const uint32_t bv = (cnt * 4 + 15) & ~15u;
     fence_proxy_async_smem();
-    mbar_arrive_expect_tx(&bar[s], bk + bv);
+    mbar_arrive_expect_tx(&bar[s], bk + (NOVAL ? 0u : bv));
     tma_load_1d(skey(s), kin + base, bk, &bar[s]);
-    tma_load_1d(sval(s), vin + base, bv, &bar[s]);
+    if (!NOVAL) tma_load_1d(sval(s), vin + base, bv, &bar[s]);
   };
 
   if (threadIdx.x == 0) {
@@ -243,7 +246,10 @@ __global__ void WJ_DS_BOUNDS k_rs_down2(const K* __restrict__ kin, const uint32_
     mbar_init(&bar[1], 1);
     fence_mbar_init();
   }
-  for (int i = threadIdx.x; i < kDsWarps * 256; i += kDsThreads) (&wcnt[0][0])[i] = (&wbins[0][0])[i] = 0;
+  for (int i = threadIdx.x; i < kDsWarps * 256; i += kDsThreads) {
+    (&wcnt[0][0])[i] = 0;
+    if (kSmemPeers) (&wbins[0][0])[i] = 0;
+  }
   if (threadIdx.x < 256) run_base[threadIdx.x] = offs[(uint64_t)threadIdx.x * gridDim.x + blockIdx.x];
   __syncthreads();
   if (threadIdx.x == 0) issue(0, lo);
@@ -268,7 +274,7 @@ __global__ void WJ_DS_BOUNDS k_rs_down2(const K* __restrict__ kin, const uint32_
       // 64-bit keys (all distinct: new-term sort): shared-memory masks; 32-bit keys (Zipf-skewed
       // ranks, many equal digits per warp -> atomic conflicts): ballots
       // (shared-memory masks for the 32-bit stream keys too: 3.31 vs 3.09 ms for the three passes)
-      rank[k] = sizeof(K) == 8 ? digit_peers_smem(wbins[w], dg[k], valid) : digit_peers(dg[k], valid);
+      rank[k] = kSmemPeers ? digit_peers_smem(wbins[kSmemPeers ? w : 0], dg[k], valid) : digit_peers(dg[k], valid);
     }
 #pragma unroll
     for (int k = 0; k < kDsItems; ++k) {
@@ -323,7 +329,7 @@ __global__ void WJ_DS_BOUNDS k_rs_down2(const K* __restrict__ kin, const uint32_
       const K kk = sk[li];
       const uint32_t pos = dig_glob[(uint32_t)((rs_dkey<K, MASK>(kk, kmask) >> shift) & 255u)] + j;
       kout[pos] = kk;
-      vout[pos] = sv[li];
+      if (!NOVAL) vout[pos] = sv[li];
     }
     for (int i = threadIdx.x; i < kDsWarps * 256; i += kDsThreads) (&wcnt[0][0])[i] = 0;
     __syncthreads();

@@ -53,6 +53,7 @@ struct EmitOut {
   uint32_t doc_base;       // global DocID of local document 0
   uint32_t* slot;          // per kept token: slot | 1 << 25 (key 0 = hole: a hot token, HOT only)
   uint32_t* doc;           // per kept token: global DocID
+  unsigned long long* elem;  // or (packed stream, no HOT): per kept token slot << 32 | global DocID
   uint32_t* dbg_start;     // optional (debug): token start
   uint32_t* dbg_len;       // optional (debug): token length
   uint32_t* overflow;      // set to 1 if a probe sequence exceeded the limit
@@ -519,8 +520,12 @@ __global__ void __launch_bounds__(kTokThreads, HOT ? WJ_EMIT_HOT_MINB : WJ_EMIT_
           else atomicAdd(&eo.hot_mat[(uint64_t)hh * eo.hot_docs + ldoc], 1u);
         }
         // branch-free stores: stream element slot | count 1 << 25, or a hole (the docID is not read)
-        __stcs(eo.slot + out, (HOT && hid) ? 0u : (slot | (1u << 25)));
-        __stcs(eo.doc + out, eo.doc_base + ldoc);
+        if (!HOT && eo.elem) {  // one 8-byte store: the sort moves (slot, docID) as one u64 key
+          __stcs(eo.elem + out, ((unsigned long long)slot << 32) | (eo.doc_base + ldoc));
+        } else {
+          __stcs(eo.slot + out, (HOT && hid) ? 0u : (slot | (1u << 25)));
+          __stcs(eo.doc + out, eo.doc_base + ldoc);
+        }
         if (eo.dbg_start) { eo.dbg_start[out] = s_abs; eo.dbg_len[out] = len; }
       }
       if (HOT && hkey != 0xFFFFFFFFu) atomicAdd(&hc[hkey], 1u);  // (a warp match first was slower)
