@@ -257,10 +257,7 @@ struct wj_index {
       cf_totb;
   uint64_t pbase = 0, nrec = 0;      // partial postings / records of the chunks so far
   uint32_t rs_ctas = kRsCtas;        // radix downsweep CTAs (ranges) of sort_pairs
-#ifndef WJ_SIDE_CTAS
-#define WJ_SIDE_CTAS kRsCtas
-#endif
-  uint32_t side_ctas = WJ_SIDE_CTAS;  // ... for the side stream's sort (148 / 222 measured slower)
+  uint32_t side_ctas = kRsCtas;      // ... for the side stream's sort (148 / 222 / 592 / 1184 measured slower)
   bool pc_pending = false;           // the last chunk's posting count is still on the device (dscal[13])
   bool pc_join = false;              // the last chunk's side-stream work is not joined yet
   uint64_t pc_U = 0, pc_Nc = 0;  // pc_Nc: tokens of the pending chunk
@@ -1037,9 +1034,18 @@ struct wj_index {
   // term's key (key & kRankMask); the posting count is left in dscal[8] (u32, no host round trip)
   // n_dev (optional): the actual element count on the device, N being an upper bound
   // pairs != nullptr: the postings go there as interleaved (docID, tf) pairs (per-run partial lists)
+  // geometry of the plain-stream run-length pass (k_rlw_*): warp ranges of `per` elements, Wg warps
+  void rlw_geometry(uint64_t N, uint64_t& per, uint32_t& grid, uint32_t& Wg) const {
+    const uint64_t W = 148ull * 3 * kRlwWarps;  // one wave at 3 CTAs per SM
+    per = rlw_per(N, W);
+    const uint32_t Wn = (uint32_t)((N + per - 1) / per);
+    grid = (Wn + kRlwWarps - 1) / kRlwWarps;
+    Wg = grid * kRlwWarps;  // warps launched (ranges past N count 0)
+  }
+  // precounted: rle_p0 already holds each warp range's posting count (the last radix pass counted them)
   void rle(const uint32_t* key, const uint32_t* docs, uint64_t N, bool counts, uint32_t* od, uint32_t* of, uint64_t* po,
            uint64_t* csp, const uint32_t* n_dev = nullptr, uint2* pairs = nullptr,
-           const unsigned long long* elem = nullptr) {
+           const unsigned long long* elem = nullptr, bool precounted = false) {
     const uint32_t ostride = pairs ? 2u : 1u;
     if (pairs) {
       od = (uint32_t*)pairs;
@@ -1051,20 +1057,17 @@ struct wj_index {
     }
     if (elem && (counts || n_dev)) throw StatusError{WJ_ERR_STATE, "packed stream with counts"};
     if (!counts && !n_dev) {  // plain stream: one warp per range (k_rlw_*)
-#ifndef WJ_RLW_WAVES
-#define WJ_RLW_WAVES 1
-#endif
-      const uint64_t W = 148ull * 3 * kRlwWarps * WJ_RLW_WAVES;  // one wave at 3 CTAs per SM
-      const uint64_t per = rlw_per(N, W);
-      const uint32_t Wn = (uint32_t)((N + per - 1) / per);
-      const unsigned grid = (Wn + kRlwWarps - 1) / kRlwWarps;
-      const uint32_t Wg = grid * kRlwWarps;  // warps launched (ranges past N count 0)
+      uint64_t per;
+      uint32_t grid, Wg;
+      rlw_geometry(N, per, grid, Wg);
       uint32_t* rc = buf<uint32_t>(rle_p0, (uint64_t)Wg + 1);
       uint32_t* rl = buf<uint32_t>(rle_lead, (uint64_t)Wg + 1);
       ktime(WJ_KERNEL_RLE_EMIT, [&] {
-        if (elem) k_rlw_count<true><<<grid, kRlwThreads, 0, st>>>(key, docs, elem, N, per, rc);
-        else k_rlw_count<false><<<grid, kRlwThreads, 0, st>>>(key, docs, elem, N, per, rc);
-        launched();
+        if (!precounted) {
+          if (elem) k_rlw_count<true><<<grid, kRlwThreads, 0, st>>>(key, docs, elem, N, per, rc);
+          else k_rlw_count<false><<<grid, kRlwThreads, 0, st>>>(key, docs, elem, N, per, rc);
+          launched();
+        }
         scan<uint32_t>(ArrayIn<uint32_t>{rc}, Wg, rc, (uint32_t*)(dscal() + 8));
         if (elem) k_rlw_write<true><<<grid, kRlwThreads, 0, st>>>(key, docs, elem, N, per, rc, od, of, ostride, po, csp, rl);
         else k_rlw_write<false><<<grid, kRlwThreads, 0, st>>>(key, docs, elem, N, per, rc, od, of, ostride, po, csp, rl);
@@ -1144,10 +1147,17 @@ struct wj_index {
       uint32_t* ns_dev = hot ? (uint32_t*)(dscal() + 13) : nullptr;
       if (packed) {  // value-less 64-bit keys, digits from the slot bits (32 ..)
         unsigned long long* e0 = (unsigned long long*)pc_key.p;
+        // the last radix pass counts the run-length heads per warp range of the run-length pass
+        uint64_t rper;
+        uint32_t rgrid, Wg;
+        rlw_geometry(Nc, rper, rgrid, Wg);
+        uint32_t* rc = buf<uint32_t>(rle_p0, (uint64_t)Wg + 1);
+        WJ_CUDA_CHECK(cudaMemsetAsync(rc, 0, ((size_t)Wg + 1) * 4, st));
         const bool in1 = sort_pairs<uint64_t>((uint64_t*)e0, nullptr, (uint64_t*)e1, nullptr, Nc, 32,
-                                              32 + std::max(bits, 1), nullptr, true);
+                                              32 + std::max(bits, 1), nullptr, true, nullptr, ~0ull, false, nullptr,
+                                              true, nullptr, nullptr, rc, (uint32_t)rper);
         phase(WJ_PHASE_POSTINGS);
-        rle(nullptr, nullptr, Nc, false, nullptr, nullptr, po, cs, nullptr, pp + pbase, in1 ? e1 : e0);
+        rle(nullptr, nullptr, Nc, false, nullptr, nullptr, po, cs, nullptr, pp + pbase, in1 ? e1 : e0, true);
       } else {
         const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, bits, nullptr, true, nullptr, kRankMask, hot, nullptr,
                                               true, nullptr, ns_dev);
@@ -1176,9 +1186,6 @@ struct wj_index {
     // the dictionary update (latency-bound small kernels with host round trips) on a high-priority
     // stream, so its CTAs are scheduled ahead of the side stream's whenever SMs free up
     WJ_CUDA_CHECK(cudaStreamWaitEvent(hp_st, ev_fork, 0));
-#ifdef WJ_SERIAL_FORK  // experiment: the dictionary update after the side stream (no overlap)
-    WJ_CUDA_CHECK(cudaStreamWaitEvent(hp_st, ev_side, 0));
-#endif
     std::swap(st, hp_st);
     try {
       dictionary_update(text, U);
@@ -1960,7 +1967,8 @@ struct wj_index {
                   const uint32_t* rank_of, bool timed,
                   const std::vector<std::pair<uint64_t, const uint32_t*>>* segs = nullptr, K kmask = ~K(0),
                   bool skip0 = false, uint64_t* n_out = nullptr, bool mask_digits = true,
-                  std::vector<uint64_t>* digit_start = nullptr, uint32_t* holes_n_dev = nullptr) {
+                  std::vector<uint64_t>* digit_start = nullptr, uint32_t* holes_n_dev = nullptr,
+                  uint32_t* head_cnt = nullptr, uint32_t head_per = 0) {
     if (n_out) *n_out = n;
     if (n == 0) return false;
     int passes = end_bit > begin_bit ? (end_bit - begin_bit + 7) / 8 : 0;
@@ -1980,6 +1988,11 @@ struct wj_index {
       }
     }
     if (passes == 0 || (n == 1 && !skip0)) {
+      if (head_cnt) {  // no pass counts the run-length heads: a single element is one head
+        if (n > 1) throw StatusError{WJ_ERR_STATE, "head counting needs a radix pass (internal)"};
+        k_fill<uint32_t><<<1, 32, 0, st>>>(head_cnt, 1, 1u);
+        launched();
+      }
       if (segs && !multi_map) {
         k_map_rank<<<grid_for(n, 256), 256, 0, st>>>((uint32_t*)k0, n, (*segs)[0].second);
         launched();
@@ -2023,7 +2036,14 @@ struct wj_index {
         const size_t sm = v0 ? ds_smem_bytes<K>() : ds_smem_bytes<K, true>();
         if (!v0) {  // value-less keys (the packed stream): no holes, no masked digits
           if (holes || masked) throw StatusError{WJ_ERR_STATE, "value-less sort with holes / masked digits"};
-          k_rs_down2<K, false, false, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
+          if (head_cnt && p == passes - 1) {  // the last pass also counts the run-length heads
+            k_rs_down2<K, false, false, true, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask,
+                                                                              n_dev, head_cnt, head_per);
+            k_head_fix<K><<<grid_for((uint64_t)256 * G, 256), 256, 0, st>>>(ko, h2, 256 * G, head_cnt, head_per);
+            launched();
+          } else {
+            k_rs_down2<K, false, false, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
+          }
         } else if (holes && masked) k_rs_down2<K, true, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
         else if (holes) k_rs_down2<K, true, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
         else if (masked) k_rs_down2<K, false, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
@@ -2447,6 +2467,8 @@ int index_init(wj_index** out, const wj_config* cfg) {
     WJ_DS_ATTR(uint64_t, true, true); WJ_DS_ATTR(uint32_t, false, false); WJ_DS_ATTR(uint32_t, true, false);
     WJ_DS_ATTR(uint32_t, false, true); WJ_DS_ATTR(uint32_t, true, true);
 #undef WJ_DS_ATTR
+    WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rs_down2<uint64_t, false, false, true, true>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ds_smem_bytes<uint64_t, true>()));
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rs_down2<uint64_t, false, false, true>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ds_smem_bytes<uint64_t, true>()));
     WJ_CUDA_CHECK(cudaFuncSetAttribute(k_rle_write_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,

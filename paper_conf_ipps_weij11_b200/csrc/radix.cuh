@@ -190,7 +190,12 @@ inline size_t ds_smem_bytes() { return 2 * (size_t)kOsTile * (sizeof(K) + (NOVAL
 
 // NOVAL: keys only (the packed stream: u64 slot << 32 | docID, digits from the slot bits), one TMA load,
 // one shared-memory gather and one 8-byte store per element instead of two of each
-template <typename K, bool HOLES, bool MASK, bool NOVAL = false>
+// HEADS (the last pass over a packed stream, NOVAL): also counts run-length heads -- elements whose
+// (slot, docID) differs from the previous one in the final order -- per run-length range of rper elements
+// into rcnt (zeroed by the caller), which replaces the run-length count pass.  The predecessor is the
+// previous lane's element (a shuffle), the previous warp's last one, or the digit's last element of an
+// earlier tile (carry); a block's first element is counted as a head and k_head_fix corrects it.
+template <typename K, bool HOLES, bool MASK, bool NOVAL = false, bool HEADS = false>
 // 64 registers (__launch_bounds__(512, 2)): with the lazy B-tree re-layout the dictionary stream
 // no longer needs room beside the persistent downsweep; the earlier 48-register cap
 // (WJ_DS_MAXREG=48) is 2.93 -> 3.09 ms for the three passes, step 8.98 vs 9.00-9.02 ms (A/B x2)
@@ -205,7 +210,8 @@ template <typename K, bool HOLES, bool MASK, bool NOVAL = false>
 __global__ void WJ_DS_BOUNDS k_rs_down2(const K* __restrict__ kin, const uint32_t* __restrict__ vin,
                                                          K* __restrict__ kout, uint32_t* __restrict__ vout, uint64_t n,
                                                          uint64_t per, int shift, const uint32_t* __restrict__ offs,
-                                                         K kmask, const uint32_t* __restrict__ n_dev) {
+                                                         K kmask, const uint32_t* __restrict__ n_dev,
+                                                         uint32_t* __restrict__ rcnt = nullptr, uint32_t rper = 0) {
   if (n_dev) {
     n = min(n, (uint64_t)*n_dev);
     per = rs_per(n, gridDim.x);
@@ -220,6 +226,9 @@ __global__ void WJ_DS_BOUNDS k_rs_down2(const K* __restrict__ kin, const uint32_
   __shared__ uint32_t run_base[256];
   __shared__ uint32_t wtot[8];
   __shared__ uint32_t s_tvalid;
+  __shared__ __align__(8) K carry[HEADS ? 2 : 1][HEADS ? 256 : 1];  // per digit: last element of an earlier tile
+  const uint32_t rmagic = HEADS ? (uint32_t)(0xFFFFFFFFull / rper + 1) : 0u;  // q = umulhi(pos, m), -1 fix
+  uint32_t tile_par = 0;
   const size_t stage_bytes = (size_t)kOsTile * (sizeof(K) + (NOVAL ? 0 : sizeof(uint32_t)));
   auto skey = [&](int s) { return (K*)(os_smem + s * stage_bytes); };
   auto sval = [&](int s) { return (uint32_t*)(os_smem + s * stage_bytes + (size_t)kOsTile * sizeof(K)); };
@@ -251,6 +260,7 @@ __global__ void WJ_DS_BOUNDS k_rs_down2(const K* __restrict__ kin, const uint32_
     if (kSmemPeers) (&wbins[0][0])[i] = 0;
   }
   if (threadIdx.x < 256) run_base[threadIdx.x] = offs[(uint64_t)threadIdx.x * gridDim.x + blockIdx.x];
+  if (HEADS && threadIdx.x < 256) carry[0][threadIdx.x] = carry[HEADS ? 1 : 0][threadIdx.x] = ~K(0);  // none
   __syncthreads();
   if (threadIdx.x == 0) issue(0, lo);
   uint32_t parity = 0u;
@@ -324,17 +334,63 @@ __global__ void WJ_DS_BOUNDS k_rs_down2(const K* __restrict__ kin, const uint32_
     }
     __syncthreads();
     const uint32_t tvalid = HOLES ? s_tvalid : tn;  // valid (non-hole) items of the tile
-    for (uint32_t j = threadIdx.x; j < tvalid; j += kDsThreads) {
-      const uint32_t li = inv[j];
-      const K kk = sk[li];
-      const uint32_t pos = dig_glob[(uint32_t)((rs_dkey<K, MASK>(kk, kmask) >> shift) & 255u)] + j;
-      kout[pos] = kk;
-      if (!NOVAL) vout[pos] = sv[li];
+    if (HEADS) {
+      const K* cprev = carry[(tile_par ^ 1) & (HEADS ? 1u : 0u)];
+      for (uint32_t j0 = 0; j0 < kOsTile; j0 += kDsThreads) {
+        const uint32_t j = j0 + threadIdx.x;
+        const bool valid = j < tvalid;
+        const K kk = valid ? sk[inv[j]] : ~K(0);
+        const uint32_t d = (uint32_t)(kk >> shift) & 255u;
+        const uint32_t pos = dig_glob[d] + j;
+        if (valid) kout[pos] = kk;
+        K pk = (K)__shfl_up_sync(0xffffffffu, (unsigned long long)kk, 1);
+        if (lane == 0) pk = (valid && j > 0) ? sk[inv[j - 1]] : ~K(0);  // (inv past tvalid is stale)
+        // the previous element of the final order: in this tile's run of digit d, else the carry
+        const K pred = (j > 0 && ((uint32_t)(pk >> shift) & 255u) == d) ? pk : cprev[d];
+        const bool head = valid && pred != kk;
+        uint32_t q = valid ? __umulhi(pos, rmagic) : 0xFFFFFFFFu;
+        if (valid && (uint64_t)q * rper > pos) --q;
+        const uint32_t qp = __shfl_up_sync(0xffffffffu, q, 1);
+        const bool leader = valid && (lane == 0 || qp != q);
+        const uint32_t lm = __ballot_sync(0xffffffffu, leader), hm = __ballot_sync(0xffffffffu, head);
+        if (leader) {
+          const uint32_t later = lm & ~((2u << lane) - 1u);
+          const uint32_t seg = (later ? (1u << (__ffs(later) - 1)) - 1u : 0xFFFFFFFFu) & ~((1u << lane) - 1u);
+          const uint32_t hc = __popc(hm & seg);
+          if (hc) atomicAdd(&rcnt[q], hc);
+        }
+      }
+    } else {
+      for (uint32_t j = threadIdx.x; j < tvalid; j += kDsThreads) {
+        const uint32_t li = inv[j];
+        const K kk = sk[li];
+        const uint32_t pos = dig_glob[(uint32_t)((rs_dkey<K, MASK>(kk, kmask) >> shift) & 255u)] + j;
+        kout[pos] = kk;
+        if (!NOVAL) vout[pos] = sv[li];
+      }
     }
+    if (HEADS && threadIdx.x < 256) {  // this tile's last element of each digit (or the earlier carry)
+      K* cur = carry[tile_par & (HEADS ? 1u : 0u)];
+      const K* prv = carry[(tile_par ^ 1) & (HEADS ? 1u : 0u)];
+      cur[threadIdx.x] = cnt ? sk[inv[dig_off[threadIdx.x] + cnt - 1]] : prv[threadIdx.x];
+    }
+    tile_par ^= 1u;
     for (int i = threadIdx.x; i < kDsWarps * 256; i += kDsThreads) (&wcnt[0][0])[i] = 0;
     __syncthreads();
     s ^= 1;
   }
+}
+
+// HEADS correction: a non-empty block (d, c) of the last pass starts at offs[d][c]; its first element was
+// counted as a head without seeing its predecessor out[pos - 1]
+template <typename K>
+__global__ void k_head_fix(const K* __restrict__ out, const uint32_t* __restrict__ offs, uint32_t blocks,
+                           uint32_t* rcnt, uint32_t rper) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= blocks) return;
+  const uint32_t p = offs[i];
+  if (offs[i + 1] == p || p == 0) return;
+  if (out[p - 1] == out[p]) atomicSub(&rcnt[p / rper], 1u);
 }
 
 }  // namespace wj
