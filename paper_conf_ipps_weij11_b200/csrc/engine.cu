@@ -253,6 +253,7 @@ struct wj_index {
   cudaEvent_t ev_fork = nullptr, ev_side = nullptr, ev_dict = nullptr;
   DevBuf side_scan, side_hist, side_hist_scan;
   DevBuf mr_key, mr_idx, mr_key2, mr_idx2, mr_dst, mr_src;  // several runs: records in destination order
+  DevBuf pc_dig;  // packed stream: one digit byte per element for the next radix pass's upsweep
   DevBuf pc_key, pc_doc, pc_po, pc_cs, u_slot, pp_pair, x_pair, rec_tid, rec_start, rec_df, rec_cf, rec_aos, rec_before, df_totb,
       cf_totb;
   uint64_t pbase = 0, nrec = 0;      // partial postings / records of the chunks so far
@@ -376,7 +377,7 @@ struct wj_index {
                      &table_s, &uid_s, &st_off, &st_text, &st_keep, &st_tidx, &st_m1, &st_slot, &st_doc, &st_tiles,
                      &st_doff, &stop_keys, &side_scan, &side_hist, &side_hist_scan, &pc_key, &pc_doc, &pc_po,
                      &pc_cs, &u_slot, &pp_pair, &x_pair, &mr_key, &mr_idx, &mr_key2, &mr_idx2, &mr_dst, &mr_src, &rec_tid, &rec_start, &rec_df, &rec_cf, &rec_aos, &rec_before, &df_totb,
-                     &cf_totb};
+                     &cf_totb, &pc_dig};
     for (DevBuf* b : all) {
       dev_free(b->p);
       b->p = nullptr;
@@ -603,6 +604,7 @@ struct wj_index {
     eo.slot = slot_out;
     eo.doc = doc_out;
     eo.elem = use_hot ? nullptr : emit_elem;
+    eo.dig0 = eo.elem ? (uint8_t*)pc_dig.p : nullptr;
     eo.dbg_start = dstart;
     eo.dbg_len = dlen;
     eo.overflow = (uint32_t*)(dscal() + 5);
@@ -1155,7 +1157,7 @@ struct wj_index {
         WJ_CUDA_CHECK(cudaMemsetAsync(rc, 0, ((size_t)Wg + 1) * 4, st));
         const bool in1 = sort_pairs<uint64_t>((uint64_t*)e0, nullptr, (uint64_t*)e1, nullptr, Nc, 32,
                                               32 + std::max(bits, 1), nullptr, true, nullptr, ~0ull, false, nullptr,
-                                              true, nullptr, nullptr, rc, (uint32_t)rper);
+                                              true, nullptr, nullptr, rc, (uint32_t)rper, (uint8_t*)pc_dig.p);
         phase(WJ_PHASE_POSTINGS);
         rle(nullptr, nullptr, Nc, false, nullptr, nullptr, po, cs, nullptr, pp + pbase, in1 ? e1 : e0, true);
       } else {
@@ -1333,6 +1335,7 @@ struct wj_index {
         pc_packed = !norm && hot_H == 0;
         if (pc_packed) {
           emit_elem = buf<unsigned long long>(pc_key, nc + 16);
+          buf<uint8_t>(pc_dig, nc + 64);  // digit bytes of the radix passes (k_rs_up_bytes)
           sp = dp = nullptr;
           return;
         }
@@ -1968,7 +1971,7 @@ struct wj_index {
                   const std::vector<std::pair<uint64_t, const uint32_t*>>* segs = nullptr, K kmask = ~K(0),
                   bool skip0 = false, uint64_t* n_out = nullptr, bool mask_digits = true,
                   std::vector<uint64_t>* digit_start = nullptr, uint32_t* holes_n_dev = nullptr,
-                  uint32_t* head_cnt = nullptr, uint32_t head_per = 0) {
+                  uint32_t* head_cnt = nullptr, uint32_t head_per = 0, uint8_t* digits = nullptr) {
     if (n_out) *n_out = n;
     if (n == 0) return false;
     int passes = end_bit > begin_bit ? (end_bit - begin_bit + 7) / 8 : 0;
@@ -2024,7 +2027,8 @@ struct wj_index {
       auto up = [&] {
         WJ_CUDA_CHECK(cudaMemsetAsync(h1, 0, (size_t)256 * G * 4, st));
         const uint32_t GU = G * kRsUpSplit;
-        if (holes && masked) k_rs_up<K, true, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, n_dev);
+        if (digits) k_rs_up_bytes<<<GU, 256, 0, st>>>(digits, cur_n, per, h1);  // this pass's digit bytes
+        else if (holes && masked) k_rs_up<K, true, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, n_dev);
         else if (holes) k_rs_up<K, true, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, n_dev);
         else if (masked) k_rs_up<K, false, true><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, n_dev);
         else k_rs_up<K, false, false><<<GU, 256, 0, st>>>(ki, cur_n, per, shift, mp, h1, kmask, n_dev);
@@ -2041,8 +2045,9 @@ struct wj_index {
                                                                               n_dev, head_cnt, head_per);
             k_head_fix<K><<<grid_for((uint64_t)256 * G, 256), 256, 0, st>>>(ko, h2, 256 * G, head_cnt, head_per);
             launched();
-          } else {
-            k_rs_down2<K, false, false, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
+          } else {  // (digits: write the next pass's digit bytes)
+            k_rs_down2<K, false, false, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev,
+                                                                        nullptr, 0, digits);
           }
         } else if (holes && masked) k_rs_down2<K, true, true><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);
         else if (holes) k_rs_down2<K, true, false><<<G, kDsThreads, sm, st>>>(ki, vi, ko, vo, cur_n, per, shift, h2, kmask, n_dev);

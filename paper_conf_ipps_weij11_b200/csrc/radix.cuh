@@ -177,6 +177,40 @@ __global__ void __launch_bounds__(256) k_rs_up(K* keys, uint64_t n, uint64_t per
   if (t) atomicAdd(&hist[(uint64_t)threadIdx.x * n_ranges + range], t);
 }
 
+// Upsweep over a digit byte array (the packed stream's passes: the emit kernel / the previous downsweep
+// wrote each element's digit of this pass as one byte at the element's position): reads 1 B per element
+// instead of the 8-byte element.  Same ranges and histogram layout as k_rs_up.
+__global__ void __launch_bounds__(256) k_rs_up_bytes(const uint8_t* __restrict__ dig, uint64_t n, uint64_t per,
+                                                     uint32_t* hist) {
+  __shared__ uint32_t h[kOsWarps][256];
+  const int w = threadIdx.x >> 5;
+  for (int x = 0; x < kOsWarps; ++x) h[x][threadIdx.x] = 0;
+  __syncthreads();
+  const uint32_t range = blockIdx.x / kRsUpSplit, part = blockIdx.x % kRsUpSplit;
+  const uint32_t n_ranges = gridDim.x / kRsUpSplit;
+  const uint64_t sub = per / kRsUpSplit;  // a multiple of 1024: 16-byte aligned parts
+  const uint64_t rhi = (uint64_t)range * per + per < n ? (uint64_t)range * per + per : n;
+  const uint64_t lo0 = (uint64_t)range * per + part * sub;
+  const uint64_t lo = lo0 < rhi ? lo0 : rhi;
+  const uint64_t hi = (part + 1 == kRsUpSplit) ? rhi : (lo0 + sub < rhi ? lo0 + sub : rhi);
+  const uint64_t nvec = (hi - lo) / 16;
+  const uint4* vp = (const uint4*)(dig + lo);
+  for (uint64_t v = threadIdx.x; v < nvec; v += 256) {
+    const uint4 x = __ldcs(vp + v);
+    const uint32_t wd[4] = {x.x, x.y, x.z, x.w};
+#pragma unroll
+    for (int q = 0; q < 4; ++q)
+#pragma unroll
+      for (int b = 0; b < 4; ++b) atomicAdd(&h[w][(wd[q] >> (8 * b)) & 255u], 1u);
+  }
+  for (uint64_t i = lo + nvec * 16 + threadIdx.x; i < hi; i += 256) atomicAdd(&h[w][dig[i]], 1u);
+  __syncthreads();
+  uint32_t t = 0;
+#pragma unroll
+  for (int x = 0; x < kOsWarps; ++x) t += h[x][threadIdx.x];
+  if (t) atomicAdd(&hist[(uint64_t)threadIdx.x * n_ranges + range], t);
+}
+
 // Downsweep v2: 512 threads x 8 items (tile 4096); the tile is never copied inside shared memory:
 // ranks produce an inverse permutation (u16) and the write-out gathers keys/values from the TMA
 // stage through it, so keys/values need no registers across barriers (occupancy: 32 warps/SM).
@@ -211,7 +245,8 @@ __global__ void WJ_DS_BOUNDS k_rs_down2(const K* __restrict__ kin, const uint32_
                                                          K* __restrict__ kout, uint32_t* __restrict__ vout, uint64_t n,
                                                          uint64_t per, int shift, const uint32_t* __restrict__ offs,
                                                          K kmask, const uint32_t* __restrict__ n_dev,
-                                                         uint32_t* __restrict__ rcnt = nullptr, uint32_t rper = 0) {
+                                                         uint32_t* __restrict__ rcnt = nullptr, uint32_t rper = 0,
+                                                         uint8_t* __restrict__ dnext = nullptr) {
   if (n_dev) {
     n = min(n, (uint64_t)*n_dev);
     per = rs_per(n, gridDim.x);
@@ -367,6 +402,7 @@ __global__ void WJ_DS_BOUNDS k_rs_down2(const K* __restrict__ kin, const uint32_
         const uint32_t pos = dig_glob[(uint32_t)((rs_dkey<K, MASK>(kk, kmask) >> shift) & 255u)] + j;
         kout[pos] = kk;
         if (!NOVAL) vout[pos] = sv[li];
+        if (NOVAL && dnext) dnext[pos] = (uint8_t)(kk >> (shift + 8));  // the next pass's digit
       }
     }
     if (HEADS && threadIdx.x < 256) {  // this tile's last element of each digit (or the earlier carry)

@@ -54,6 +54,7 @@ struct EmitOut {
   uint32_t* slot;          // per kept token: slot | 1 << 25 (key 0 = hole: a hot token, HOT only)
   uint32_t* doc;           // per kept token: global DocID
   unsigned long long* elem;  // or (packed stream, no HOT): per kept token slot << 32 | global DocID
+  uint8_t* dig0;           // packed stream: per kept token the first radix pass's digit (slot & 255)
   uint32_t* dbg_start;     // optional (debug): token start
   uint32_t* dbg_len;       // optional (debug): token length
   uint32_t* overflow;      // set to 1 if a probe sequence exceeded the limit
@@ -522,6 +523,7 @@ __global__ void __launch_bounds__(kTokThreads, HOT ? WJ_EMIT_HOT_MINB : WJ_EMIT_
         // branch-free stores: stream element slot | count 1 << 25, or a hole (the docID is not read)
         if (!HOT && eo.elem) {  // one 8-byte store: the sort moves (slot, docID) as one u64 key
           __stcs(eo.elem + out, ((unsigned long long)slot << 32) | (eo.doc_base + ldoc));
+          eo.dig0[out] = (uint8_t)slot;
         } else {
           __stcs(eo.slot + out, (HOT && hid) ? 0u : (slot | (1u << 25)));
           __stcs(eo.doc + out, eo.doc_base + ldoc);
