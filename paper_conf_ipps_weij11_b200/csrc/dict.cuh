@@ -391,7 +391,8 @@ __global__ void k_tie_fix(const uint64_t* key, uint32_t* val, uint32_t N, const 
 __global__ void k_new_terms(uint32_t U, const uint32_t* aoff, uint64_t arena_base, const uint8_t* text,
                             const uint4* u_w, const uint32_t* u_ref, const uint32_t* u_len, const uint32_t* u_bucket,
                             const uint32_t* u_cache, uint32_t* u_tid, const uint32_t* miss_idx, uint32_t V0,
-                            uint8_t* arena, uint32_t* t_arena, uint32_t* t_cache, uint32_t* t_bucket) {
+                            uint8_t* arena, uint32_t* t_arena, uint32_t* t_cache, uint32_t* t_bucket,
+                            const uint32_t* u_rank, uint4* u_pack) {
   const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
   if (u >= U || u_tid[u] != kMiss) return;
   const uint32_t tid = V0 + miss_idx[u];
@@ -404,6 +405,8 @@ __global__ void k_new_terms(uint32_t U, const uint32_t* aoff, uint64_t arena_bas
   t_cache[tid] = u_cache[u];
   t_bucket[tid] = b;
   u_tid[u] = tid;
+  // what k_ns_fill gathers in sorted order, as one 16-byte line (one sector per gathered term)
+  u_pack[u] = make_uint4(tid, b | u_len[u] << 16, u_rank[u], (uint32_t)off);
 }
 
 // E (the per-collection sorted key order) carries, besides termIDs, each term's arena offset and
@@ -411,18 +414,16 @@ __global__ void k_new_terms(uint32_t U, const uint32_t* aoff, uint64_t arena_bas
 __host__ __device__ __forceinline__ uint32_t e_info(uint32_t bucket, uint32_t full_len) { return bucket | full_len << 16; }
 __host__ __device__ __forceinline__ uint32_t e_info_bucket(uint32_t info) { return info & 0xFFFFu; }
 
-__global__ void k_ns_fill(const uint32_t* sorted_u, uint32_t N, const uint32_t* u_tid, const uint32_t* u_bucket,
-                          const uint32_t* u_rank, const uint32_t* u_len, const uint32_t* aoff, uint64_t arena_base,
-                          uint32_t* ns_tid, uint32_t* ns_bucket, uint32_t* ns_rank, uint32_t* ns_info, uint32_t* ns_arena) {
+__global__ void k_ns_fill(const uint32_t* sorted_u, uint32_t N, const uint4* __restrict__ u_pack, uint32_t* ns_tid,
+                          uint32_t* ns_bucket, uint32_t* ns_rank, uint32_t* ns_info, uint32_t* ns_arena) {
   const uint32_t k = blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= N) return;
-  const uint32_t u = sorted_u[k];
-  ns_tid[k] = u_tid[u];
-  const uint32_t b = u_bucket[u];
-  ns_bucket[k] = b;
-  ns_rank[k] = u_rank[u];
-  ns_info[k] = e_info(b, u_len[u]);
-  ns_arena[k] = (uint32_t)(arena_base + aoff[u]);
+  const uint4 x = u_pack[sorted_u[k]];  // {tid, e_info(bucket, full length), insertion rank, arena offset}
+  ns_tid[k] = x.x;
+  ns_bucket[k] = e_info_bucket(x.y);
+  ns_rank[k] = x.z;
+  ns_info[k] = x.y;
+  ns_arena[k] = x.w;
 }
 
 // per-collection [lo, hi) of the sorted new terms

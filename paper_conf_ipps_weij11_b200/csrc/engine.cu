@@ -253,6 +253,7 @@ struct wj_index {
   cudaEvent_t ev_fork = nullptr, ev_side = nullptr, ev_dict = nullptr;
   DevBuf side_scan, side_hist, side_hist_scan;
   DevBuf mr_key, mr_idx, mr_key2, mr_idx2, mr_dst, mr_src;  // several runs: records in destination order
+  DevBuf u_pack;  // per unique term {tid, info, insertion rank, arena offset} for k_ns_fill
   DevBuf pc_dig;  // packed stream: one digit byte per element for the next radix pass's upsweep
   DevBuf pc_key, pc_doc, pc_po, pc_cs, u_slot, pp_pair, x_pair, rec_tid, rec_start, rec_df, rec_cf, rec_aos, rec_before, df_totb,
       cf_totb;
@@ -377,7 +378,7 @@ struct wj_index {
                      &table_s, &uid_s, &st_off, &st_text, &st_keep, &st_tidx, &st_m1, &st_slot, &st_doc, &st_tiles,
                      &st_doff, &stop_keys, &side_scan, &side_hist, &side_hist_scan, &pc_key, &pc_doc, &pc_po,
                      &pc_cs, &u_slot, &pp_pair, &x_pair, &mr_key, &mr_idx, &mr_key2, &mr_idx2, &mr_dst, &mr_src, &rec_tid, &rec_start, &rec_df, &rec_cf, &rec_aos, &rec_before, &df_totb,
-                     &cf_totb, &pc_dig};
+                     &cf_totb, &pc_dig, &u_pack};
     for (DevBuf* b : all) {
       dev_free(b->p);
       b->p = nullptr;
@@ -1878,13 +1879,12 @@ struct wj_index {
     k_new_terms<<<grid_for(U, 256), 256, 0, st>>>((uint32_t)U, ao, arena_used, text, (const uint4*)u_w.p,
                                                   (const uint32_t*)u_ref.p, (const uint32_t*)u_len.p,
                                                   (const uint32_t*)u_bucket.p, (const uint32_t*)u_cache.p,
-                                                  (uint32_t*)u_tid.p, (const uint32_t*)midx.p, V, ar, ta, tc, tb);
+                                                  (uint32_t*)u_tid.p, (const uint32_t*)midx.p, V, ar, ta, tc, tb,
+                                                  (const uint32_t*)u_rank.p, buf<uint4>(u_pack, U));
     launched();
     uint32_t* ni = buf<uint32_t>(ns_info, Nn);
     uint32_t* na = buf<uint32_t>(ns_arena, Nn);
-    k_ns_fill<<<grid_for(Nn, 256), 256, 0, st>>>(sv, (uint32_t)Nn, (const uint32_t*)u_tid.p,
-                                                 (const uint32_t*)u_bucket.p, (const uint32_t*)u_rank.p,
-                                                 (const uint32_t*)u_len.p, ao, arena_used, nt, nb, nr, ni, na);
+    k_ns_fill<<<grid_for(Nn, 256), 256, 0, st>>>(sv, (uint32_t)Nn, (const uint4*)u_pack.p, nt, nb, nr, ni, na);
     launched();
     if (defer) arena_pending = true;
     else arena_used += A;
