@@ -1846,14 +1846,9 @@ struct wj_index {
     k_miss_compact<<<grid_for(U, 256), 256, 0, st>>>((const uint32_t*)u_tid.p, (const uint32_t*)midx.p,
                                                      (const uint64_t*)u_key.p, (uint32_t)U, kk, kv);
     launched();
-    // sort new terms by (collection, suffix): 8-bit LSD over the kSortKeyBits-bit key, then tie runs
-    const bool in2 = sort_pairs<uint64_t>(kk, kv, kk2, kv2, Nn, 0, kSortKeyBits, nullptr, false);
-    uint64_t* sk = in2 ? kk2 : kk;
-    uint32_t* sv = in2 ? kv2 : kv;
-    k_tie_fix<<<grid_for(Nn, 256), 256, 0, st>>>(sk, sv, (uint32_t)Nn, text, (const uint4*)u_w.p, (const uint32_t*)u_ref.p,
-                                                 (const uint32_t*)u_len.p);
-    launched();
-    // arena offsets, in unique order (only misses take space)
+    // arena offsets, in unique order (only misses take space); the new terms' columns and arena bytes
+    // need no sorted order, so they go ahead of the sort (the dictionary stream's tail is the step's
+    // critical path once the side stream is done)
     uint32_t* ao = buf<uint32_t>(aoff, U);
     scan<uint32_t>(ArenaSizeU{(const uint32_t*)u_tid.p, (const uint32_t*)u_len.p, (const uint32_t*)u_bucket.p}, U, ao,
                    (uint32_t*)(dscal() + 4));
@@ -1881,6 +1876,13 @@ struct wj_index {
                                                   (const uint32_t*)u_bucket.p, (const uint32_t*)u_cache.p,
                                                   (uint32_t*)u_tid.p, (const uint32_t*)midx.p, V, ar, ta, tc, tb,
                                                   (const uint32_t*)u_rank.p, buf<uint4>(u_pack, U));
+    launched();
+    // sort new terms by (collection, suffix): 8-bit LSD over the kSortKeyBits-bit key, then tie runs
+    const bool in2 = sort_pairs<uint64_t>(kk, kv, kk2, kv2, Nn, 0, kSortKeyBits, nullptr, false);
+    uint64_t* sk = in2 ? kk2 : kk;
+    uint32_t* sv = in2 ? kv2 : kv;
+    k_tie_fix<<<grid_for(Nn, 256), 256, 0, st>>>(sk, sv, (uint32_t)Nn, text, (const uint4*)u_w.p, (const uint32_t*)u_ref.p,
+                                                 (const uint32_t*)u_len.p);
     launched();
     uint32_t* ni = buf<uint32_t>(ns_info, Nn);
     uint32_t* na = buf<uint32_t>(ns_arena, Nn);
