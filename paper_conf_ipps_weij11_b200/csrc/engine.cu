@@ -1148,19 +1148,8 @@ struct wj_index {
       // holes (hot tokens, key 0) are dropped by the first pass; the count left stays on the device
       // (*ns_dev) and the later passes and the run-length pass are launched for the upper bound Nc
       uint32_t* ns_dev = hot ? (uint32_t*)(dscal() + 13) : nullptr;
-      if (packed) {  // value-less 64-bit keys, digits from the slot bits (32 ..)
-        unsigned long long* e0 = (unsigned long long*)pc_key.p;
-        // the last radix pass counts the run-length heads per warp range of the run-length pass
-        uint64_t rper;
-        uint32_t rgrid, Wg;
-        rlw_geometry(Nc, rper, rgrid, Wg);
-        uint32_t* rc = buf<uint32_t>(rle_p0, (uint64_t)Wg + 1);
-        WJ_CUDA_CHECK(cudaMemsetAsync(rc, 0, ((size_t)Wg + 1) * 4, st));
-        const bool in1 = sort_pairs<uint64_t>((uint64_t*)e0, nullptr, (uint64_t*)e1, nullptr, Nc, 32,
-                                              32 + std::max(bits, 1), nullptr, true, nullptr, ~0ull, false, nullptr,
-                                              true, nullptr, nullptr, rc, (uint32_t)rper, (uint8_t*)pc_dig.p);
-        phase(WJ_PHASE_POSTINGS);
-        rle(nullptr, nullptr, Nc, false, nullptr, nullptr, po, cs, nullptr, pp + pbase, in1 ? e1 : e0, true);
+      if (packed) {
+        sort_rle_packed(Nc, bits, e1, po, cs, pp + pbase);
       } else {
         const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, bits, nullptr, true, nullptr, kRankMask, hot, nullptr,
                                               true, nullptr, ns_dev);
@@ -1204,6 +1193,23 @@ struct wj_index {
     pc_U = U;
     pc_Nc = Nc;
     pc_hot = hot;
+  }
+
+  // The packed chunk stream (pc_key, Nc elements of C <= 2^bits slots) sorted by slot and run-length
+  // encoded into partial lists at pp: value-less 64-bit radix passes (digits from bit 32, upsweeps over
+  // the digit bytes in pc_dig), the last pass counting the run-length heads per warp range
+  void sort_rle_packed(uint64_t Nc, int bits, unsigned long long* e1, uint64_t* po, uint64_t* cs, uint2* pp) {
+    unsigned long long* e0 = (unsigned long long*)pc_key.p;
+    uint64_t rper;
+    uint32_t rgrid, Wg;
+    rlw_geometry(Nc, rper, rgrid, Wg);
+    uint32_t* rc = buf<uint32_t>(rle_p0, (uint64_t)Wg + 1);
+    WJ_CUDA_CHECK(cudaMemsetAsync(rc, 0, ((size_t)Wg + 1) * 4, st));
+    const bool in1 = sort_pairs<uint64_t>((uint64_t*)e0, nullptr, (uint64_t*)e1, nullptr, Nc, 32, 32 + std::max(bits, 1),
+                                          nullptr, true, nullptr, ~0ull, false, nullptr, true, nullptr, nullptr, rc,
+                                          (uint32_t)rper, (uint8_t*)pc_dig.p);
+    phase(WJ_PHASE_POSTINGS);
+    rle(nullptr, nullptr, Nc, false, nullptr, nullptr, po, cs, nullptr, pp, in1 ? e1 : e0, true);
   }
 
   // Join the last chunk's side-stream work and write its records; runs before the next chunk's
@@ -1416,11 +1422,14 @@ struct wj_index {
     uint32_t *lslot = nullptr, *ldoc = nullptr;
     if (nd > 0 && n_bytes > 0) {
       ChunkView cv{text, n_bytes, off, nd};
+      emit_elem = nullptr;
       Nc = tokenize_dedup(cv, (uint32_t)base, [&](uint64_t nc, uint32_t*& sp, uint32_t*& dp) {
         if (nc > 0xFFFFFFFFull) throw StatusError{WJ_ERR_CAPACITY, "more than 2^32-1 tokens in one chunk"};
-        sp = buf<uint32_t>(pc_key, nc + 16);
-        dp = buf<uint32_t>(pc_doc, nc + 16);
+        emit_elem = buf<unsigned long long>(pc_key, nc + 16);  // the packed stream (chunk_partials)
+        buf<uint8_t>(pc_dig, nc + 64);
+        sp = dp = nullptr;
       }, C, U, lslot, ldoc, false, (uint32_t)K);  // table partitioned by owner (slot order = owner order)
+      emit_elem = nullptr;
     }
     std::vector<uint64_t> t_off(K + 1, 0), b_off(K + 1, 0), p_off(K + 1, 0), c_off(K + 1, 0);
     uint8_t* send_terms = (uint8_t*)grow(x_send, 16);
@@ -1488,10 +1497,7 @@ struct wj_index {
     if (U > 0) {
       int bits = 0;
       while (bits < 32 && ((uint64_t)1 << bits) < C) ++bits;
-      uint32_t* kt = (uint32_t*)pc_key.p;
-      uint32_t* dt = (uint32_t*)pc_doc.p;
-      uint32_t* k1 = buf<uint32_t>(sk1, Nc + 16);
-      uint32_t* v1 = buf<uint32_t>(sv1, Nc + 16);
+      unsigned long long* e1 = buf<unsigned long long>(sk1, Nc + 16);
       uint64_t* po = buf<uint64_t>(pc_po, C + 1);
       uint64_t* cs = buf<uint64_t>(pc_cs, C + 1);
       WJ_CUDA_CHECK(cudaMemcpyAsync(us, u_slot.p, U * 4, cudaMemcpyDeviceToDevice, st));
@@ -1501,9 +1507,7 @@ struct wj_index {
       swap_side();
       try {
         phase(WJ_PHASE_SORT);
-        const bool in1 = sort_pairs<uint32_t>(kt, dt, k1, v1, Nc, 0, std::max(bits, 1), nullptr, true);
-        phase(WJ_PHASE_POSTINGS);
-        rle(in1 ? k1 : kt, in1 ? v1 : dt, Nc, false, nullptr, nullptr, po, cs, nullptr, opp);
+        sort_rle_packed(Nc, bits, e1, po, cs, opp);
         k_term_hdr<<<grid_for(U, 256), 256, 0, st>>>(us, (uint32_t)U, po, cs, (const uint32_t*)(dscal() + 8), Nc, hdf, hcf);
         k_owner_bounds<<<grid_for(K + 1, 256), 256, 0, st>>>(us, po, cs, toff_d, (uint32_t)K, (uint32_t)U,
                                                             (const uint32_t*)(dscal() + 8), Nc, bnd, bnd + K + 1);
