@@ -2097,7 +2097,8 @@ struct wj_index {
       sync();
       TB = h_scal[9];
       uint8_t* tbp = buf<uint8_t>(term_bytes, TB);
-      k_term_bytes<<<grid_for(V, 256), 256, 0, st>>>(ta, V, (const uint8_t*)arena.p, to, tbp);
+      k_term_bytes<<<(unsigned)std::min<uint64_t>(grid_for(V, 256), 148ull * 2), 256, 0, st>>>(  // 2 CTAs per SM
+          ta, V, (const uint8_t*)arena.p, to, tbp);
       launched();
     } else {
       WJ_CUDA_CHECK(cudaMemsetAsync(to, 0, 8, st));

@@ -595,15 +595,17 @@ struct TermFullLen {  // full length of the term of rank r (rank_info written by
 };
 
 // final dictionary bytes: trie prefix (restored) + stored suffix
+// (grid-stride: launched with a few CTAs per SM, so that the finalize copy of the postings, queued right
+// after it on the other stream, runs beside it instead of behind it)
 __global__ void k_term_bytes(const uint2* rank_info, uint32_t V, const uint8_t* arena, const uint64_t* term_off,
                              uint8_t* out) {
-  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r >= V) return;
-  const uint2 ri = rank_info[r];
-  const uint32_t b = ri.y & 0xFFFFu, plen = bucket_plen(b), a = ri.x, slen = (ri.y >> 16) - plen;
-  uint8_t* o = out + term_off[r];
-  for (uint32_t i = 0; i < plen; ++i) o[i] = (uint8_t)prefix_byte(b, i);
-  for (uint32_t i = 0; i < slen; ++i) o[plen + i] = arena[a + 1 + i];
+  for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < V; r += gridDim.x * blockDim.x) {
+    const uint2 ri = rank_info[r];
+    const uint32_t b = ri.y & 0xFFFFu, plen = bucket_plen(b), a = ri.x, slen = (ri.y >> 16) - plen;
+    uint8_t* o = out + term_off[r];
+    for (uint32_t i = 0; i < plen; ++i) o[i] = (uint8_t)prefix_byte(b, i);
+    for (uint32_t i = 0; i < slen; ++i) o[plen + i] = arena[a + 1 + i];
+  }
 }
 
 // ------------------------------------------------------------------ debug token dump
