@@ -249,8 +249,10 @@ struct wj_index {
   // pass reads it back (one 8-byte access per element everywhere instead of two 4-byte ones)
   unsigned long long* emit_elem = nullptr;
   bool pc_packed = false;
+  bool side_launched = false;  // the current chunk's side-stream work is enqueued (side_launch)
   cudaStream_t side_st = nullptr, hp_st = nullptr;  // side: lowest priority; hp: dictionary, highest
   cudaEvent_t ev_fork = nullptr, ev_side = nullptr, ev_dict = nullptr;
+  cudaEvent_t ev_dfork = nullptr;  // the dictionary stream's fork (after the unique terms are gathered)
   DevBuf side_scan, side_hist, side_hist_scan;
   DevBuf mr_key, mr_idx, mr_key2, mr_idx2, mr_dst, mr_src;  // several runs: records in destination order
   DevBuf u_pack;  // per unique term {tid, info, insertion rank, arena offset} for k_ns_fill
@@ -500,6 +502,7 @@ struct wj_index {
     pbase = nrec = 0;
     pm_merged = 0;
     pc_pending = pc_join = false;
+    side_launched = false;
     rec_end.clear();
     unique_last = new_last = n_nodes = height_max = 0;
     btree_dirty = false;
@@ -817,6 +820,7 @@ struct wj_index {
         launched();
       }
       emit_tokens(cv, n_segs, slot_out, doc_out, doc_base, C, nullptr, nullptr, hot_H > 0, false);
+      if (pc_packed && Nc > 0) side_launch(Nc, C, false);  // the sort needs the stream only
       phase(WJ_PHASE_UNIQUE);
       slot_uid = buf<uint32_t>(uid, C);
       scan<uint32_t>(NonZeroSlot{(const Slot*)table.p}, C, slot_uid, (uint32_t*)(dscal() + 2));
@@ -824,7 +828,12 @@ struct wj_index {
       readback(2, 4);
       U = (uint32_t)h_scal[2];
       if (((uint32_t)h_scal[5]) == 0) break;
-      // probe sequence overflow: retry with a larger table
+      // probe sequence overflow: retry with a larger table (an early-forked sort reads the stream the
+      // retry rewrites: drained first, then forked again)
+      if (side_launched) {
+        WJ_CUDA_CHECK(cudaStreamSynchronize(side_st));
+        side_launched = false;
+      }
       if (C >= kMaxC / parts * parts) {
         tab_parts = 1;
         throw StatusError{WJ_ERR_CAPACITY, "more than ~2^25 distinct terms in one index_add_stream call: pass smaller chunks"};
@@ -1124,10 +1133,39 @@ struct wj_index {
   // st; then one record per unique term.
   // hot: the stream holds merged hot-term elements (counts) and holes (hot.cuh)
   void chunk_partials(const uint8_t* text, uint64_t Nc, uint64_t C, uint64_t U, bool hot) {
-    settle_partials();  // the previous chunk is joined (add_chunk), its posting count read here
     // the first chunk into an empty dictionary: every unique term is new and takes termID = its unique
     // index (k_new_terms), so its records (k_chunk_records, record u = unique term u) are indexed by termID
     recs_by_tid = nrec == 0 && V == 0 && !hot;
+    if (!side_launched) side_launch(Nc, C, hot);
+    side_launched = false;
+    // the dictionary update (latency-bound small kernels with host round trips) on a high-priority
+    // stream, so its CTAs are scheduled ahead of the side stream's whenever SMs free up; it forks here,
+    // after the unique terms it reads are gathered (the side stream may have forked at the emit kernel)
+    WJ_CUDA_CHECK(cudaEventRecord(ev_dfork, st));
+    WJ_CUDA_CHECK(cudaStreamWaitEvent(hp_st, ev_dfork, 0));
+    std::swap(st, hp_st);
+    try {
+      dictionary_update(text, U);
+      phase(-1);
+      WJ_CUDA_CHECK(cudaEventRecord(ev_dict, st));
+    } catch (...) {
+      std::swap(st, hp_st);
+      throw;
+    }
+    std::swap(st, hp_st);
+    WJ_CUDA_CHECK(cudaStreamWaitEvent(st, ev_dict, 0));
+    pc_join = true;
+    pc_U = U;
+    pc_Nc = Nc;
+    pc_hot = hot;
+  }
+
+  // The chunk's stream sorted by slot and run-length encoded on side_st (forked from st here).  The packed
+  // path forks right after the emit kernel (tokenize_dedup), ahead of the unique-term scan and gather,
+  // which the sort does not need.
+  void side_launch(uint64_t Nc, uint64_t C, bool hot) {
+    settle_partials();  // the previous chunk is joined (add_chunk), its posting count read here
+    side_launched = true;
     const bool packed = pc_packed;
     uint32_t* kt = (uint32_t*)pc_key.p;
     uint32_t* dt = (uint32_t*)pc_doc.p;
@@ -1175,24 +1213,6 @@ struct wj_index {
       throw;
     }
     swap_side();
-    // the dictionary update (latency-bound small kernels with host round trips) on a high-priority
-    // stream, so its CTAs are scheduled ahead of the side stream's whenever SMs free up
-    WJ_CUDA_CHECK(cudaStreamWaitEvent(hp_st, ev_fork, 0));
-    std::swap(st, hp_st);
-    try {
-      dictionary_update(text, U);
-      phase(-1);
-      WJ_CUDA_CHECK(cudaEventRecord(ev_dict, st));
-    } catch (...) {
-      std::swap(st, hp_st);
-      throw;
-    }
-    std::swap(st, hp_st);
-    WJ_CUDA_CHECK(cudaStreamWaitEvent(st, ev_dict, 0));
-    pc_join = true;
-    pc_U = U;
-    pc_Nc = Nc;
-    pc_hot = hot;
   }
 
   // The packed chunk stream (pc_key, Nc elements of C <= 2^bits slots) sorted by slot and run-length
@@ -2461,6 +2481,7 @@ int index_init(wj_index** out, const wj_config* cfg) {
       WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->ev_fork, cudaEventDisableTiming));
       WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->ev_side, cudaEventDisableTiming));
       WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->ev_dict, cudaEventDisableTiming));
+      WJ_CUDA_CHECK(cudaEventCreateWithFlags(&ix->ev_dfork, cudaEventDisableTiming));
     }
     if (cfg->world > 1 || cfg->nccl_unique_id) {  // a transport at world 1 runs the same distributed path
       try {
@@ -2868,6 +2889,7 @@ void index_destroy(wj_index* ix) {
     cudaStreamDestroy(ix->hp_st);
   }
   if (ix->ev_dict) cudaEventDestroy(ix->ev_dict);
+  if (ix->ev_dfork) cudaEventDestroy(ix->ev_dfork);
   if (ix->ev_fork) cudaEventDestroy(ix->ev_fork);
   if (ix->ev_side) cudaEventDestroy(ix->ev_side);
   delete ix->xport;
