@@ -411,11 +411,20 @@ struct wj_index {
   }
 
   // ---------------------------------------------------------------- launch bookkeeping
+#ifdef WJ_DEBUG_LAUNCH  // debug build: every launch synchronised, a fault reported with its call site
+  void launched(int n = 1, int line = __builtin_LINE()) {
+    launches += n;
+    cudaError_t e = cudaDeviceSynchronize();
+    if (e == cudaSuccess) e = cudaGetLastError();
+    if (e != cudaSuccess) throw CudaError(e, "kernel launch", __FILE__, line);
+  }
+#else
   void launched(int n = 1) {
     launches += n;
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) throw CudaError(e, "kernel launch", __FILE__, __LINE__);
   }
+#endif
   void sync() {
     WJ_CUDA_CHECK(cudaStreamSynchronize(st));
     ++syncs;

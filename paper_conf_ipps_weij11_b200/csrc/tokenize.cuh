@@ -522,8 +522,11 @@ __global__ void __launch_bounds__(kTokThreads, HOT ? WJ_EMIT_HOT_MINB : WJ_EMIT_
         }
         // branch-free stores: stream element slot | count 1 << 25, or a hole (the docID is not read)
         if (!HOT && eo.elem) {  // one 8-byte store: the sort moves (slot, docID) as one u64 key
-          __stcs(eo.elem + out, ((unsigned long long)slot << 32) | (eo.doc_base + ldoc));
-          eo.dig0[out] = (uint8_t)slot;
+          // (a probe-sequence overflow (kMiss) makes the host retry with a larger table; the sort forked
+          // early on this stream must still stay in bounds: slot 0 instead)
+          const uint32_t ps = slot == kMiss ? 0u : slot;
+          __stcs(eo.elem + out, ((unsigned long long)ps << 32) | (eo.doc_base + ldoc));
+          eo.dig0[out] = (uint8_t)ps;
         } else {
           __stcs(eo.slot + out, (HOT && hid) ? 0u : (slot | (1u << 25)));
           __stcs(eo.doc + out, eo.doc_base + ldoc);
