@@ -8,10 +8,10 @@ WJ_BENCH_FORCE_DIST=1 python -m torch.distributed.run --nnodes=1 --nproc-per-nod
 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/ref.json 2> gpurun_out/ref.err; head -c 300 gpurun_out/ref.json; echo
 timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv --log-file gpurun_out/launches.csv python bench.py --steps 2 --warmup 1 --e2e-steps 0 --no-cpu-baseline --steady-chunks 0 > /dev/null 2>&1
 python tools/launch_summary.py gpurun_out/launches.csv 1 --json gpurun_out/ncu_traffic.json --bmin 1976511937 > gpurun_out/launch_summary.txt 2>&1; head -14 gpurun_out/launch_summary.txt
-for k in k_tok_emit "k_rs_down2<unsigned.long,.false,.false,.true" k_rlw_write k_tok_count k_copy_by_rank; do
+for k in k_tok_emit "k_rs_down2<unsigned.long,..bool.0,..bool.0,..bool.1,..bool.0" k_rlw_write k_tok_count k_copy_by_rank; do
   n=$(echo $k | tr -c 'a-zA-Z0-9_\n' '_' | cut -c1-40)
   K="$k" NAME="e_$n" bash tools/ncu_one.sh > /dev/null 2>&1
   python tools/ncu_summary.py gpurun_out/e_$n.ncu-rep
 done
 python tools/trace_step.py > gpurun_out/trace_head.txt 2>/dev/null; tail -1 gpurun_out/trace_head.txt
-TOOLS="memcheck racecheck synccheck" bash tools/call_sanitize.sh
+timeout 2400 python -m pytest tests -m gpu -q --timeout 900 > gpurun_out/t_full.log 2>&1; tail -2 gpurun_out/t_full.log
