@@ -71,8 +71,8 @@ __device__ __forceinline__ uint32_t tokmask4(uint32_t x) {
   const uint32_t ge0 = fma_add(lo, 0x50505050u);  // bit7: lo >= '0'
   const uint32_t le9 = ~fma_add(lo, 0x46464646u); // bit7: lo <  ':'
   const uint32_t l = lo | 0x20202020u;
-  const uint32_t gea = l + 0x1F1F1F1Fu;           // bit7: l >= 'a'
-  const uint32_t lez = ~(l + 0x05050505u);        // bit7: l <  '{'
+  const uint32_t gea = fma_add(l, 0x1F1F1F1Fu);   // bit7: l >= 'a'
+  const uint32_t lez = ~fma_add(l, 0x05050505u);  // bit7: l <  '{'
   const uint32_t t = (hi | ((ge0 & le9) | (gea & lez))) & 0x80808080u;
   // bits 7, 15, 23, 31 -> bits 0..3 in one multiply-high (no carries: the partial products are disjoint)
   return __umulhi(t, (1u << 25) | (1u << 18) | (1u << 11) | (1u << 4)) & 15u;
