@@ -65,6 +65,12 @@ __device__ __forceinline__ uint32_t fma_add(uint32_t a, uint32_t c) {
   asm("mad.lo.u32 %0, %1, 1, %2;" : "=r"(r) : "r"(a), "r"(c));
   return r;
 }
+// a * m + c as one multiply-add (FMA pipe)
+__device__ __forceinline__ uint32_t fma_mad(uint32_t a, uint32_t m, uint32_t c) {
+  uint32_t r;
+  asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(m), "r"(c));
+  return r;
+}
 __device__ __forceinline__ uint32_t tokmask4(uint32_t x) {
   const uint32_t hi = x & 0x80808080u;
   const uint32_t lo = x & 0x7F7F7F7Fu;

@@ -321,13 +321,14 @@ __device__ __forceinline__ uint32_t win_word(const uint32_t* win32, uint32_t s, 
 // kernel is instruction-bound).  First slot = mulhi(h, capacity) (any capacity, so the table can be
 // sized to the expected unique terms instead of the next power of two); the slot tag is a second mix.
 __device__ __forceinline__ uint32_t hash_init(uint32_t len) { return len * 0x9E3779B1u + 0x7F4A7C15u; }
-__device__ __forceinline__ uint32_t hash_mix(uint32_t h, uint32_t w) {
-  h = (h ^ w) * 0x85EBCA77u;
-  return h ^ (h >> 15);
-}
+// polynomial over the words (one multiply-add per word, FMA pipe; the xor-multiply-xorshift mix per word
+// cost 3 ALU instructions each: emit 2.39 -> 2.31 ms) + murmur3's 32-bit finaliser for the slot bits
+__device__ __forceinline__ uint32_t hash_mix(uint32_t h, uint32_t w) { return fma_mad(h, 0x85EBCA77u, w); }
 __device__ __forceinline__ uint32_t hash_fin(uint32_t h) {
+  h ^= h >> 16;
+  h *= 0x85EBCA6Bu;
   h ^= h >> 13;
-  h *= 0xC2B2AE3Du;
+  h *= 0xC2B2AE35u;
   return h ^ (h >> 16);
 }
 __device__ __forceinline__ uint32_t hash_tag(uint32_t h) { return (h * 0x9E3779B1u) >> 8; }
